@@ -1,0 +1,312 @@
+"""Pins of the FP64 oracle against things other than itself (CPU only).
+
+Each test names what fixes the expected value: a hand-computed fixture under
+tests/golden/ (with its citation), a value printed in PAPER.md, a closed form,
+an invariant, or an independent library routine (scipy / numpy).
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+from scipy import signal
+
+import synth
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _load(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+# ----------------------------------------------------------------- conv
+def test_conv_tiny_hand_computed(orc):
+    g = _load("conv_tiny.json")
+    x = np.array(g["x"], float)[None, None]
+    w = np.array(g["w"], float)[None, None]
+    for case in g["cases"]:
+        y = orc.conv2d(x, w, np.array([case["bias"]]), case["stride"],
+                       case["pad"], 1, False, threads=1)
+        np.testing.assert_array_equal(y[0, 0], np.array(case["y"], float))
+        y2 = orc.conv2d_im2col_gemm(x, w, np.array([case["bias"]]),
+                                    case["stride"], case["pad"], 1, False)
+        np.testing.assert_array_equal(y2[0, 0], np.array(case["y"], float))
+
+
+def test_conv_grouped_hand_computed(orc):
+    g = _load("conv_tiny.json")
+    x = np.stack([np.array(g["x"], float), np.array(g["grouped"]["x1"], float)])[None]
+    w = np.stack([np.array(g["w"], float), np.array(g["grouped"]["w1"], float)])[:, None]
+    y = orc.conv2d(x, w, np.zeros(2), 1, 0, 2, False, threads=1)
+    np.testing.assert_array_equal(y[0, 0], np.array(g["grouped"]["y0"], float))
+    np.testing.assert_array_equal(y[0, 1], np.array(g["grouped"]["y1"], float))
+
+
+def _scipy_conv(x, w, b, stride, pad, groups, relu):
+    """Independent reference: scipy.signal.correlate2d per (filter, channel)."""
+    B, C, H, W = x.shape
+    F, Cg, S, _ = w.shape
+    Fg = F // groups
+    xp = np.pad(x, ((0, 0), (0, 0), (pad, pad), (pad, pad)))
+    out = []
+    for n in range(B):
+        per_f = []
+        for f in range(F):
+            g = f // Fg
+            acc = 0.0
+            for c in range(Cg):
+                acc = acc + signal.correlate2d(xp[n, g * Cg + c], w[f, c], mode="valid")
+            acc = acc[::stride, ::stride] + b[f]
+            per_f.append(np.maximum(acc, 0) if relu else acc)
+        out.append(np.stack(per_f))
+    return np.stack(out)
+
+
+@pytest.mark.parametrize("shape", [
+    # B, C, H, W, F, S, stride, pad, groups
+    (2, 3, 9, 7, 4, 3, 1, 1, 1),
+    (1, 4, 11, 11, 6, 5, 2, 2, 2),
+    (2, 3, 15, 15, 2, 11, 4, 0, 1),
+    (1, 6, 6, 6, 6, 3, 1, 1, 3),
+])
+def test_conv_matches_scipy_and_fig2(orc, shape):
+    B, C, H, W, F, S, st, pad, g = shape
+    rng = np.random.default_rng(1)
+    x = rng.standard_normal((B, C, H, W))
+    w = rng.standard_normal((F, C // g, S, S))
+    b = rng.standard_normal(F)
+    for relu in (False, True):
+        y = orc.conv2d(x, w, b, st, pad, g, relu, threads=3)
+        ref = _scipy_conv(x, w, b, st, pad, g, relu)
+        assert y.shape == ref.shape
+        np.testing.assert_allclose(y, ref, rtol=1e-12, atol=1e-12)
+        y2 = orc.conv2d_im2col_gemm(x, w, b, st, pad, g, relu)
+        np.testing.assert_allclose(y, y2, rtol=1e-13, atol=1e-13)
+        if relu:
+            assert (y >= 0).all()
+
+
+def test_conv_thread_count_invariant(orc):
+    rng = np.random.default_rng(2)
+    x = rng.standard_normal((5, 4, 8, 8))
+    w = rng.standard_normal((6, 2, 3, 3))
+    b = rng.standard_normal(6)
+    y1 = orc.conv2d(x, w, b, 1, 1, 2, True, threads=1)
+    y8 = orc.conv2d(x, w, b, 1, 1, 2, True, threads=8)
+    np.testing.assert_array_equal(y1, y8)
+
+
+def test_output_sizes_pin_paper_shapes(orc):
+    p = _load("paper_pins.json")["alexnet_shapes"]
+    h = orc.conv_out_size(227, 11, 4, 0)
+    assert h == p["conv1"]
+    h = orc.pool_out_size(h, 3, 2)
+    assert h == p["pool1"]
+    h = orc.conv_out_size(h, 5, 1, 2)
+    assert h == p["conv2"]
+    h = orc.pool_out_size(h, 3, 2)
+    assert h == p["pool2"]
+    h = orc.conv_out_size(h, 3, 1, 1)
+    assert h == p["conv5"]
+    assert orc.pool_out_size(h, 3, 2) == p["pool5"]
+    # VGG: 224 -> 112 -> 56 -> 28 -> 14 -> 7 (2x2 s2 pools), 3x3 p1 convs keep size
+    h = 224
+    for _ in range(5):
+        assert orc.conv_out_size(h, 3, 1, 1) == h
+        h = orc.pool_out_size(h, 2, 2)
+    assert h == 7
+
+
+def test_alexnet_per_group_gemm_dims_table_iv(orc):
+    """T4: per-group GEMM N_f/g x W_oH_o of AlexNet at batch 1 (Table IV)."""
+    p = _load("paper_pins.json")["alexnet_per_group_gemm"]
+    net = synth.alexnet()
+    h = 227
+    ci = 0
+    for L in net["layers"]:
+        if L["kind"] == "conv":
+            h = orc.conv_out_size(h, L["k"], L["stride"], L["pad"])
+            ci += 1
+            assert [L["out"] // L["groups"], h * h] == p["conv%d" % ci]
+        elif L["kind"] == "maxpool":
+            h = orc.pool_out_size(h, L["k"], L["stride"])
+
+
+# ----------------------------------------------------------------- pool
+def test_maxpool_hand_computed(orc):
+    g = _load("conv_tiny.json")["maxpool"]
+    x = np.array(g["x"], float)[None, None]
+    y = orc.maxpool(x, 3, 2, threads=1)
+    np.testing.assert_array_equal(y[0, 0], np.array(g["y"], float))
+
+
+def test_avgpool_closed_forms(orc):
+    x = np.full((2, 3, 8, 8), 2.5)
+    np.testing.assert_array_equal(orc.avgpool(x, 2, 2), np.full((2, 3, 4, 4), 2.5))
+    x = np.arange(16, dtype=float).reshape(1, 1, 4, 4)
+    y = orc.avgpool(x, 2, 2)
+    np.testing.assert_allclose(y[0, 0], [[2.5, 4.5], [10.5, 12.5]])
+
+
+def test_maxpool_matches_numpy_reduce(orc):
+    rng = np.random.default_rng(3)
+    x = rng.standard_normal((2, 5, 8, 8))
+    y = orc.maxpool(x, 2, 2)
+    ref = x.reshape(2, 5, 4, 2, 4, 2).max(axis=(3, 5))
+    np.testing.assert_array_equal(y, ref)
+
+
+# ----------------------------------------------------------------- LRN
+@pytest.mark.parametrize("a", [1.0, 30.0, 128.0])
+def test_lrn_constant_input_closed_form(orc, a):
+    """Closed form on constant input: interior channels see 5 equal terms,
+    channel 0 / C-1 see 3, channel 1 / C-2 see 4 (Caffe window, reading R3)."""
+    C = 8
+    x = np.full((1, C, 2, 3), a)
+    y = orc.lrn(x, 5, 1e-4, 0.75, 1.0)
+    n_terms = [3, 4, 5, 5, 5, 5, 4, 3]
+    for c in range(C):
+        expect = a / (1.0 + 1e-4 / 5 * n_terms[c] * a * a) ** 0.75
+        np.testing.assert_allclose(y[0, c], expect, rtol=1e-14)
+
+
+def test_lrn_single_channel_spike(orc):
+    """A lone non-zero channel normalises itself only through its own square;
+    neighbours stay exactly zero."""
+    x = np.zeros((1, 6, 1, 1))
+    x[0, 2] = 10.0
+    y = orc.lrn(x, 5, 1e-4, 0.75, 2.0)
+    np.testing.assert_allclose(y[0, 2, 0, 0], 10.0 / (2.0 + 1e-4 / 5 * 100.0) ** 0.75, rtol=1e-14)
+    assert np.count_nonzero(y) == 1
+
+
+# ----------------------------------------------------------------- FC
+def test_fc_single_column_probe(orc):
+    N, K = 7, 12
+    w = np.zeros((N, K))
+    w[:, 5] = np.arange(1, N + 1)
+    x = np.arange(K, dtype=float)[None] + 1.0
+    b = np.full(N, -0.25)
+    y = orc.fc(x, w, b, relu=False)
+    np.testing.assert_array_equal(y[0], np.arange(1, N + 1) * 6.0 - 0.25)
+
+
+def test_fc_matches_numpy_matmul_and_chw_flatten(orc):
+    rng = np.random.default_rng(4)
+    x = rng.standard_normal((3, 4, 2, 5))
+    w = rng.standard_normal((9, 40))
+    b = rng.standard_normal(9)
+    y = orc.fc(x, w, b, relu=True)
+    ref = np.maximum(x.reshape(3, 40) @ w.T + b, 0)   # C,H,W flatten
+    np.testing.assert_allclose(y, ref, rtol=1e-13, atol=1e-13)
+
+
+# ----------------------------------------------------------------- softmax / entropy
+def test_entropy_paper_example(orc):
+    e = _load("paper_pins.json")["entropy_example"]
+    h1, h2 = orc.entropy(np.array(e["P1"])), orc.entropy(np.array(e["P2"]))
+    assert abs(h1 - e["H1"]) < 5e-5 and abs(h2 - e["H2"]) < 5e-5
+    assert h1 > h2
+
+
+def test_softmax_closed_forms(orc):
+    p, H = orc.softmax_entropy(np.zeros((2, 1000)))
+    np.testing.assert_allclose(p, 1e-3, rtol=1e-14)
+    np.testing.assert_allclose(H, math.log(1000.0), rtol=1e-12)   # 6.9078 (1000-term sum rounding)
+    p, H = orc.softmax_entropy(np.array([[0.0, math.log(2.0)]]))
+    np.testing.assert_allclose(p[0], [1 / 3, 2 / 3], rtol=1e-14)
+    rng = np.random.default_rng(5)
+    z = rng.standard_normal((4, 50)) * 20
+    p, H = orc.softmax_entropy(z)
+    np.testing.assert_allclose(p.sum(1), 1.0, rtol=1e-14)
+    p2, _ = orc.softmax_entropy(z + 1234.5)           # shift invariance
+    np.testing.assert_allclose(p, p2, rtol=1e-9)
+    # one-hot limit: H -> 0
+    _, H = orc.softmax_entropy(np.array([[0.0, 800.0, 0.0]]))
+    assert H[0] < 1e-300 or H[0] == 0.0
+
+
+# ----------------------------------------------------------------- rank-r
+def test_rank_r_against_numpy_svd(orc):
+    rng = np.random.default_rng(6)
+    Wm = rng.standard_normal((24, 40))
+    U, s, Vt = np.linalg.svd(Wm, full_matrices=False)
+    for r in (1, 5, 12, 24):
+        Wr, sig, uniq = orc.rank_r(Wm, r)
+        assert uniq
+        np.testing.assert_allclose(sig, s, rtol=1e-10, atol=1e-10)
+        ref = (U[:, :r] * s[:r]) @ Vt[:r]
+        np.testing.assert_allclose(Wr, ref, atol=1e-10)
+        # Eckart-Young: ||W - W_r||_F^2 = sum_{i>r} sigma_i^2
+        np.testing.assert_allclose(np.sum((Wm - Wr) ** 2), np.sum(s[r:] ** 2),
+                                   rtol=1e-9, atol=1e-9)
+    # full rank reproduces W
+    Wr, _, _ = orc.rank_r(Wm, 24)
+    np.testing.assert_allclose(Wr, Wm, atol=1e-12)
+
+
+def test_rank_r_exact_on_rank_one(orc):
+    u = np.arange(1.0, 9.0)
+    v = np.linspace(-1, 1, 13)
+    Wm = np.outer(u, v)
+    Wr, sig, _ = orc.rank_r(Wm, 1)
+    np.testing.assert_allclose(Wr, Wm, atol=1e-12)
+    assert sig[1] < 1e-6 * sig[0]
+
+
+def test_rank_r_conv_linearity(orc):
+    """conv with W_r == stage-1 conv (filters V_r^T) then 1x1 conv (U_r S_r):
+    the two-stage identity the CUDA variant uses (reading R7)."""
+    rng = np.random.default_rng(7)
+    x = rng.standard_normal((1, 4, 7, 7))
+    w = rng.standard_normal((6, 4, 3, 3))
+    b = rng.standard_normal(6)
+    r = 3
+    Wr, _ = orc.rank_r_conv_weight(w, 1, r)
+    y = orc.conv2d(x, Wr, b, 1, 1, 1, True)
+    U, s, Vt = np.linalg.svd(w.reshape(6, -1), full_matrices=False)
+    st1 = orc.conv2d(x, Vt[:r].reshape(r, 4, 3, 3), None, 1, 1, 1, False)
+    st2 = orc.conv2d(st1, (U[:, :r] * s[:r]).reshape(6, r, 1, 1), b, 1, 0, 1, True)
+    np.testing.assert_allclose(y, st2, rtol=1e-10, atol=1e-10)
+
+
+# ----------------------------------------------------------------- analytical models
+def test_table_v_util_all_cells(orc):
+    """T1: all 15 Util cells of Table V from eqs. 4 and 6 (reading R8)."""
+    pins = _load("paper_pins.json")
+    dims = pins["alexnet_per_group_gemm"]
+    for gpu, cfg in pins["table_v_util"].items():
+        if gpu.startswith("_"):
+            continue
+        for i, want in enumerate(cfg["util"]):
+            nf, wh = dims["conv%d" % (i + 1)]
+            G = orc.grid_size(nf, wh, cfg["tile_nf"], cfg["tile_wh"])
+            assert abs(orc.util(G, cfg["max_blocks"]) - want) < 0.006, (gpu, i)
+
+
+def test_table_iv_grid_and_max_blocks(orc):
+    """T2: Table IV grid sizes (eq. 4) and maxBlocks (eq. 5)."""
+    p = _load("paper_pins.json")
+    dims = p["alexnet_per_group_gemm"]
+    for name, t in p["table_iv"].items():
+        if name.startswith("_"):
+            continue
+        assert orc.max_blocks(t["n_sms"], 65536, t["block"], t["regs"]) == t["max_blocks"]
+        assert orc.grid_size(*dims["conv2"], t["tile_nf"], t["tile_wh"]) == t["grid_conv2"]
+        assert orc.grid_size(*dims["conv5"], t["tile_nf"], t["tile_wh"]) == t["grid_conv5"]
+
+
+def test_eq11_worked_example(orc):
+    e = _load("paper_pins.json")["eq11_example"]
+    assert orc.opt_sm(e["grid"], e["opt_tlp"], e["num_sms"]) == e["opt_sm"]
+    # eq. 8 consistency: optSM keeps the invocation count
+    assert orc.n_invocations(40, 3, 7) == orc.n_invocations(40, 3, 10) == 2
+
+
+def test_rec_eq9_closed_forms(orc):
+    assert orc.rec(256, 256, 128, 128) == 1.0
+    assert orc.rec(100, 128, 128, 128) == 100 / 128
+    assert abs(orc.rec(169, 128, 128, 128) - 169 / 256) < 1e-15
