@@ -1,0 +1,228 @@
+/*
+ * pcnn.h -- C ABI of the B200-native P-CNN batched-inference hot path.
+ *
+ * The operations are the ones PAPER.md (Song et al., HPCA'17) states as the
+ * problem (cited P:<line>):
+ *   - deploy a trained CNN without retraining
+ *   - execute inference: conv = im2col + GEMM (F_m x D_m)       P:53-61, Fig. 2
+ *     max-pooling and classifier layers
+ *     output probabilities and their entropy (eq. 2)
+ *   - choose per layer a faster, less precise kernel variant
+ *     (here: rank-r factorisation, north_star; R7)
+ *   - give each layer optSM SMs x optTLP CTAs
+ *
+ * Conventions for every function:
+ *   - Returns a pcnn_status; nothing throws across the ABI.  On failure a
+ *     thread-local message is available from pcnn_last_error_message().
+ *   - Layer indices are 0-based positions in the descriptor list.
+ *   - "host" pointers are ordinary CPU memory; "device" pointers are CUDA
+ *     device memory on the net's device.  The caller keeps ownership of every
+ *     pointer it passes; host weight/bias arrays are read during the call and
+ *     never retained.  The library owns packed weights, factor caches, the
+ *     activation arena and its CUDA graphs, all released by pcnn_destroy_net.
+ *   - Streams are passed as `void*` holding a cudaStream_t (NULL = legacy
+ *     default stream), so this header needs no CUDA headers.
+ *   - Argument and shape errors are reported synchronously, before anything
+ *     is enqueued.  Kernel launch failures return PCNN_ERR_CUDA; device faults
+ *     surface at the caller's next synchronisation (CUDA convention).
+ *   - A net is not re-entrant: at most one pcnn_infer* in flight per net, and
+ *     pcnn_set_* must not be called while one is in flight.
+ *   - There is no CPU fallback: every compute step runs in the library's CUDA
+ *     kernels for sm_100a; without a usable B200 pcnn_create_net fails with
+ *     PCNN_ERR_CUDA.
+ */
+#ifndef PCNN_H
+#define PCNN_H
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    PCNN_OK = 0,
+    PCNN_ERR_INVALID_ARGUMENT = 1,
+    PCNN_ERR_SHAPE = 2,
+    PCNN_ERR_UNSUPPORTED = 3,
+    PCNN_ERR_OUT_OF_MEMORY = 4,
+    PCNN_ERR_CUDA = 5,
+    PCNN_ERR_BATCH_TOO_LARGE = 6
+} pcnn_status;
+
+typedef enum {
+    PCNN_CONV = 0,     /* conv + bias (+ReLU): Fig. 2             */
+    PCNN_LRN = 1,      /* across-channel LRN (Caffe; R3)          */
+    PCNN_MAXPOOL = 2,  /* max pooling, no padding (R4)                */
+    PCNN_AVGPOOL = 3,  /* average pooling, no padding (R4)                  */
+    PCNN_FC = 4        /* classifier layer y = Wx + b (+ReLU) (R5)    */
+} pcnn_layer_kind;
+
+typedef enum {
+    PCNN_FP32_SIMT = 0, /* FP32 FFMA check path (the paper's SGEMM)  */
+    PCNN_TF32 = 1,      /* tcgen05 kind::tf32, operands RN-rounded (R9)     */
+    PCNN_BF16 = 2       /* tcgen05 kind::f16 with BF16 operands (R9)        */
+} pcnn_precision;
+
+typedef enum {
+    PCNN_VARIANT_EXACT = 0, /* the exact layer                              */
+    PCNN_VARIANT_RANK = 1   /* rank-r two-stage factorisation (R7)          */
+} pcnn_variant;
+
+/* One layer.  Unused fields are ignored for a kind.
+ *   CONV  : out_channels = N_f, kernel = S_f, stride, pad, groups (Caffe
+ *           groups: N_f and the input channels must be divisible), relu.
+ *   FC    : out_channels = output features, relu.  Input is the previous
+ *           activation flattened in C,H,W order (R5).
+ *   LRN   : kernel = local size n (odd), lrn_alpha, lrn_beta, lrn_k.
+ *   POOLS : kernel = window k, stride. */
+typedef struct {
+    int kind;
+    int out_channels;
+    int kernel;
+    int stride;
+    int pad;
+    int groups;
+    int relu;
+    float lrn_alpha;
+    float lrn_beta;
+    float lrn_k;
+} pcnn_layer_desc;
+
+typedef struct {
+    int in_channels;   /* C of the NCHW input images                        */
+    int in_height;     /* H                                                  */
+    int in_width;      /* W                                                  */
+    int max_batch;     /* largest batch pcnn_infer* will be called with      */
+    int precision;     /* pcnn_precision                                     */
+    int device;        /* CUDA device ordinal                                */
+} pcnn_net_desc;
+
+/* Per-layer geometry / plan, for a given batch (pcnn_query_layer,
+ * pcnn_describe_net).  GEMM dims are per group (eq. 4 M x N, K). */
+typedef struct {
+    int kind;
+    int in_c, in_h, in_w;
+    int out_c, out_h, out_w;
+    int groups;
+    long long gemm_m;   /* B * H_o * W_o (GEMM rows = output pixels)         */
+    int gemm_n;         /* N_f / g                                           */
+    int gemm_k;         /* S_f^2 * C / g                                     */
+    double flops;       /* algorithmic FLOPs of the active variant (eq. 1)  */
+    double flops_exact; /* eq. 1 FLOPs of the exact layer                    */
+    double bytes;       /* algorithmic bytes: in + out activations at storage
+                           precision + weights once                          */
+    int variant;        /* pcnn_variant in effect                            */
+    int rank;           /* r when variant == RANK, else 0                    */
+    int n_sms;          /* SM budget in effect (0 = all)                     */
+    int tlp;            /* CTAs per SM in effect                             */
+    int engine;         /* 0 = SIMT kernel, 1 = tcgen05 kernel, 2 = no GEMM  */
+    int tile_m, tile_n; /* GEMM tile (sub-matrix m x n)               */
+    long long tiles;    /* GridSize, eq. 4 (all groups)                      */
+    int grid;           /* CTAs launched                                     */
+    double util;        /* eq. 6 with maxBlocks = n_sms * tlp                */
+    double rec;         /* eq. 9 (tile-padding efficiency)                   */
+} pcnn_layer_info;
+
+typedef struct pcnn_net pcnn_net;
+
+/* Build a net: validate descriptors, infer shapes, pack weights into the
+ * kernel layouts (K-major, NHWC order, precision-rounded), allocate the
+ * activation arena for max_batch and plan every layer.
+ *   weights[i] : host fp32; CONV in OIHW [N_f][C/g][S][S], FC in
+ *                [out][in] with `in` in C,H,W order; NULL for weightless kinds.
+ *   biases[i]  : host fp32 [out_channels]; NULL = zero bias.
+ * Errors: INVALID_ARGUMENT / SHAPE / UNSUPPORTED (a layer shape the kernels
+ * cannot take), OUT_OF_MEMORY, CUDA (no device / not sm_100). */
+pcnn_status pcnn_create_net(const pcnn_net_desc *desc,
+                            const pcnn_layer_desc *layers, int n_layers,
+                            const float *const *weights,
+                            const float *const *biases, pcnn_net **out);
+
+pcnn_status pcnn_destroy_net(pcnn_net *net);
+
+/* Select a layer's variant (P:335 accuracy tuning picks, P:345 calibration
+ * backtracks).  RANK: rank in [1, min(N_f/g, S^2 C/g)]; the library computes a
+ * truncated SVD of each group's F_m on the host (FP64 one-sided Jacobi) the
+ * first time, caches it, and runs stage 1 (S x S conv, r filters) then stage 2
+ * (1x1, r -> N_f/g, + bias + ReLU).  rank == min(...) is full rank.
+ * EXACT ignores `rank`.  Errors: UNSUPPORTED for LRN / pool layers,
+ * INVALID_ARGUMENT for a bad rank. */
+pcnn_status pcnn_set_variant(pcnn_net *net, int layer, int variant, int rank);
+
+/* Test hook: install explicit factors for a RANK variant.
+ *   A : host fp32 [groups][N_f/g][rank]   (stage-2 1x1 weights)
+ *   B : host fp32 [groups][rank][C/g][S][S] (stage-1 filters, OIHW)
+ * so that the layer computes conv(x, A_g B_g) + bias. */
+pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank,
+                                     const float *A, const float *B);
+
+/* Per-layer SM / CTA budget (P:213 PSM, P:341 optSM x optTLP): the layer's
+ * kernels run on at most n_sms SMs with at most ctas_per_sm CTAs each.
+ * n_sms = 0 means all SMs; values above the device count are clamped.
+ * ctas_per_sm = 0 means the kernel's natural occupancy.  tcgen05 kernels are
+ * 1 CTA/SM by construction (their tlp is reported as 1).  The budget changes
+ * placement only: results are bitwise identical for every budget (R11). */
+pcnn_status pcnn_set_sm_budget(pcnn_net *net, int layer, int n_sms,
+                               int ctas_per_sm);
+
+/* The hot path.  Asynchronous on `stream`.
+ *   d_images  : device fp32 [batch][C][H][W] (NCHW)
+ *   d_out     : device fp32 [batch][pcnn_output_size()] -- the last layer's
+ *               output flattened in C,H,W order (logits for a classifier)
+ *   d_probs   : device fp32 [batch][pcnn_output_size()] softmax, or NULL
+ *   d_entropy : device fp32 [batch] entropy (eq. 2, natural log), or NULL
+ * 1 <= batch <= max_batch (else BATCH_TOO_LARGE / INVALID_ARGUMENT).  The
+ * launch sequence is captured once per (batch, pointers, variant/budget
+ * state) into a CUDA graph and replayed. */
+pcnn_status pcnn_infer(pcnn_net *net, const float *d_images, int batch,
+                       float *d_out, float *d_probs, float *d_entropy,
+                       void *stream);
+
+/* End-to-end form of pcnn_infer with HOST buffers: copies h_images to a
+ * library-owned device buffer, runs the hot path, copies the outputs back and
+ * synchronises `stream` before returning.  Host buffers should be pinned for
+ * full PCIe bandwidth.  h_probs / h_entropy may be NULL. */
+pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch,
+                            float *h_out, float *h_probs, float *h_entropy,
+                            void *stream);
+
+/* Elements per image of d_out (C*H*W of the last layer). */
+pcnn_status pcnn_output_size(const pcnn_net *net, int *out_elems);
+
+/* Number of layers and the plan of one layer for `batch` images. */
+pcnn_status pcnn_num_layers(const pcnn_net *net, int *n_layers);
+pcnn_status pcnn_query_layer(const pcnn_net *net, int layer, int batch,
+                             pcnn_layer_info *info);
+
+/* Host-only shape inference + FLOP/byte accounting of a descriptor list,
+ * no device needed (used by CPU tests and by planners).  infos[n_layers]. */
+pcnn_status pcnn_describe_net(const pcnn_net_desc *desc,
+                              const pcnn_layer_desc *layers, int n_layers,
+                              int batch, pcnn_layer_info *infos);
+
+/* Per-layer latency: run the net `reps` times (not graph-captured) with CUDA
+ * events around every layer on `stream`; layer_ms[n_layers] receives the mean
+ * milliseconds per layer, *total_ms (nullable) the mean whole pass (staging
+ * and softmax included).  Synchronises `stream`. */
+pcnn_status pcnn_profile_layers(pcnn_net *net, const float *d_images,
+                                int batch, float *d_out, int reps,
+                                float *layer_ms, float *total_ms,
+                                void *stream);
+
+/* Test hook: when enabled, every admitted CTA of every layer kernel records
+ * its %smid; pcnn_get_sm_census returns the 256-bit SM mask (8 words) seen
+ * by `layer` during the last pcnn_infer.  Disabling frees the buffers. */
+pcnn_status pcnn_enable_sm_census(pcnn_net *net, int enable);
+pcnn_status pcnn_get_sm_census(pcnn_net *net, int layer,
+                               unsigned int mask_out[8]);
+
+/* Number of SMs of `device` (0 if none), and the library's version string. */
+int pcnn_device_sm_count(int device);
+const char *pcnn_version(void);
+
+const char *pcnn_status_string(pcnn_status status);
+const char *pcnn_last_error_message(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PCNN_H */

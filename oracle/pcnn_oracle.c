@@ -14,7 +14,7 @@
 #include <string.h>
 
 /* ------------------------------------------------------------------ */
-/* batch parallelism: one image per work item, sequential inside       */
+/* work-item parallelism: every output value is computed sequentially  */
 /* ------------------------------------------------------------------ */
 typedef void (*image_fn)(void *ctx, int n);
 
@@ -84,31 +84,31 @@ typedef struct {
     int C, H, W, F, S, stride, pad, groups, relu, Ho, Wo;
 } conv_ctx;
 
-static void conv_image(void *vctx, int n) {
+/* one work item = one output channel f of one image n */
+static void conv_item(void *vctx, int item) {
     const conv_ctx *c = (const conv_ctx *)vctx;
+    const int n = item / c->F, f = item % c->F;
     const int Cg = c->C / c->groups, Fg = c->F / c->groups;
-    for (int f = 0; f < c->F; ++f) {
-        const int g = f / Fg;                       /* g(f) = floor(f / (N_f/g)) */
-        for (int p = 0; p < c->Ho; ++p) {
-            for (int q = 0; q < c->Wo; ++q) {
-                double acc = 0.0;
-                for (int ci = 0; ci < Cg; ++ci) {
-                    const int cin = g * Cg + ci;
-                    for (int r = 0; r < c->S; ++r) {
-                        const int ih = p * c->stride + r - c->pad;
-                        if (ih < 0 || ih >= c->H) continue;      /* zero padding */
-                        for (int s = 0; s < c->S; ++s) {
-                            const int iw = q * c->stride + s - c->pad;
-                            if (iw < 0 || iw >= c->W) continue;
-                            acc += c->w[(((size_t)f * Cg + ci) * c->S + r) * c->S + s] *
-                                   c->x[(((size_t)n * c->C + cin) * c->H + ih) * c->W + iw];
-                        }
+    const int g = f / Fg;                           /* g(f) = floor(f / (N_f/g)) */
+    for (int p = 0; p < c->Ho; ++p) {
+        for (int q = 0; q < c->Wo; ++q) {
+            double acc = 0.0;
+            for (int ci = 0; ci < Cg; ++ci) {
+                const int cin = g * Cg + ci;
+                for (int r = 0; r < c->S; ++r) {
+                    const int ih = p * c->stride + r - c->pad;
+                    if (ih < 0 || ih >= c->H) continue;      /* zero padding */
+                    for (int s = 0; s < c->S; ++s) {
+                        const int iw = q * c->stride + s - c->pad;
+                        if (iw < 0 || iw >= c->W) continue;
+                        acc += c->w[(((size_t)f * Cg + ci) * c->S + r) * c->S + s] *
+                               c->x[(((size_t)n * c->C + cin) * c->H + ih) * c->W + iw];
                     }
                 }
-                double v = acc + (c->bias ? c->bias[f] : 0.0);
-                if (c->relu && v < 0.0) v = 0.0;         /* reading R2 */
-                c->y[(((size_t)n * c->F + f) * c->Ho + p) * c->Wo + q] = v;
             }
+            double v = acc + (c->bias ? c->bias[f] : 0.0);
+            if (c->relu && v < 0.0) v = 0.0;         /* reading R2 */
+            c->y[(((size_t)n * c->F + f) * c->Ho + p) * c->Wo + q] = v;
         }
     }
 }
@@ -122,7 +122,7 @@ int orc_conv2d(const double *x, int B, int C, int H, int W, const double *w,
     int Wo = orc_conv_out_size(W, S, stride, pad);
     if (Ho <= 0 || Wo <= 0) return -2;
     conv_ctx c = {x, w, bias, y, C, H, W, F, S, stride, pad, groups, relu, Ho, Wo};
-    for_each_image(conv_image, &c, B, nthreads);
+    for_each_image(conv_item, &c, B * F, nthreads);
     return 0;
 }
 
@@ -272,23 +272,23 @@ typedef struct {
     int K, N, relu;
 } fc_ctx;
 
-static void fc_image(void *vctx, int n) {
+/* one work item = one output feature j of one image n */
+static void fc_item(void *vctx, int item) {
     const fc_ctx *c = (const fc_ctx *)vctx;
-    for (int j = 0; j < c->N; ++j) {
-        double acc = 0.0;
-        for (int i = 0; i < c->K; ++i)
-            acc += c->w[(size_t)j * c->K + i] * c->x[(size_t)n * c->K + i];
-        double v = acc + (c->bias ? c->bias[j] : 0.0);
-        if (c->relu && v < 0.0) v = 0.0;
-        c->y[(size_t)n * c->N + j] = v;
-    }
+    const int n = item / c->N, j = item % c->N;
+    double acc = 0.0;
+    for (int i = 0; i < c->K; ++i)
+        acc += c->w[(size_t)j * c->K + i] * c->x[(size_t)n * c->K + i];
+    double v = acc + (c->bias ? c->bias[j] : 0.0);
+    if (c->relu && v < 0.0) v = 0.0;
+    c->y[(size_t)n * c->N + j] = v;
 }
 
 int orc_fc(const double *x, int B, int K, const double *w, const double *bias,
            int N, int relu, double *y, int nthreads) {
     if (!x || !w || !y || K <= 0 || N <= 0) return -1;
     fc_ctx c = {x, w, bias, y, K, N, relu};
-    for_each_image(fc_image, &c, B, nthreads);
+    for_each_image(fc_item, &c, B * N, nthreads);
     return 0;
 }
 

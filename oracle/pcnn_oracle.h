@@ -12,9 +12,10 @@
  * conv weights OIHW (F_m of Fig. 2 row-major = [N_f][N_c/g][S_f][S_f]),
  * FC weights [out][in] with the input flattened in C,H,W order.
  *
- * Threading: functions taking `nthreads` split the batch over pthreads
- * (one image per work item); each image's arithmetic is sequential, so the
- * result does not depend on nthreads.
+ * Threading: functions taking `nthreads` split independent work items
+ * (an image, or one output channel / feature of one image) over pthreads;
+ * every output value is computed by one sequential loop, so the result does
+ * not depend on nthreads.
  *
  * Return value: 0 on success, negative on bad arguments.
  */

@@ -1,0 +1,457 @@
+// kernels_tc.cu -- tcgen05 implicit-GEMM convolution / FC for sm_100a (K1/K2).
+//
+// What it computes (Fig. 2; eq. 1): for every group g,
+//   O_g[M x Nfg] = im2col(X)_g[M x K] * F_m,g[Nfg x K]^T  (+bias, ReLU)
+// with M = B*Ho*Wo output pixels (NHWC rows), K = (r, s, c) taps x channels.
+// D_m (the im2col matrix) is never materialised: producer warps gather each
+// A tile row -- one output pixel's (r, s, c-chunk) input run -- straight from
+// the NHWC activations into the 128B-swizzled shared-memory layout the UMMA
+// descriptor expects (cp.async 16 B chunks, zero-fill for padding / ragged
+// tails).  The weight tile (B operand) arrives by TMA.  One elected thread
+// issues tcgen05.mma (BF16 kind::f16 or kind::tf32, FP32 accumulate) into a
+// double-buffered TMEM accumulator; four epilogue warps drain it with
+// tcgen05.ld, add bias, apply ReLU, round to the storage precision and store
+// NHWC rows.  The kernel is persistent: grid = min(tiles, SM budget) CTAs,
+// 1 CTA per SM (smem + TMEM), static round-robin tile schedule -- the grid cap
+// IS the per-layer SM budget.
+//
+// CTA = 14 warps (448 threads):
+//   warp 0       : TMA producer for B (weights)
+//   warp 1       : TMEM allocator + MMA issuer
+//   warps 2..5   : epilogue (TMEM lane quarter = warp % 4)
+//   warps 6..13  : im2col gather producers for A (256 threads)
+#include "budget.cuh"
+#include "pcnn_internal.h"
+
+namespace pcnn {
+
+constexpr int TC_BM = 128;              // UMMA M (cta_group::1)
+constexpr int TC_BN_MAX = 256;          // max UMMA N
+constexpr int TC_ROW_BYTES = 128;       // one K-block row = one 128B swizzle row
+constexpr int TC_STAGES = 4;
+constexpr int TC_LAG = 2;               // producer arrive lag (< TC_STAGES)
+constexpr int TC_A_STAGE = TC_BM * TC_ROW_BYTES;          // 16 KB
+constexpr int TC_B_STAGE = TC_BN_MAX * TC_ROW_BYTES;      // 32 KB
+constexpr int TC_MAX_KTAB = 4096;       // chunk-table entries kept in smem
+constexpr int TC_THREADS = 448;
+constexpr int TC_PRODUCER0 = 192;       // first A-producer thread
+constexpr int TC_NPROD = 256;
+constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
+
+// smem layout (bytes from the 1024-aligned base)
+constexpr int SM_A = 0;
+constexpr int SM_B = SM_A + TC_STAGES * TC_A_STAGE;
+constexpr int SM_BAR = SM_B + TC_STAGES * TC_B_STAGE;     // 196608
+constexpr int SM_FULL = SM_BAR;
+constexpr int SM_EMPTY = SM_FULL + 8 * TC_STAGES;
+constexpr int SM_TFULL = SM_EMPTY + 8 * TC_STAGES;
+constexpr int SM_TEMPTY = SM_TFULL + 16;
+constexpr int SM_TMEMPTR = SM_TEMPTY + 16;
+constexpr int SM_KTAB = SM_BAR + 128;
+constexpr int SM_TOTAL = SM_KTAB + 4 * TC_MAX_KTAB;
+constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
+
+size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
+int tc_max_ktab() { return TC_MAX_KTAB; }
+int tc_block_k_elems(int st) { return st == ST_BF16 ? 64 : 32; }
+
+// ------------------------------------------------------------ PTX wrappers
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra WAIT_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map,
+                                            uint32_t bar, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
+      : "memory");
+}
+
+__device__ __forceinline__ void cp_async_16(uint32_t dst, const void *src, int nbytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
+               "r"(nbytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() {
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_commit(uint32_t bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+          bar)
+      : "memory");
+}
+
+template <int ST>
+__device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
+                                       uint32_t idesc, uint32_t accum) {
+  if constexpr (ST == ST_BF16) {
+    asm volatile(
+        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
+  } else {
+    asm volatile(
+        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
+  }
+}
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
+        "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]),
+        "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_ld_wait() {
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+// UMMA shared-memory descriptor, K-major, 128B swizzle: 8-row x 128 B atoms
+// stacked along M/N every 1024 B (SBO), version 1 (sm_100), layout 2 = SW128.
+__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)1 << 16;                  // LBO (unused for swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;        // SBO
+  d |= (uint64_t)1 << 46;                  // descriptor version (sm_100)
+  d |= (uint64_t)2 << 61;                  // SWIZZLE_128B
+  return d;
+}
+
+// Instruction descriptor: D fp32, A/B = BF16 (1) or TF32 (2), K-major, M=128.
+template <int ST>
+__device__ __forceinline__ uint32_t umma_idesc(int bn) {
+  const uint32_t fmt = ST == ST_BF16 ? 1u : 2u;
+  return (1u << 4) | (fmt << 7) | (fmt << 10) | ((uint32_t)(bn >> 3) << 17) |
+         ((uint32_t)(TC_BM >> 4) << 24);
+}
+
+__device__ __forceinline__ float tf32_rna_tc(float v) {
+  unsigned r;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(v));
+  return __uint_as_float(r);
+}
+
+struct TcArgs {
+  ConvGeom g;
+  const void *x;
+  void *y;
+  const float *bias;
+  const int *ktab;      // per-element (r,s,c) table (nullptr when S == 1)
+  int bn;
+  int mtiles, ntiles, tiles;
+  int kblocks;
+  Budget b;
+};
+
+template <int ST>
+__global__ void __launch_bounds__(TC_THREADS, 1)
+conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const uint32_t sbase = smem_u32(smem);
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31;
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  constexpr int CH = 16 / ESZ;                 // elements per 16 B chunk
+  const ConvGeom &g = a.g;
+
+  uint32_t *ktab_s = (uint32_t *)(smem + SM_KTAB);
+  const bool use_tab = a.ktab != nullptr;
+  const int nchunks = g.Kpad / CH;
+  if (use_tab) {
+    for (int i = tid; i < nchunks && i < TC_MAX_KTAB; i += TC_THREADS) {
+      const int k = i * CH;
+      ktab_s[i] = k < g.K ? (uint32_t)__ldg(&a.ktab[k]) : 0xFF000000u;
+    }
+  }
+  if (tid == 0) {
+    for (int s = 0; s < TC_STAGES; ++s) {
+      mbar_init(sbase + SM_FULL + 8 * s, 1 + TC_NPROD);
+      mbar_init(sbase + SM_EMPTY + 8 * s, 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(sbase + SM_TFULL + 8 * i, 1);
+      mbar_init(sbase + SM_TEMPTY + 8 * i, 128);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    census_mark(a.b);
+  }
+  if (warp == 1) {
+    asm volatile(
+        "tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+            sbase + SM_TMEMPTR),
+        "n"(TC_TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *(volatile uint32_t *)(smem + SM_TMEMPTR);
+
+  const int HoWo = g.Ho * g.Wo;
+
+  if (warp == 0) {
+    // ------------------------------------------------ B (weights) TMA producer
+    if (lane == 0) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
+      uint32_t it = 0;
+      for (int t = blockIdx.x; t < a.tiles; t += gridDim.x) {
+        const int rest = t / a.mtiles;
+        const int nt = rest % a.ntiles, grp = rest / a.ntiles;
+        const int nrow = grp * g.Nfg + nt * a.bn;
+        for (int kb = 0; kb < a.kblocks; ++kb, ++it) {
+          const uint32_t s = it % TC_STAGES, ph = (it / TC_STAGES) & 1;
+          mbar_wait(sbase + SM_EMPTY + 8 * s, ph ^ 1);
+          mbar_arrive_expect_tx(sbase + SM_FULL + 8 * s, (uint32_t)a.bn * TC_ROW_BYTES);
+          tma_load_2d(sbase + SM_B + s * TC_B_STAGE, &tmap_w, sbase + SM_FULL + 8 * s,
+                      kb * (TC_ROW_BYTES / ESZ), nrow);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------ MMA issuer
+    if (lane == 0) {
+      const uint32_t idesc = umma_idesc<ST>(a.bn);
+      uint32_t it = 0, lt = 0;
+      for (int t = blockIdx.x; t < a.tiles; t += gridDim.x, ++lt) {
+        const uint32_t buf = lt & 1, use = lt >> 1;
+        mbar_wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
+        for (int kb = 0; kb < a.kblocks; ++kb, ++it) {
+          const uint32_t s = it % TC_STAGES, ph = (it / TC_STAGES) & 1;
+          mbar_wait(sbase + SM_FULL + 8 * s, ph);
+          tc_fence_after();
+          const uint64_t ad = umma_desc_sw128(sbase + SM_A + s * TC_A_STAGE);
+          const uint64_t bd = umma_desc_sw128(sbase + SM_B + s * TC_B_STAGE);
+#pragma unroll
+          for (int k = 0; k < 4; ++k)   // 4 x 32 B along K inside the 128 B row
+            tc_mma<ST>(dcol, ad + 2 * k, bd + 2 * k, idesc, (kb | k) != 0);
+          tc_commit(sbase + SM_EMPTY + 8 * s);
+        }
+        tc_commit(sbase + SM_TFULL + 8 * buf);
+      }
+    }
+  } else if (warp < 6) {
+    // ------------------------------------------------ epilogue
+    const int quarter = warp & 3;
+    const int row = quarter * 32 + lane;
+    uint32_t lt = 0;
+    for (int t = blockIdx.x; t < a.tiles; t += gridDim.x, ++lt) {
+      const int mt = t % a.mtiles, rest = t / a.mtiles;
+      const int nt = rest % a.ntiles, grp = rest / a.ntiles;
+      const uint32_t buf = lt & 1, use = lt >> 1;
+      mbar_wait(sbase + SM_TFULL + 8 * buf, use & 1);
+      tc_fence_after();
+      const int m = mt * TC_BM + row;
+      const bool mok = m < g.M;
+      const size_t orow = (size_t)m * g.out_cs;
+      for (int c0 = 0; c0 < a.bn; c0 += 16) {
+        __syncwarp();
+        uint32_t v[16];
+        tmem_ld16(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0, v);
+        tmem_ld_wait();
+        const int n = nt * a.bn + c0;          // column within the group
+        if (mok && n < g.Nfg) {
+          const int col = grp * g.Nfg + n;
+          float f[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            float x = __uint_as_float(v[i]);
+            if (a.bias && n + i < g.Nfg) x += __ldg(&a.bias[col + i]);
+            if (g.relu) x = fmaxf(x, 0.f);
+            f[i] = x;
+          }
+          if (g.out_mode == OUT_BF16) {
+            __nv_bfloat16 *yp = (__nv_bfloat16 *)a.y + orow + col;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              if (n + 8 * h < g.Nfg) {
+                uint4 pk;
+                uint32_t *pw = (uint32_t *)&pk;
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                  __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * h + 2 * i], f[8 * h + 2 * i + 1]);
+                  pw[i] = *(uint32_t *)&b2;
+                }
+                *(uint4 *)(yp + 8 * h) = pk;
+              }
+            }
+          } else {
+            float *yp = (float *)a.y + orow + col;
+#pragma unroll
+            for (int h = 0; h < 4; ++h) {
+              if (n + 4 * h < g.Nfg) {
+                float4 q;
+                if (g.out_mode == OUT_F32_TF32) {
+                  q = make_float4(tf32_rna_tc(f[4 * h]), tf32_rna_tc(f[4 * h + 1]),
+                                  tf32_rna_tc(f[4 * h + 2]), tf32_rna_tc(f[4 * h + 3]));
+                } else {
+                  q = make_float4(f[4 * h], f[4 * h + 1], f[4 * h + 2], f[4 * h + 3]);
+                }
+                *(float4 *)(yp + 4 * h) = q;
+              }
+            }
+          }
+        }
+      }
+      __syncwarp();
+      tc_fence_before();
+      mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
+    }
+  } else {
+    // ------------------------------------------------ A (im2col) gather producers
+    const int p = tid - TC_PRODUCER0;          // 0..255
+    const int j = p & 7;                       // 16 B chunk within the 128 B row
+    const int rb = p >> 3;                     // rows rb, rb+32, rb+64, rb+96
+    const uint32_t swz = (uint32_t)((j ^ (rb & 7)) << 4);
+    const char *xb = (const char *)a.x;
+    uint32_t it = 0;
+    for (int t = blockIdx.x; t < a.tiles; t += gridDim.x) {
+      const int mt = t % a.mtiles, rest = t / a.mtiles;
+      const int grp = (rest / a.ntiles);
+      long long base[4];
+      int ih0[4], iw0[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int m = mt * TC_BM + rb + 32 * i;
+        if (m < g.M) {
+          const int n = m / HoWo, pq = m % HoWo;
+          const int pp = pq / g.Wo, q = pq % g.Wo;
+          base[i] = ((long long)n * g.H * g.W * g.Cs + (long long)grp * g.Cg) * ESZ;
+          ih0[i] = pp * g.stride - g.pad;
+          iw0[i] = q * g.stride - g.pad;
+        } else {
+          base[i] = -1;
+          ih0[i] = 0;
+          iw0[i] = 0;
+        }
+      }
+      for (int kb = 0; kb < a.kblocks; ++kb, ++it) {
+        const uint32_t s = it % TC_STAGES, ph = (it / TC_STAGES) & 1;
+        mbar_wait(sbase + SM_EMPTY + 8 * s, ph ^ 1);
+        const int kc = kb * 8 + j;
+        int r = 0, sx = 0, c = kc * CH;
+        bool kok = c < g.K;
+        if (use_tab) {
+          const uint32_t e = kc < TC_MAX_KTAB ? ktab_s[kc] : 0xFF000000u;
+          r = (e >> 24) & 0xFF;
+          sx = (e >> 16) & 0xFF;
+          c = e & 0xFFFF;
+          kok = kok && r != 0xFF;
+        }
+        const uint32_t dst_stage = sbase + SM_A + s * TC_A_STAGE;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int row = rb + 32 * i;
+          const int ih = ih0[i] + r, iw = iw0[i] + sx;
+          const bool ok = kok && base[i] >= 0 && ih >= 0 && ih < g.H && iw >= 0 && iw < g.W;
+          const char *src = ok ? xb + base[i] + (((long long)ih * g.W + iw) * g.Cs + c) * ESZ : xb;
+          cp_async_16(dst_stage + row * TC_ROW_BYTES + swz, src, ok ? 16 : 0);
+        }
+        cp_async_commit();
+        if (it >= TC_LAG) {
+          cp_async_wait<TC_LAG>();
+          fence_proxy_async();
+          mbar_arrive(sbase + SM_FULL + 8 * ((it - TC_LAG) % TC_STAGES));
+        }
+      }
+    }
+    // flush the last TC_LAG stages
+    cp_async_wait<0>();
+    fence_proxy_async();
+    const uint32_t first = it > TC_LAG ? it - TC_LAG : 0;
+    for (uint32_t k = first; k < it; ++k) mbar_arrive(sbase + SM_FULL + 8 * (k % TC_STAGES));
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                 "n"(TC_TMEM_COLS));
+  }
+}
+
+cudaError_t tc_init() {
+  cudaError_t e = cudaFuncSetAttribute(conv_tc_kernel<ST_BF16>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)TC_SMEM_BYTES);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(conv_tc_kernel<ST_F32>,
+                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM_BYTES);
+}
+
+template <int ST>
+static cudaError_t launch_tc_impl(const TcArgs &args, const CUtensorMap *tmap, int grid,
+                                  cudaStream_t s) {
+  conv_tc_kernel<ST><<<grid, TC_THREADS, TC_SMEM_BYTES, s>>>(*tmap, args);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
+                           const CUtensorMap *tmap_w, const float *bias, void *y,
+                           const int *ktab, const TcPlan &p, const Budget &b,
+                           cudaStream_t s) {
+  TcArgs args;
+  args.g = g;
+  args.x = x;
+  args.y = y;
+  args.bias = bias;
+  args.ktab = ktab;
+  args.bn = p.bn;
+  args.mtiles = p.mtiles;
+  args.ntiles = p.ntiles;
+  args.tiles = p.tiles;
+  args.kblocks = g.Kpad / tc_block_k_elems(st);
+  args.b = b;
+  if (st == ST_BF16) return launch_tc_impl<ST_BF16>(args, tmap_w, p.grid, s);
+  return launch_tc_impl<ST_F32>(args, tmap_w, p.grid, s);
+}
+
+}  // namespace pcnn

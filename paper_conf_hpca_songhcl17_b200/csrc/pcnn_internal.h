@@ -1,0 +1,103 @@
+// pcnn_internal.h -- shared declarations of the runtime and its kernels.
+// Part of libpcnn.so (the CUDA product path).  Never includes oracle/.
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+namespace pcnn {
+
+constexpr int kMaxSMs = 256;          // census mask width
+
+// Element storage types of activations / packed weights.
+enum StoreType : int { ST_F32 = 0, ST_BF16 = 1 };
+// Epilogue output modes.
+enum OutMode : int { OUT_BF16 = 0, OUT_F32_TF32 = 1, OUT_F32 = 2 };
+
+// SM / CTA budget handed to every layer kernel (P:213 PSM).
+//   gated == 0 : no budget (static schedule over all SMs)
+//   gated == 1 : CTA admitted iff %smid < n_sms and fewer than tlp CTAs of
+//                this launch were admitted on its SM; admitted CTAs pull
+//                tiles from an atomic counter (ctr[0]).  ctr[1 + smid] counts
+//                admissions.  ctr must be zeroed before the launch.
+struct Budget {
+  int gated;
+  int n_sms;
+  int tlp;
+  int pad_;
+  unsigned long long *ctr;
+  unsigned int *census;   // 8 words or nullptr
+};
+
+// Implicit-GEMM convolution geometry (one launch, all groups).
+// GEMM per group g:  O[M x Nfg] = A[M x K] * B_g[Nfg x K]^T  with
+//   M = B*Ho*Wo output pixels, A = im2col(X) (never materialised),
+//   K ordered (r, s, c) over the Cg stored channels of group g.
+struct ConvGeom {
+  int M;            // B*Ho*Wo
+  int H, W, Cs;     // input spatial size, stored channels per pixel
+  int Cg;           // stored channels per group read by the GEMM
+  int S, stride, pad;
+  int Ho, Wo;
+  int Nfg;          // output channels per group
+  int groups;
+  int out_cs;       // output pixel stride in elements (channels stored)
+  int K;            // S*S*Cg
+  int Kpad;         // K rounded up to the kernel's K-block
+  int relu;
+  int out_mode;     // OutMode
+};
+
+// ---------------------------------------------------------------- launchers
+// All return cudaSuccess or the launch error; they never synchronise.
+
+// a1: NCHW fp32 -> NHWC storage (channels zero-padded to Cs).
+cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C,
+                               int H, int W, int Cs, int tf32_round,
+                               cudaStream_t s);
+// final NHWC storage -> NCHW fp32 flatten
+cudaError_t launch_unstage_output(const void *x, int st, float *y, int B,
+                                  int C, int H, int W, int Cs, cudaStream_t s);
+
+// FP32 SIMT implicit-GEMM conv / FC (check path, K3).
+cudaError_t launch_conv_simt(const ConvGeom &g, const float *x,
+                             const float *w, const float *bias, float *y,
+                             const int *ktab, const Budget &b, int grid,
+                             cudaStream_t s);
+int conv_simt_tiles(const ConvGeom &g);
+void conv_simt_tile_shape(int *tm, int *tn);
+
+// tcgen05 implicit-GEMM conv / FC (K1/K2).
+struct TcPlan {
+  int bn;          // N tile (16..256, multiple of 16)
+  int mtiles, ntiles, tiles;
+  int grid;
+};
+cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
+                           const CUtensorMap *tmap_w, const float *bias,
+                           void *y, const int *ktab, const TcPlan &p,
+                           const Budget &b, cudaStream_t s);
+int tc_block_k_elems(int st);          // K-block in elements (128 B)
+cudaError_t tc_init();                 // sets the kernels' smem attributes
+size_t tc_smem_bytes();
+int tc_max_ktab();
+
+// a4 / a5 / a7
+cudaError_t launch_lrn(const void *x, void *y, int st, int tf32_round,
+                       long pixels, int C, int size, float alpha, float beta,
+                       float k, const Budget &b, int grid, cudaStream_t s);
+cudaError_t launch_pool(const void *x, void *y, int st, int B, int H, int W,
+                        int C, int k, int stride, int Ho, int Wo, int is_max,
+                        int tf32_round, const Budget &b, int grid,
+                        cudaStream_t s);
+cudaError_t launch_softmax_entropy(const float *z, float *p, float *h, int B,
+                                   int N, cudaStream_t s);
+
+// occupancy helpers for gated launches
+int simt_conv_occupancy();
+int lrn_occupancy();
+int pool_occupancy();
+
+}  // namespace pcnn

@@ -1,0 +1,1051 @@
+// runtime.cu -- libpcnn host runtime and C ABI (include/pcnn.h).
+//
+// Responsibilities: validate layer descriptors, infer shapes, pack weights
+// into the kernels' K-major (r, s, c) layouts in the storage precision, own
+// the activation arena, plan each layer (engine, tile, grid, SM budget), run
+// the rank-r variant's SVD, and enqueue the hot path (optionally through a
+// cached CUDA graph).  No arithmetic of the hot path runs on the host.
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/pcnn.h"
+#include "pcnn_internal.h"
+#include "svd.h"
+
+using namespace pcnn;
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+
+static pcnn_status fail(pcnn_status s, const std::string &msg) {
+  g_err = msg;
+  return s;
+}
+
+#define CUDA_TRY(expr)                                                          \
+  do {                                                                          \
+    cudaError_t e_ = (expr);                                                    \
+    if (e_ != cudaSuccess)                                                      \
+      return fail(PCNN_ERR_CUDA, std::string(#expr) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+// ------------------------------------------------------------------ host rounding
+static inline uint16_t f32_to_bf16_rne(float f) {
+  uint32_t u;
+  std::memcpy(&u, &f, 4);
+  if ((u & 0x7F800000u) == 0x7F800000u) return (uint16_t)(u >> 16);  // inf/nan
+  u += 0x7FFFu + ((u >> 16) & 1u);
+  return (uint16_t)(u >> 16);
+}
+static inline float tf32_rna_host(float f) {
+  uint32_t u;
+  std::memcpy(&u, &f, 4);
+  if ((u & 0x7F800000u) != 0x7F800000u) {
+    u += 0x1000u;
+    u &= 0xFFFFE000u;
+  }
+  float r;
+  std::memcpy(&r, &u, 4);
+  return r;
+}
+
+// ------------------------------------------------------------------ driver entry
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode_tiled() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+  });
+  return fn;
+}
+
+// ------------------------------------------------------------------ net state
+namespace {
+
+struct GemmStage {           // one implicit-GEMM launch
+  ConvGeom g{};              // M filled per batch
+  int in_c = 0, in_h = 0, in_w = 0;
+  int st = ST_F32;           // storage type of input / weights
+  int engine = 0;            // 0 SIMT, 1 tcgen05
+  void *d_w = nullptr;       // packed [groups*Nfg][Kpad]
+  float *d_bias = nullptr;
+  int *d_ktab = nullptr;     // per-element (r,s,c) table
+  std::map<int, CUtensorMap> tmaps;  // by N tile
+  size_t w_bytes = 0;
+  void release() {
+    if (d_w) cudaFree(d_w);
+    if (d_bias) cudaFree(d_bias);
+    if (d_ktab) cudaFree(d_ktab);
+    d_w = nullptr;
+    d_bias = nullptr;
+    d_ktab = nullptr;
+    tmaps.clear();
+  }
+};
+
+struct Layer {
+  pcnn_layer_desc d{};
+  int in_c = 0, in_h = 0, in_w = 0, in_cs = 0;
+  int out_c = 0, out_h = 0, out_w = 0, out_cs = 0;
+  int gemm = 0;             // conv or fc
+  GemmStage exact;
+  // rank-r variant
+  int variant = PCNN_VARIANT_EXACT, rank = 0;
+  GemmStage r1, r2;
+  std::vector<float> host_w;   // OIHW copy kept for the SVD (conv only)
+  std::vector<Svd> svd;        // per group (lazily computed)
+  // budget
+  int n_sms = 0, tlp = 0;
+  unsigned long long *d_ctr = nullptr;   // 3 launch slots x (1 + kMaxSMs)
+  unsigned int *d_census = nullptr;      // 8 words
+};
+
+}  // namespace
+
+struct pcnn_net {
+  pcnn_net_desc desc{};
+  int device = 0;
+  int num_sms = 148;
+  int st = ST_F32;
+  int in_cs = 4;
+  std::vector<Layer> layers;
+  size_t act_bytes = 0;     // per arena buffer
+  void *d_act[3] = {nullptr, nullptr, nullptr};
+  float *d_host_in = nullptr, *d_host_out = nullptr, *d_host_p = nullptr,
+        *d_host_h = nullptr;
+  int out_elems = 0;
+  int occ_simt = 1, occ_lrn = 1, occ_pool = 1;
+  bool census = false;
+  // CUDA graph cache
+  uint64_t version = 1;
+  struct GraphKey {
+    int batch;
+    const void *in, *out, *p, *h;
+    cudaStream_t s;
+    uint64_t version;
+    bool operator<(const GraphKey &o) const {
+      return std::tie(batch, in, out, p, h, s, version) <
+             std::tie(o.batch, o.in, o.out, o.p, o.h, o.s, o.version);
+    }
+  };
+  std::map<GraphKey, cudaGraphExec_t> graphs;
+  bool use_graphs = true;
+};
+
+// ------------------------------------------------------------------ geometry
+static int conv_out(int in, int k, int st, int pad) {
+  if (st <= 0 || in + 2 * pad < k) return -1;
+  return (in + 2 * pad - k) / st + 1;
+}
+static int pool_out(int in, int k, int st) {
+  if (st <= 0 || in < k) return -1;
+  int o = (in - k + st - 1) / st + 1;
+  if ((o - 1) * st >= in) --o;
+  return o;
+}
+static int round_up(int a, int b) { return (a + b - 1) / b * b; }
+static int esz_of(int st) { return st == ST_BF16 ? 2 : 4; }
+
+static int storage_of(int precision) {
+  return precision == PCNN_BF16 ? ST_BF16 : ST_F32;
+}
+static int chunk_elems(int precision) {
+  // channel padding unit of stored activations: 16 B for tcgen05 chunks
+  return precision == PCNN_BF16 ? 8 : 4;
+}
+
+// Shape inference over the descriptor list (host only).  Fills in/out dims.
+static pcnn_status infer_shapes(const pcnn_net_desc *d, const pcnn_layer_desc *L, int n,
+                                std::vector<Layer> &out) {
+  if (!d || !L || n <= 0) return fail(PCNN_ERR_INVALID_ARGUMENT, "null descriptor or no layers");
+  if (d->in_channels <= 0 || d->in_height <= 0 || d->in_width <= 0)
+    return fail(PCNN_ERR_SHAPE, "bad input shape");
+  if (d->precision < PCNN_FP32_SIMT || d->precision > PCNN_BF16)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad precision");
+  const int ch = chunk_elems(d->precision);
+  out.assign(n, Layer());
+  int c = d->in_channels, h = d->in_height, w = d->in_width;
+  int cs = round_up(c, ch);
+  for (int i = 0; i < n; ++i) {
+    Layer &ly = out[i];
+    ly.d = L[i];
+    ly.in_c = c;
+    ly.in_h = h;
+    ly.in_w = w;
+    ly.in_cs = cs;
+    const auto &li = L[i];
+    char buf[160];
+    switch (li.kind) {
+      case PCNN_CONV: {
+        const int g = li.groups <= 0 ? 1 : li.groups;
+        ly.d.groups = g;
+        if (li.out_channels <= 0 || li.kernel <= 0 || li.stride <= 0 || li.pad < 0 ||
+            c % g || li.out_channels % g) {
+          snprintf(buf, sizeof buf, "layer %d: bad conv descriptor", i);
+          return fail(PCNN_ERR_SHAPE, buf);
+        }
+        if (li.kernel > 255) return fail(PCNN_ERR_UNSUPPORTED, "kernel > 255");
+        if (i == 0 && g > 1 && cs != c)
+          return fail(PCNN_ERR_UNSUPPORTED, "grouped first layer needs C multiple of 8");
+        const int ho = conv_out(h, li.kernel, li.stride, li.pad);
+        const int wo = conv_out(w, li.kernel, li.stride, li.pad);
+        if (ho <= 0 || wo <= 0) {
+          snprintf(buf, sizeof buf, "layer %d: conv output empty", i);
+          return fail(PCNN_ERR_SHAPE, buf);
+        }
+        ly.gemm = 1;
+        c = li.out_channels;
+        h = ho;
+        w = wo;
+        break;
+      }
+      case PCNN_FC:
+        if (li.out_channels <= 0) return fail(PCNN_ERR_SHAPE, "bad fc descriptor");
+        ly.gemm = 1;
+        ly.d.groups = 1;
+        c = li.out_channels;
+        h = 1;
+        w = 1;
+        break;
+      case PCNN_LRN:
+        if (li.kernel <= 0 || (li.kernel % 2) == 0)
+          return fail(PCNN_ERR_SHAPE, "LRN size must be odd");
+        if (c > 1024) return fail(PCNN_ERR_UNSUPPORTED, "LRN with > 1024 channels");
+        break;
+      case PCNN_MAXPOOL:
+      case PCNN_AVGPOOL: {
+        const int ho = pool_out(h, li.kernel, li.stride);
+        const int wo = pool_out(w, li.kernel, li.stride);
+        if (li.kernel <= 0 || ho <= 0 || wo <= 0) return fail(PCNN_ERR_SHAPE, "bad pool");
+        h = ho;
+        w = wo;
+        break;
+      }
+      default:
+        return fail(PCNN_ERR_INVALID_ARGUMENT, "unknown layer kind");
+    }
+    ly.out_c = c;
+    ly.out_h = h;
+    ly.out_w = w;
+    // stored channels: GEMM outputs keep exactly out_c (must be chunk-aligned to
+    // feed the next GEMM); pool / LRN keep their input's storage.
+    ly.out_cs = ly.gemm ? c : cs;
+    cs = ly.out_cs;
+  }
+  return PCNN_OK;
+}
+
+static double layer_flops_exact(const Layer &ly, int B) {
+  const auto &d = ly.d;
+  if (d.kind == PCNN_CONV)
+    return 2.0 * B * (double)ly.out_h * ly.out_w * d.out_channels *
+           ((double)d.kernel * d.kernel * (ly.in_c / d.groups));   // eq. 1
+  if (d.kind == PCNN_FC)
+    return 2.0 * B * (double)d.out_channels * ((double)ly.in_c * ly.in_h * ly.in_w);
+  return 0.0;
+}
+
+static double layer_flops_variant(const Layer &ly, int B) {
+  if (ly.variant != PCNN_VARIANT_RANK) return layer_flops_exact(ly, B);
+  const auto &d = ly.d;
+  const double P = (double)B * ly.out_h * ly.out_w;
+  const double K = (double)d.kernel * d.kernel * (ly.in_c / d.groups);
+  const double Nfg = d.out_channels / d.groups;
+  return 2.0 * P * ly.rank * (K + Nfg) * d.groups;
+}
+
+static double layer_bytes(const Layer &ly, int B, int precision, bool last) {
+  const double e = precision == PCNN_BF16 ? 2.0 : 4.0;
+  const double in = (double)B * ly.in_c * ly.in_h * ly.in_w * e;
+  const double oe = last && ly.d.kind == PCNN_FC ? 4.0 : e;
+  const double out = (double)B * ly.out_c * ly.out_h * ly.out_w * oe;
+  double w = 0;
+  if (ly.d.kind == PCNN_CONV)
+    w = (double)ly.d.out_channels * (ly.in_c / ly.d.groups) * ly.d.kernel * ly.d.kernel * e;
+  if (ly.d.kind == PCNN_FC) w = (double)ly.d.out_channels * ly.in_c * ly.in_h * ly.in_w * e;
+  if (ly.variant == PCNN_VARIANT_RANK && ly.d.kind == PCNN_CONV) {
+    const double K = (double)ly.d.kernel * ly.d.kernel * (ly.in_c / ly.d.groups);
+    const double Nfg = ly.d.out_channels / ly.d.groups;
+    w = (double)ly.d.groups * ly.rank * (K + Nfg) * e;
+    // the stage-1 intermediate is written and read once
+    w += 2.0 * B * ly.out_h * ly.out_w * (double)ly.d.groups * ly.rank * e;
+  }
+  return in + out + w;
+}
+
+// ------------------------------------------------------------------ packing
+// F_m of Fig. 2 in the kernels' layout: row n = g*Nfg + f, column
+// k = (r*S + s)*Cg_stored + c, zero for padded channels and k >= K.
+static std::vector<float> pack_conv(const float *w, int Nf, int Cg_log, int Cg_st, int S,
+                                    int Kpad) {
+  std::vector<float> p((size_t)Nf * Kpad, 0.f);
+  for (int n = 0; n < Nf; ++n)
+    for (int c = 0; c < Cg_log; ++c)
+      for (int r = 0; r < S; ++r)
+        for (int s = 0; s < S; ++s)
+          p[(size_t)n * Kpad + (size_t)(r * S + s) * Cg_st + c] =
+              w[(((size_t)n * Cg_log + c) * S + r) * S + s];
+  return p;
+}
+
+// FC weight [N][C*H*W] (C,H,W order) -> [N][Kpad] over the stored NHWC
+// flatten (h, w, c_stored).
+static std::vector<float> pack_fc(const float *w, int N, int C, int H, int W, int Cs,
+                                  int Kpad) {
+  std::vector<float> p((size_t)N * Kpad, 0.f);
+  const size_t Kin = (size_t)C * H * W;
+  for (int n = 0; n < N; ++n)
+    for (int c = 0; c < C; ++c)
+      for (int h = 0; h < H; ++h)
+        for (int x = 0; x < W; ++x)
+          p[(size_t)n * Kpad + ((size_t)h * W + x) * Cs + c] =
+              w[(size_t)n * Kin + ((size_t)c * H + h) * W + x];
+  return p;
+}
+
+static pcnn_status upload_weights(GemmStage &gs, const std::vector<float> &packed,
+                                  int precision) {
+  const size_t n = packed.size();
+  if (precision == PCNN_BF16) {
+    std::vector<uint16_t> b(n);
+    for (size_t i = 0; i < n; ++i) b[i] = f32_to_bf16_rne(packed[i]);
+    gs.w_bytes = n * 2;
+    CUDA_TRY(cudaMalloc(&gs.d_w, gs.w_bytes));
+    CUDA_TRY(cudaMemcpy(gs.d_w, b.data(), gs.w_bytes, cudaMemcpyHostToDevice));
+  } else {
+    std::vector<float> f(packed);
+    if (precision == PCNN_TF32)
+      for (auto &v : f) v = tf32_rna_host(v);
+    gs.w_bytes = n * 4;
+    CUDA_TRY(cudaMalloc(&gs.d_w, gs.w_bytes));
+    CUDA_TRY(cudaMemcpy(gs.d_w, f.data(), gs.w_bytes, cudaMemcpyHostToDevice));
+  }
+  return PCNN_OK;
+}
+
+static int k_align(int precision) {
+  if (precision == PCNN_BF16) return 64;   // one 128 B K-block
+  if (precision == PCNN_TF32) return 32;
+  return 16;                               // SIMT BK
+}
+
+// Build a GEMM stage.  w_oihw: [Nf][Cg_log][S][S]; for fc (is_fc) w is
+// [N][C*H*W] and the geometry is a 1x1 conv on a 1x1 "image" of K features.
+static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, int Nf,
+                               int groups, int S, int stride, int pad, int relu,
+                               int in_c, int in_h, int in_w, int in_cs, bool is_fc,
+                               const float *w, const float *bias, int out_mode) {
+  gs.release();
+  gs.st = storage_of(precision);
+  gs.engine = precision == PCNN_FP32_SIMT ? 0 : 1;
+  gs.in_c = in_c;
+  gs.in_h = in_h;
+  gs.in_w = in_w;
+  ConvGeom &g = gs.g;
+  std::memset(&g, 0, sizeof g);
+  const int ch = chunk_elems(precision);
+  std::vector<float> packed;
+  if (is_fc) {
+    const int K = in_h * in_w * in_cs;
+    g.H = g.W = 1;
+    g.Cs = K;
+    g.Cg = K;
+    g.S = 1;
+    g.stride = 1;
+    g.pad = 0;
+    g.Ho = g.Wo = 1;
+    g.groups = 1;
+    g.Nfg = Nf;
+    g.K = K;
+    g.Kpad = round_up(K, k_align(precision));
+    packed = pack_fc(w, Nf, in_c, in_h, in_w, in_cs, g.Kpad);
+  } else {
+    const int Cg_log = in_c / groups;
+    const int Cg_st = groups == 1 ? in_cs : Cg_log;
+    if (gs.engine == 1 && (Cg_st % ch)) return fail(PCNN_ERR_UNSUPPORTED,
+        "tcgen05 conv needs channels per group multiple of 16 bytes");
+    g.H = in_h;
+    g.W = in_w;
+    g.Cs = in_cs;
+    g.Cg = Cg_st;
+    g.S = S;
+    g.stride = stride;
+    g.pad = pad;
+    g.Ho = conv_out(in_h, S, stride, pad);
+    g.Wo = conv_out(in_w, S, stride, pad);
+    g.groups = groups;
+    g.Nfg = Nf / groups;
+    g.K = S * S * Cg_st;
+    g.Kpad = round_up(g.K, k_align(precision));
+    packed = pack_conv(w, Nf, Cg_log, Cg_st, S, g.Kpad);
+    if (S > 1) {
+      if (gs.engine == 1 && g.Kpad / ch > tc_max_ktab())
+        return fail(PCNN_ERR_UNSUPPORTED, "conv K too large for the tap table");
+      std::vector<int> tab(g.K);
+      for (int k = 0; k < g.K; ++k) {
+        const int tap = k / Cg_st, c = k % Cg_st;
+        tab[k] = ((tap / S) << 24) | ((tap % S) << 16) | c;
+      }
+      CUDA_TRY(cudaMalloc(&gs.d_ktab, sizeof(int) * g.K));
+      CUDA_TRY(cudaMemcpy(gs.d_ktab, tab.data(), sizeof(int) * g.K, cudaMemcpyHostToDevice));
+    }
+  }
+  if (gs.engine == 1 && (g.Nfg % 8))
+    return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 path needs N_f/g multiple of 8");
+  g.relu = relu;
+  g.out_mode = out_mode;
+  g.out_cs = Nf;
+  pcnn_status st = upload_weights(gs, packed, precision);
+  if (st != PCNN_OK) return st;
+  std::vector<float> b(Nf, 0.f);
+  if (bias) std::memcpy(b.data(), bias, sizeof(float) * Nf);
+  CUDA_TRY(cudaMalloc(&gs.d_bias, sizeof(float) * Nf));
+  CUDA_TRY(cudaMemcpy(gs.d_bias, b.data(), sizeof(float) * Nf, cudaMemcpyHostToDevice));
+  (void)ly;
+  return PCNN_OK;
+}
+
+static const CUtensorMap *stage_tmap(GemmStage &gs, int bn) {
+  auto it = gs.tmaps.find(bn);
+  if (it != gs.tmaps.end()) return &it->second;
+  auto enc = get_encode_tiled();
+  if (!enc) return nullptr;
+  CUtensorMap m;
+  const int esz = esz_of(gs.st);
+  const cuuint64_t dims[2] = {(cuuint64_t)gs.g.Kpad, (cuuint64_t)gs.g.Nfg * gs.g.groups};
+  const cuuint64_t strides[1] = {(cuuint64_t)gs.g.Kpad * esz};
+  const cuuint32_t box[2] = {(cuuint32_t)(128 / esz), (cuuint32_t)bn};
+  const cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                   2, gs.d_w, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return nullptr;
+  return &(gs.tmaps[bn] = m);
+}
+
+// ------------------------------------------------------------------ planning
+// Tile selection (the paper's sub-matrix choice):
+// pick the N tile minimising  waves * kblocks * cost(bn), where one K-block
+// costs max(MMA cycles ~ 2 bn, gather ~ 256 cycles) -- small tiles raise Util
+// (eq. 6) and rEC (eq. 9) but lower the computation density.
+static TcPlan plan_tc(const ConvGeom &g, int n_sms) {
+  TcPlan best{};
+  double best_cost = 1e300;
+  const int mtiles = (g.M + 127) / 128;
+  const int nmax = std::min(256, round_up(g.Nfg, 16));
+  for (int bn = 16; bn <= nmax; bn += 16) {
+    const int ntiles = (g.Nfg + bn - 1) / bn;
+    const long long tiles = (long long)mtiles * ntiles * g.groups;
+    const long long waves = (tiles + n_sms - 1) / n_sms;
+    const double cost = (double)waves * (std::max(2.05 * bn, 256.0) + 40.0);
+    if (cost < best_cost * 0.999 || (cost <= best_cost * 1.001 && bn > best.bn)) {
+      best_cost = cost;
+      best.bn = bn;
+      best.mtiles = mtiles;
+      best.ntiles = ntiles;
+      best.tiles = (int)tiles;
+    }
+  }
+  best.grid = std::min(best.tiles, n_sms);
+  return best;
+}
+
+static int effective_sms(const pcnn_net *net, const Layer &ly) {
+  int n = ly.n_sms <= 0 ? net->num_sms : std::min(ly.n_sms, net->num_sms);
+  return std::max(n, 1);
+}
+
+static bool is_gated(const pcnn_net *net, const Layer &ly) {
+  return (ly.n_sms > 0 && ly.n_sms < net->num_sms) || ly.tlp > 0;
+}
+
+static Budget make_budget(const pcnn_net *net, const Layer &ly, int slot, bool gated_kernel) {
+  Budget b{};
+  b.gated = gated_kernel && is_gated(net, ly) ? 1 : 0;
+  b.n_sms = effective_sms(net, ly);
+  b.tlp = ly.tlp > 0 ? ly.tlp : 1 << 20;
+  b.ctr = ly.d_ctr + (size_t)slot * (1 + kMaxSMs);
+  b.census = net->census ? ly.d_census : nullptr;
+  return b;
+}
+
+// ------------------------------------------------------------------ enqueue
+static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, const void *x,
+                             void *y, int slot, cudaStream_t s, pcnn_layer_info *info) {
+  ConvGeom g = gs.g;
+  g.M = B * g.Ho * g.Wo;
+  if (gs.engine == 1) {
+    TcPlan p = plan_tc(g, effective_sms(net, ly));
+    const CUtensorMap *tm = stage_tmap(gs, p.bn);
+    if (!tm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeTiled failed");
+    if (info) {
+      info->tile_m = 128;
+      info->tile_n = p.bn;
+      info->tiles = p.tiles;
+      info->grid = p.grid;
+      info->tlp = 1;
+      info->engine = 1;
+    }
+    if (!x) return PCNN_OK;   // planning only
+    Budget b = make_budget(net, ly, slot, false);
+    CUDA_TRY(launch_conv_tc(g, gs.st, x, tm, gs.d_bias, y, gs.d_ktab, p, b, s));
+  } else {
+    const int tiles = conv_simt_tiles(g);
+    const bool gated = is_gated(net, ly);
+    int grid = gated ? net->num_sms * net->occ_simt : tiles;
+    if (!gated) grid = std::min(grid, 1 << 30);
+    if (info) {
+      int tm, tn;
+      conv_simt_tile_shape(&tm, &tn);
+      info->tile_m = tm;
+      info->tile_n = tn;
+      info->tiles = tiles;
+      info->grid = grid;
+      info->tlp = ly.tlp > 0 ? ly.tlp : net->occ_simt;
+      info->engine = 0;
+    }
+    if (!x) return PCNN_OK;
+    Budget b = make_budget(net, ly, slot, true);
+    if (b.gated)
+      CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
+    CUDA_TRY(launch_conv_simt(g, (const float *)x, (const float *)gs.d_w, gs.d_bias,
+                              (float *)y, gs.d_ktab, b, grid, s));
+  }
+  return PCNN_OK;
+}
+
+// Enqueue one layer.  x / y are arena buffers (or the user's output for a
+// final FC).  r_buf is the rank-r intermediate buffer.
+static pcnn_status run_layer(pcnn_net *net, int i, int B, const void *x, void *y, void *r_buf,
+                             cudaStream_t s) {
+  Layer &ly = net->layers[i];
+  const int st = net->st;
+  const int tf32 = net->desc.precision == PCNN_TF32;
+  switch (ly.d.kind) {
+    case PCNN_CONV:
+    case PCNN_FC:
+      if (ly.variant == PCNN_VARIANT_RANK) {
+        pcnn_status r = run_stage(net, ly, ly.r1, B, x, r_buf, 0, s, nullptr);
+        if (r != PCNN_OK) return r;
+        return run_stage(net, ly, ly.r2, B, r_buf, y, 1, s, nullptr);
+      }
+      return run_stage(net, ly, ly.exact, B, x, y, 0, s, nullptr);
+    case PCNN_LRN: {
+      const long pixels = (long)B * ly.in_h * ly.in_w;
+      const bool gated = is_gated(net, ly);
+      int grid = gated ? net->num_sms * net->occ_lrn : (int)std::min<long>((pixels + 7) / 8, 1 << 30);
+      Budget b = make_budget(net, ly, 0, true);
+      if (b.gated)
+        CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
+      CUDA_TRY(launch_lrn(x, y, st, tf32, pixels, ly.in_cs, ly.d.kernel, ly.d.lrn_alpha,
+                          ly.d.lrn_beta, ly.d.lrn_k, b, grid, s));
+      return PCNN_OK;
+    }
+    case PCNN_MAXPOOL:
+    case PCNN_AVGPOOL: {
+      const long long total = (long long)B * ly.out_h * ly.out_w * ly.in_cs;
+      const bool gated = is_gated(net, ly);
+      int grid = gated ? net->num_sms * net->occ_pool : (int)std::min<long long>((total + 255) / 256, 1 << 30);
+      Budget b = make_budget(net, ly, 0, true);
+      if (b.gated)
+        CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
+      CUDA_TRY(launch_pool(x, y, st, B, ly.in_h, ly.in_w, ly.in_cs, ly.d.kernel, ly.d.stride,
+                           ly.out_h, ly.out_w, ly.d.kind == PCNN_MAXPOOL, tf32, b, grid, s));
+      return PCNN_OK;
+    }
+  }
+  return fail(PCNN_ERR_INVALID_ARGUMENT, "bad layer kind");
+}
+
+static bool last_is_fc(const pcnn_net *net) { return net->layers.back().d.kind == PCNN_FC; }
+
+// The full pass: staging, every layer, unstaging, softmax + entropy.
+static pcnn_status enqueue_all(pcnn_net *net, const float *d_images, int B, float *d_out,
+                               float *d_p, float *d_h, cudaStream_t s,
+                               std::vector<cudaEvent_t> *evs) {
+  const int st = net->st;
+  const int tf32 = net->desc.precision == PCNN_TF32;
+  if (net->census)
+    for (auto &ly : net->layers) CUDA_TRY(cudaMemsetAsync(ly.d_census, 0, 32, s));
+  CUDA_TRY(launch_stage_input(d_images, net->d_act[0], st, B, net->desc.in_channels,
+                              net->desc.in_height, net->desc.in_width, net->in_cs, tf32, s));
+  if (evs) CUDA_TRY(cudaEventRecord((*evs)[0], s));
+  int cur = 0;
+  const int n = (int)net->layers.size();
+  for (int i = 0; i < n; ++i) {
+    const bool final_fc = (i == n - 1) && last_is_fc(net);
+    void *dst = final_fc ? (void *)d_out : net->d_act[cur ^ 1];
+    pcnn_status r = run_layer(net, i, B, net->d_act[cur], dst, net->d_act[2], s);
+    if (r != PCNN_OK) return r;
+    if (evs) CUDA_TRY(cudaEventRecord((*evs)[i + 1], s));
+    if (!final_fc) cur ^= 1;
+  }
+  if (!last_is_fc(net)) {
+    const Layer &l = net->layers.back();
+    CUDA_TRY(launch_unstage_output(net->d_act[cur], st, d_out, B, l.out_c, l.out_h, l.out_w,
+                                   l.out_cs, s));
+  }
+  if (d_p || d_h) CUDA_TRY(launch_softmax_entropy(d_out, d_p, d_h, B, net->out_elems, s));
+  return PCNN_OK;
+}
+
+// ------------------------------------------------------------------ rank-r
+static pcnn_status build_rank_stages(pcnn_net *net, Layer &ly, int r, const float *A,
+                                     const float *Bf) {
+  // A: [g][Nfg][r], Bf: [g][r][Cg][S][S]
+  const auto &d = ly.d;
+  const int g = d.groups, Nfg = d.out_channels / g, Cg = ly.in_c / g, S = d.kernel;
+  const int prec = net->desc.precision;
+  const int st = net->st;
+  const int ch = chunk_elems(prec);
+  // stage-1 output channels: g*r stored as groups of r; keep each group's r
+  // chunk-aligned for the stage-2 gather (pad r with zero filters).
+  const int rs = round_up(r, ch);
+  std::vector<float> w1((size_t)g * rs * Cg * S * S, 0.f);
+  for (int gi = 0; gi < g; ++gi)
+    for (int a = 0; a < r; ++a)
+      std::memcpy(&w1[((size_t)gi * rs + a) * Cg * S * S], &Bf[((size_t)gi * r + a) * Cg * S * S],
+                  sizeof(float) * Cg * S * S);
+  std::vector<float> w2((size_t)g * Nfg * rs, 0.f);   // [g*Nfg][rs][1][1]
+  for (int gi = 0; gi < g; ++gi)
+    for (int f = 0; f < Nfg; ++f)
+      for (int a = 0; a < r; ++a)
+        w2[((size_t)gi * Nfg + f) * rs + a] = A[((size_t)gi * Nfg + f) * r + a];
+  const int mode1 = st == ST_BF16 ? OUT_BF16 : (prec == PCNN_TF32 ? OUT_F32_TF32 : OUT_F32);
+  pcnn_status s1 = build_stage(ly.r1, ly, prec, g * rs, g, S, d.stride, d.pad, 0, ly.in_c,
+                               ly.in_h, ly.in_w, ly.in_cs, false, w1.data(), nullptr, mode1);
+  if (s1 != PCNN_OK) return s1;
+  const int ho = ly.out_h, wo = ly.out_w;
+  const GemmStage &ex = ly.exact;
+  pcnn_status s2 = build_stage(ly.r2, ly, prec, d.out_channels, g, 1, 1, 0, d.relu, g * rs, ho,
+                               wo, g * rs, false, w2.data(), nullptr, ex.g.out_mode);
+  if (s2 != PCNN_OK) return s2;
+  // stage 2 carries the layer's bias: copy it from the exact stage.
+  CUDA_TRY(cudaMemcpy(ly.r2.d_bias, ex.d_bias, sizeof(float) * d.out_channels,
+                      cudaMemcpyDeviceToDevice));
+  ly.rank = r;
+  ly.variant = PCNN_VARIANT_RANK;
+  net->version++;
+  return PCNN_OK;
+}
+
+// ------------------------------------------------------------------ C ABI
+extern "C" {
+
+const char *pcnn_version(void) { return "pcnn-b200 0.1 (sm_100a)"; }
+
+const char *pcnn_status_string(pcnn_status s) {
+  switch (s) {
+    case PCNN_OK: return "ok";
+    case PCNN_ERR_INVALID_ARGUMENT: return "invalid argument";
+    case PCNN_ERR_SHAPE: return "shape error";
+    case PCNN_ERR_UNSUPPORTED: return "unsupported";
+    case PCNN_ERR_OUT_OF_MEMORY: return "out of memory";
+    case PCNN_ERR_CUDA: return "CUDA error";
+    case PCNN_ERR_BATCH_TOO_LARGE: return "batch too large";
+  }
+  return "unknown status";
+}
+
+const char *pcnn_last_error_message(void) { return g_err.c_str(); }
+
+int pcnn_device_sm_count(int device) {
+  int n = 0;
+  if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return n;
+}
+
+pcnn_status pcnn_describe_net(const pcnn_net_desc *desc, const pcnn_layer_desc *layers,
+                              int n_layers, int batch, pcnn_layer_info *infos) {
+  if (!infos || batch <= 0) return fail(PCNN_ERR_INVALID_ARGUMENT, "null infos / bad batch");
+  std::vector<Layer> ls;
+  pcnn_status s = infer_shapes(desc, layers, n_layers, ls);
+  if (s != PCNN_OK) return s;
+  for (int i = 0; i < n_layers; ++i) {
+    const Layer &ly = ls[i];
+    pcnn_layer_info &f = infos[i];
+    std::memset(&f, 0, sizeof f);
+    f.kind = ly.d.kind;
+    f.in_c = ly.in_c;
+    f.in_h = ly.in_h;
+    f.in_w = ly.in_w;
+    f.out_c = ly.out_c;
+    f.out_h = ly.out_h;
+    f.out_w = ly.out_w;
+    f.groups = ly.gemm ? ly.d.groups : 1;
+    if (ly.d.kind == PCNN_CONV) {
+      f.gemm_m = (long long)batch * ly.out_h * ly.out_w;
+      f.gemm_n = ly.d.out_channels / ly.d.groups;
+      f.gemm_k = ly.d.kernel * ly.d.kernel * (ly.in_c / ly.d.groups);
+    } else if (ly.d.kind == PCNN_FC) {
+      f.gemm_m = batch;
+      f.gemm_n = ly.d.out_channels;
+      f.gemm_k = ly.in_c * ly.in_h * ly.in_w;
+    }
+    f.flops = f.flops_exact = layer_flops_exact(ly, batch);
+    f.bytes = layer_bytes(ly, batch, desc->precision, i == n_layers - 1);
+    f.engine = ly.gemm ? (desc->precision == PCNN_FP32_SIMT ? 0 : 1) : 2;
+  }
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *layers,
+                            int n_layers, const float *const *weights,
+                            const float *const *biases, pcnn_net **out) {
+  if (!out) return fail(PCNN_ERR_INVALID_ARGUMENT, "out is null");
+  *out = nullptr;
+  if (!desc || desc->max_batch <= 0) return fail(PCNN_ERR_INVALID_ARGUMENT, "bad max_batch");
+  std::unique_ptr<pcnn_net> net(new pcnn_net());
+  net->desc = *desc;
+  pcnn_status s = infer_shapes(desc, layers, n_layers, net->layers);
+  if (s != PCNN_OK) return s;
+  for (int i = 0; i < n_layers; ++i)
+    if (net->layers[i].gemm && (!weights || !weights[i]))
+      return fail(PCNN_ERR_INVALID_ARGUMENT, "missing weights for layer " + std::to_string(i));
+  // device
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= desc->device || desc->device < 0) {
+    cudaGetLastError();
+    return fail(PCNN_ERR_CUDA, "no CUDA device " + std::to_string(desc->device));
+  }
+  CUDA_TRY(cudaSetDevice(desc->device));
+  cudaDeviceProp prop;
+  CUDA_TRY(cudaGetDeviceProperties(&prop, desc->device));
+  if (prop.major != 10)
+    return fail(PCNN_ERR_CUDA, std::string("device is not sm_100 (Blackwell): ") + prop.name);
+  net->device = desc->device;
+  net->num_sms = std::min(prop.multiProcessorCount, kMaxSMs);
+  net->st = storage_of(desc->precision);
+  net->in_cs = round_up(desc->in_channels, chunk_elems(desc->precision));
+  net->occ_simt = simt_conv_occupancy();
+  net->occ_lrn = lrn_occupancy();
+  net->occ_pool = pool_occupancy();
+  if (desc->precision != PCNN_FP32_SIMT) {
+    if (!get_encode_tiled())
+      return fail(PCNN_ERR_CUDA, "driver entry point cuTensorMapEncodeTiled unavailable");
+    CUDA_TRY(tc_init());
+  }
+
+  const int prec = desc->precision;
+  const int esz = esz_of(net->st);
+  const int B = desc->max_batch;
+  size_t act = (size_t)B * desc->in_height * desc->in_width * net->in_cs * esz;
+  const int n = n_layers;
+  for (int i = 0; i < n; ++i) {
+    Layer &ly = net->layers[i];
+    act = std::max(act, (size_t)B * ly.out_h * ly.out_w * ly.out_cs * esz);
+    if (ly.gemm) {
+      const bool final_fc = (i == n - 1) && ly.d.kind == PCNN_FC;
+      const int mode = final_fc ? OUT_F32
+                                : (net->st == ST_BF16 ? OUT_BF16
+                                                      : (prec == PCNN_TF32 ? OUT_F32_TF32 : OUT_F32));
+      const bool is_fc = ly.d.kind == PCNN_FC;
+      s = build_stage(ly.exact, ly, prec, ly.d.out_channels, is_fc ? 1 : ly.d.groups,
+                      is_fc ? 1 : ly.d.kernel, is_fc ? 1 : ly.d.stride, is_fc ? 0 : ly.d.pad,
+                      ly.d.relu, ly.in_c, ly.in_h, ly.in_w, ly.in_cs, is_fc, weights[i],
+                      biases ? biases[i] : nullptr, mode);
+      if (s != PCNN_OK) {
+        for (auto &l2 : net->layers) l2.exact.release();
+        return fail(s, "layer " + std::to_string(i) + ": " + g_err);
+      }
+      if (ly.d.kind == PCNN_CONV) {
+        const size_t cnt = (size_t)ly.d.out_channels * (ly.in_c / ly.d.groups) * ly.d.kernel *
+                           ly.d.kernel;
+        ly.host_w.assign(weights[i], weights[i] + cnt);
+      }
+    }
+    CUDA_TRY(cudaMalloc(&ly.d_ctr, sizeof(unsigned long long) * 3 * (1 + kMaxSMs)));
+    CUDA_TRY(cudaMemset(ly.d_ctr, 0, sizeof(unsigned long long) * 3 * (1 + kMaxSMs)));
+    CUDA_TRY(cudaMalloc(&ly.d_census, 32));
+    CUDA_TRY(cudaMemset(ly.d_census, 0, 32));
+  }
+  net->act_bytes = act;
+  for (int k = 0; k < 3; ++k) {
+    if (cudaMalloc(&net->d_act[k], act) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(PCNN_ERR_OUT_OF_MEMORY, "activation arena");
+    }
+  }
+  const Layer &last = net->layers.back();
+  net->out_elems = last.out_c * last.out_h * last.out_w;
+  *out = net.release();
+  return PCNN_OK;
+}
+
+static void destroy_graphs(pcnn_net *net) {
+  for (auto &kv : net->graphs) cudaGraphExecDestroy(kv.second);
+  net->graphs.clear();
+}
+
+pcnn_status pcnn_destroy_net(pcnn_net *net) {
+  if (!net) return PCNN_OK;
+  cudaSetDevice(net->device);
+  destroy_graphs(net);
+  for (auto &ly : net->layers) {
+    ly.exact.release();
+    ly.r1.release();
+    ly.r2.release();
+    if (ly.d_ctr) cudaFree(ly.d_ctr);
+    if (ly.d_census) cudaFree(ly.d_census);
+  }
+  for (auto &p : net->d_act)
+    if (p) cudaFree(p);
+  if (net->d_host_in) cudaFree(net->d_host_in);
+  if (net->d_host_out) cudaFree(net->d_host_out);
+  if (net->d_host_p) cudaFree(net->d_host_p);
+  if (net->d_host_h) cudaFree(net->d_host_h);
+  delete net;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_num_layers(const pcnn_net *net, int *n) {
+  if (!net || !n) return fail(PCNN_ERR_INVALID_ARGUMENT, "null");
+  *n = (int)net->layers.size();
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_output_size(const pcnn_net *net, int *n) {
+  if (!net || !n) return fail(PCNN_ERR_INVALID_ARGUMENT, "null");
+  *n = net->out_elems;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_set_variant(pcnn_net *net, int layer, int variant, int rank) {
+  if (!net || layer < 0 || layer >= (int)net->layers.size())
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad net / layer");
+  Layer &ly = net->layers[layer];
+  if (variant == PCNN_VARIANT_EXACT) {
+    if (ly.variant != PCNN_VARIANT_EXACT) net->version++;
+    ly.variant = PCNN_VARIANT_EXACT;
+    ly.rank = 0;
+    return PCNN_OK;
+  }
+  if (variant != PCNN_VARIANT_RANK) return fail(PCNN_ERR_INVALID_ARGUMENT, "bad variant");
+  if (ly.d.kind != PCNN_CONV)
+    return fail(PCNN_ERR_UNSUPPORTED, "rank variant is implemented for conv layers");
+  const int g = ly.d.groups, Nfg = ly.d.out_channels / g, Cg = ly.in_c / g,
+            S = ly.d.kernel, K = Cg * S * S;
+  const int rmax = std::min(Nfg, K);
+  if (rank < 1 || rank > rmax)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "rank out of [1, min(N_f/g, K)]");
+  CUDA_TRY(cudaSetDevice(net->device));
+  if (ly.svd.empty()) {
+    for (int gi = 0; gi < g; ++gi) {
+      std::vector<double> Wg((size_t)Nfg * K);
+      for (size_t i = 0; i < Wg.size(); ++i) Wg[i] = ly.host_w[(size_t)gi * Nfg * K + i];
+      ly.svd.push_back(svd_rows(Wg, Nfg, K));
+    }
+  }
+  // A = U_r Sigma_r  [g][Nfg][r],  B = V_r^T  [g][r][K]  (K in OIHW (c, r, s) order)
+  std::vector<float> A((size_t)g * Nfg * rank), Bm((size_t)g * rank * K);
+  for (int gi = 0; gi < g; ++gi) {
+    const Svd &sv = ly.svd[gi];
+    for (int f = 0; f < Nfg; ++f)
+      for (int a = 0; a < rank; ++a)
+        A[((size_t)gi * Nfg + f) * rank + a] = (float)(sv.U[(size_t)f * Nfg + a] * sv.sigma[a]);
+    for (int a = 0; a < rank; ++a)
+      for (int k = 0; k < K; ++k)
+        Bm[((size_t)gi * rank + a) * K + k] = (float)sv.Vt[(size_t)a * K + k];
+  }
+  return build_rank_stages(net, ly, rank, A.data(), Bm.data());
+}
+
+pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank, const float *A,
+                                     const float *B) {
+  if (!net || layer < 0 || layer >= (int)net->layers.size() || !A || !B)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  Layer &ly = net->layers[layer];
+  if (ly.d.kind != PCNN_CONV) return fail(PCNN_ERR_UNSUPPORTED, "conv layers only");
+  if (rank < 1 || rank > 4096) return fail(PCNN_ERR_INVALID_ARGUMENT, "bad rank");
+  CUDA_TRY(cudaSetDevice(net->device));
+  return build_rank_stages(net, ly, rank, A, B);
+}
+
+pcnn_status pcnn_set_sm_budget(pcnn_net *net, int layer, int n_sms, int ctas_per_sm) {
+  if (!net || layer < 0 || layer >= (int)net->layers.size() || n_sms < 0 || ctas_per_sm < 0)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  Layer &ly = net->layers[layer];
+  ly.n_sms = n_sms >= net->num_sms ? 0 : n_sms;
+  ly.tlp = ctas_per_sm;
+  net->version++;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_query_layer(const pcnn_net *cnet, int layer, int batch, pcnn_layer_info *f) {
+  pcnn_net *net = const_cast<pcnn_net *>(cnet);
+  if (!net || !f || layer < 0 || layer >= (int)net->layers.size() || batch <= 0)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  Layer &ly = net->layers[layer];
+  std::memset(f, 0, sizeof *f);
+  f->kind = ly.d.kind;
+  f->in_c = ly.in_c;
+  f->in_h = ly.in_h;
+  f->in_w = ly.in_w;
+  f->out_c = ly.out_c;
+  f->out_h = ly.out_h;
+  f->out_w = ly.out_w;
+  f->groups = ly.gemm ? ly.d.groups : 1;
+  f->flops_exact = layer_flops_exact(ly, batch);
+  f->flops = layer_flops_variant(ly, batch);
+  f->bytes = layer_bytes(ly, batch, net->desc.precision, layer == (int)net->layers.size() - 1);
+  f->variant = ly.variant;
+  f->rank = ly.rank;
+  f->n_sms = effective_sms(net, ly);
+  f->tlp = ly.tlp;
+  f->engine = 2;
+  if (ly.gemm) {
+    GemmStage &gs = ly.variant == PCNN_VARIANT_RANK ? ly.r1 : ly.exact;
+    f->gemm_m = (long long)batch * gs.g.Ho * gs.g.Wo;
+    f->gemm_n = ly.exact.g.Nfg;
+    f->gemm_k = ly.d.kind == PCNN_CONV ? ly.d.kernel * ly.d.kernel * (ly.in_c / ly.d.groups)
+                                       : ly.in_c * ly.in_h * ly.in_w;
+    pcnn_status s = run_stage(net, ly, ly.variant == PCNN_VARIANT_RANK ? ly.r2 : ly.exact,
+                              batch, nullptr, nullptr, 0, nullptr, f);
+    if (s != PCNN_OK) return s;
+    const long long maxb = (long long)f->n_sms * std::max(f->tlp, 1);
+    const long long waves = (f->tiles + maxb - 1) / maxb;
+    f->util = (double)f->tiles / ((double)waves * maxb);                 // eq. 6
+    const long long M = f->gemm_m, N = f->gemm_n;
+    const long long mt = (M + f->tile_m - 1) / f->tile_m, nt = (N + f->tile_n - 1) / f->tile_n;
+    f->rec = (double)M * N / ((double)mt * nt * f->tile_m * f->tile_n);   // eq. 9
+  }
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_infer(pcnn_net *net, const float *d_images, int batch, float *d_out,
+                       float *d_probs, float *d_entropy, void *stream) {
+  if (!net || !d_images || !d_out) return fail(PCNN_ERR_INVALID_ARGUMENT, "null pointer");
+  if (batch <= 0) return fail(PCNN_ERR_INVALID_ARGUMENT, "batch must be positive");
+  if (batch > net->desc.max_batch) return fail(PCNN_ERR_BATCH_TOO_LARGE, "batch > max_batch");
+  CUDA_TRY(cudaSetDevice(net->device));
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!net->use_graphs || net->census || s == nullptr)
+    return enqueue_all(net, d_images, batch, d_out, d_probs, d_entropy, s, nullptr);
+  pcnn_net::GraphKey key{batch, d_images, d_out, d_probs, d_entropy, s, net->version};
+  auto it = net->graphs.find(key);
+  if (it == net->graphs.end()) {
+    if (net->graphs.size() > 64) destroy_graphs(net);
+    CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    pcnn_status r = enqueue_all(net, d_images, batch, d_out, d_probs, d_entropy, s, nullptr);
+    cudaGraph_t graph = nullptr;
+    cudaError_t ce = cudaStreamEndCapture(s, &graph);
+    if (r != PCNN_OK) {
+      if (graph) cudaGraphDestroy(graph);
+      return r;
+    }
+    if (ce != cudaSuccess) return fail(PCNN_ERR_CUDA, std::string("graph capture: ") + cudaGetErrorString(ce));
+    cudaGraphExec_t exec = nullptr;
+    ce = cudaGraphInstantiate(&exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (ce != cudaSuccess) return fail(PCNN_ERR_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(ce));
+    it = net->graphs.emplace(key, exec).first;
+  }
+  CUDA_TRY(cudaGraphLaunch(it->second, s));
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch, float *h_out,
+                            float *h_probs, float *h_entropy, void *stream) {
+  if (!net || !h_images || !h_out) return fail(PCNN_ERR_INVALID_ARGUMENT, "null pointer");
+  if (batch <= 0 || batch > net->desc.max_batch)
+    return fail(PCNN_ERR_BATCH_TOO_LARGE, "bad batch");
+  CUDA_TRY(cudaSetDevice(net->device));
+  const size_t in_elems = (size_t)net->desc.in_channels * net->desc.in_height * net->desc.in_width;
+  const size_t maxb = net->desc.max_batch;
+  if (!net->d_host_in) {
+    CUDA_TRY(cudaMalloc(&net->d_host_in, sizeof(float) * in_elems * maxb));
+    CUDA_TRY(cudaMalloc(&net->d_host_out, sizeof(float) * net->out_elems * maxb));
+    CUDA_TRY(cudaMalloc(&net->d_host_p, sizeof(float) * net->out_elems * maxb));
+    CUDA_TRY(cudaMalloc(&net->d_host_h, sizeof(float) * maxb));
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  CUDA_TRY(cudaMemcpyAsync(net->d_host_in, h_images, sizeof(float) * in_elems * batch,
+                           cudaMemcpyHostToDevice, s));
+  pcnn_status r = pcnn_infer(net, net->d_host_in, batch, net->d_host_out,
+                             h_probs ? net->d_host_p : nullptr,
+                             h_entropy ? net->d_host_h : nullptr, stream);
+  if (r != PCNN_OK) return r;
+  CUDA_TRY(cudaMemcpyAsync(h_out, net->d_host_out, sizeof(float) * net->out_elems * batch,
+                           cudaMemcpyDeviceToHost, s));
+  if (h_probs)
+    CUDA_TRY(cudaMemcpyAsync(h_probs, net->d_host_p, sizeof(float) * net->out_elems * batch,
+                             cudaMemcpyDeviceToHost, s));
+  if (h_entropy)
+    CUDA_TRY(cudaMemcpyAsync(h_entropy, net->d_host_h, sizeof(float) * batch,
+                             cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_profile_layers(pcnn_net *net, const float *d_images, int batch, float *d_out,
+                                int reps, float *layer_ms, float *total_ms, void *stream) {
+  if (!net || !d_images || !d_out || !layer_ms || reps <= 0)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  if (batch <= 0 || batch > net->desc.max_batch) return fail(PCNN_ERR_BATCH_TOO_LARGE, "bad batch");
+  CUDA_TRY(cudaSetDevice(net->device));
+  cudaStream_t s = (cudaStream_t)stream;
+  const int n = (int)net->layers.size();
+  std::vector<cudaEvent_t> ev(n + 1);
+  cudaEvent_t e_begin, e_end;
+  for (auto &e : ev) CUDA_TRY(cudaEventCreate(&e));
+  CUDA_TRY(cudaEventCreate(&e_begin));
+  CUDA_TRY(cudaEventCreate(&e_end));
+  std::vector<double> acc(n, 0.0);
+  double tot = 0;
+  for (int r = 0; r < reps; ++r) {
+    CUDA_TRY(cudaEventRecord(e_begin, s));
+    pcnn_status st = enqueue_all(net, d_images, batch, d_out, nullptr, nullptr, s, &ev);
+    if (st != PCNN_OK) return st;
+    CUDA_TRY(cudaEventRecord(e_end, s));
+    CUDA_TRY(cudaEventSynchronize(e_end));
+    for (int i = 0; i < n; ++i) {
+      float ms = 0;
+      CUDA_TRY(cudaEventElapsedTime(&ms, ev[i], ev[i + 1]));
+      acc[i] += ms;
+    }
+    float t = 0;
+    CUDA_TRY(cudaEventElapsedTime(&t, e_begin, e_end));
+    tot += t;
+  }
+  for (int i = 0; i < n; ++i) layer_ms[i] = (float)(acc[i] / reps);
+  if (total_ms) *total_ms = (float)(tot / reps);
+  for (auto &e : ev) cudaEventDestroy(e);
+  cudaEventDestroy(e_begin);
+  cudaEventDestroy(e_end);
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_enable_sm_census(pcnn_net *net, int enable) {
+  if (!net) return fail(PCNN_ERR_INVALID_ARGUMENT, "null net");
+  net->census = enable != 0;
+  net->version++;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_get_sm_census(pcnn_net *net, int layer, unsigned int mask_out[8]) {
+  if (!net || !mask_out || layer < 0 || layer >= (int)net->layers.size())
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  CUDA_TRY(cudaSetDevice(net->device));
+  CUDA_TRY(cudaMemcpy(mask_out, net->layers[layer].d_census, 32, cudaMemcpyDeviceToHost));
+  return PCNN_OK;
+}
+
+}  // extern "C"

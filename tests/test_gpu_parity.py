@@ -1,0 +1,174 @@
+"""Parity of the CUDA path (through the C ABI) against the FP64 oracle on the
+same seeded inputs.  Tolerances from north_star (R10):
+max|err|/max|ref| <= 1e-4 (FP32 SIMT), 5e-3 (TF32), 2e-2 (BF16); max-pool
+bitwise; top-1 identical (margin-aware on iid inputs)."""
+import numpy as np
+import pytest
+
+import synth
+from tests.helpers import TOL, conv_layer, gpu_run, params, rel_err, small_inputs
+
+pytestmark = pytest.mark.gpu
+PRECS = ["fp32", "tf32", "bf16"]
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    from paper_conf_hpca_songhcl17_b200 import pcnn  # noqa: F401  (fails loudly if unbuilt)
+
+
+# ------------------------------------------------------------ config 0 (CIFAR-quick)
+@pytest.mark.parametrize("prec", PRECS)
+def test_cifar_quick_config0(orc, prec):
+    net = synth.cifar_quick()
+    w, b = params(net)
+    x = synth.images(0, 1, net["in_shape"], lo=-1, hi=1)
+    ref = orc.run_net(net, w, b, x).reshape(1, -1)
+    out = gpu_run(net, w, b, x, prec)["out"]
+    assert rel_err(out, ref) <= TOL[prec]
+    assert (out >= 0).all()
+
+
+# ------------------------------------------------------------ layer-isolated conv
+CONV_CASES = [
+    # (out, k, in_c, stride, pad, groups, H, W, B)
+    (16, 5, 3, 1, 2, 1, 32, 32, 1),        # configs[0] geometry
+    (96, 11, 3, 4, 0, 1, 67, 67, 2),       # AlexNet conv1 geometry, smaller image
+    (256, 5, 96, 1, 2, 2, 27, 27, 1),      # AlexNet conv2 (groups 2, C/g = 48)
+    (384, 3, 256, 1, 1, 1, 13, 13, 3),     # conv3: ragged M (507 rows), N = 384
+    (192, 3, 192, 1, 1, 2, 13, 13, 2),     # conv4-like, groups 2
+    (64, 3, 64, 1, 1, 1, 20, 18, 2),       # VGG conv1_2-like, ragged tiles
+    (40, 3, 16, 2, 1, 1, 17, 15, 3),       # N not a tile multiple, stride 2
+    (128, 1, 64, 1, 0, 1, 9, 9, 2),        # 1x1 conv
+]
+
+
+@pytest.mark.parametrize("prec", PRECS)
+@pytest.mark.parametrize("case", CONV_CASES, ids=lambda c: "x".join(map(str, c)))
+def test_conv_layer_parity(orc, prec, case):
+    out_c, k, in_c, st, pad, g, H, W, B = case
+    net = dict(in_shape=(in_c, H, W),
+               layers=[conv_layer(out_c, k, in_c, st, pad, g, relu=False)])
+    w, b = params(net, seed=31)
+    x = small_inputs((in_c, H, W), B)
+    ref = orc.run_net(net, w, b, x).reshape(B, -1)
+    out = gpu_run(net, w, b, x, prec)["out"]
+    assert rel_err(out, ref) <= TOL[prec] / 4
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_fc_layer_parity_and_chw_flatten(orc, prec):
+    # FC directly on a spatial input: columns permuted CHW -> HWC at create.
+    net = dict(in_shape=(16, 3, 5), layers=[dict(kind="fc", out=40, in_f=16 * 15, relu=False)])
+    w, b = params(net, seed=5)
+    x = small_inputs((16, 3, 5), 5)
+    ref = orc.run_net(net, w, b, x)
+    out = gpu_run(net, w, b, x, prec)["out"]
+    assert rel_err(out, ref) <= TOL[prec] / 4
+    # single-column probe: only input element (c=7, h=2, w=1) matters
+    wp = np.zeros_like(w[0])
+    col = 7 * 15 + 2 * 5 + 1
+    wp[:, col] = synth.round_to_bf16(np.linspace(-1, 1, 40))
+    out = gpu_run(net, [wp], [np.zeros(40, np.float32)], x, prec)["out"]
+    np.testing.assert_allclose(out, x[:, 7, 2, 1][:, None] * wp[:, col][None, :],
+                               rtol=1e-2 if prec == "bf16" else 1e-6, atol=1e-6)
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_maxpool_bitwise(orc, prec):
+    net = dict(in_shape=(24, 27, 27), layers=[dict(kind="maxpool", k=3, stride=2)])
+    x = small_inputs((24, 27, 27), 3, lo=-100, hi=100)
+    ref = orc.run_net(net, [None], [None], x).reshape(3, -1)
+    out = gpu_run(net, [None], [None], x, prec)["out"]
+    np.testing.assert_array_equal(out, ref.astype(np.float32))
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_avgpool(orc, prec):
+    net = dict(in_shape=(16, 14, 14), layers=[dict(kind="avgpool", k=2, stride=2)])
+    x = small_inputs((16, 14, 14), 2)
+    ref = orc.run_net(net, [None], [None], x).reshape(2, -1)
+    out = gpu_run(net, [None], [None], x, prec)["out"]
+    assert rel_err(out, ref) <= TOL[prec] / 4
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_lrn_parity(orc, prec):
+    # Caffe-scale inputs make the LRN term O(1) (reading R3), C = 96 like norm1
+    L = dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0)
+    net = dict(in_shape=(96, 9, 7), layers=[L])
+    x = small_inputs((96, 9, 7), 2, lo=-128, hi=128)
+    ref = orc.run_net(net, [None], [None], x).reshape(2, -1)
+    out = gpu_run(net, [None], [None], x, prec)["out"]
+    assert rel_err(out, ref) <= TOL[prec] / 4
+    assert np.abs(ref - x.reshape(2, -1)).max() > 1.0      # LRN is active
+
+
+# ------------------------------------------------------------ softmax + entropy
+def test_softmax_entropy_parity(orc):
+    net = synth.cifar_quick()
+    net = dict(in_shape=(8, 4, 4), layers=[dict(kind="fc", out=1000, in_f=128, relu=False)])
+    w, b = params(net, seed=9)
+    x = small_inputs((8, 4, 4), 6, lo=-30, hi=30)
+    r = gpu_run(net, w, b, x, "fp32", probs=True)
+    p_ref, h_ref = orc.softmax_entropy(r["out"].astype(np.float64))
+    np.testing.assert_allclose(r["probs"], p_ref, rtol=2e-5, atol=1e-9)
+    np.testing.assert_allclose(r["entropy"], h_ref, rtol=2e-5, atol=2e-6)
+    np.testing.assert_allclose(r["probs"].sum(1), 1.0, rtol=1e-5)
+
+
+# ------------------------------------------------------------ end to end
+def _top1_agreement(out, ref, tol):
+    top_g, top_r = out.argmax(1), ref.argmax(1)
+    srt = np.sort(ref, axis=1)
+    margin = srt[:, -1] - srt[:, -2]
+    near_tie = margin < 2 * tol * np.abs(ref).max()
+    agree = (top_g == top_r) | near_tie
+    return agree.mean(), (top_g == top_r).mean()
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_alexnet_end_to_end(orc, prec):
+    net = synth.alexnet()
+    w, b = params(net)
+    B = 4
+    x = synth.images(0, B, net["in_shape"])
+    ref = orc.run_net(net, w, b, x)
+    r = gpu_run(net, w, b, x, prec, probs=True)
+    err = rel_err(r["out"], ref)
+    assert err <= TOL[prec], err
+    aware, raw = _top1_agreement(r["out"], ref, TOL[prec])
+    assert aware == 1.0
+    p_ref, h_ref = orc.softmax_entropy(ref)
+    assert np.abs(r["entropy"] - h_ref).max() < 0.05 + 10 * err
+
+
+@pytest.mark.parametrize("prec", ["tf32", "bf16"])
+def test_vgg16_end_to_end(orc, prec):
+    net = synth.vgg16()
+    w, b = params(net)
+    x = synth.images(0, 2, net["in_shape"])
+    ref = orc.run_net(net, w, b, x)
+    out = gpu_run(net, w, b, x, prec)["out"]
+    assert rel_err(out, ref) <= TOL[prec]
+    aware, _ = _top1_agreement(out, ref, TOL[prec])
+    assert aware == 1.0
+
+
+def test_infer_host_matches_device(orc):
+    import torch
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    net = synth.alexnet()
+    w, b = params(net)
+    x = synth.images(0, 3, net["in_shape"])
+    n = pcnn.Net(net, w, b, 4, "bf16")
+    xd = torch.from_numpy(x).cuda()
+    out, _, _ = n.infer(xd)
+    torch.cuda.synchronize()
+    xh = torch.from_numpy(x).pin_memory()
+    oh = torch.empty((3, 1000)).pin_memory()
+    n.infer_host(xh, oh)
+    np.testing.assert_array_equal(oh.numpy(), out.cpu().numpy())
