@@ -120,6 +120,7 @@ typedef struct {
     int grid;           /* CTAs launched                                     */
     double util;        /* eq. 6 with maxBlocks = n_sms * tlp                */
     double rec;         /* eq. 9 (tile-padding efficiency)                   */
+    int splits;         /* split-K factor of the GEMM (1 = none)             */
 } pcnn_layer_info;
 
 typedef struct pcnn_net pcnn_net;
@@ -207,6 +208,19 @@ pcnn_status pcnn_profile_layers(pcnn_net *net, const float *d_images,
                                 int batch, float *d_out, int reps,
                                 float *layer_ms, float *total_ms,
                                 void *stream);
+
+/* Live per-layer timing.  While enabled, pcnn_infer runs without CUDA graphs
+ * and records a CUDA event on the caller's stream after input staging and
+ * after every layer.  pcnn_read_layer_timing synchronises those events and
+ * returns, per layer, the milliseconds summed over all pcnn_infer calls since
+ * the previous read (*n_steps = number of calls), then resets. */
+pcnn_status pcnn_set_layer_timing(pcnn_net *net, int enable);
+pcnn_status pcnn_read_layer_timing(pcnn_net *net, float *layer_ms,
+                                   int *n_steps);
+
+/* Number of CUDA kernels the last pcnn_infer enqueue launched (a graph
+ * replay launches the same kernels as the capture that built it). */
+pcnn_status pcnn_last_launch_count(const pcnn_net *net, int *launches);
 
 /* Test hook: when enabled, every admitted CTA of every layer kernel records
  * its %smid; pcnn_get_sm_census returns the 256-bit SM mask (8 words) seen

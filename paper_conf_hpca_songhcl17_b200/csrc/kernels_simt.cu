@@ -1,7 +1,10 @@
 // kernels_simt.cu -- SIMT kernels of the hot path (sm_100a):
-//   a1 input staging, final unstaging, FP32 implicit-GEMM conv/FC check path
-//   (the paper's SGEMM), a4 LRN, a5 pooling, a7 softmax + entropy.
+//   a1 input staging (incl. space-to-depth), final unstaging, FP32 implicit-GEMM
+//   conv/FC check path
+//   (the paper's SGEMM), a4/a5 LRN + pooling (fused), a7 softmax + entropy.
 // Activations are NHWC; all arithmetic is fp32; storage is bf16 or fp32.
+#include <algorithm>
+
 #include "budget.cuh"
 #include "pcnn_internal.h"
 
@@ -27,42 +30,100 @@ __device__ __forceinline__ void store_act(void *p, int st, size_t i, float v,
     ((float *)p)[i] = tf32_round ? tf32_rna(v) : v;
 }
 
+// ------------------------------------------------------------ vector helpers
+// 16 B of storage = 8 bf16 or 4 fp32 values, converted to / from fp32.
+template <int ST>
+struct Vec16 {
+  static constexpr int N = ST == ST_BF16 ? 8 : 4;
+  float v[N];
+  __device__ __forceinline__ void load(const void *p) {
+    const uint4 raw = *(const uint4 *)p;
+    if constexpr (ST == ST_BF16) {
+      const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float2 f = __bfloat1622float2(h[i]);
+        v[2 * i] = f.x;
+        v[2 * i + 1] = f.y;
+      }
+    } else {
+      const float *f = (const float *)&raw;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[i] = f[i];
+    }
+  }
+  __device__ __forceinline__ void store(void *p, int tf32_round) const {
+    uint4 raw;
+    if constexpr (ST == ST_BF16) {
+      __nv_bfloat162 *h = (__nv_bfloat162 *)&raw;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) h[i] = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+    } else {
+      float *f = (float *)&raw;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) f[i] = tf32_round ? tf32_rna(v[i]) : v[i];
+    }
+    *(uint4 *)p = raw;
+  }
+};
+
 // ------------------------------------------------------------ a1: staging
-// One thread per (pixel, 4-channel group): reads NCHW (coalesced along W per
-// channel), writes NHWC with zero-filled channel padding.
-__global__ void stage_input_kernel(const float *__restrict__ x, void *y, int st,
-                                   int B, int C, int H, int W, int Cs,
-                                   int tf32_round) {
+// NCHW fp32 -> NHWC storage [B][Hs][Ws][Cs].  Output channel c' < blk^2*C is
+// (dr, ds, c) = (c' / C / blk, c' / C % blk, c' % C) and reads input pixel
+// (h'*blk - pad + dr, w'*blk - pad + ds); blk = 1 is the plain layout with
+// zero channel padding, blk = stride is space-to-depth for a strided first
+// conv (turns AlexNet's 11x11/4 conv on 3 channels into a 3x3/1 conv on 48,
+// so the GEMM's K is 432 instead of 968 with 8-channel padding).  Rounded to
+// the storage precision (BF16 RN-even, TF32 RN-away).  One thread per
+// (pixel, 16 B chunk); chunk index fastest so the stores are coalesced.
+template <int ST>
+__global__ void __launch_bounds__(256)
+stage_input_kernel(const float *__restrict__ x, void *y, int B, int C, int H, int W, int Hs,
+                   int Ws, int Cs, int blk, int pad, int tf32_round) {
+  constexpr int VN = Vec16<ST>::N;
+  const int chunks = Cs / VN;
+  const long long total = (long long)B * Hs * Ws * chunks;
   const long long HW = (long long)H * W;
-  const int groups4 = Cs / 4;
-  const long long total = (long long)B * HW * groups4;
+  const int creal = blk * blk * C;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
        i += (long long)gridDim.x * blockDim.x) {
-    const long long pix = i % (B * HW);
-    const int cg = (int)(i / (B * HW));
-    const long long n = pix / HW, hw = pix % HW;
+    const int ch = (int)(i % chunks);
+    const long long pix = i / chunks;
+    const int ws = (int)(pix % Ws);
+    const long long t = pix / Ws;
+    const int hs = (int)(t % Hs);
+    const long long n = t / Hs;
+    Vec16<ST> o;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int c = cg * 4 + j;
+    for (int j = 0; j < VN; ++j) {
+      const int cp = ch * VN + j;
       float v = 0.f;
-      if (c < C) v = __ldg(&x[(n * C + c) * HW + hw]);
-      store_act(y, st, (size_t)pix * Cs + c, v, tf32_round);
+      if (cp < creal) {
+        const int b = cp / C, c = cp - b * C;
+        const int ih = hs * blk - pad + b / blk, iw = ws * blk - pad + b % blk;
+        if (ih >= 0 && ih < H && iw >= 0 && iw < W) v = __ldg(&x[(n * C + c) * HW + (long long)ih * W + iw]);
+      }
+      o.v[j] = v;
     }
+    o.store((char *)y + (size_t)i * 16, tf32_round);
   }
 }
 
-cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C,
-                               int H, int W, int Cs, int tf32_round,
+cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
+                               int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {
-  const long long total = (long long)B * H * W * (Cs / 4);
-  int grid = (int)((total + 255) / 256);
-  if (grid > 148 * 16) grid = 148 * 16;
-  if (grid < 1) grid = 1;
-  stage_input_kernel<<<grid, 256, 0, s>>>(x, y, st, B, C, H, W, Cs, tf32_round);
+  const int vn = st == ST_BF16 ? 8 : 4;
+  const long long total = (long long)B * Hs * Ws * (Cs / vn);
+  const int grid = (int)std::max<long long>(1, std::min<long long>((total + 255) / 256, 148 * 16));
+  if (st == ST_BF16)
+    stage_input_kernel<ST_BF16><<<grid, 256, 0, s>>>(x, y, B, C, H, W, Hs, Ws, Cs, blk, pad, 0);
+  else
+    stage_input_kernel<ST_F32><<<grid, 256, 0, s>>>(x, y, B, C, H, W, Hs, Ws, Cs, blk, pad,
+                                                    tf32_round);
   return cudaGetLastError();
 }
 
-// final NHWC storage -> NCHW fp32 (C,H,W flatten order, reading R5)
+// final NHWC storage -> NCHW fp32 flatten (C,H,W order, reading R5)
 __global__ void unstage_output_kernel(const void *x, int st, float *y, int B,
                                       int C, int H, int W, int Cs) {
   const long long HW = (long long)H * W;
@@ -218,100 +279,181 @@ cudaError_t launch_conv_simt(const ConvGeom &g, const float *x, const float *w,
   return cudaGetLastError();
 }
 
-// ------------------------------------------------------------ a4: LRN
-// Across-channel LRN (reading R3) on NHWC: one warp per pixel; the pixel's
-// channel vector is staged in smem and each lane sums its 5-channel window.
-constexpr int LRN_WARPS = 8;
-constexpr int LRN_MAXC = 1024;
+// ------------------------------------------------------------ a4 + a5: LRN and pooling
+// One kernel for LRN (reading R3), max / avg pooling (R4), and the fused
+// LRN -> max-pool pair of AlexNet (norm1 -> pool1, norm2 -> pool2).  NHWC.
+// A tile is (image n, output row p, output columns [q0, q0 + Q)): the pool
+// window rows [p*s, p*s + k) x the columns they cover are contiguous runs of
+// C channels in memory, loaded into smem with coalesced 16 B vectors.  LRN
+// (when enabled) transforms every staged pixel's channel vector -- rounded to
+// the storage precision exactly as the stand-alone layer would store it -- and
+// the pool reduces k x k windows of 16 B channel chunks.  Without pooling
+// (k = s = 1) the kernel is the stand-alone LRN; without LRN it is the pool.
+struct LrnPoolArgs {
+  const void *x;
+  void *y;
+  int B, H, W, C;
+  int lrn_size;            // 0 = no LRN
+  float lrn_alpha_over_n, lrn_beta, lrn_k;
+  int k, s, is_max;        // pool window / stride (1, 1 = no pool)
+  int Ho, Wo;
+  int Q, nqt;              // output columns per tile, tiles per row
+  int tf32_round;
+  Budget b;
+};
 
-__global__ void __launch_bounds__(LRN_WARPS * 32)
-lrn_kernel(const void *x, void *y, int st, int tf32_round, long long pixels,
-           int C, int size, float alpha, float beta, float k, Budget b) {
-  __shared__ float buf[LRN_WARPS][LRN_MAXC];
-  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int half = size / 2;
-  const float a_over_n = alpha / (float)size;
-  const long long tiles = (pixels + LRN_WARPS - 1) / LRN_WARPS;
-  for_each_tile(b, tiles, [&](long long t) {
-    const long long pix = t * LRN_WARPS + warp;
-    if (pix < pixels) {
-      const size_t base = (size_t)pix * C;
-      for (int c = lane; c < C; c += 32) buf[warp][c] = load_act(x, st, base + c);
-      __syncwarp();
-      for (int c = lane; c < C; c += 32) {
-        const int lo = c - half < 0 ? 0 : c - half;
-        const int hi = c + half > C - 1 ? C - 1 : c + half;
-        float sq = 0.f;
-        for (int cc = lo; cc <= hi; ++cc) sq = fmaf(buf[warp][cc], buf[warp][cc], sq);
-        const float scale = k + a_over_n * sq;
-        store_act(y, st, base + c, buf[warp][c] * powf(scale, -beta), tf32_round);
-      }
-      __syncwarp();
+template <int ST>
+__global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
+  extern __shared__ __align__(16) uint8_t lp_smem[];
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  constexpr int VN = Vec16<ST>::N;
+  const int C = a.C, chunks = C / VN;
+  const int wc_max = (a.Q - 1) * a.s + a.k;
+  const size_t tile_elems = (size_t)a.k * wc_max * C;
+  uint8_t *T = lp_smem;                                  // staged input
+  uint8_t *U = a.lrn_size > 0 ? lp_smem + tile_elems * ESZ : lp_smem;   // LRN output
+  const long long tiles = (long long)a.B * a.Ho * a.nqt;
+  const int half = a.lrn_size / 2;
+
+  for_each_tile(a.b, tiles, [&](long long t) {
+    const int qt = (int)(t % a.nqt);
+    const long long r2 = t / a.nqt;
+    const int p = (int)(r2 % a.Ho);
+    const long long n = r2 / a.Ho;
+    const int q0 = qt * a.Q, q1 = min(q0 + a.Q, a.Wo);
+    const int h0 = p * a.s, h1 = min(h0 + a.k, a.H);
+    const int w0 = q0 * a.s, w1 = min((q1 - 1) * a.s + a.k, a.W);
+    const int nr = h1 - h0, wc = w1 - w0;
+    __syncthreads();
+    // stage rows [h0, h1) x cols [w0, w1): each row segment is contiguous
+    const int vec_per_row = wc * chunks;
+    for (int v = threadIdx.x; v < nr * vec_per_row; v += blockDim.x) {
+      const int r = v / vec_per_row, rem = v - r * vec_per_row;
+      const size_t src = (((size_t)n * a.H + h0 + r) * a.W + w0) * C + (size_t)rem * VN;
+      *(uint4 *)(T + ((size_t)r * wc_max * C + (size_t)rem * VN) * ESZ) =
+          __ldg((const uint4 *)((const char *)a.x + src * ESZ));
     }
-  });
-}
-
-int lrn_occupancy() {
-  int n = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lrn_kernel, LRN_WARPS * 32, 0);
-  return n > 0 ? n : 1;
-}
-
-cudaError_t launch_lrn(const void *x, void *y, int st, int tf32_round,
-                       long pixels, int C, int size, float alpha, float beta,
-                       float k, const Budget &b, int grid, cudaStream_t s) {
-  if (C > LRN_MAXC) return cudaErrorInvalidValue;
-  lrn_kernel<<<grid, LRN_WARPS * 32, 0, s>>>(x, y, st, tf32_round, pixels, C,
-                                             size, alpha, beta, k, b);
-  return cudaGetLastError();
-}
-
-// ------------------------------------------------------------ a5: pooling
-// One thread per (output pixel, channel); consecutive threads walk channels
-// (contiguous in NHWC) so loads and stores are coalesced.
-constexpr int POOL_THREADS = 256;
-
-__global__ void __launch_bounds__(POOL_THREADS)
-pool_kernel(const void *x, void *y, int st, int B, int H, int W, int C, int k,
-            int stride, int Ho, int Wo, int is_max, int tf32_round, Budget b) {
-  const long long total = (long long)B * Ho * Wo * C;
-  const long long tiles = (total + POOL_THREADS - 1) / POOL_THREADS;
-  for_each_tile(b, tiles, [&](long long t) {
-    const long long i = t * POOL_THREADS + threadIdx.x;
-    if (i < total) {
-      const int c = (int)(i % C);
-      const long long op = i / C;
-      const int q = (int)(op % Wo);
-      const long long np = op / Wo;
-      const int p = (int)(np % Ho);
-      const long long n = np / Ho;
-      const int h0 = p * stride, w0 = q * stride;
-      const int h1 = min(h0 + k, H), w1 = min(w0 + k, W);
-      float m = -INFINITY, sum = 0.f;
-      for (int h = h0; h < h1; ++h)
-        for (int w = w0; w < w1; ++w) {
-          const float v = load_act(x, st, (size_t)(((n * H + h) * W + w) * C + c));
-          m = fmaxf(m, v);
-          sum += v;
+    __syncthreads();
+    if (a.lrn_size > 0) {
+      for (int v = threadIdx.x; v < nr * wc * chunks; v += blockDim.x) {
+        const int ch = v % chunks, pix = v / chunks;
+        const int r = pix / wc, col = pix - r * wc;
+        const size_t base = ((size_t)r * wc_max + col) * C;
+        const int c0 = ch * VN;
+        float sq[VN + 16];
+        const int lo = c0 - half;
+#pragma unroll
+        for (int j = 0; j < VN + 16; ++j) {
+          if (j < VN + 2 * half) {
+            const int c = lo + j;
+            float xv = 0.f;
+            if (c >= 0 && c < C) {
+              xv = ST == ST_BF16 ? __bfloat162float(((const __nv_bfloat16 *)T)[base + c])
+                                 : ((const float *)T)[base + c];
+            }
+            sq[j] = xv * xv;
+          }
         }
-      const float out = is_max ? m : sum / (float)(k * k);
-      store_act(y, st, (size_t)i, out, is_max ? 0 : tf32_round);
+        Vec16<ST> in, out;
+        in.load(T + (base + c0) * ESZ);
+#pragma unroll
+        for (int j = 0; j < VN; ++j) {
+          float acc = 0.f;
+          for (int w = 0; w < a.lrn_size; ++w) acc += sq[j + w];
+          const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
+          out.v[j] = in.v[j] * exp2f(-a.lrn_beta * __log2f(scale));
+        }
+        out.store(U + (base + c0) * ESZ, a.tf32_round);
+      }
+      __syncthreads();
+    }
+    // pool the staged (and normalised) rows
+    const float inv = 1.f / (float)(a.k * a.k);
+    for (int v = threadIdx.x; v < (q1 - q0) * chunks; v += blockDim.x) {
+      const int ch = v % chunks, q = q0 + v / chunks;
+      const int cs = q * a.s - w0, ce = min(cs + a.k, wc);
+      Vec16<ST> acc, cur;
+#pragma unroll
+      for (int j = 0; j < VN; ++j) acc.v[j] = a.is_max ? -INFINITY : 0.f;
+      for (int r = 0; r < nr; ++r)
+        for (int col = cs; col < ce; ++col) {
+          cur.load(U + (((size_t)r * wc_max + col) * C + ch * VN) * ESZ);
+#pragma unroll
+          for (int j = 0; j < VN; ++j)
+            acc.v[j] = a.is_max ? fmaxf(acc.v[j], cur.v[j]) : acc.v[j] + cur.v[j];
+        }
+      if (!a.is_max)
+#pragma unroll
+        for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
+      acc.store((char *)a.y + ((((size_t)n * a.Ho + p) * a.Wo + q) * C + ch * VN) * ESZ,
+                a.is_max ? 0 : a.tf32_round);
     }
   });
 }
 
-int pool_occupancy() {
+constexpr int LP_SMEM_BUDGET = 48 * 1024;
+
+// Output columns per tile so that the staged rows fit the smem budget.
+static int lrn_pool_cols(int st, int W, int C, int lrn, int k, int s, int Wo) {
+  const int esz = st == ST_BF16 ? 2 : 4;
+  const size_t per_col = (size_t)k * C * esz * (lrn ? 2 : 1);
+  int Q = Wo;
+  while (Q > 1 && (size_t)((Q - 1) * s + k) * per_col > LP_SMEM_BUDGET) Q = (Q + 1) / 2;
+  (void)W;
+  return Q;
+}
+
+int lrn_pool_occupancy(int st) {
   int n = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, pool_kernel, POOL_THREADS, 0);
+  if (st == ST_BF16)
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lrn_pool_kernel<ST_BF16>, 256, LP_SMEM_BUDGET);
+  else
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lrn_pool_kernel<ST_F32>, 256, LP_SMEM_BUDGET);
   return n > 0 ? n : 1;
 }
 
-cudaError_t launch_pool(const void *x, void *y, int st, int B, int H, int W,
-                        int C, int k, int stride, int Ho, int Wo, int is_max,
-                        int tf32_round, const Budget &b, int grid,
-                        cudaStream_t s) {
-  pool_kernel<<<grid, POOL_THREADS, 0, s>>>(x, y, st, B, H, W, C, k, stride, Ho,
-                                            Wo, is_max, tf32_round, b);
+long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int Ho, int Wo) {
+  const int Q = lrn_pool_cols(st, W, C, lrn, k, s, Wo);
+  return (long long)B * Ho * ((Wo + Q - 1) / Q);
+}
+
+cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int B, int H, int W,
+                            int C, int lrn_size, float alpha, float beta, float kk, int k,
+                            int s, int is_max, int Ho, int Wo, const Budget &b, int grid,
+                            cudaStream_t stream) {
+  const int vn = st == ST_BF16 ? 8 : 4;
+  if (C % vn) return cudaErrorInvalidValue;
+  LrnPoolArgs a;
+  a.x = x;
+  a.y = y;
+  a.B = B;
+  a.H = H;
+  a.W = W;
+  a.C = C;
+  a.lrn_size = lrn_size;
+  a.lrn_alpha_over_n = lrn_size > 0 ? alpha / (float)lrn_size : 0.f;
+  a.lrn_beta = beta;
+  a.lrn_k = kk;
+  a.k = k;
+  a.s = s;
+  a.is_max = is_max;
+  a.Ho = Ho;
+  a.Wo = Wo;
+  a.Q = lrn_pool_cols(st, W, C, lrn_size > 0, k, s, Wo);
+  a.nqt = (Wo + a.Q - 1) / a.Q;
+  a.tf32_round = tf32_round;
+  a.b = b;
+  const int esz = st == ST_BF16 ? 2 : 4;
+  const size_t smem = (size_t)k * ((a.Q - 1) * s + k) * C * esz * (lrn_size > 0 ? 2 : 1);
+  if (smem > 200 * 1024 || lrn_size > 17) return cudaErrorInvalidValue;
+  if (smem > 48 * 1024) {
+    cudaFuncSetAttribute(lrn_pool_kernel<ST_BF16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(lrn_pool_kernel<ST_F32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  }
+  if (st == ST_BF16)
+    lrn_pool_kernel<ST_BF16><<<grid, 256, smem, stream>>>(a);
+  else
+    lrn_pool_kernel<ST_F32><<<grid, 256, smem, stream>>>(a);
   return cudaGetLastError();
 }
 

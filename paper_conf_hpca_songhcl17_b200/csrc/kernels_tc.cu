@@ -7,19 +7,25 @@
 // A tile row -- one output pixel's (r, s, c-chunk) input run -- straight from
 // the NHWC activations into the 128B-swizzled shared-memory layout the UMMA
 // descriptor expects (cp.async 16 B chunks, zero-fill for padding / ragged
-// tails).  The weight tile (B operand) arrives by TMA.  One elected thread
-// issues tcgen05.mma (BF16 kind::f16 or kind::tf32, FP32 accumulate) into a
-// double-buffered TMEM accumulator; four epilogue warps drain it with
-// tcgen05.ld, add bias, apply ReLU, round to the storage precision and store
-// NHWC rows.  The kernel is persistent: grid = min(tiles, SM budget) CTAs,
-// 1 CTA per SM (smem + TMEM), static round-robin tile schedule -- the grid cap
-// IS the per-layer SM budget.
+// tails; completion signalled with cp.async.mbarrier.arrive.noinc so the
+// producers never block on their own loads).  The weight tile (B operand)
+// arrives by TMA.  One elected thread issues tcgen05.mma (BF16 kind::f16 or
+// kind::tf32, FP32 accumulate) into a double-buffered TMEM accumulator; four
+// epilogue warps drain it with tcgen05.ld, add bias, apply ReLU, round to the
+// storage precision and store NHWC rows (or, for split-K work units, store
+// FP32 partial sums that a deterministic reduction kernel adds in split order).
+// The kernel is persistent: grid = min(work units, SM budget) CTAs, 1 CTA per
+// SM (smem + TMEM), static round-robin schedule -- the grid cap IS the
+// per-layer SM budget.  The pipeline depth is sized at launch from
+// the N tile so that ~200 KB of operand stages are in flight per SM.
 //
 // CTA = 14 warps (448 threads):
 //   warp 0       : TMA producer for B (weights)
 //   warp 1       : TMEM allocator + MMA issuer
 //   warps 2..5   : epilogue (TMEM lane quarter = warp % 4)
 //   warps 6..13  : im2col gather producers for A (256 threads)
+#include <algorithm>
+
 #include "budget.cuh"
 #include "pcnn_internal.h"
 
@@ -28,32 +34,37 @@ namespace pcnn {
 constexpr int TC_BM = 128;              // UMMA M (cta_group::1)
 constexpr int TC_BN_MAX = 256;          // max UMMA N
 constexpr int TC_ROW_BYTES = 128;       // one K-block row = one 128B swizzle row
-constexpr int TC_STAGES = 4;
-constexpr int TC_LAG = 2;               // producer arrive lag (< TC_STAGES)
+constexpr int TC_MAX_STAGES = 12;
 constexpr int TC_A_STAGE = TC_BM * TC_ROW_BYTES;          // 16 KB
-constexpr int TC_B_STAGE = TC_BN_MAX * TC_ROW_BYTES;      // 32 KB
+constexpr int TC_STAGE_BUDGET = 200 * 1024;               // operand stages per CTA
 constexpr int TC_MAX_KTAB = 4096;       // chunk-table entries kept in smem
 constexpr int TC_THREADS = 448;
 constexpr int TC_PRODUCER0 = 192;       // first A-producer thread
 constexpr int TC_NPROD = 256;
 constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 
-// smem layout (bytes from the 1024-aligned base)
-constexpr int SM_A = 0;
-constexpr int SM_B = SM_A + TC_STAGES * TC_A_STAGE;
-constexpr int SM_BAR = SM_B + TC_STAGES * TC_B_STAGE;     // 196608
+// smem layout (bytes from the 1024-aligned base):
+//   [0, TC_STAGE_BUDGET)   A stages, then B stages (runtime count)
+//   SM_BAR                 barriers + TMEM pointer
+//   SM_KTAB                (r, s, c) chunk table
+constexpr int SM_BAR = TC_STAGE_BUDGET;
 constexpr int SM_FULL = SM_BAR;
-constexpr int SM_EMPTY = SM_FULL + 8 * TC_STAGES;
-constexpr int SM_TFULL = SM_EMPTY + 8 * TC_STAGES;
+constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_STAGES;
+constexpr int SM_TFULL = SM_EMPTY + 8 * TC_MAX_STAGES;
 constexpr int SM_TEMPTY = SM_TFULL + 16;
 constexpr int SM_TMEMPTR = SM_TEMPTY + 16;
-constexpr int SM_KTAB = SM_BAR + 128;
+constexpr int SM_KTAB = SM_BAR + 256;
 constexpr int SM_TOTAL = SM_KTAB + 4 * TC_MAX_KTAB;
 constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
 
 size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
 int tc_max_ktab() { return TC_MAX_KTAB; }
 int tc_block_k_elems(int st) { return st == ST_BF16 ? 64 : 32; }
+int tc_stages_for(int bn) {
+  const int per = TC_A_STAGE + bn * TC_ROW_BYTES;
+  const int n = TC_STAGE_BUDGET / per;
+  return n > TC_MAX_STAGES ? TC_MAX_STAGES : n;
+}
 
 // ------------------------------------------------------------ PTX wrappers
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -97,12 +108,10 @@ __device__ __forceinline__ void cp_async_16(uint32_t dst, const void *src, int n
                "r"(nbytes)
                : "memory");
 }
-__device__ __forceinline__ void cp_async_commit() {
-  asm volatile("cp.async.commit_group;" ::: "memory");
-}
-template <int N>
-__device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+// Arrive on `bar` once every cp.async this thread issued so far has landed
+// (the arrival counts against the barrier's expected count: .noinc).
+__device__ __forceinline__ void cp_async_arrive_noinc(uint32_t bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
 }
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -180,13 +189,22 @@ struct TcArgs {
   ConvGeom g;
   const void *x;
   void *y;
+  float *ws;            // split-K partials [splits][M][out_cs] fp32 (splits > 1)
   const float *bias;
   const int *ktab;      // per-element (r,s,c) table (nullptr when S == 1)
   int bn;
-  int mtiles, ntiles, tiles;
-  int kblocks;
+  int mtiles, ntiles, splits, units;
+  int kblocks, kb_per_split;
+  int stages;
   Budget b;
 };
+
+__device__ __forceinline__ void advance(uint32_t &stage, uint32_t &phase, int stages) {
+  if (++stage == (uint32_t)stages) {
+    stage = 0;
+    phase ^= 1;
+  }
+}
 
 template <int ST>
 __global__ void __launch_bounds__(TC_THREADS, 1)
@@ -199,6 +217,10 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
   constexpr int CH = 16 / ESZ;                 // elements per 16 B chunk
   const ConvGeom &g = a.g;
+  const int stages = a.stages;
+  const uint32_t sA = sbase;                                     // A stages
+  const uint32_t sB = sbase + (uint32_t)stages * TC_A_STAGE;     // B stages
+  const uint32_t b_stage = (uint32_t)a.bn * TC_ROW_BYTES;
 
   uint32_t *ktab_s = (uint32_t *)(smem + SM_KTAB);
   const bool use_tab = a.ktab != nullptr;
@@ -210,7 +232,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     }
   }
   if (tid == 0) {
-    for (int s = 0; s < TC_STAGES; ++s) {
+    for (int s = 0; s < stages; ++s) {
       mbar_init(sbase + SM_FULL + 8 * s, 1 + TC_NPROD);
       mbar_init(sbase + SM_EMPTY + 8 * s, 1);
     }
@@ -234,22 +256,37 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   const uint32_t tmem_base = *(volatile uint32_t *)(smem + SM_TMEMPTR);
 
   const int HoWo = g.Ho * g.Wo;
+  // work unit u -> (m tile, n tile, group, split); m fastest so CTAs running
+  // concurrently share one weight slice in L2.
+  auto decode = [&](int u, int &mt, int &nt, int &grp, int &sp) {
+    mt = u % a.mtiles;
+    int r = u / a.mtiles;
+    nt = r % a.ntiles;
+    r /= a.ntiles;
+    grp = r % g.groups;
+    sp = r / g.groups;
+  };
+  auto kb_range = [&](int sp, int &k0, int &k1) {
+    k0 = sp * a.kb_per_split;
+    k1 = min(a.kblocks, k0 + a.kb_per_split);
+  };
 
   if (warp == 0) {
     // ------------------------------------------------ B (weights) TMA producer
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
-      uint32_t it = 0;
-      for (int t = blockIdx.x; t < a.tiles; t += gridDim.x) {
-        const int rest = t / a.mtiles;
-        const int nt = rest % a.ntiles, grp = rest / a.ntiles;
+      uint32_t stage = 0, phase = 0;
+      for (int u = blockIdx.x; u < a.units; u += gridDim.x) {
+        int mt, nt, grp, sp, k0, k1;
+        decode(u, mt, nt, grp, sp);
+        kb_range(sp, k0, k1);
         const int nrow = grp * g.Nfg + nt * a.bn;
-        for (int kb = 0; kb < a.kblocks; ++kb, ++it) {
-          const uint32_t s = it % TC_STAGES, ph = (it / TC_STAGES) & 1;
-          mbar_wait(sbase + SM_EMPTY + 8 * s, ph ^ 1);
-          mbar_arrive_expect_tx(sbase + SM_FULL + 8 * s, (uint32_t)a.bn * TC_ROW_BYTES);
-          tma_load_2d(sbase + SM_B + s * TC_B_STAGE, &tmap_w, sbase + SM_FULL + 8 * s,
+        for (int kb = k0; kb < k1; ++kb) {
+          mbar_wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
+          mbar_arrive_expect_tx(sbase + SM_FULL + 8 * stage, b_stage);
+          tma_load_2d(sB + stage * b_stage, &tmap_w, sbase + SM_FULL + 8 * stage,
                       kb * (TC_ROW_BYTES / ESZ), nrow);
+          advance(stage, phase, stages);
         }
       }
     }
@@ -257,22 +294,26 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     // ------------------------------------------------ MMA issuer
     if (lane == 0) {
       const uint32_t idesc = umma_idesc<ST>(a.bn);
-      uint32_t it = 0, lt = 0;
-      for (int t = blockIdx.x; t < a.tiles; t += gridDim.x, ++lt) {
+      uint32_t stage = 0, phase = 0, lt = 0;
+      for (int u = blockIdx.x; u < a.units; u += gridDim.x, ++lt) {
+        int mt, nt, grp, sp, k0, k1;
+        decode(u, mt, nt, grp, sp);
+        kb_range(sp, k0, k1);
         const uint32_t buf = lt & 1, use = lt >> 1;
         mbar_wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
         tc_fence_after();
         const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
-        for (int kb = 0; kb < a.kblocks; ++kb, ++it) {
-          const uint32_t s = it % TC_STAGES, ph = (it / TC_STAGES) & 1;
-          mbar_wait(sbase + SM_FULL + 8 * s, ph);
+        for (int kb = k0; kb < k1; ++kb) {
+          mbar_wait(sbase + SM_FULL + 8 * stage, phase);
+          fence_proxy_async();   // cp.async (generic proxy) writes -> UMMA reads
           tc_fence_after();
-          const uint64_t ad = umma_desc_sw128(sbase + SM_A + s * TC_A_STAGE);
-          const uint64_t bd = umma_desc_sw128(sbase + SM_B + s * TC_B_STAGE);
+          const uint64_t ad = umma_desc_sw128(sA + stage * TC_A_STAGE);
+          const uint64_t bd = umma_desc_sw128(sB + stage * b_stage);
 #pragma unroll
           for (int k = 0; k < 4; ++k)   // 4 x 32 B along K inside the 128 B row
-            tc_mma<ST>(dcol, ad + 2 * k, bd + 2 * k, idesc, (kb | k) != 0);
-          tc_commit(sbase + SM_EMPTY + 8 * s);
+            tc_mma<ST>(dcol, ad + 2 * k, bd + 2 * k, idesc, (kb > k0) || (k > 0));
+          tc_commit(sbase + SM_EMPTY + 8 * stage);
+          advance(stage, phase, stages);
         }
         tc_commit(sbase + SM_TFULL + 8 * buf);
       }
@@ -281,10 +322,11 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     // ------------------------------------------------ epilogue
     const int quarter = warp & 3;
     const int row = quarter * 32 + lane;
+    const bool partial = a.splits > 1;
     uint32_t lt = 0;
-    for (int t = blockIdx.x; t < a.tiles; t += gridDim.x, ++lt) {
-      const int mt = t % a.mtiles, rest = t / a.mtiles;
-      const int nt = rest % a.ntiles, grp = rest / a.ntiles;
+    for (int u = blockIdx.x; u < a.units; u += gridDim.x, ++lt) {
+      int mt, nt, grp, sp;
+      decode(u, mt, nt, grp, sp);
       const uint32_t buf = lt & 1, use = lt >> 1;
       mbar_wait(sbase + SM_TFULL + 8 * buf, use & 1);
       tc_fence_after();
@@ -303,11 +345,20 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
             float x = __uint_as_float(v[i]);
-            if (a.bias && n + i < g.Nfg) x += __ldg(&a.bias[col + i]);
-            if (g.relu) x = fmaxf(x, 0.f);
+            if (!partial) {
+              if (a.bias && n + i < g.Nfg) x += __ldg(&a.bias[col + i]);
+              if (g.relu) x = fmaxf(x, 0.f);
+            }
             f[i] = x;
           }
-          if (g.out_mode == OUT_BF16) {
+          if (partial) {
+            float *yp = a.ws + (size_t)sp * g.M * g.out_cs + orow + col;
+#pragma unroll
+            for (int h = 0; h < 4; ++h)
+              if (n + 4 * h < g.Nfg)
+                *(float4 *)(yp + 4 * h) =
+                    make_float4(f[4 * h], f[4 * h + 1], f[4 * h + 2], f[4 * h + 3]);
+          } else if (g.out_mode == OUT_BF16) {
             __nv_bfloat16 *yp = (__nv_bfloat16 *)a.y + orow + col;
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
@@ -316,7 +367,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
                 uint32_t *pw = (uint32_t *)&pk;
 #pragma unroll
                 for (int i = 0; i < 4; ++i) {
-                  __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * h + 2 * i], f[8 * h + 2 * i + 1]);
+                  __nv_bfloat162 b2 =
+                      __floats2bfloat162_rn(f[8 * h + 2 * i], f[8 * h + 2 * i + 1]);
                   pw[i] = *(uint32_t *)&b2;
                 }
                 *(uint4 *)(yp + 8 * h) = pk;
@@ -351,10 +403,11 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     const int rb = p >> 3;                     // rows rb, rb+32, rb+64, rb+96
     const uint32_t swz = (uint32_t)((j ^ (rb & 7)) << 4);
     const char *xb = (const char *)a.x;
-    uint32_t it = 0;
-    for (int t = blockIdx.x; t < a.tiles; t += gridDim.x) {
-      const int mt = t % a.mtiles, rest = t / a.mtiles;
-      const int grp = (rest / a.ntiles);
+    uint32_t stage = 0, phase = 0;
+    for (int u = blockIdx.x; u < a.units; u += gridDim.x) {
+      int mt, nt, grp, sp, k0, k1;
+      decode(u, mt, nt, grp, sp);
+      kb_range(sp, k0, k1);
       long long base[4];
       int ih0[4], iw0[4];
 #pragma unroll
@@ -372,9 +425,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
           iw0[i] = 0;
         }
       }
-      for (int kb = 0; kb < a.kblocks; ++kb, ++it) {
-        const uint32_t s = it % TC_STAGES, ph = (it / TC_STAGES) & 1;
-        mbar_wait(sbase + SM_EMPTY + 8 * s, ph ^ 1);
+      for (int kb = k0; kb < k1; ++kb) {
+        mbar_wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
         const int kc = kb * 8 + j;
         int r = 0, sx = 0, c = kc * CH;
         bool kok = c < g.K;
@@ -385,28 +437,22 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
           c = e & 0xFFFF;
           kok = kok && r != 0xFF;
         }
-        const uint32_t dst_stage = sbase + SM_A + s * TC_A_STAGE;
+        const uint32_t dst_stage = sA + stage * TC_A_STAGE;
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           const int row = rb + 32 * i;
           const int ih = ih0[i] + r, iw = iw0[i] + sx;
           const bool ok = kok && base[i] >= 0 && ih >= 0 && ih < g.H && iw >= 0 && iw < g.W;
-          const char *src = ok ? xb + base[i] + (((long long)ih * g.W + iw) * g.Cs + c) * ESZ : xb;
+          const char *src =
+              ok ? xb + base[i] + (((long long)ih * g.W + iw) * g.Cs + c) * ESZ : xb;
           cp_async_16(dst_stage + row * TC_ROW_BYTES + swz, src, ok ? 16 : 0);
         }
-        cp_async_commit();
-        if (it >= TC_LAG) {
-          cp_async_wait<TC_LAG>();
-          fence_proxy_async();
-          mbar_arrive(sbase + SM_FULL + 8 * ((it - TC_LAG) % TC_STAGES));
-        }
+        cp_async_arrive_noinc(sbase + SM_FULL + 8 * stage);
+        advance(stage, phase, stages);
       }
     }
-    // flush the last TC_LAG stages
-    cp_async_wait<0>();
-    fence_proxy_async();
-    const uint32_t first = it > TC_LAG ? it - TC_LAG : 0;
-    for (uint32_t k = first; k < it; ++k) mbar_arrive(sbase + SM_FULL + 8 * (k % TC_STAGES));
+    // keep the CTA (and its smem) alive until every in-flight copy has landed
+    asm volatile("cp.async.wait_all;" ::: "memory");
   }
 
   tc_fence_before();
@@ -415,6 +461,42 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   if (warp == 1) {
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
                  "n"(TC_TMEM_COLS));
+  }
+}
+
+// Deterministic split-K reduction: y = act(sum_s ws[s] + bias), s ascending.
+__global__ void splitk_reduce_kernel(const float *__restrict__ ws, void *y,
+                                     const float *__restrict__ bias, int M, int N, int splits,
+                                     int relu, int out_mode) {
+  const long long total = (long long)M * N / 4;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    const long long e = i * 4;
+    const int col = (int)(e % N);
+    float4 acc = *(const float4 *)(ws + e);
+    for (int s = 1; s < splits; ++s) {
+      const float4 v = *(const float4 *)(ws + (size_t)s * M * N + e);
+      acc.x += v.x;
+      acc.y += v.y;
+      acc.z += v.z;
+      acc.w += v.w;
+    }
+    float f[4] = {acc.x, acc.y, acc.z, acc.w};
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      if (bias) f[t] += __ldg(&bias[col + t]);
+      if (relu) f[t] = fmaxf(f[t], 0.f);
+    }
+    if (out_mode == OUT_BF16) {
+      __nv_bfloat162 lo = __floats2bfloat162_rn(f[0], f[1]);
+      __nv_bfloat162 hi = __floats2bfloat162_rn(f[2], f[3]);
+      uint2 pk = make_uint2(*(uint32_t *)&lo, *(uint32_t *)&hi);
+      *(uint2 *)((__nv_bfloat16 *)y + e) = pk;
+    } else {
+      if (out_mode == OUT_F32_TF32)
+        for (int t = 0; t < 4; ++t) f[t] = tf32_rna_tc(f[t]);
+      *(float4 *)((float *)y + e) = make_float4(f[0], f[1], f[2], f[3]);
+    }
   }
 }
 
@@ -427,31 +509,37 @@ cudaError_t tc_init() {
                               cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM_BYTES);
 }
 
-template <int ST>
-static cudaError_t launch_tc_impl(const TcArgs &args, const CUtensorMap *tmap, int grid,
-                                  cudaStream_t s) {
-  conv_tc_kernel<ST><<<grid, TC_THREADS, TC_SMEM_BYTES, s>>>(*tmap, args);
-  return cudaGetLastError();
-}
-
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
                            const CUtensorMap *tmap_w, const float *bias, void *y,
-                           const int *ktab, const TcPlan &p, const Budget &b,
+                           const int *ktab, const TcPlan &p, float *ws, const Budget &b,
                            cudaStream_t s) {
   TcArgs args;
   args.g = g;
   args.x = x;
   args.y = y;
+  args.ws = ws;
   args.bias = bias;
   args.ktab = ktab;
   args.bn = p.bn;
   args.mtiles = p.mtiles;
   args.ntiles = p.ntiles;
-  args.tiles = p.tiles;
+  args.splits = p.splits;
+  args.units = p.units;
   args.kblocks = g.Kpad / tc_block_k_elems(st);
+  args.kb_per_split = p.kb_per_split;
+  args.stages = tc_stages_for(p.bn);
   args.b = b;
-  if (st == ST_BF16) return launch_tc_impl<ST_BF16>(args, tmap_w, p.grid, s);
-  return launch_tc_impl<ST_F32>(args, tmap_w, p.grid, s);
+  if (st == ST_BF16)
+    conv_tc_kernel<ST_BF16><<<p.grid, TC_THREADS, TC_SMEM_BYTES, s>>>(*tmap_w, args);
+  else
+    conv_tc_kernel<ST_F32><<<p.grid, TC_THREADS, TC_SMEM_BYTES, s>>>(*tmap_w, args);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess || p.splits <= 1) return e;
+  const long long total = (long long)g.M * g.out_cs / 4;
+  const int grid = (int)std::min<long long>((total + 255) / 256, 148 * 8);
+  splitk_reduce_kernel<<<grid, 256, 0, s>>>(ws, y, bias, g.M, g.out_cs, p.splits, g.relu,
+                                            g.out_mode);
+  return cudaGetLastError();
 }
 
 }  // namespace pcnn

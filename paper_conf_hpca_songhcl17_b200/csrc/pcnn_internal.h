@@ -53,10 +53,11 @@ struct ConvGeom {
 // ---------------------------------------------------------------- launchers
 // All return cudaSuccess or the launch error; they never synchronise.
 
-// a1: NCHW fp32 -> NHWC storage (channels zero-padded to Cs).
+// a1: NCHW fp32 [B][C][H][W] -> NHWC storage [B][Hs][Ws][Cs]; blk > 1 is
+// space-to-depth by blk with the conv's padding `pad` folded in.
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C,
-                               int H, int W, int Cs, int tf32_round,
-                               cudaStream_t s);
+                               int H, int W, int Hs, int Ws, int Cs, int blk,
+                               int pad, int tf32_round, cudaStream_t s);
 // final NHWC storage -> NCHW fp32 flatten
 cudaError_t launch_unstage_output(const void *x, int st, float *y, int B,
                                   int C, int H, int W, int Cs, cudaStream_t s);
@@ -72,32 +73,40 @@ void conv_simt_tile_shape(int *tm, int *tn);
 // tcgen05 implicit-GEMM conv / FC (K1/K2).
 struct TcPlan {
   int bn;          // N tile (16..256, multiple of 16)
-  int mtiles, ntiles, tiles;
-  int grid;
+  int mtiles, ntiles, tiles;   // output tiles (eq. 4 grid size)
+  int splits;      // split-K factor (1 = none); chosen from the shape only
+  int kb_per_split;
+  int units;       // tiles * splits work units
+  int grid;        // CTAs = min(units, SM budget)
 };
+// Launches the GEMM and, when p.splits > 1, the deterministic split-K
+// reduction (ws must hold splits * M * out_cs floats; a split-K output must
+// be packed, out_cs == groups * Nfg, with out_cs % 4 == 0).
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
                            const CUtensorMap *tmap_w, const float *bias,
-                           void *y, const int *ktab, const TcPlan &p,
+                           void *y, const int *ktab, const TcPlan &p, float *ws,
                            const Budget &b, cudaStream_t s);
+int tc_stages_for(int bn);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)
 cudaError_t tc_init();                 // sets the kernels' smem attributes
 size_t tc_smem_bytes();
 int tc_max_ktab();
 
-// a4 / a5 / a7
-cudaError_t launch_lrn(const void *x, void *y, int st, int tf32_round,
-                       long pixels, int C, int size, float alpha, float beta,
-                       float k, const Budget &b, int grid, cudaStream_t s);
-cudaError_t launch_pool(const void *x, void *y, int st, int B, int H, int W,
-                        int C, int k, int stride, int Ho, int Wo, int is_max,
-                        int tf32_round, const Budget &b, int grid,
-                        cudaStream_t s);
+// a4 / a5: LRN (lrn_size > 0) followed by pooling (k x k, stride s; k = s =
+// 1 for no pooling), NHWC with C stored channels.
+cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int B,
+                            int H, int W, int C, int lrn_size, float alpha,
+                            float beta, float kk, int k, int s, int is_max,
+                            int Ho, int Wo, const Budget &b, int grid,
+                            cudaStream_t stream);
+long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s,
+                         int Ho, int Wo);
+int lrn_pool_occupancy(int st);
+// a7
 cudaError_t launch_softmax_entropy(const float *z, float *p, float *h, int B,
                                    int N, cudaStream_t s);
 
 // occupancy helpers for gated launches
 int simt_conv_occupancy();
-int lrn_occupancy();
-int pool_occupancy();
 
 }  // namespace pcnn

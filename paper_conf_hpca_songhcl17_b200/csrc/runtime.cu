@@ -38,6 +38,13 @@ static pcnn_status fail(pcnn_status s, const std::string &msg) {
       return fail(PCNN_ERR_CUDA, std::string(#expr) + ": " + cudaGetErrorString(e_)); \
   } while (0)
 
+// every kernel launch of the hot path goes through this counter
+static thread_local int g_launches = 0;
+static inline cudaError_t counted(cudaError_t e) {
+  ++g_launches;
+  return e;
+}
+
 // ------------------------------------------------------------------ host rounding
 static inline uint16_t f32_to_bf16_rne(float f) {
   uint32_t u;
@@ -128,7 +135,10 @@ struct pcnn_net {
   float *d_host_in = nullptr, *d_host_out = nullptr, *d_host_p = nullptr,
         *d_host_h = nullptr;
   int out_elems = 0;
-  int occ_simt = 1, occ_lrn = 1, occ_pool = 1;
+  int occ_simt = 1, occ_lp = 1;
+  // input staging geometry (space-to-depth by `blk` for a strided first conv)
+  int stage_h = 0, stage_w = 0, stage_blk = 1, stage_pad = 0;
+  bool fuse_lrn_pool = true;
   bool census = false;
   // CUDA graph cache
   uint64_t version = 1;
@@ -144,6 +154,13 @@ struct pcnn_net {
   };
   std::map<GraphKey, cudaGraphExec_t> graphs;
   bool use_graphs = true;
+  int launches_per_infer = 0;
+  float *d_ws = nullptr;    // split-K partials
+  size_t ws_bytes = 0;
+  // live per-layer timing (pcnn_set_layer_timing)
+  bool timing = false;
+  std::vector<std::vector<cudaEvent_t>> timing_sets;   // recorded, unread
+  std::vector<std::vector<cudaEvent_t>> timing_free;   // reusable
 };
 
 // ------------------------------------------------------------------ geometry
@@ -439,29 +456,50 @@ static const CUtensorMap *stage_tmap(GemmStage &gs, int bn) {
 }
 
 // ------------------------------------------------------------------ planning
-// Tile selection (the paper's sub-matrix choice):
-// pick the N tile minimising  waves * kblocks * cost(bn), where one K-block
-// costs max(MMA cycles ~ 2 bn, gather ~ 256 cycles) -- small tiles raise Util
-// (eq. 6) and rEC (eq. 9) but lower the computation density.
-static TcPlan plan_tc(const ConvGeom &g, int n_sms) {
+// Tile / split selection (the paper's sub-matrix choice, P:223,
+// P:267).  For every N tile bn (multiple of 16, <= 256):
+//   tiles  = ceil(M/128) * ceil(Nfg/bn) * groups          (eq. 4)
+//   splits = K split when the tiles cannot fill half the GPU
+//   time   = max(waves * kblocks/splits * cycles(bn) / f, weight bytes / HBM)
+//            + split-K reduction traffic
+// where one K-block costs max(MMA ~2.05*bn, A gather ~256) + 40 cycles.  Small
+// tiles raise Util (eq. 6) and rEC (eq. 9), big tiles raise the computation
+// density -- the trade-off of P:223.  The plan depends on the problem shape and
+// the device's SM count only, never on the SM budget, so every budget runs the
+// same tiles and K order (bitwise-identical results, R11).
+static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
   TcPlan best{};
-  double best_cost = 1e300;
+  double best_t = 1e300;
   const int mtiles = (g.M + 127) / 128;
   const int nmax = std::min(256, round_up(g.Nfg, 16));
+  const double f = 1.9e9, hbm = 6.0e12;
+  const double wbytes = (double)g.Nfg * g.groups * g.Kpad * esz;
   for (int bn = 16; bn <= nmax; bn += 16) {
     const int ntiles = (g.Nfg + bn - 1) / bn;
     const long long tiles = (long long)mtiles * ntiles * g.groups;
-    const long long waves = (tiles + n_sms - 1) / n_sms;
-    const double cost = (double)waves * (std::max(2.05 * bn, 256.0) + 40.0);
-    if (cost < best_cost * 0.999 || (cost <= best_cost * 1.001 && bn > best.bn)) {
-      best_cost = cost;
+    int splits = 1;
+    if (tiles * 2 < device_sms && kblocks >= 8) {
+      splits = (int)std::min<long long>((device_sms + tiles - 1) / tiles, 16);
+      splits = std::max(1, std::min(splits, kblocks / 4));
+    }
+    const int kbs = (kblocks + splits - 1) / splits;
+    splits = (kblocks + kbs - 1) / kbs;
+    const long long units = tiles * splits;
+    const long long waves = (units + device_sms - 1) / device_sms;
+    double t = (double)waves * kbs * (std::max(2.05 * bn, 256.0) + 40.0) / f;
+    t = std::max(t, wbytes / hbm);
+    if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
+    if (t < best_t * 0.999 || (t <= best_t * 1.001 && bn > best.bn)) {
+      best_t = t;
       best.bn = bn;
       best.mtiles = mtiles;
       best.ntiles = ntiles;
       best.tiles = (int)tiles;
+      best.splits = splits;
+      best.kb_per_split = kbs;
+      best.units = (int)units;
     }
   }
-  best.grid = std::min(best.tiles, n_sms);
   return best;
 }
 
@@ -486,11 +524,13 @@ static Budget make_budget(const pcnn_net *net, const Layer &ly, int slot, bool g
 
 // ------------------------------------------------------------------ enqueue
 static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, const void *x,
-                             void *y, int slot, cudaStream_t s, pcnn_layer_info *info) {
+                             void *y, int slot, cudaStream_t s, pcnn_layer_info *info,
+                             size_t *ws_need = nullptr) {
   ConvGeom g = gs.g;
   g.M = B * g.Ho * g.Wo;
   if (gs.engine == 1) {
-    TcPlan p = plan_tc(g, effective_sms(net, ly));
+    TcPlan p = plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st));
+    p.grid = std::min(p.units, effective_sms(net, ly));
     const CUtensorMap *tm = stage_tmap(gs, p.bn);
     if (!tm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeTiled failed");
     if (info) {
@@ -500,10 +540,16 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->grid = p.grid;
       info->tlp = 1;
       info->engine = 1;
+      info->splits = p.splits;
     }
+    if (ws_need) *ws_need = std::max(*ws_need, p.splits > 1 ? (size_t)p.splits * g.M * g.out_cs * 4 : 0);
     if (!x) return PCNN_OK;   // planning only
     Budget b = make_budget(net, ly, slot, false);
-    CUDA_TRY(launch_conv_tc(g, gs.st, x, tm, gs.d_bias, y, gs.d_ktab, p, b, s));
+    if (p.splits > 1 && (size_t)p.splits * g.M * g.out_cs * 4 > net->ws_bytes)
+      return fail(PCNN_ERR_OUT_OF_MEMORY, "split-K workspace not reserved");
+    g_launches += p.splits > 1 ? 1 : 0;   // the reduction kernel
+    CUDA_TRY(counted(launch_conv_tc(g, gs.st, x, tm, gs.d_bias, y, gs.d_ktab, p, net->d_ws,
+                                    b, s)));
   } else {
     const int tiles = conv_simt_tiles(g);
     const bool gated = is_gated(net, ly);
@@ -523,9 +569,43 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
     Budget b = make_budget(net, ly, slot, true);
     if (b.gated)
       CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
-    CUDA_TRY(launch_conv_simt(g, (const float *)x, (const float *)gs.d_w, gs.d_bias,
-                              (float *)y, gs.d_ktab, b, grid, s));
+    CUDA_TRY(counted(launch_conv_simt(g, (const float *)x, (const float *)gs.d_w, gs.d_bias,
+                              (float *)y, gs.d_ktab, b, grid, s)));
   }
+  return PCNN_OK;
+}
+
+// LRN layer `li` and / or pooling layer `pi` (-1 = absent) in one launch
+// (the fused pair runs under the LRN layer's budget).
+static pcnn_status run_lrn_pool(pcnn_net *net, int li, int pi, int B, const void *x, void *y,
+                                cudaStream_t s) {
+  Layer &ly = net->layers[li >= 0 ? li : pi];
+  const int C = ly.in_cs, H = ly.in_h, W = ly.in_w;
+  int lrn = 0, k = 1, st = 1, is_max = 1, Ho = H, Wo = W;
+  float alpha = 0.f, beta = 0.f, kk = 1.f;
+  if (li >= 0) {
+    const auto &d = net->layers[li].d;
+    lrn = d.kernel;
+    alpha = d.lrn_alpha;
+    beta = d.lrn_beta;
+    kk = d.lrn_k;
+  }
+  if (pi >= 0) {
+    const Layer &p = net->layers[pi];
+    k = p.d.kernel;
+    st = p.d.stride;
+    is_max = p.d.kind == PCNN_MAXPOOL;
+    Ho = p.out_h;
+    Wo = p.out_w;
+  }
+  const long long tiles = lrn_pool_tiles(net->st, B, W, C, lrn > 0, k, st, Ho, Wo);
+  const bool gated = is_gated(net, ly);
+  const int grid = gated ? net->num_sms * net->occ_lp : (int)std::min<long long>(tiles, 1 << 30);
+  Budget b = make_budget(net, ly, 0, true);
+  if (b.gated)
+    CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
+  CUDA_TRY(counted(launch_lrn_pool(x, y, net->st, net->desc.precision == PCNN_TF32, B, H, W, C,
+                                   lrn, alpha, beta, kk, k, st, is_max, Ho, Wo, b, grid, s)));
   return PCNN_OK;
 }
 
@@ -545,29 +625,11 @@ static pcnn_status run_layer(pcnn_net *net, int i, int B, const void *x, void *y
         return run_stage(net, ly, ly.r2, B, r_buf, y, 1, s, nullptr);
       }
       return run_stage(net, ly, ly.exact, B, x, y, 0, s, nullptr);
-    case PCNN_LRN: {
-      const long pixels = (long)B * ly.in_h * ly.in_w;
-      const bool gated = is_gated(net, ly);
-      int grid = gated ? net->num_sms * net->occ_lrn : (int)std::min<long>((pixels + 7) / 8, 1 << 30);
-      Budget b = make_budget(net, ly, 0, true);
-      if (b.gated)
-        CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
-      CUDA_TRY(launch_lrn(x, y, st, tf32, pixels, ly.in_cs, ly.d.kernel, ly.d.lrn_alpha,
-                          ly.d.lrn_beta, ly.d.lrn_k, b, grid, s));
-      return PCNN_OK;
-    }
+    case PCNN_LRN:
+      return run_lrn_pool(net, i, -1, B, x, y, s);
     case PCNN_MAXPOOL:
-    case PCNN_AVGPOOL: {
-      const long long total = (long long)B * ly.out_h * ly.out_w * ly.in_cs;
-      const bool gated = is_gated(net, ly);
-      int grid = gated ? net->num_sms * net->occ_pool : (int)std::min<long long>((total + 255) / 256, 1 << 30);
-      Budget b = make_budget(net, ly, 0, true);
-      if (b.gated)
-        CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
-      CUDA_TRY(launch_pool(x, y, st, B, ly.in_h, ly.in_w, ly.in_cs, ly.d.kernel, ly.d.stride,
-                           ly.out_h, ly.out_w, ly.d.kind == PCNN_MAXPOOL, tf32, b, grid, s));
-      return PCNN_OK;
-    }
+    case PCNN_AVGPOOL:
+      return run_lrn_pool(net, -1, i, B, x, y, s);
   }
   return fail(PCNN_ERR_INVALID_ARGUMENT, "bad layer kind");
 }
@@ -580,16 +642,31 @@ static pcnn_status enqueue_all(pcnn_net *net, const float *d_images, int B, floa
                                std::vector<cudaEvent_t> *evs) {
   const int st = net->st;
   const int tf32 = net->desc.precision == PCNN_TF32;
+  g_launches = 0;
   if (net->census)
     for (auto &ly : net->layers) CUDA_TRY(cudaMemsetAsync(ly.d_census, 0, 32, s));
-  CUDA_TRY(launch_stage_input(d_images, net->d_act[0], st, B, net->desc.in_channels,
-                              net->desc.in_height, net->desc.in_width, net->in_cs, tf32, s));
+  CUDA_TRY(counted(launch_stage_input(d_images, net->d_act[0], st, B, net->desc.in_channels,
+                                      net->desc.in_height, net->desc.in_width, net->stage_h,
+                                      net->stage_w, net->in_cs, net->stage_blk, net->stage_pad,
+                                      tf32, s)));
   if (evs) CUDA_TRY(cudaEventRecord((*evs)[0], s));
   int cur = 0;
   const int n = (int)net->layers.size();
   for (int i = 0; i < n; ++i) {
     const bool final_fc = (i == n - 1) && last_is_fc(net);
     void *dst = final_fc ? (void *)d_out : net->d_act[cur ^ 1];
+    if (net->fuse_lrn_pool && net->layers[i].d.kind == PCNN_LRN && i + 1 < n &&
+        (net->layers[i + 1].d.kind == PCNN_MAXPOOL || net->layers[i + 1].d.kind == PCNN_AVGPOOL)) {
+      pcnn_status r = run_lrn_pool(net, i, i + 1, B, net->d_act[cur], dst, s);
+      if (r != PCNN_OK) return r;
+      if (evs) {
+        CUDA_TRY(cudaEventRecord((*evs)[i + 1], s));
+        CUDA_TRY(cudaEventRecord((*evs)[i + 2], s));
+      }
+      cur ^= 1;
+      ++i;
+      continue;
+    }
     pcnn_status r = run_layer(net, i, B, net->d_act[cur], dst, net->d_act[2], s);
     if (r != PCNN_OK) return r;
     if (evs) CUDA_TRY(cudaEventRecord((*evs)[i + 1], s));
@@ -597,10 +674,11 @@ static pcnn_status enqueue_all(pcnn_net *net, const float *d_images, int B, floa
   }
   if (!last_is_fc(net)) {
     const Layer &l = net->layers.back();
-    CUDA_TRY(launch_unstage_output(net->d_act[cur], st, d_out, B, l.out_c, l.out_h, l.out_w,
-                                   l.out_cs, s));
+    CUDA_TRY(counted(launch_unstage_output(net->d_act[cur], st, d_out, B, l.out_c, l.out_h, l.out_w,
+                                   l.out_cs, s)));
   }
-  if (d_p || d_h) CUDA_TRY(launch_softmax_entropy(d_out, d_p, d_h, B, net->out_elems, s));
+  if (d_p || d_h) CUDA_TRY(counted(launch_softmax_entropy(d_out, d_p, d_h, B, net->out_elems, s)));
+  net->launches_per_infer = g_launches;
   return PCNN_OK;
 }
 
@@ -641,6 +719,34 @@ static pcnn_status build_rank_stages(pcnn_net *net, Layer &ly, int r, const floa
   ly.rank = r;
   ly.variant = PCNN_VARIANT_RANK;
   net->version++;
+  return PCNN_OK;
+}
+
+// Reserve the split-K workspace for `batch` (outside any graph capture).
+static pcnn_status ensure_workspace(pcnn_net *net, int batch) {
+  size_t need = 0;
+  for (auto &ly : net->layers) {
+    if (!ly.gemm) continue;
+    if (ly.variant == PCNN_VARIANT_RANK) {
+      run_stage(net, ly, ly.r1, batch, nullptr, nullptr, 0, nullptr, nullptr, &need);
+      run_stage(net, ly, ly.r2, batch, nullptr, nullptr, 0, nullptr, nullptr, &need);
+    } else {
+      run_stage(net, ly, ly.exact, batch, nullptr, nullptr, 0, nullptr, nullptr, &need);
+    }
+  }
+  if (need <= net->ws_bytes) return PCNN_OK;
+  if (net->d_ws) {
+    CUDA_TRY(cudaDeviceSynchronize());
+    cudaFree(net->d_ws);
+    net->d_ws = nullptr;
+    net->ws_bytes = 0;
+  }
+  if (cudaMalloc(&net->d_ws, need) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(PCNN_ERR_OUT_OF_MEMORY, "split-K workspace");
+  }
+  net->ws_bytes = need;
+  net->version++;          // cached graphs captured the old pointer
   return PCNN_OK;
 }
 
@@ -736,8 +842,13 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   net->st = storage_of(desc->precision);
   net->in_cs = round_up(desc->in_channels, chunk_elems(desc->precision));
   net->occ_simt = simt_conv_occupancy();
-  net->occ_lrn = lrn_occupancy();
-  net->occ_pool = pool_occupancy();
+  net->occ_lp = lrn_pool_occupancy(net->st);
+  net->stage_h = desc->in_height;
+  net->stage_w = desc->in_width;
+  {
+    const char *e = getenv("PCNN_NO_FUSE");
+    net->fuse_lrn_pool = !(e && e[0] == '1');
+  }
   if (desc->precision != PCNN_FP32_SIMT) {
     if (!get_encode_tiled())
       return fail(PCNN_ERR_CUDA, "driver entry point cuTensorMapEncodeTiled unavailable");
@@ -747,7 +858,33 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   const int prec = desc->precision;
   const int esz = esz_of(net->st);
   const int B = desc->max_batch;
-  size_t act = (size_t)B * desc->in_height * desc->in_width * net->in_cs * esz;
+  // Space-to-depth for a strided first conv (layout transform of a1): the
+  // conv S x S / st on C channels becomes ceil(S/st) x ceil(S/st) / 1 on
+  // st^2 C channels over an (Ho - 1 + S') x (Wo - 1 + S') grid whose origin
+  // is shifted by -pad.  Same products, no K padding waste.
+  std::vector<float> s2d_w;
+  const Layer &l0 = net->layers[0];
+  const char *no_s2d = getenv("PCNN_NO_S2D");
+  if (l0.d.kind == PCNN_CONV && l0.d.groups == 1 && l0.d.stride >= 2 && l0.d.stride <= 8 &&
+      !(no_s2d && no_s2d[0] == '1')) {
+    const int st2 = l0.d.stride, S = l0.d.kernel, Sp = (S + st2 - 1) / st2;
+    const int C = desc->in_channels, Cp = st2 * st2 * C, F = l0.d.out_channels;
+    net->stage_blk = st2;
+    net->stage_pad = l0.d.pad;
+    net->stage_h = l0.out_h - 1 + Sp;
+    net->stage_w = l0.out_w - 1 + Sp;
+    net->in_cs = round_up(Cp, chunk_elems(prec));
+    s2d_w.assign((size_t)F * Cp * Sp * Sp, 0.f);
+    for (int f = 0; f < F; ++f)
+      for (int c = 0; c < C; ++c)
+        for (int r = 0; r < S; ++r)
+          for (int q = 0; q < S; ++q) {
+            const int cp = ((r % st2) * st2 + (q % st2)) * C + c;
+            s2d_w[(((size_t)f * Cp + cp) * Sp + r / st2) * Sp + q / st2] =
+                weights[0][(((size_t)f * C + c) * S + r) * S + q];
+          }
+  }
+  size_t act = (size_t)B * net->stage_h * net->stage_w * net->in_cs * esz;
   const int n = n_layers;
   for (int i = 0; i < n; ++i) {
     Layer &ly = net->layers[i];
@@ -758,10 +895,17 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
                                 : (net->st == ST_BF16 ? OUT_BF16
                                                       : (prec == PCNN_TF32 ? OUT_F32_TF32 : OUT_F32));
       const bool is_fc = ly.d.kind == PCNN_FC;
-      s = build_stage(ly.exact, ly, prec, ly.d.out_channels, is_fc ? 1 : ly.d.groups,
-                      is_fc ? 1 : ly.d.kernel, is_fc ? 1 : ly.d.stride, is_fc ? 0 : ly.d.pad,
-                      ly.d.relu, ly.in_c, ly.in_h, ly.in_w, ly.in_cs, is_fc, weights[i],
-                      biases ? biases[i] : nullptr, mode);
+      if (i == 0 && net->stage_blk > 1) {
+        const int Sp = (ly.d.kernel + net->stage_blk - 1) / net->stage_blk;
+        s = build_stage(ly.exact, ly, prec, ly.d.out_channels, 1, Sp, 1, 0, ly.d.relu,
+                        net->in_cs, net->stage_h, net->stage_w, net->in_cs, false,
+                        s2d_w.data(), biases ? biases[i] : nullptr, mode);
+      } else {
+        s = build_stage(ly.exact, ly, prec, ly.d.out_channels, is_fc ? 1 : ly.d.groups,
+                        is_fc ? 1 : ly.d.kernel, is_fc ? 1 : ly.d.stride,
+                        is_fc ? 0 : ly.d.pad, ly.d.relu, ly.in_c, ly.in_h, ly.in_w,
+                        ly.in_cs, is_fc, weights[i], biases ? biases[i] : nullptr, mode);
+      }
       if (s != PCNN_OK) {
         for (auto &l2 : net->layers) l2.exact.release();
         return fail(s, "layer " + std::to_string(i) + ": " + g_err);
@@ -799,6 +943,9 @@ pcnn_status pcnn_destroy_net(pcnn_net *net) {
   if (!net) return PCNN_OK;
   cudaSetDevice(net->device);
   destroy_graphs(net);
+  for (auto *lst : {&net->timing_sets, &net->timing_free})
+    for (auto &ev : *lst)
+      for (auto e : ev) cudaEventDestroy(e);
   for (auto &ly : net->layers) {
     ly.exact.release();
     ly.r1.release();
@@ -808,6 +955,7 @@ pcnn_status pcnn_destroy_net(pcnn_net *net) {
   }
   for (auto &p : net->d_act)
     if (p) cudaFree(p);
+  if (net->d_ws) cudaFree(net->d_ws);
   if (net->d_host_in) cudaFree(net->d_host_in);
   if (net->d_host_out) cudaFree(net->d_host_out);
   if (net->d_host_p) cudaFree(net->d_host_p);
@@ -895,6 +1043,7 @@ pcnn_status pcnn_query_layer(const pcnn_net *cnet, int layer, int batch, pcnn_la
     return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
   Layer &ly = net->layers[layer];
   std::memset(f, 0, sizeof *f);
+  f->splits = 1;
   f->kind = ly.d.kind;
   f->in_c = ly.in_c;
   f->in_h = ly.in_h;
@@ -936,7 +1085,24 @@ pcnn_status pcnn_infer(pcnn_net *net, const float *d_images, int batch, float *d
   if (batch <= 0) return fail(PCNN_ERR_INVALID_ARGUMENT, "batch must be positive");
   if (batch > net->desc.max_batch) return fail(PCNN_ERR_BATCH_TOO_LARGE, "batch > max_batch");
   CUDA_TRY(cudaSetDevice(net->device));
+  {
+    pcnn_status r = ensure_workspace(net, batch);
+    if (r != PCNN_OK) return r;
+  }
   cudaStream_t s = (cudaStream_t)stream;
+  if (net->timing) {
+    std::vector<cudaEvent_t> ev;
+    if (!net->timing_free.empty()) {
+      ev = std::move(net->timing_free.back());
+      net->timing_free.pop_back();
+    } else {
+      ev.resize(net->layers.size() + 1);
+      for (auto &e : ev) CUDA_TRY(cudaEventCreate(&e));
+    }
+    pcnn_status r = enqueue_all(net, d_images, batch, d_out, d_probs, d_entropy, s, &ev);
+    net->timing_sets.push_back(std::move(ev));
+    return r;
+  }
   if (!net->use_graphs || net->census || s == nullptr)
     return enqueue_all(net, d_images, batch, d_out, d_probs, d_entropy, s, nullptr);
   pcnn_net::GraphKey key{batch, d_images, d_out, d_probs, d_entropy, s, net->version};
@@ -1001,6 +1167,10 @@ pcnn_status pcnn_profile_layers(pcnn_net *net, const float *d_images, int batch,
     return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
   if (batch <= 0 || batch > net->desc.max_batch) return fail(PCNN_ERR_BATCH_TOO_LARGE, "bad batch");
   CUDA_TRY(cudaSetDevice(net->device));
+  {
+    pcnn_status r = ensure_workspace(net, batch);
+    if (r != PCNN_OK) return r;
+  }
   cudaStream_t s = (cudaStream_t)stream;
   const int n = (int)net->layers.size();
   std::vector<cudaEvent_t> ev(n + 1);
@@ -1030,6 +1200,38 @@ pcnn_status pcnn_profile_layers(pcnn_net *net, const float *d_images, int batch,
   for (auto &e : ev) cudaEventDestroy(e);
   cudaEventDestroy(e_begin);
   cudaEventDestroy(e_end);
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_set_layer_timing(pcnn_net *net, int enable) {
+  if (!net) return fail(PCNN_ERR_INVALID_ARGUMENT, "null net");
+  net->timing = enable != 0;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_read_layer_timing(pcnn_net *net, float *layer_ms, int *n_steps) {
+  if (!net || !layer_ms) return fail(PCNN_ERR_INVALID_ARGUMENT, "null argument");
+  CUDA_TRY(cudaSetDevice(net->device));
+  const int n = (int)net->layers.size();
+  std::vector<double> acc(n, 0.0);
+  for (auto &ev : net->timing_sets) {
+    CUDA_TRY(cudaEventSynchronize(ev[n]));
+    for (int i = 0; i < n; ++i) {
+      float ms = 0;
+      CUDA_TRY(cudaEventElapsedTime(&ms, ev[i], ev[i + 1]));
+      acc[i] += ms;
+    }
+  }
+  for (int i = 0; i < n; ++i) layer_ms[i] = (float)acc[i];
+  if (n_steps) *n_steps = (int)net->timing_sets.size();
+  for (auto &ev : net->timing_sets) net->timing_free.push_back(std::move(ev));
+  net->timing_sets.clear();
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_last_launch_count(const pcnn_net *net, int *launches) {
+  if (!net || !launches) return fail(PCNN_ERR_INVALID_ARGUMENT, "null argument");
+  *launches = net->launches_per_infer;
   return PCNN_OK;
 }
 

@@ -52,7 +52,7 @@ class LayerInfo(ctypes.Structure):
                 ("variant", ctypes.c_int), ("rank", ctypes.c_int), ("n_sms", ctypes.c_int),
                 ("tlp", ctypes.c_int), ("engine", ctypes.c_int), ("tile_m", ctypes.c_int),
                 ("tile_n", ctypes.c_int), ("tiles", ctypes.c_longlong), ("grid", ctypes.c_int),
-                ("util", ctypes.c_double), ("rec", ctypes.c_double)]
+                ("util", ctypes.c_double), ("rec", ctypes.c_double), ("splits", ctypes.c_int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -75,6 +75,9 @@ _lib.pcnn_query_layer.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.POINTER
 _lib.pcnn_describe_net.argtypes = [ctypes.POINTER(NetDesc), ctypes.POINTER(LayerDesc),
                                    ctypes.c_int, ctypes.c_int, ctypes.POINTER(LayerInfo)]
 _lib.pcnn_profile_layers.argtypes = [_P, _P, ctypes.c_int, _P, ctypes.c_int, _FP, _FP, _P]
+_lib.pcnn_set_layer_timing.argtypes = [_P, ctypes.c_int]
+_lib.pcnn_read_layer_timing.argtypes = [_P, _FP, ctypes.POINTER(ctypes.c_int)]
+_lib.pcnn_last_launch_count.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.pcnn_enable_sm_census.argtypes = [_P, ctypes.c_int]
 _lib.pcnn_get_sm_census.argtypes = [_P, ctypes.c_int, ctypes.POINTER(ctypes.c_uint)]
 _lib.pcnn_device_sm_count.argtypes = [ctypes.c_int]
@@ -87,14 +90,16 @@ for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_infer",
            "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer",
            "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
-           "pcnn_get_sm_census"):
+           "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
+           "pcnn_last_launch_count"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
             "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_infer",
             "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer",
             "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
-            "pcnn_get_sm_census", "pcnn_device_sm_count", "pcnn_version",
+            "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
+            "pcnn_last_launch_count", "pcnn_device_sm_count", "pcnn_version",
             "pcnn_status_string", "pcnn_last_error_message"]
 
 
@@ -267,6 +272,22 @@ class Net:
                                         ctypes.byref(tot), _stream_ptr(stream)),
                "pcnn_profile_layers")
         return list(ms), tot.value
+
+    def set_layer_timing(self, enable=True):
+        _check(_lib.pcnn_set_layer_timing(self._h, int(enable)), "pcnn_set_layer_timing")
+
+    def read_layer_timing(self):
+        """(per-layer ms summed over the recorded infers, number of infers)."""
+        ms = (ctypes.c_float * self.n_layers)()
+        n = ctypes.c_int()
+        _check(_lib.pcnn_read_layer_timing(self._h, ms, ctypes.byref(n)),
+               "pcnn_read_layer_timing")
+        return list(ms), n.value
+
+    def last_launch_count(self):
+        n = ctypes.c_int()
+        _check(_lib.pcnn_last_launch_count(self._h, ctypes.byref(n)), "pcnn_last_launch_count")
+        return n.value
 
     def enable_sm_census(self, enable=True):
         _check(_lib.pcnn_enable_sm_census(self._h, int(enable)), "pcnn_enable_sm_census")

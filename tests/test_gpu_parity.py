@@ -172,3 +172,36 @@ def test_infer_host_matches_device(orc):
     oh = torch.empty((3, 1000)).pin_memory()
     n.infer_host(xh, oh)
     np.testing.assert_array_equal(oh.numpy(), out.cpu().numpy())
+
+
+# ------------------------------------------------------------ layout transforms
+def test_fused_lrn_pool_bitwise_equals_unfused(orc, monkeypatch):
+    """norm -> pool fusion changes scheduling only: the LRN output is rounded
+    to the storage precision before the max in both paths."""
+    net = dict(in_shape=(96, 27, 27), layers=[
+        dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0),
+        dict(kind="maxpool", k=3, stride=2)])
+    x = small_inputs((96, 27, 27), 3, lo=-128, hi=128)
+    for prec in PRECS:
+        fused = gpu_run(net, [None, None], [None, None], x, prec)["out"]
+        monkeypatch.setenv("PCNN_NO_FUSE", "1")
+        plain = gpu_run(net, [None, None], [None, None], x, prec)["out"]
+        monkeypatch.delenv("PCNN_NO_FUSE")
+        np.testing.assert_array_equal(fused, plain)
+        ref = orc.run_net(net, [None, None], [None, None], x).reshape(3, -1)
+        assert rel_err(fused, ref) <= TOL[prec] / 4
+
+
+@pytest.mark.parametrize("prec", PRECS)
+def test_space_to_depth_first_conv(orc, prec, monkeypatch):
+    """The strided first conv runs as a space-to-depth 3x3/1 conv; the plain
+    channel-padded path must agree with it and with the oracle."""
+    net = dict(in_shape=(3, 51, 47), layers=[conv_layer(32, 11, 3, 4, 2, 1, relu=True)])
+    w, b = params(net, seed=3)
+    x = small_inputs((3, 51, 47), 2, lo=-128, hi=128)
+    ref = orc.run_net(net, w, b, x).reshape(2, -1)
+    s2d = gpu_run(net, w, b, x, prec)["out"]
+    monkeypatch.setenv("PCNN_NO_S2D", "1")
+    plain = gpu_run(net, w, b, x, prec)["out"]
+    assert rel_err(s2d, ref) <= TOL[prec] / 4
+    assert rel_err(plain, ref) <= TOL[prec] / 4
