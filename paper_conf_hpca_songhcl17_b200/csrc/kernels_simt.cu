@@ -302,7 +302,7 @@ struct LrnPoolArgs {
   Budget b;
 };
 
-template <int ST>
+template <int ST, int LS>
 __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
   extern __shared__ __align__(16) uint8_t lp_smem[];
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
@@ -311,9 +311,8 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
   const int wc_max = (a.Q - 1) * a.s + a.k;
   const size_t tile_elems = (size_t)a.k * wc_max * C;
   uint8_t *T = lp_smem;                                  // staged input
-  uint8_t *U = a.lrn_size > 0 ? lp_smem + tile_elems * ESZ : lp_smem;   // LRN output
+  uint8_t *U = LS > 0 ? lp_smem + tile_elems * ESZ : lp_smem;   // LRN output
   const long long tiles = (long long)a.B * a.Ho * a.nqt;
-  const int half = a.lrn_size / 2;
 
   for_each_tile(a.b, tiles, [&](long long t) {
     const int qt = (int)(t % a.nqt);
@@ -334,36 +333,42 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
           __ldg((const uint4 *)((const char *)a.x + src * ESZ));
     }
     __syncthreads();
-    if (a.lrn_size > 0) {
+    if (LS > 0) {
+      // each thread: one 16 B channel chunk of one staged pixel; the window
+      // needs HALF channels of the neighbouring chunks, read as whole vectors
+      constexpr int HALF = LS / 2;
+      static_assert(HALF <= VN, "LRN window wider than one neighbouring chunk");
       for (int v = threadIdx.x; v < nr * wc * chunks; v += blockDim.x) {
         const int ch = v % chunks, pix = v / chunks;
         const int r = pix / wc, col = pix - r * wc;
-        const size_t base = ((size_t)r * wc_max + col) * C;
-        const int c0 = ch * VN;
-        float sq[VN + 16];
-        const int lo = c0 - half;
+        const uint8_t *px = T + ((size_t)r * wc_max + col) * C * ESZ;
+        Vec16<ST> prev, cur, next;
+        cur.load(px + (size_t)ch * 16);
+        if (ch > 0) prev.load(px + (size_t)(ch - 1) * 16);
+        else
 #pragma unroll
-        for (int j = 0; j < VN + 16; ++j) {
-          if (j < VN + 2 * half) {
-            const int c = lo + j;
-            float xv = 0.f;
-            if (c >= 0 && c < C) {
-              xv = ST == ST_BF16 ? __bfloat162float(((const __nv_bfloat16 *)T)[base + c])
-                                 : ((const float *)T)[base + c];
-            }
-            sq[j] = xv * xv;
-          }
+          for (int j = 0; j < VN; ++j) prev.v[j] = 0.f;
+        if (ch + 1 < chunks) next.load(px + (size_t)(ch + 1) * 16);
+        else
+#pragma unroll
+          for (int j = 0; j < VN; ++j) next.v[j] = 0.f;
+        float sq[VN + 2 * HALF];
+#pragma unroll
+        for (int j = 0; j < VN + 2 * HALF; ++j) {
+          const int t = j - HALF;            // channel offset from the chunk start
+          const float xv = t < 0 ? prev.v[VN + t] : (t < VN ? cur.v[t] : next.v[t - VN]);
+          sq[j] = xv * xv;
         }
-        Vec16<ST> in, out;
-        in.load(T + (base + c0) * ESZ);
+        Vec16<ST> out;
 #pragma unroll
         for (int j = 0; j < VN; ++j) {
           float acc = 0.f;
-          for (int w = 0; w < a.lrn_size; ++w) acc += sq[j + w];
+#pragma unroll
+          for (int w = 0; w < LS; ++w) acc += sq[j + w];
           const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
-          out.v[j] = in.v[j] * exp2f(-a.lrn_beta * __log2f(scale));
+          out.v[j] = cur.v[j] * exp2f(-a.lrn_beta * __log2f(scale));
         }
-        out.store(U + (base + c0) * ESZ, a.tf32_round);
+        out.store(U + ((size_t)r * wc_max + col) * C * ESZ + (size_t)ch * 16, a.tf32_round);
       }
       __syncthreads();
     }
@@ -406,10 +411,32 @@ static int lrn_pool_cols(int st, int W, int C, int lrn, int k, int s, int Wo) {
 int lrn_pool_occupancy(int st) {
   int n = 0;
   if (st == ST_BF16)
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lrn_pool_kernel<ST_BF16>, 256, LP_SMEM_BUDGET);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lrn_pool_kernel<ST_BF16, 5>, 256, LP_SMEM_BUDGET);
   else
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lrn_pool_kernel<ST_F32>, 256, LP_SMEM_BUDGET);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, lrn_pool_kernel<ST_F32, 5>, 256, LP_SMEM_BUDGET);
   return n > 0 ? n : 1;
+}
+
+template <int ST, int LS>
+static cudaError_t lrn_pool_launch(const LrnPoolArgs &a, int grid, size_t smem, cudaStream_t s) {
+  if (smem > 48 * 1024)
+    cudaFuncSetAttribute(lrn_pool_kernel<ST, LS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)smem);
+  lrn_pool_kernel<ST, LS><<<grid, 256, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+template <int ST>
+static cudaError_t lrn_pool_dispatch(const LrnPoolArgs &a, int grid, size_t smem, cudaStream_t s) {
+  switch (a.lrn_size) {
+    case 0: return lrn_pool_launch<ST, 0>(a, grid, smem, s);
+    case 1: return lrn_pool_launch<ST, 1>(a, grid, smem, s);
+    case 3: return lrn_pool_launch<ST, 3>(a, grid, smem, s);
+    case 5: return lrn_pool_launch<ST, 5>(a, grid, smem, s);
+    case 7: return lrn_pool_launch<ST, 7>(a, grid, smem, s);
+    case 9: return lrn_pool_launch<ST, 9>(a, grid, smem, s);
+  }
+  return cudaErrorInvalidValue;
 }
 
 long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int Ho, int Wo) {
@@ -445,16 +472,10 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
   const size_t smem = (size_t)k * ((a.Q - 1) * s + k) * C * esz * (lrn_size > 0 ? 2 : 1);
-  if (smem > 200 * 1024 || lrn_size > 17) return cudaErrorInvalidValue;
-  if (smem > 48 * 1024) {
-    cudaFuncSetAttribute(lrn_pool_kernel<ST_BF16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaFuncSetAttribute(lrn_pool_kernel<ST_F32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  }
-  if (st == ST_BF16)
-    lrn_pool_kernel<ST_BF16><<<grid, 256, smem, stream>>>(a);
-  else
-    lrn_pool_kernel<ST_F32><<<grid, 256, smem, stream>>>(a);
-  return cudaGetLastError();
+  if (smem > 200 * 1024) return cudaErrorInvalidValue;
+  if (st == ST_BF16) return lrn_pool_dispatch<ST_BF16>(a, grid, smem, stream);
+  if (lrn_size > 9) return cudaErrorInvalidValue;   // fp32 chunk holds 4 channels
+  return lrn_pool_dispatch<ST_F32>(a, grid, smem, stream);
 }
 
 // ------------------------------------------------------------ a7: softmax + entropy

@@ -19,6 +19,15 @@
 // per-layer SM budget.  The pipeline depth is sized at launch from
 // the N tile so that ~200 KB of operand stages are in flight per SM.
 //
+// CG = 2 runs the same pipeline on a CTA pair (cluster of 2, cta_group::2):
+// one 256 x N tile per pair, each CTA gathering its 128 A rows and loading
+// half of the weight tile, the leader CTA issuing M = 256 UMMAs whose
+// accumulator rows are split across both CTAs' TMEM.  Per SM this halves the
+// operand bytes moved per FLOP (smem and L2 bandwidth were the limit of the
+// 128 x N single-CTA tile).  The peer's A-gather completion is relayed to the
+// leader's full barrier by one peer thread; MMA commits multicast to both
+// CTAs' empty / accumulator-full barriers.
+//
 // CTA = 14 warps (448 threads):
 //   warp 0       : TMA producer for B (weights)
 //   warp 1       : TMEM allocator + MMA issuer
@@ -60,8 +69,8 @@ constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
 size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
 int tc_max_ktab() { return TC_MAX_KTAB; }
 int tc_block_k_elems(int st) { return st == ST_BF16 ? 64 : 32; }
-int tc_stages_for(int bn) {
-  const int per = TC_A_STAGE + bn * TC_ROW_BYTES;
+int tc_stages_for(int bn, int cg) {
+  const int per = TC_A_STAGE + bn / cg * TC_ROW_BYTES;
   const int n = TC_STAGE_BUDGET / per;
   return n > TC_MAX_STAGES ? TC_MAX_STAGES : n;
 }
@@ -123,25 +132,74 @@ __device__ __forceinline__ void tc_fence_before() {
 __device__ __forceinline__ void tc_fence_after() {
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 }
+template <int CG>
 __device__ __forceinline__ void tc_commit(uint32_t bar) {
+  if constexpr (CG == 1) {
+    asm volatile(
+        "tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+            bar)
+        : "memory");
+  } else {   // arrive on the barrier at this offset in both CTAs of the pair
+    asm volatile(
+        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
+        " [%0], %1;" ::"r"(bar),
+        "h"((uint16_t)0x3)
+        : "memory");
+  }
+}
+
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n"
+               "barrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// address of the same smem offset in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr)
+               : "memory");
+}
+// 2-SM TMA load: data lands in this CTA's smem, bytes are counted on the
+// leader CTA's barrier (peer bit cleared).
+__device__ __forceinline__ void tma_load_2d_2sm(uint32_t dst, const CUtensorMap *map,
+                                                uint32_t bar, int c0, int c1) {
   asm volatile(
-      "tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-          bar)
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c0), "r"(c1)
       : "memory");
 }
 
-template <int ST>
+template <int ST, int CG>
 __device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
                                        uint32_t idesc, uint32_t accum) {
-  if constexpr (ST == ST_BF16) {
+  if constexpr (ST == ST_BF16 && CG == 1) {
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
-  } else {
+  } else if constexpr (ST == ST_BF16 && CG == 2) {
+    asm volatile(
+        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
+  } else if constexpr (CG == 1) {
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
+  } else {
+    asm volatile(
+        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+        "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
   }
 }
@@ -171,12 +229,13 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
   return d;
 }
 
-// Instruction descriptor: D fp32, A/B = BF16 (1) or TF32 (2), K-major, M=128.
-template <int ST>
+// Instruction descriptor: D fp32, A/B = BF16 (1) or TF32 (2), K-major,
+// M = 128 * CG, N = bn.
+template <int ST, int CG>
 __device__ __forceinline__ uint32_t umma_idesc(int bn) {
   const uint32_t fmt = ST == ST_BF16 ? 1u : 2u;
   return (1u << 4) | (fmt << 7) | (fmt << 10) | ((uint32_t)(bn >> 3) << 17) |
-         ((uint32_t)(TC_BM >> 4) << 24);
+         ((uint32_t)((TC_BM * CG) >> 4) << 24);
 }
 
 __device__ __forceinline__ float tf32_rna_tc(float v) {
@@ -206,7 +265,7 @@ __device__ __forceinline__ void advance(uint32_t &stage, uint32_t &phase, int st
   }
 }
 
-template <int ST>
+template <int ST, int CG>
 __global__ void __launch_bounds__(TC_THREADS, 1)
 conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   extern __shared__ uint8_t smem_raw[];
@@ -218,9 +277,12 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   constexpr int CH = 16 / ESZ;                 // elements per 16 B chunk
   const ConvGeom &g = a.g;
   const int stages = a.stages;
+  const uint32_t rank = CG == 2 ? cluster_ctarank() : 0;   // 0 = leader
+  const int pair = blockIdx.x / CG, npairs = gridDim.x / CG;
+  const int b_rows = a.bn / CG;                            // weight rows per CTA
   const uint32_t sA = sbase;                                     // A stages
   const uint32_t sB = sbase + (uint32_t)stages * TC_A_STAGE;     // B stages
-  const uint32_t b_stage = (uint32_t)a.bn * TC_ROW_BYTES;
+  const uint32_t b_stage = (uint32_t)b_rows * TC_ROW_BYTES;
 
   uint32_t *ktab_s = (uint32_t *)(smem + SM_KTAB);
   const bool use_tab = a.ktab != nullptr;
@@ -232,26 +294,37 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     }
   }
   if (tid == 0) {
+    // leader full: its B producer + 256 gather threads (+ the peer's relay);
+    // peer full: its 256 gather threads (watched by the relay thread)
+    const uint32_t full_count = rank == 0 ? 1 + TC_NPROD + (CG == 2 ? 1 : 0) : TC_NPROD;
     for (int s = 0; s < stages; ++s) {
-      mbar_init(sbase + SM_FULL + 8 * s, 1 + TC_NPROD);
+      mbar_init(sbase + SM_FULL + 8 * s, full_count);
       mbar_init(sbase + SM_EMPTY + 8 * s, 1);
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(sbase + SM_TFULL + 8 * i, 1);
-      mbar_init(sbase + SM_TEMPTY + 8 * i, 128);
+      mbar_init(sbase + SM_TEMPTY + 8 * i, 4 * CG);   // one arrive per epilogue warp
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     census_mark(a.b);
   }
   if (warp == 1) {
-    asm volatile(
-        "tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-            sbase + SM_TMEMPTR),
-        "n"(TC_TMEM_COLS));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    if constexpr (CG == 1) {
+      asm volatile(
+          "tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+              sbase + SM_TMEMPTR),
+          "n"(TC_TMEM_COLS));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    } else {
+      asm volatile(
+          "tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+              sbase + SM_TMEMPTR),
+          "n"(TC_TMEM_COLS));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    }
   }
   tc_fence_before();
-  __syncthreads();
+  if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *(volatile uint32_t *)(smem + SM_TMEMPTR);
 
@@ -276,26 +349,31 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
       uint32_t stage = 0, phase = 0;
-      for (int u = blockIdx.x; u < a.units; u += gridDim.x) {
+      for (int u = pair; u < a.units; u += npairs) {
         int mt, nt, grp, sp, k0, k1;
         decode(u, mt, nt, grp, sp);
         kb_range(sp, k0, k1);
-        const int nrow = grp * g.Nfg + nt * a.bn;
+        const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
         for (int kb = k0; kb < k1; ++kb) {
           mbar_wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
-          mbar_arrive_expect_tx(sbase + SM_FULL + 8 * stage, b_stage);
-          tma_load_2d(sB + stage * b_stage, &tmap_w, sbase + SM_FULL + 8 * stage,
-                      kb * (TC_ROW_BYTES / ESZ), nrow);
+          const uint32_t fb = sbase + SM_FULL + 8 * stage;
+          if constexpr (CG == 1) {
+            mbar_arrive_expect_tx(fb, b_stage);
+            tma_load_2d(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
+          } else {
+            if (rank == 0) mbar_arrive_expect_tx(fb, 2 * b_stage);   // both halves
+            tma_load_2d_2sm(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
+          }
           advance(stage, phase, stages);
         }
       }
     }
   } else if (warp == 1) {
-    // ------------------------------------------------ MMA issuer
-    if (lane == 0) {
-      const uint32_t idesc = umma_idesc<ST>(a.bn);
+    if (lane == 0 && rank == 0) {
+      // ---------------------------------------------- MMA issuer (leader)
+      const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
       uint32_t stage = 0, phase = 0, lt = 0;
-      for (int u = blockIdx.x; u < a.units; u += gridDim.x, ++lt) {
+      for (int u = pair; u < a.units; u += npairs, ++lt) {
         int mt, nt, grp, sp, k0, k1;
         decode(u, mt, nt, grp, sp);
         kb_range(sp, k0, k1);
@@ -311,11 +389,26 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
           const uint64_t bd = umma_desc_sw128(sB + stage * b_stage);
 #pragma unroll
           for (int k = 0; k < 4; ++k)   // 4 x 32 B along K inside the 128 B row
-            tc_mma<ST>(dcol, ad + 2 * k, bd + 2 * k, idesc, (kb > k0) || (k > 0));
-          tc_commit(sbase + SM_EMPTY + 8 * stage);
+            tc_mma<ST, CG>(dcol, ad + 2 * k, bd + 2 * k, idesc, (kb > k0) || (k > 0));
+          tc_commit<CG>(sbase + SM_EMPTY + 8 * stage);
           advance(stage, phase, stages);
         }
-        tc_commit(sbase + SM_TFULL + 8 * buf);
+        tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
+      }
+    } else if (CG == 2 && lane == 0) {
+      // ---------------------------------------------- relay (peer): its gather
+      // threads' completion -> one arrive on the leader's full barrier
+      uint32_t stage = 0, phase = 0;
+      for (int u = pair; u < a.units; u += npairs) {
+        int mt, nt, grp, sp, k0, k1;
+        decode(u, mt, nt, grp, sp);
+        kb_range(sp, k0, k1);
+        for (int kb = k0; kb < k1; ++kb) {
+          mbar_wait(sbase + SM_FULL + 8 * stage, phase);
+          fence_proxy_async();
+          mbar_arrive_cluster(mapa(sbase + SM_FULL + 8 * stage, 0));
+          advance(stage, phase, stages);
+        }
       }
     }
   } else if (warp < 6) {
@@ -323,14 +416,16 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     const int quarter = warp & 3;
     const int row = quarter * 32 + lane;
     const bool partial = a.splits > 1;
+    const uint32_t tempty_leader =
+        CG == 2 ? mapa(sbase + SM_TEMPTY, 0) : sbase + SM_TEMPTY;
     uint32_t lt = 0;
-    for (int u = blockIdx.x; u < a.units; u += gridDim.x, ++lt) {
+    for (int u = pair; u < a.units; u += npairs, ++lt) {
       int mt, nt, grp, sp;
       decode(u, mt, nt, grp, sp);
       const uint32_t buf = lt & 1, use = lt >> 1;
       mbar_wait(sbase + SM_TFULL + 8 * buf, use & 1);
       tc_fence_after();
-      const int m = mt * TC_BM + row;
+      const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
       const bool mok = m < g.M;
       const size_t orow = (size_t)m * g.out_cs;
       for (int c0 = 0; c0 < a.bn; c0 += 16) {
@@ -392,9 +487,12 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
           }
         }
       }
-      __syncwarp();
       tc_fence_before();
-      mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
+      __syncwarp();
+      if (lane == 0) {
+        if constexpr (CG == 2) mbar_arrive_cluster(tempty_leader + 8 * buf);
+        else mbar_arrive(tempty_leader + 8 * buf);
+      }
     }
   } else {
     // ------------------------------------------------ A (im2col) gather producers
@@ -404,7 +502,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     const uint32_t swz = (uint32_t)((j ^ (rb & 7)) << 4);
     const char *xb = (const char *)a.x;
     uint32_t stage = 0, phase = 0;
-    for (int u = blockIdx.x; u < a.units; u += gridDim.x) {
+    for (int u = pair; u < a.units; u += npairs) {
       int mt, nt, grp, sp, k0, k1;
       decode(u, mt, nt, grp, sp);
       kb_range(sp, k0, k1);
@@ -412,7 +510,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
       int ih0[4], iw0[4];
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
-        const int m = mt * TC_BM + rb + 32 * i;
+        const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + rb + 32 * i;
         if (m < g.M) {
           const int n = m / HoWo, pq = m % HoWo;
           const int pp = pq / g.Wo, q = pq % g.Wo;
@@ -456,11 +554,15 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   }
 
   tc_fence_before();
-  __syncthreads();
+  if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   if (warp == 1) {
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
-                 "n"(TC_TMEM_COLS));
+    if constexpr (CG == 1)
+      asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                   "n"(TC_TMEM_COLS));
+    else
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                   "n"(TC_TMEM_COLS));
   }
 }
 
@@ -500,13 +602,36 @@ __global__ void splitk_reduce_kernel(const float *__restrict__ ws, void *y,
   }
 }
 
-cudaError_t tc_init() {
-  cudaError_t e = cudaFuncSetAttribute(conv_tc_kernel<ST_BF16>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)TC_SMEM_BYTES);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(conv_tc_kernel<ST_F32>,
+template <int ST, int CG>
+static cudaError_t set_smem_attr() {
+  return cudaFuncSetAttribute(conv_tc_kernel<ST, CG>,
                               cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM_BYTES);
+}
+
+cudaError_t tc_init() {
+  cudaError_t e;
+  if ((e = set_smem_attr<ST_BF16, 1>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_BF16, 2>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_F32, 1>()) != cudaSuccess) return e;
+  return set_smem_attr<ST_F32, 2>();
+}
+
+template <int ST, int CG>
+static cudaError_t launch_tc(const CUtensorMap *tmap, const TcArgs &args, int grid,
+                             cudaStream_t s) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(TC_THREADS);
+  cfg.dynamicSmemBytes = TC_SMEM_BYTES;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG>, *tmap, args);
 }
 
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
@@ -527,13 +652,17 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
   args.units = p.units;
   args.kblocks = g.Kpad / tc_block_k_elems(st);
   args.kb_per_split = p.kb_per_split;
-  args.stages = tc_stages_for(p.bn);
+  args.stages = tc_stages_for(p.bn, p.cg);
   args.b = b;
+  cudaError_t e;
   if (st == ST_BF16)
-    conv_tc_kernel<ST_BF16><<<p.grid, TC_THREADS, TC_SMEM_BYTES, s>>>(*tmap_w, args);
+    e = p.cg == 2 ? launch_tc<ST_BF16, 2>(tmap_w, args, p.grid, s)
+                  : launch_tc<ST_BF16, 1>(tmap_w, args, p.grid, s);
   else
-    conv_tc_kernel<ST_F32><<<p.grid, TC_THREADS, TC_SMEM_BYTES, s>>>(*tmap_w, args);
-  cudaError_t e = cudaGetLastError();
+    e = p.cg == 2 ? launch_tc<ST_F32, 2>(tmap_w, args, p.grid, s)
+                  : launch_tc<ST_F32, 1>(tmap_w, args, p.grid, s);
+  if (e != cudaSuccess) return e;
+  e = cudaGetLastError();
   if (e != cudaSuccess || p.splits <= 1) return e;
   const long long total = (long long)g.M * g.out_cs / 4;
   const int grid = (int)std::min<long long>((total + 255) / 256, 148 * 8);

@@ -72,12 +72,13 @@ void conv_simt_tile_shape(int *tm, int *tn);
 
 // tcgen05 implicit-GEMM conv / FC (K1/K2).
 struct TcPlan {
+  int cg;          // CTAs per tile: 1 (M = 128) or 2 (CTA pair, M = 256)
   int bn;          // N tile (16..256, multiple of 16)
   int mtiles, ntiles, tiles;   // output tiles (eq. 4 grid size)
   int splits;      // split-K factor (1 = none); chosen from the shape only
   int kb_per_split;
   int units;       // tiles * splits work units
-  int grid;        // CTAs = min(units, SM budget)
+  int grid;        // CTAs = cg * min(units, SM budget / cg)
 };
 // Launches the GEMM and, when p.splits > 1, the deterministic split-K
 // reduction (ws must hold splits * M * out_cs floats; a split-K output must
@@ -86,7 +87,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
                            const CUtensorMap *tmap_w, const float *bias,
                            void *y, const int *ktab, const TcPlan &p, float *ws,
                            const Budget &b, cudaStream_t s);
-int tc_stages_for(int bn);
+int tc_stages_for(int bn, int cg);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)
 cudaError_t tc_init();                 // sets the kernels' smem attributes
 size_t tc_smem_bytes();

@@ -241,7 +241,7 @@ static pcnn_status infer_shapes(const pcnn_net_desc *d, const pcnn_layer_desc *L
       case PCNN_LRN:
         if (li.kernel <= 0 || (li.kernel % 2) == 0)
           return fail(PCNN_ERR_SHAPE, "LRN size must be odd");
-        if (c > 1024) return fail(PCNN_ERR_UNSUPPORTED, "LRN with > 1024 channels");
+        if (li.kernel > 9) return fail(PCNN_ERR_UNSUPPORTED, "LRN local size > 9");
         break;
       case PCNN_MAXPOOL:
       case PCNN_AVGPOOL: {
@@ -457,47 +457,60 @@ static const CUtensorMap *stage_tmap(GemmStage &gs, int bn) {
 
 // ------------------------------------------------------------------ planning
 // Tile / split selection (the paper's sub-matrix choice, P:223,
-// P:267).  For every N tile bn (multiple of 16, <= 256):
-//   tiles  = ceil(M/128) * ceil(Nfg/bn) * groups          (eq. 4)
+// P:267).  For every CTA grouping cg (1 CTA, M = 128 / CTA pair, M = 256) and
+// N tile bn (multiple of 16, <= 256):
+//   tiles  = ceil(M / (128 cg)) * ceil(Nfg / bn) * groups       (eq. 4)
 //   splits = K split when the tiles cannot fill half the GPU
-//   time   = max(waves * kblocks/splits * cycles(bn) / f, weight bytes / HBM)
+//   K-block cost (cycles, per SM) = max(MMA 2.05 bn, operand bytes per SM /
+//            kOperandBytesPerCycle) + 40
+//   time   = max(waves * kblocks/splits * cost / f, weight bytes / HBM)
 //            + split-K reduction traffic
-// where one K-block costs max(MMA ~2.05*bn, A gather ~256) + 40 cycles.  Small
-// tiles raise Util (eq. 6) and rEC (eq. 9), big tiles raise the computation
-// density -- the trade-off of P:223.  The plan depends on the problem shape and
-// the device's SM count only, never on the SM budget, so every budget runs the
-// same tiles and K order (bitwise-identical results, R11).
+// Small tiles raise Util (eq. 6) and rEC (eq. 9), big tiles raise the
+// computation density per operand byte -- the trade-off of P:223.  The plan
+// depends on the problem shape and the device's SM count only, never on the
+// SM budget, so every budget runs the same tiles and K order (R11).
+static constexpr double kOperandBytesPerCycle = 23.5;   // measured L2->SM feed per SM
+
 static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
   TcPlan best{};
   double best_t = 1e300;
-  const int mtiles = (g.M + 127) / 128;
   const int nmax = std::min(256, round_up(g.Nfg, 16));
   const double f = 1.9e9, hbm = 6.0e12;
   const double wbytes = (double)g.Nfg * g.groups * g.Kpad * esz;
-  for (int bn = 16; bn <= nmax; bn += 16) {
-    const int ntiles = (g.Nfg + bn - 1) / bn;
-    const long long tiles = (long long)mtiles * ntiles * g.groups;
-    int splits = 1;
-    if (tiles * 2 < device_sms && kblocks >= 8) {
-      splits = (int)std::min<long long>((device_sms + tiles - 1) / tiles, 16);
-      splits = std::max(1, std::min(splits, kblocks / 4));
-    }
-    const int kbs = (kblocks + splits - 1) / splits;
-    splits = (kblocks + kbs - 1) / kbs;
-    const long long units = tiles * splits;
-    const long long waves = (units + device_sms - 1) / device_sms;
-    double t = (double)waves * kbs * (std::max(2.05 * bn, 256.0) + 40.0) / f;
-    t = std::max(t, wbytes / hbm);
-    if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
-    if (t < best_t * 0.999 || (t <= best_t * 1.001 && bn > best.bn)) {
-      best_t = t;
-      best.bn = bn;
-      best.mtiles = mtiles;
-      best.ntiles = ntiles;
-      best.tiles = (int)tiles;
-      best.splits = splits;
-      best.kb_per_split = kbs;
-      best.units = (int)units;
+  const char *force_cg = getenv("PCNN_FORCE_CG");
+  for (int cg = 1; cg <= 2; ++cg) {
+    if (force_cg && atoi(force_cg) != cg) continue;
+    const int mtiles = (g.M + 128 * cg - 1) / (128 * cg);
+    const int slots = device_sms / cg;          // concurrent units
+    for (int bn = 16; bn <= nmax; bn += 16) {
+      if (cg == 2 && (bn / 2) % 8) continue;
+      const int ntiles = (g.Nfg + bn - 1) / bn;
+      const long long tiles = (long long)mtiles * ntiles * g.groups;
+      int splits = 1;
+      if (tiles * 2 < slots && kblocks >= 8) {
+        splits = (int)std::min<long long>((slots + tiles - 1) / tiles, 16);
+        splits = std::max(1, std::min(splits, kblocks / 4));
+      }
+      const int kbs = (kblocks + splits - 1) / splits;
+      splits = (kblocks + kbs - 1) / kbs;
+      const long long units = tiles * splits;
+      const long long waves = (units + slots - 1) / slots;
+      const double bytes_sm = 128.0 * 128 + (double)bn / cg * 128;   // A + B per SM per K-block
+      const double kb_cycles = std::max(2.05 * bn, bytes_sm / kOperandBytesPerCycle) + 40.0;
+      double t = (double)waves * kbs * kb_cycles / f;
+      t = std::max(t, wbytes / hbm);
+      if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
+      if (t < best_t * 0.999 || (t <= best_t * 1.001 && bn * cg > best.bn * best.cg)) {
+        best_t = t;
+        best.cg = cg;
+        best.bn = bn;
+        best.mtiles = mtiles;
+        best.ntiles = ntiles;
+        best.tiles = (int)tiles;
+        best.splits = splits;
+        best.kb_per_split = kbs;
+        best.units = (int)units;
+      }
     }
   }
   return best;
@@ -530,17 +543,20 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
   g.M = B * g.Ho * g.Wo;
   if (gs.engine == 1) {
     TcPlan p = plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st));
-    p.grid = std::min(p.units, effective_sms(net, ly));
+    // the budget caps concurrent units; a CTA pair needs at least 2 SMs
+    const int slots = std::max(1, effective_sms(net, ly) / p.cg);
+    p.grid = p.cg * std::min(p.units, slots);
     const CUtensorMap *tm = stage_tmap(gs, p.bn);
     if (!tm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeTiled failed");
     if (info) {
-      info->tile_m = 128;
+      info->tile_m = 128 * p.cg;
       info->tile_n = p.bn;
       info->tiles = p.tiles;
       info->grid = p.grid;
       info->tlp = 1;
       info->engine = 1;
       info->splits = p.splits;
+      info->n_sms = std::max(info->n_sms, p.grid);   // pair granularity
     }
     if (ws_need) *ws_need = std::max(*ws_need, p.splits > 1 ? (size_t)p.splits * g.M * g.out_cs * 4 : 0);
     if (!x) return PCNN_OK;   // planning only

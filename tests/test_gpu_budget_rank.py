@@ -1,0 +1,131 @@
+"""Per-layer SM budget (P:213 PSM, P:341 optSM x optTLP) and the rank-r
+variant (north_star; R7) on the GPU, through the C ABI."""
+import numpy as np
+import pytest
+
+import synth
+from tests.helpers import TOL, conv_layer, gpu_run, params, rel_err, small_inputs
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+
+
+@pytest.fixture(scope="module")
+def alex():
+    net = synth.alexnet()
+    w, b = params(net)
+    x = synth.images(0, 2, net["in_shape"])
+    return net, w, b, x
+
+
+# ------------------------------------------------------------------ SM budget
+@pytest.mark.parametrize("prec", ["bf16", "fp32"])
+def test_budget_is_bitwise_invariant_and_census_bounded(alex, prec):
+    """R11: the budget changes placement only.  Every budget gives bitwise
+    identical logits; the %smid census of each layer stays within the budget
+    (tcgen05 CTA pairs round the budget up to 2 SMs)."""
+    net, w, b, x = alex
+    gemm_layers = [i for i, L in enumerate(net["layers"]) if L["kind"] in ("conv", "fc")]
+    base = gpu_run(net, w, b, x, prec)["out"]
+    for n_sms, tlp in [(1, 0), (2, 0), (7, 1), (37, 2), (74, 0), (148, 0)]:
+        budgets = {i: (n_sms, tlp) for i in range(len(net["layers"]))}
+        r = gpu_run(net, w, b, x, prec, budgets=budgets, census=True)
+        np.testing.assert_array_equal(r["out"], base, err_msg="budget %d/%d" % (n_sms, tlp))
+        for i in gemm_layers:
+            used = r["census"][i]
+            assert 0 < len(used) <= max(n_sms, 2), (i, n_sms, used)
+
+
+def test_budget_simt_tlp_gating(alex):
+    """SIMT kernels: CTAs admitted only on SMs with %smid < n, at most tlp
+    CTAs each (Priority-SM packing, Fig. 7)."""
+    net, w, b, x = alex
+    r = gpu_run(net, w, b, x, "fp32", budgets={3: (4, 2)}, census=True)
+    assert set(r["census"][3]) <= {0, 1, 2, 3}
+
+
+def test_query_layer_reports_plan(alex):
+    net, w, b, x = alex
+    r = gpu_run(net, w, b, x, "bf16", budgets={6: (37, 0)})
+    info = r["net"].query_layer(6, 64)
+    assert info["engine"] == 1 and info["n_sms"] == 37
+    assert 0 < info["util"] <= 1 and 0 < info["rec"] <= 1
+    assert info["tiles"] >= 1 and info["grid"] <= 37
+    assert info["flops"] == info["flops_exact"] == 2 * 64 * 13 * 13 * 384 * 9 * 256
+
+
+# ------------------------------------------------------------------ rank-r variant
+def test_rank_identity_factors_bitwise_fp32(alex):
+    """Identity factorisation (A = I, B = W) reproduces the exact layer
+    bitwise on the FP32 path: stage 1 sums the same K terms in the same order,
+    stage 2 multiplies by exact ones and zeros."""
+    net = dict(in_shape=(32, 13, 13), layers=[conv_layer(64, 3, 32, 1, 1, 2, relu=True)])
+    w, b = params(net, seed=11)
+    x = small_inputs((32, 13, 13), 3)
+    import torch
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    n = pcnn.Net(net, w, b, 3, "fp32")
+    xd = torch.from_numpy(x).cuda()
+    exact = n.infer(xd)[0].cpu().numpy()
+    g, Nfg = 2, 32
+    A = np.stack([np.eye(Nfg, dtype=np.float32)] * g)             # [g][Nfg][r]
+    B = w[0].reshape(g, Nfg, 16, 3, 3)                             # [g][r][C/g][S][S]
+    n.set_variant_factors(0, Nfg, A, B)
+    fact = n.infer(xd)[0].cpu().numpy()
+    np.testing.assert_array_equal(fact, exact)
+    n.set_variant(0, "exact")
+    np.testing.assert_array_equal(n.infer(xd)[0].cpu().numpy(), exact)
+
+
+@pytest.mark.parametrize("prec", ["fp32", "tf32", "bf16"])
+def test_rank_r_conv_matches_rank_oracle(orc, prec):
+    """The two-stage rank-r conv equals the oracle's W_r = U_r U_r^T W conv."""
+    net = dict(in_shape=(48, 15, 15), layers=[conv_layer(64, 3, 48, 1, 1, 1, relu=True)])
+    w, b = params(net, seed=13)
+    x = small_inputs((48, 15, 15), 2)
+    for r in (8, 24, 64):
+        ref = orc.run_net(net, w, b, x, ranks={0: r}).reshape(2, -1)
+        out = gpu_run(net, w, b, x, prec, variants={0: ("rank", r)})["out"]
+        assert rel_err(out, ref) <= TOL[prec] / 2, (prec, r)
+    # full rank == exact layer
+    ref = orc.run_net(net, w, b, x).reshape(2, -1)
+    out = gpu_run(net, w, b, x, prec, variants={0: ("rank", 64)})["out"]
+    assert rel_err(out, ref) <= TOL[prec] / 2
+
+
+@pytest.mark.parametrize("prec", ["tf32", "bf16"])
+def test_alexnet_rank_ladder(orc, alex, prec):
+    """configs[2]: the accuracy-tuning ladder -- each
+    rung matches the rank-r oracle end to end."""
+    net, w, b, x = alex
+    ladder = [{}, {3: 64}, {3: 64, 8: 64}, {3: 64, 8: 64, 7: 96},
+              {3: 64, 8: 64, 7: 96, 6: 192}]
+    for rung in ladder[1:]:
+        ref = orc.run_net(net, w, b, x, ranks=rung)
+        out = gpu_run(net, w, b, x, prec,
+                      variants={i: ("rank", r) for i, r in rung.items()})["out"]
+        assert rel_err(out, ref) <= TOL[prec], (prec, rung)
+
+
+def test_rank_variant_rejects_bad_requests(alex):
+    net, w, b, x = alex
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    n = pcnn.Net(net, w, b, 2, "bf16")
+    with pytest.raises(pcnn.PcnnError):
+        n.set_variant(1, "rank", 8)         # LRN layer
+    with pytest.raises(pcnn.PcnnError):
+        n.set_variant(3, "rank", 0)
+    with pytest.raises(pcnn.PcnnError):
+        n.set_variant(3, "rank", 129)       # > min(N_f/g, K) = 128
+    info = n.query_layer(3, 2)
+    assert info["variant"] == 0
+    n.set_variant(3, "rank", 32)
+    info = n.query_layer(3, 2)
+    assert info["variant"] == 1 and info["rank"] == 32
+    assert info["flops"] < info["flops_exact"]
