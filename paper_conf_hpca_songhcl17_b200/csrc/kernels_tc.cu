@@ -3,36 +3,32 @@
 // What it computes (Fig. 2; eq. 1): for every group g,
 //   O_g[M x Nfg] = im2col(X)_g[M x K] * F_m,g[Nfg x K]^T  (+bias, ReLU)
 // with M = B*Ho*Wo output pixels (NHWC rows), K = (r, s, c) taps x channels.
-// D_m (the im2col matrix) is never materialised: producer warps gather each
-// A tile row -- one output pixel's (r, s, c-chunk) input run -- straight from
-// the NHWC activations into the 128B-swizzled shared-memory layout the UMMA
-// descriptor expects (cp.async 16 B chunks, zero-fill for padding / ragged
-// tails; completion signalled with cp.async.mbarrier.arrive.noinc so the
-// producers never block on their own loads).  The weight tile (B operand)
-// arrives by TMA.  One elected thread issues tcgen05.mma (BF16 kind::f16 or
-// kind::tf32, FP32 accumulate) into a double-buffered TMEM accumulator; four
-// epilogue warps drain it with tcgen05.ld, add bias, apply ReLU, round to the
-// storage precision and store NHWC rows (or, for split-K work units, store
-// FP32 partial sums that a deterministic reduction kernel adds in split order).
+// D_m (the im2col matrix) is never materialised: the A tile of every K-block
+// is fetched by TMA in im2col mode -- 128 consecutive output pixels x one
+// filter tap (r, s) x a channel slab, with conv padding and ragged tails
+// zero-filled by the TMA unit -- straight into the swizzled shared-memory
+// layout the UMMA descriptor expects.  A K-block is 128 B of K per row: one
+// 64-channel slab (SW128), or 2 / 4 narrower slabs (SW64 / SW32) when the
+// channels per group are not a multiple of 64 (AlexNet conv2: 48).  The
+// weight tile (B operand) arrives by a tiled TMA load.  One thread issues all
+// loads, one thread issues tcgen05.mma (BF16 kind::f16 or kind::tf32, FP32
+// accumulate) into a double-buffered TMEM accumulator, and four epilogue
+// warps drain it with tcgen05.ld, add bias, apply ReLU, round to the storage
+// precision and store NHWC rows (or, for split-K work units, FP32 partial
+// sums that a deterministic reduction kernel adds in split order).
 // The kernel is persistent: grid = min(work units, SM budget) CTAs, 1 CTA per
 // SM (smem + TMEM), static round-robin schedule -- the grid cap IS the
 // per-layer SM budget.  The pipeline depth is sized at launch from
-// the N tile so that ~200 KB of operand stages are in flight per SM.
+// the N tile (~200 KB of operand stages per SM).
 //
 // CG = 2 runs the same pipeline on a CTA pair (cluster of 2, cta_group::2):
-// one 256 x N tile per pair, each CTA gathering its 128 A rows and loading
-// half of the weight tile, the leader CTA issuing M = 256 UMMAs whose
-// accumulator rows are split across both CTAs' TMEM.  Per SM this halves the
-// operand bytes moved per FLOP (smem and L2 bandwidth were the limit of the
-// 128 x N single-CTA tile).  The peer's A-gather completion is relayed to the
-// leader's full barrier by one peer thread; MMA commits multicast to both
-// CTAs' empty / accumulator-full barriers.
+// one 256 x N tile per pair, each CTA loading its 128 A rows and half of the
+// weight tile into its own smem with the loads' bytes counted on the leader's
+// barrier; the leader issues M = 256 UMMAs whose accumulator rows are split
+// across both CTAs' TMEM, and its commits multicast to both CTAs' barriers.
 //
-// CTA = 14 warps (448 threads):
-//   warp 0       : TMA producer for B (weights)
-//   warp 1       : TMEM allocator + MMA issuer
-//   warps 2..5   : epilogue (TMEM lane quarter = warp % 4)
-//   warps 6..13  : im2col gather producers for A (256 threads)
+// CTA = 6 warps: warp 0 TMA producer, warp 1 TMEM allocator + MMA issuer,
+// warps 2..5 epilogue (TMEM lane quarter = warp % 4).
 #include <algorithm>
 
 #include "budget.cuh"
@@ -46,16 +42,14 @@ constexpr int TC_ROW_BYTES = 128;       // one K-block row = one 128B swizzle ro
 constexpr int TC_MAX_STAGES = 12;
 constexpr int TC_A_STAGE = TC_BM * TC_ROW_BYTES;          // 16 KB
 constexpr int TC_STAGE_BUDGET = 200 * 1024;               // operand stages per CTA
-constexpr int TC_MAX_KTAB = 4096;       // chunk-table entries kept in smem
-constexpr int TC_THREADS = 448;
-constexpr int TC_PRODUCER0 = 192;       // first A-producer thread
-constexpr int TC_NPROD = 256;
+constexpr int TC_MAX_KTAB = 4096;       // slab-table entries kept in smem
+constexpr int TC_THREADS = 192;
 constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 
 // smem layout (bytes from the 1024-aligned base):
 //   [0, TC_STAGE_BUDGET)   A stages, then B stages (runtime count)
 //   SM_BAR                 barriers + TMEM pointer
-//   SM_KTAB                (r, s, c) chunk table
+//   SM_KTAB                (r, s, c) table, one entry per A slab
 constexpr int SM_BAR = TC_STAGE_BUDGET;
 constexpr int SM_FULL = SM_BAR;
 constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_STAGES;
@@ -112,15 +106,28 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map
       : "memory");
 }
 
-__device__ __forceinline__ void cp_async_16(uint32_t dst, const void *src, int nbytes) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
-               "r"(nbytes)
-               : "memory");
+// TMA im2col load of one A slab: 128 output pixels starting at (w, h, n)
+// (input-space corner of the first pixel), channels [c, c + slab), filter tap
+// offsets (ow, oh); padding / out-of-range pixels are zero-filled.
+__device__ __forceinline__ void tma_im2col(uint32_t dst, const CUtensorMap *map, uint32_t bar,
+                                           int c, int w, int h, int n, uint16_t ow,
+                                           uint16_t oh) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ow), "h"(oh)
+      : "memory");
 }
-// Arrive on `bar` once every cp.async this thread issued so far has landed
-// (the arrival counts against the barrier's expected count: .noinc).
-__device__ __forceinline__ void cp_async_arrive_noinc(uint32_t bar) {
-  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
+// 2-SM form: lands in this CTA's smem, bytes counted on the leader's barrier.
+__device__ __forceinline__ void tma_im2col_2sm(uint32_t dst, const CUtensorMap *map,
+                                               uint32_t bar, int c, int w, int h, int n,
+                                               uint16_t ow, uint16_t oh) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.im2col.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
+      "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ow),
+      "h"(oh)
+      : "memory");
 }
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -217,17 +224,20 @@ __device__ __forceinline__ void tmem_ld_wait() {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
-// UMMA shared-memory descriptor, K-major, 128B swizzle: 8-row x 128 B atoms
-// stacked along M/N every 1024 B (SBO), version 1 (sm_100), layout 2 = SW128.
-__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
+// UMMA shared-memory descriptor, K-major, swizzled rows of `row_bytes`
+// (128 / 64 / 32 B): 8-row atoms stacked along M/N every 8*row_bytes (SBO),
+// version 1 (sm_100), layout SW128 = 2, SW64 = 4, SW32 = 6.
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t row_bytes) {
+  const uint64_t layout = row_bytes == 128 ? 2 : (row_bytes == 64 ? 4 : 6);
   uint64_t d = 0;
   d |= (uint64_t)((saddr >> 4) & 0x3FFF);
-  d |= (uint64_t)1 << 16;                  // LBO (unused for swizzled K-major)
-  d |= (uint64_t)(1024 >> 4) << 32;        // SBO
-  d |= (uint64_t)1 << 46;                  // descriptor version (sm_100)
-  d |= (uint64_t)2 << 61;                  // SWIZZLE_128B
+  d |= (uint64_t)1 << 16;                        // LBO (unused for swizzled K-major)
+  d |= (uint64_t)((8 * row_bytes) >> 4) << 32;   // SBO
+  d |= (uint64_t)1 << 46;                        // descriptor version (sm_100)
+  d |= layout << 61;
   return d;
 }
+__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) { return umma_desc(saddr, 128); }
 
 // Instruction descriptor: D fp32, A/B = BF16 (1) or TF32 (2), K-major,
 // M = 128 * CG, N = bn.
@@ -246,7 +256,6 @@ __device__ __forceinline__ float tf32_rna_tc(float v) {
 
 struct TcArgs {
   ConvGeom g;
-  const void *x;
   void *y;
   float *ws;            // split-K partials [splits][M][out_cs] fp32 (splits > 1)
   const float *bias;
@@ -255,6 +264,7 @@ struct TcArgs {
   int mtiles, ntiles, splits, units;
   int kblocks, kb_per_split;
   int stages;
+  int slab_bytes;       // 128 / 64 / 32: A K-block = 128 / slab_bytes TMA slabs
   Budget b;
 };
 
@@ -267,14 +277,14 @@ __device__ __forceinline__ void advance(uint32_t &stage, uint32_t &phase, int st
 
 template <int ST, int CG>
 __global__ void __launch_bounds__(TC_THREADS, 1)
-conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
+conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
+               const __grid_constant__ CUtensorMap tmap_x, const TcArgs a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const uint32_t sbase = smem_u32(smem);
   const int tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31;
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
-  constexpr int CH = 16 / ESZ;                 // elements per 16 B chunk
   const ConvGeom &g = a.g;
   const int stages = a.stages;
   const uint32_t rank = CG == 2 ? cluster_ctarank() : 0;   // 0 = leader
@@ -283,22 +293,22 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   const uint32_t sA = sbase;                                     // A stages
   const uint32_t sB = sbase + (uint32_t)stages * TC_A_STAGE;     // B stages
   const uint32_t b_stage = (uint32_t)b_rows * TC_ROW_BYTES;
+  const int slab_bytes = a.slab_bytes;
+  const int nslab = TC_ROW_BYTES / slab_bytes;
+  const int slab_elems = slab_bytes / ESZ;
 
   uint32_t *ktab_s = (uint32_t *)(smem + SM_KTAB);
   const bool use_tab = a.ktab != nullptr;
-  const int nchunks = g.Kpad / CH;
+  const int nent = g.Kpad / slab_elems;
   if (use_tab) {
-    for (int i = tid; i < nchunks && i < TC_MAX_KTAB; i += TC_THREADS) {
-      const int k = i * CH;
+    for (int i = tid; i < nent && i < TC_MAX_KTAB; i += TC_THREADS) {
+      const int k = i * slab_elems;
       ktab_s[i] = k < g.K ? (uint32_t)__ldg(&a.ktab[k]) : 0xFF000000u;
     }
   }
   if (tid == 0) {
-    // leader full: its B producer + 256 gather threads (+ the peer's relay);
-    // peer full: its 256 gather threads (watched by the relay thread)
-    const uint32_t full_count = rank == 0 ? 1 + TC_NPROD + (CG == 2 ? 1 : 0) : TC_NPROD;
     for (int s = 0; s < stages; ++s) {
-      mbar_init(sbase + SM_FULL + 8 * s, full_count);
+      mbar_init(sbase + SM_FULL + 8 * s, 1);
       mbar_init(sbase + SM_EMPTY + 8 * s, 1);
     }
     for (int i = 0; i < 2; ++i) {
@@ -345,25 +355,48 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
   };
 
   if (warp == 0) {
-    // ------------------------------------------------ B (weights) TMA producer
+    // ------------------------------------------------ TMA producer (A im2col + B)
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
       uint32_t stage = 0, phase = 0;
       for (int u = pair; u < a.units; u += npairs) {
         int mt, nt, grp, sp, k0, k1;
         decode(u, mt, nt, grp, sp);
         kb_range(sp, k0, k1);
         const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
+        // input-space corner of this CTA's first output pixel
+        const int m0 = mt * (TC_BM * CG) + (int)rank * TC_BM;
+        const int n0 = m0 / HoWo, pq = m0 % HoWo;
+        const int w0 = (pq % g.Wo) * g.stride - g.pad, h0 = (pq / g.Wo) * g.stride - g.pad;
         for (int kb = k0; kb < k1; ++kb) {
           mbar_wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
           const uint32_t fb = sbase + SM_FULL + 8 * stage;
-          if constexpr (CG == 1) {
-            mbar_arrive_expect_tx(fb, b_stage);
-            tma_load_2d(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
-          } else {
-            if (rank == 0) mbar_arrive_expect_tx(fb, 2 * b_stage);   // both halves
-            tma_load_2d_2sm(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
+          if (rank == 0) mbar_arrive_expect_tx(fb, CG * (TC_A_STAGE + b_stage));
+          const uint32_t dA = sA + stage * TC_A_STAGE;
+          for (int sl = 0; sl < nslab; ++sl) {
+            const int ke = kb * (TC_ROW_BYTES / ESZ) + sl * slab_elems;   // K element
+            int r = 0, s = 0, c = ke;
+            if (use_tab) {
+              const uint32_t e = ktab_s[ke / slab_elems];
+              r = (e >> 24) & 0xFF;
+              s = (e >> 16) & 0xFF;
+              c = e & 0xFFFF;
+              if (r == 0xFF) { r = 0; s = 0; c = g.Cs; }   // beyond K: zero-fill
+            } else if (ke >= g.K) {
+              c = g.Cs;
+            }
+            const int cc = c >= g.Cs ? g.Cs : grp * g.Cg + c;
+            const uint32_t dst = dA + sl * (TC_BM * slab_bytes);
+            if constexpr (CG == 1)
+              tma_im2col(dst, &tmap_x, fb, cc, w0, h0, n0, (uint16_t)s, (uint16_t)r);
+            else
+              tma_im2col_2sm(dst, &tmap_x, fb, cc, w0, h0, n0, (uint16_t)s, (uint16_t)r);
           }
+          if constexpr (CG == 1)
+            tma_load_2d(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
+          else
+            tma_load_2d_2sm(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
           advance(stage, phase, stages);
         }
       }
@@ -372,6 +405,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
     if (lane == 0 && rank == 0) {
       // ---------------------------------------------- MMA issuer (leader)
       const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
+      const int mma_per_slab = slab_bytes / 32;      // K = 32 B per UMMA
       uint32_t stage = 0, phase = 0, lt = 0;
       for (int u = pair; u < a.units; u += npairs, ++lt) {
         int mt, nt, grp, sp, k0, k1;
@@ -383,36 +417,23 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
         const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
         for (int kb = k0; kb < k1; ++kb) {
           mbar_wait(sbase + SM_FULL + 8 * stage, phase);
-          fence_proxy_async();   // cp.async (generic proxy) writes -> UMMA reads
           tc_fence_after();
-          const uint64_t ad = umma_desc_sw128(sA + stage * TC_A_STAGE);
+          const uint32_t aS = sA + stage * TC_A_STAGE;
           const uint64_t bd = umma_desc_sw128(sB + stage * b_stage);
 #pragma unroll
-          for (int k = 0; k < 4; ++k)   // 4 x 32 B along K inside the 128 B row
-            tc_mma<ST, CG>(dcol, ad + 2 * k, bd + 2 * k, idesc, (kb > k0) || (k > 0));
+          for (int k = 0; k < 4; ++k) {   // 4 x 32 B of K per 128 B K-block
+            const int sl = k / mma_per_slab, kin = k % mma_per_slab;
+            const uint64_t ad = umma_desc(aS + sl * (TC_BM * slab_bytes), slab_bytes) + 2 * kin;
+            tc_mma<ST, CG>(dcol, ad, bd + 2 * k, idesc, (kb > k0) || (k > 0));
+          }
           tc_commit<CG>(sbase + SM_EMPTY + 8 * stage);
           advance(stage, phase, stages);
         }
         tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
       }
-    } else if (CG == 2 && lane == 0) {
-      // ---------------------------------------------- relay (peer): its gather
-      // threads' completion -> one arrive on the leader's full barrier
-      uint32_t stage = 0, phase = 0;
-      for (int u = pair; u < a.units; u += npairs) {
-        int mt, nt, grp, sp, k0, k1;
-        decode(u, mt, nt, grp, sp);
-        kb_range(sp, k0, k1);
-        for (int kb = k0; kb < k1; ++kb) {
-          mbar_wait(sbase + SM_FULL + 8 * stage, phase);
-          fence_proxy_async();
-          mbar_arrive_cluster(mapa(sbase + SM_FULL + 8 * stage, 0));
-          advance(stage, phase, stages);
-        }
-      }
     }
-  } else if (warp < 6) {
-    // ------------------------------------------------ epilogue
+  } else {
+    // ------------------------------------------------ epilogue (warps 2..5)
     const int quarter = warp & 3;
     const int row = quarter * 32 + lane;
     const bool partial = a.splits > 1;
@@ -494,63 +515,6 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const TcArgs a) {
         else mbar_arrive(tempty_leader + 8 * buf);
       }
     }
-  } else {
-    // ------------------------------------------------ A (im2col) gather producers
-    const int p = tid - TC_PRODUCER0;          // 0..255
-    const int j = p & 7;                       // 16 B chunk within the 128 B row
-    const int rb = p >> 3;                     // rows rb, rb+32, rb+64, rb+96
-    const uint32_t swz = (uint32_t)((j ^ (rb & 7)) << 4);
-    const char *xb = (const char *)a.x;
-    uint32_t stage = 0, phase = 0;
-    for (int u = pair; u < a.units; u += npairs) {
-      int mt, nt, grp, sp, k0, k1;
-      decode(u, mt, nt, grp, sp);
-      kb_range(sp, k0, k1);
-      long long base[4];
-      int ih0[4], iw0[4];
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + rb + 32 * i;
-        if (m < g.M) {
-          const int n = m / HoWo, pq = m % HoWo;
-          const int pp = pq / g.Wo, q = pq % g.Wo;
-          base[i] = ((long long)n * g.H * g.W * g.Cs + (long long)grp * g.Cg) * ESZ;
-          ih0[i] = pp * g.stride - g.pad;
-          iw0[i] = q * g.stride - g.pad;
-        } else {
-          base[i] = -1;
-          ih0[i] = 0;
-          iw0[i] = 0;
-        }
-      }
-      for (int kb = k0; kb < k1; ++kb) {
-        mbar_wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
-        const int kc = kb * 8 + j;
-        int r = 0, sx = 0, c = kc * CH;
-        bool kok = c < g.K;
-        if (use_tab) {
-          const uint32_t e = kc < TC_MAX_KTAB ? ktab_s[kc] : 0xFF000000u;
-          r = (e >> 24) & 0xFF;
-          sx = (e >> 16) & 0xFF;
-          c = e & 0xFFFF;
-          kok = kok && r != 0xFF;
-        }
-        const uint32_t dst_stage = sA + stage * TC_A_STAGE;
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int row = rb + 32 * i;
-          const int ih = ih0[i] + r, iw = iw0[i] + sx;
-          const bool ok = kok && base[i] >= 0 && ih >= 0 && ih < g.H && iw >= 0 && iw < g.W;
-          const char *src =
-              ok ? xb + base[i] + (((long long)ih * g.W + iw) * g.Cs + c) * ESZ : xb;
-          cp_async_16(dst_stage + row * TC_ROW_BYTES + swz, src, ok ? 16 : 0);
-        }
-        cp_async_arrive_noinc(sbase + SM_FULL + 8 * stage);
-        advance(stage, phase, stages);
-      }
-    }
-    // keep the CTA (and its smem) alive until every in-flight copy has landed
-    asm volatile("cp.async.wait_all;" ::: "memory");
   }
 
   tc_fence_before();
@@ -616,9 +580,16 @@ cudaError_t tc_init() {
   return set_smem_attr<ST_F32, 2>();
 }
 
+int tc_slab_bytes(int st, int cg_channels) {
+  const int esz = st == ST_BF16 ? 2 : 4;
+  for (int sb = 128; sb >= 32; sb >>= 1)
+    if ((cg_channels * esz) % sb == 0) return sb;
+  return 0;   // channels per group must be a multiple of 32 bytes
+}
+
 template <int ST, int CG>
-static cudaError_t launch_tc(const CUtensorMap *tmap, const TcArgs &args, int grid,
-                             cudaStream_t s) {
+static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_x,
+                             const TcArgs &args, int grid, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(TC_THREADS);
@@ -631,16 +602,15 @@ static cudaError_t launch_tc(const CUtensorMap *tmap, const TcArgs &args, int gr
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG>, *tmap, args);
+  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG>, *tmap_w, *tmap_x, args);
 }
 
-cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
+cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias, void *y,
                            const int *ktab, const TcPlan &p, float *ws, const Budget &b,
                            cudaStream_t s) {
   TcArgs args;
   args.g = g;
-  args.x = x;
   args.y = y;
   args.ws = ws;
   args.bias = bias;
@@ -653,14 +623,16 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
   args.kblocks = g.Kpad / tc_block_k_elems(st);
   args.kb_per_split = p.kb_per_split;
   args.stages = tc_stages_for(p.bn, p.cg);
+  args.slab_bytes = tc_slab_bytes(st, g.Cg);
   args.b = b;
+  if (args.slab_bytes == 0) return cudaErrorInvalidValue;
   cudaError_t e;
   if (st == ST_BF16)
-    e = p.cg == 2 ? launch_tc<ST_BF16, 2>(tmap_w, args, p.grid, s)
-                  : launch_tc<ST_BF16, 1>(tmap_w, args, p.grid, s);
+    e = p.cg == 2 ? launch_tc<ST_BF16, 2>(tmap_w, tmap_x, args, p.grid, s)
+                  : launch_tc<ST_BF16, 1>(tmap_w, tmap_x, args, p.grid, s);
   else
-    e = p.cg == 2 ? launch_tc<ST_F32, 2>(tmap_w, args, p.grid, s)
-                  : launch_tc<ST_F32, 1>(tmap_w, args, p.grid, s);
+    e = p.cg == 2 ? launch_tc<ST_F32, 2>(tmap_w, tmap_x, args, p.grid, s)
+                  : launch_tc<ST_F32, 1>(tmap_w, tmap_x, args, p.grid, s);
   if (e != cudaSuccess) return e;
   e = cudaGetLastError();
   if (e != cudaSuccess || p.splits <= 1) return e;

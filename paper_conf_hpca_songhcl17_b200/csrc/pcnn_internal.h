@@ -83,10 +83,16 @@ struct TcPlan {
 // Launches the GEMM and, when p.splits > 1, the deterministic split-K
 // reduction (ws must hold splits * M * out_cs floats; a split-K output must
 // be packed, out_cs == groups * Nfg, with out_cs % 4 == 0).
-cudaError_t launch_conv_tc(const ConvGeom &g, int st, const void *x,
+// tmap_x: TMA im2col map of the NHWC input ({Cs, W, H, N}, corners -pad /
+// pad-(S-1), channelsPerPixel = slab, 128 pixels per column, swizzle =
+// slab bytes); tmap_w: tiled map of the packed weights (box 64|32 x bn/cg).
+cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias,
                            void *y, const int *ktab, const TcPlan &p, float *ws,
                            const Budget &b, cudaStream_t s);
+// A-slab width in bytes (128 / 64 / 32) for Cg channels per group, 0 if the
+// group width is not a multiple of 32 bytes.
+int tc_slab_bytes(int st, int cg_channels);
 int tc_stages_for(int bn, int cg);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)
 cudaError_t tc_init();                 // sets the kernels' smem attributes

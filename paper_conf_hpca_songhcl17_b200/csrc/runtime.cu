@@ -66,6 +66,20 @@ static inline float tf32_rna_host(float f) {
 }
 
 // ------------------------------------------------------------------ driver entry
+static PFN_cuTensorMapEncodeIm2col_v12000 get_encode_im2col() {
+  static PFN_cuTensorMapEncodeIm2col_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &p, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeIm2col_v12000)p;
+  });
+  return fn;
+}
+
 static PFN_cuTensorMapEncodeTiled_v12000 get_encode_tiled() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   static std::once_flag once;
@@ -91,7 +105,8 @@ struct GemmStage {           // one implicit-GEMM launch
   void *d_w = nullptr;       // packed [groups*Nfg][Kpad]
   float *d_bias = nullptr;
   int *d_ktab = nullptr;     // per-element (r,s,c) table
-  std::map<int, CUtensorMap> tmaps;  // by N tile
+  std::map<int, CUtensorMap> tmaps;  // weight maps by box rows
+  std::map<std::pair<const void *, int>, CUtensorMap> xmaps;   // im2col maps by (input, batch)
   size_t w_bytes = 0;
   void release() {
     if (d_w) cudaFree(d_w);
@@ -101,6 +116,7 @@ struct GemmStage {           // one implicit-GEMM launch
     d_bias = nullptr;
     d_ktab = nullptr;
     tmaps.clear();
+    xmaps.clear();
   }
 };
 
@@ -181,8 +197,9 @@ static int storage_of(int precision) {
   return precision == PCNN_BF16 ? ST_BF16 : ST_F32;
 }
 static int chunk_elems(int precision) {
-  // channel padding unit of stored activations: 16 B for tcgen05 chunks
-  return precision == PCNN_BF16 ? 8 : 4;
+  // channel padding unit of stored activations: 32 B, the narrowest TMA
+  // im2col slab of the tcgen05 path
+  return precision == PCNN_BF16 ? 16 : 8;
 }
 
 // Shape inference over the descriptor list (host only).  Fills in/out dims.
@@ -393,8 +410,8 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
   } else {
     const int Cg_log = in_c / groups;
     const int Cg_st = groups == 1 ? in_cs : Cg_log;
-    if (gs.engine == 1 && (Cg_st % ch)) return fail(PCNN_ERR_UNSUPPORTED,
-        "tcgen05 conv needs channels per group multiple of 16 bytes");
+    if (gs.engine == 1 && tc_slab_bytes(gs.st, Cg_st) == 0)
+      return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 conv needs channels per group multiple of 32 bytes");
     g.H = in_h;
     g.W = in_w;
     g.Cs = in_cs;
@@ -421,6 +438,9 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
       CUDA_TRY(cudaMemcpy(gs.d_ktab, tab.data(), sizeof(int) * g.K, cudaMemcpyHostToDevice));
     }
   }
+  (void)ch;
+  if (gs.engine == 1 && is_fc && tc_slab_bytes(gs.st, g.Cg) == 0)
+    return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 FC needs K multiple of 32 bytes");
   if (gs.engine == 1 && (g.Nfg % 8))
     return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 path needs N_f/g multiple of 8");
   g.relu = relu;
@@ -436,7 +456,8 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
   return PCNN_OK;
 }
 
-static const CUtensorMap *stage_tmap(GemmStage &gs, int bn) {
+static const CUtensorMap *stage_tmap(GemmStage &gs, int rows) {
+  const int bn = rows;
   auto it = gs.tmaps.find(bn);
   if (it != gs.tmaps.end()) return &it->second;
   auto enc = get_encode_tiled();
@@ -453,6 +474,38 @@ static const CUtensorMap *stage_tmap(GemmStage &gs, int bn) {
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return nullptr;
   return &(gs.tmaps[bn] = m);
+}
+
+// TMA im2col map of a stage's NHWC input for `batch` images.
+static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch) {
+  const auto key = std::make_pair(x, batch);
+  auto it = gs.xmaps.find(key);
+  if (it != gs.xmaps.end()) return &it->second;
+  auto enc = get_encode_im2col();
+  if (!enc) return nullptr;
+  const ConvGeom &g = gs.g;
+  const int esz = esz_of(gs.st);
+  const int slab = tc_slab_bytes(gs.st, g.Cg);
+  CUtensorMap m;
+  const cuuint64_t dims[4] = {(cuuint64_t)g.Cs, (cuuint64_t)g.W, (cuuint64_t)g.H,
+                              (cuuint64_t)batch};
+  const cuuint64_t strides[3] = {(cuuint64_t)g.Cs * esz, (cuuint64_t)g.W * g.Cs * esz,
+                                 (cuuint64_t)g.H * g.W * g.Cs * esz};
+  // bounding box of the conv's input corners (square kernels: W and H equal)
+  const int lower[2] = {-g.pad, -g.pad};
+  const int upper[2] = {g.pad - (g.S - 1), g.pad - (g.S - 1)};
+  const cuuint32_t estr[4] = {1, (cuuint32_t)g.stride, (cuuint32_t)g.stride, 1};
+  const CUtensorMapSwizzle sw = slab == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                : slab == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                             : CU_TENSOR_MAP_SWIZZLE_32B;
+  CUresult r = enc(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                        : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                   4, const_cast<void *>(x), dims, strides, lower, upper,
+                   (cuuint32_t)(slab / esz), 128, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return nullptr;
+  if (gs.xmaps.size() > 64) gs.xmaps.clear();
+  return &(gs.xmaps[key] = m);
 }
 
 // ------------------------------------------------------------------ planning
@@ -546,7 +599,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
     // the budget caps concurrent units; a CTA pair needs at least 2 SMs
     const int slots = std::max(1, effective_sms(net, ly) / p.cg);
     p.grid = p.cg * std::min(p.units, slots);
-    const CUtensorMap *tm = stage_tmap(gs, p.bn);
+    const CUtensorMap *tm = stage_tmap(gs, p.bn / p.cg);   // weight rows per CTA
     if (!tm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeTiled failed");
     if (info) {
       info->tile_m = 128 * p.cg;
@@ -560,11 +613,13 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
     }
     if (ws_need) *ws_need = std::max(*ws_need, p.splits > 1 ? (size_t)p.splits * g.M * g.out_cs * 4 : 0);
     if (!x) return PCNN_OK;   // planning only
+    const CUtensorMap *xm = stage_xmap(gs, x, B);
+    if (!xm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeIm2col failed");
     Budget b = make_budget(net, ly, slot, false);
     if (p.splits > 1 && (size_t)p.splits * g.M * g.out_cs * 4 > net->ws_bytes)
       return fail(PCNN_ERR_OUT_OF_MEMORY, "split-K workspace not reserved");
     g_launches += p.splits > 1 ? 1 : 0;   // the reduction kernel
-    CUDA_TRY(counted(launch_conv_tc(g, gs.st, x, tm, gs.d_bias, y, gs.d_ktab, p, net->d_ws,
+    CUDA_TRY(counted(launch_conv_tc(g, gs.st, xm, tm, gs.d_bias, y, gs.d_ktab, p, net->d_ws,
                                     b, s)));
   } else {
     const int tiles = conv_simt_tiles(g);
@@ -866,8 +921,8 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
     net->fuse_lrn_pool = !(e && e[0] == '1');
   }
   if (desc->precision != PCNN_FP32_SIMT) {
-    if (!get_encode_tiled())
-      return fail(PCNN_ERR_CUDA, "driver entry point cuTensorMapEncodeTiled unavailable");
+    if (!get_encode_tiled() || !get_encode_im2col())
+      return fail(PCNN_ERR_CUDA, "driver entry points cuTensorMapEncode{Tiled,Im2col} unavailable");
     CUDA_TRY(tc_init());
   }
 
