@@ -299,6 +299,9 @@ struct LrnPoolArgs {
   int Ho, Wo;
   int Q, nqt;              // output columns per tile, tiles per row
   int tf32_round;
+  int Cout;                // stored output channels
+  int ocg, ocp;            // output group layout: ocg real channels padded to
+                           // ocp per group (0 = compact, Cout == C)
   Budget b;
 };
 
@@ -372,25 +375,37 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
       }
       __syncthreads();
     }
-    // pool the staged (and normalised) rows
+    // pool the staged (and normalised) rows; output chunk oc maps to input
+    // chunk ch through the (optional) per-group channel padding
     const float inv = 1.f / (float)(a.k * a.k);
-    for (int v = threadIdx.x; v < (q1 - q0) * chunks; v += blockDim.x) {
-      const int ch = v % chunks, q = q0 + v / chunks;
-      const int cs = q * a.s - w0, ce = min(cs + a.k, wc);
+    const int ochunks = a.Cout / VN;
+    const int grp_real = a.ocg / VN, grp_pad = a.ocp / VN;
+    for (int v = threadIdx.x; v < (q1 - q0) * ochunks; v += blockDim.x) {
+      const int oc = v % ochunks, q = q0 + v / ochunks;
+      int ch = oc;
+      bool pad = false;
+      if (grp_pad > 0) {
+        const int gi = oc / grp_pad, j = oc % grp_pad;
+        pad = j >= grp_real;
+        ch = gi * grp_real + j;
+      }
       Vec16<ST> acc, cur;
 #pragma unroll
-      for (int j = 0; j < VN; ++j) acc.v[j] = a.is_max ? -INFINITY : 0.f;
-      for (int r = 0; r < nr; ++r)
-        for (int col = cs; col < ce; ++col) {
-          cur.load(U + (((size_t)r * wc_max + col) * C + ch * VN) * ESZ);
+      for (int j = 0; j < VN; ++j) acc.v[j] = pad ? 0.f : (a.is_max ? -INFINITY : 0.f);
+      if (!pad) {
+        const int cs = q * a.s - w0, ce = min(cs + a.k, wc);
+        for (int r = 0; r < nr; ++r)
+          for (int col = cs; col < ce; ++col) {
+            cur.load(U + (((size_t)r * wc_max + col) * C + ch * VN) * ESZ);
 #pragma unroll
-          for (int j = 0; j < VN; ++j)
-            acc.v[j] = a.is_max ? fmaxf(acc.v[j], cur.v[j]) : acc.v[j] + cur.v[j];
-        }
-      if (!a.is_max)
+            for (int j = 0; j < VN; ++j)
+              acc.v[j] = a.is_max ? fmaxf(acc.v[j], cur.v[j]) : acc.v[j] + cur.v[j];
+          }
+        if (!a.is_max)
 #pragma unroll
-        for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
-      acc.store((char *)a.y + ((((size_t)n * a.Ho + p) * a.Wo + q) * C + ch * VN) * ESZ,
+          for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
+      }
+      acc.store((char *)a.y + ((((size_t)n * a.Ho + p) * a.Wo + q) * a.Cout + oc * VN) * ESZ,
                 a.is_max ? 0 : a.tf32_round);
     }
   });
@@ -446,10 +461,14 @@ long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int
 
 cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int B, int H, int W,
                             int C, int lrn_size, float alpha, float beta, float kk, int k,
-                            int s, int is_max, int Ho, int Wo, const Budget &b, int grid,
-                            cudaStream_t stream) {
+                            int s, int is_max, int Ho, int Wo, int out_groups, int out_cg_pad,
+                            const Budget &b, int grid, cudaStream_t stream) {
   const int vn = st == ST_BF16 ? 8 : 4;
   if (C % vn) return cudaErrorInvalidValue;
+  const int ocg = out_groups > 0 ? C / out_groups : 0;
+  const int ocp = out_groups > 0 ? out_cg_pad : 0;
+  if (out_groups > 0 && (C % out_groups || ocg % vn || ocp % vn || ocp < ocg))
+    return cudaErrorInvalidValue;
   LrnPoolArgs a;
   a.x = x;
   a.y = y;
@@ -469,6 +488,9 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.Q = lrn_pool_cols(st, W, C, lrn_size > 0, k, s, Wo);
   a.nqt = (Wo + a.Q - 1) / a.Q;
   a.tf32_round = tf32_round;
+  a.ocg = ocg;
+  a.ocp = ocp;
+  a.Cout = out_groups > 0 ? out_groups * ocp : C;
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
   const size_t smem = (size_t)k * ((a.Q - 1) * s + k) * C * esz * (lrn_size > 0 ? 2 : 1);

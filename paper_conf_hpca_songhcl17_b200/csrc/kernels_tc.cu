@@ -30,6 +30,7 @@
 // CTA = 6 warps: warp 0 TMA producer, warp 1 TMEM allocator + MMA issuer,
 // warps 2..5 epilogue (TMEM lane quarter = warp % 4).
 #include <algorithm>
+#include <cstdlib>
 
 #include "budget.cuh"
 #include "pcnn_internal.h"
@@ -65,8 +66,11 @@ int tc_max_ktab() { return TC_MAX_KTAB; }
 int tc_block_k_elems(int st) { return st == ST_BF16 ? 64 : 32; }
 int tc_stages_for(int bn, int cg) {
   const int per = TC_A_STAGE + bn / cg * TC_ROW_BYTES;
-  const int n = TC_STAGE_BUDGET / per;
-  return n > TC_MAX_STAGES ? TC_MAX_STAGES : n;
+  int n = TC_STAGE_BUDGET / per;
+  if (n > TC_MAX_STAGES) n = TC_MAX_STAGES;
+  static const char *ov = getenv("PCNN_STAGES");     // tuning experiments only
+  if (ov && atoi(ov) >= 2 && atoi(ov) < n) n = atoi(ov);
+  return n;
 }
 
 // ------------------------------------------------------------ PTX wrappers
@@ -170,8 +174,12 @@ __device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
   return r;
 }
+// Remote arrive carrying no data dependency (only TMEM-read completion,
+// ordered by tcgen05.fence::before_thread_sync): relaxed is enough and avoids
+// a GPU-scope MEMBAR.
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr)
+  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(
+                   cluster_addr)
                : "memory");
 }
 // 2-SM TMA load: data lands in this CTA's smem, bytes are counted on the
@@ -218,6 +226,19 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
       : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
         "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]),
         "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
+        "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]),
+        "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]),
+        "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+        "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]),
+        "=r"(v[30]), "=r"(v[31])
       : "r"(taddr));
 }
 __device__ __forceinline__ void tmem_ld_wait() {
@@ -449,35 +470,43 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
       const bool mok = m < g.M;
       const size_t orow = (size_t)m * g.out_cs;
-      for (int c0 = 0; c0 < a.bn; c0 += 16) {
+      // bias is zero-padded on the device, so whole float4s can be read
+      for (int c0 = 0; c0 < a.bn; c0 += 32) {
         __syncwarp();
-        uint32_t v[16];
-        tmem_ld16(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0, v);
+        uint32_t v[32];
+        tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0, v);
         tmem_ld_wait();
         const int n = nt * a.bn + c0;          // column within the group
         if (mok && n < g.Nfg) {
           const int col = grp * g.Nfg + n;
-          float f[16];
+          float f[32];
 #pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            float x = __uint_as_float(v[i]);
-            if (!partial) {
-              if (a.bias && n + i < g.Nfg) x += __ldg(&a.bias[col + i]);
-              if (g.relu) x = fmaxf(x, 0.f);
+          for (int i = 0; i < 32; ++i) f[i] = __uint_as_float(v[i]);
+          if (!partial) {
+            const float4 *bp = (const float4 *)(a.bias + col);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              const float4 bb = __ldg(bp + q);
+              f[4 * q] += bb.x;
+              f[4 * q + 1] += bb.y;
+              f[4 * q + 2] += bb.z;
+              f[4 * q + 3] += bb.w;
             }
-            f[i] = x;
+            if (g.relu)
+#pragma unroll
+              for (int i = 0; i < 32; ++i) f[i] = fmaxf(f[i], 0.f);
           }
           if (partial) {
             float *yp = a.ws + (size_t)sp * g.M * g.out_cs + orow + col;
 #pragma unroll
-            for (int h = 0; h < 4; ++h)
+            for (int h = 0; h < 8; ++h)
               if (n + 4 * h < g.Nfg)
                 *(float4 *)(yp + 4 * h) =
                     make_float4(f[4 * h], f[4 * h + 1], f[4 * h + 2], f[4 * h + 3]);
           } else if (g.out_mode == OUT_BF16) {
             __nv_bfloat16 *yp = (__nv_bfloat16 *)a.y + orow + col;
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
+            for (int h = 0; h < 4; ++h) {
               if (n + 8 * h < g.Nfg) {
                 uint4 pk;
                 uint32_t *pw = (uint32_t *)&pk;
@@ -493,7 +522,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           } else {
             float *yp = (float *)a.y + orow + col;
 #pragma unroll
-            for (int h = 0; h < 4; ++h) {
+            for (int h = 0; h < 8; ++h) {
               if (n + 4 * h < g.Nfg) {
                 float4 q;
                 if (g.out_mode == OUT_F32_TF32) {
@@ -511,8 +540,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       tc_fence_before();
       __syncwarp();
       if (lane == 0) {
-        if constexpr (CG == 2) mbar_arrive_cluster(tempty_leader + 8 * buf);
-        else mbar_arrive(tempty_leader + 8 * buf);
+        if (CG == 2 && rank != 0) mbar_arrive_cluster(tempty_leader + 8 * buf);
+        else mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
       }
     }
   }

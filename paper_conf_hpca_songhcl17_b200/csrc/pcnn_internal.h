@@ -100,12 +100,15 @@ size_t tc_smem_bytes();
 int tc_max_ktab();
 
 // a4 / a5: LRN (lrn_size > 0) followed by pooling (k x k, stride s; k = s =
-// 1 for no pooling), NHWC with C stored channels.
+// 1 for no pooling), NHWC with C stored input channels.  out_groups > 0
+// writes the output with each of the out_groups channel groups padded to
+// out_cg_pad channels (zeros), the layout a following grouped conv loads
+// with full 128-byte TMA slabs.
 cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int B,
                             int H, int W, int C, int lrn_size, float alpha,
                             float beta, float kk, int k, int s, int is_max,
-                            int Ho, int Wo, const Budget &b, int grid,
-                            cudaStream_t stream);
+                            int Ho, int Wo, int out_groups, int out_cg_pad,
+                            const Budget &b, int grid, cudaStream_t stream);
 long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s,
                          int Ho, int Wo);
 int lrn_pool_occupancy(int st);

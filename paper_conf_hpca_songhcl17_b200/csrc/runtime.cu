@@ -133,6 +133,7 @@ struct Layer {
   std::vector<Svd> svd;        // per group (lazily computed)
   // budget
   int n_sms = 0, tlp = 0;
+  int out_groups = 0, out_cg_pad = 0;    // padded-group output layout (lrn/pool)
   unsigned long long *d_ctr = nullptr;   // 3 launch slots x (1 + kMaxSMs)
   unsigned int *d_census = nullptr;      // 8 words
 };
@@ -153,7 +154,7 @@ struct pcnn_net {
   int out_elems = 0;
   int occ_simt = 1, occ_lp = 1;
   // input staging geometry (space-to-depth by `blk` for a strided first conv)
-  int stage_h = 0, stage_w = 0, stage_blk = 1, stage_pad = 0;
+  int stage_h = 0, stage_w = 0, stage_blk = 1, stage_pad = 0, stage_c = 0;
   bool fuse_lrn_pool = true;
   bool census = false;
   // CUDA graph cache
@@ -409,7 +410,7 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
     packed = pack_fc(w, Nf, in_c, in_h, in_w, in_cs, g.Kpad);
   } else {
     const int Cg_log = in_c / groups;
-    const int Cg_st = groups == 1 ? in_cs : Cg_log;
+    const int Cg_st = in_cs / groups;      // stored (possibly padded) channels per group
     if (gs.engine == 1 && tc_slab_bytes(gs.st, Cg_st) == 0)
       return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 conv needs channels per group multiple of 32 bytes");
     g.H = in_h;
@@ -448,10 +449,12 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
   g.out_cs = Nf;
   pcnn_status st = upload_weights(gs, packed, precision);
   if (st != PCNN_OK) return st;
-  std::vector<float> b(Nf, 0.f);
+  // zero-padded so the epilogue can read whole 32-column slices unguarded
+  const size_t nb = (size_t)round_up(Nf, 256) + 256;
+  std::vector<float> b(nb, 0.f);
   if (bias) std::memcpy(b.data(), bias, sizeof(float) * Nf);
-  CUDA_TRY(cudaMalloc(&gs.d_bias, sizeof(float) * Nf));
-  CUDA_TRY(cudaMemcpy(gs.d_bias, b.data(), sizeof(float) * Nf, cudaMemcpyHostToDevice));
+  CUDA_TRY(cudaMalloc(&gs.d_bias, sizeof(float) * nb));
+  CUDA_TRY(cudaMemcpy(gs.d_bias, b.data(), sizeof(float) * nb, cudaMemcpyHostToDevice));
   (void)ly;
   return PCNN_OK;
 }
@@ -527,7 +530,7 @@ static constexpr double kOperandBytesPerCycle = 23.5;   // measured L2->SM feed 
 static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
   TcPlan best{};
   double best_t = 1e300;
-  const int nmax = std::min(256, round_up(g.Nfg, 16));
+  const int nmax = std::min(256, round_up(g.Nfg, 32));
   const double f = 1.9e9, hbm = 6.0e12;
   const double wbytes = (double)g.Nfg * g.groups * g.Kpad * esz;
   const char *force_cg = getenv("PCNN_FORCE_CG");
@@ -535,8 +538,7 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
     if (force_cg && atoi(force_cg) != cg) continue;
     const int mtiles = (g.M + 128 * cg - 1) / (128 * cg);
     const int slots = device_sms / cg;          // concurrent units
-    for (int bn = 16; bn <= nmax; bn += 16) {
-      if (cg == 2 && (bn / 2) % 8) continue;
+    for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {   // epilogue drains 32 columns
       const int ntiles = (g.Nfg + bn - 1) / bn;
       const long long tiles = (long long)mtiles * ntiles * g.groups;
       int splits = 1;
@@ -671,12 +673,16 @@ static pcnn_status run_lrn_pool(pcnn_net *net, int li, int pi, int B, const void
   }
   const long long tiles = lrn_pool_tiles(net->st, B, W, C, lrn > 0, k, st, Ho, Wo);
   const bool gated = is_gated(net, ly);
-  const int grid = gated ? net->num_sms * net->occ_lp : (int)std::min<long long>(tiles, 1 << 30);
+  // persistent: one wave of resident CTAs walks the tiles
+  const int grid = gated ? net->num_sms * net->occ_lp
+                         : (int)std::min<long long>(tiles, (long long)net->num_sms * net->occ_lp);
   Budget b = make_budget(net, ly, 0, true);
   if (b.gated)
     CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
+  const Layer &last = net->layers[pi >= 0 ? pi : li];
   CUDA_TRY(counted(launch_lrn_pool(x, y, net->st, net->desc.precision == PCNN_TF32, B, H, W, C,
-                                   lrn, alpha, beta, kk, k, st, is_max, Ho, Wo, b, grid, s)));
+                                   lrn, alpha, beta, kk, k, st, is_max, Ho, Wo, last.out_groups,
+                                   last.out_cg_pad, b, grid, s)));
   return PCNN_OK;
 }
 
@@ -929,6 +935,26 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   const int prec = desc->precision;
   const int esz = esz_of(net->st);
   const int B = desc->max_batch;
+  // TMA slab alignment: a grouped conv whose channels per group are not a
+  // multiple of 128 bytes reads its input with narrow (SW64/SW32) slabs.  When
+  // its producer is an LRN / pooling layer, that producer writes each group
+  // padded to a multiple of 128 bytes instead (zeros; packed weights are zero
+  // there too), so the conv loads full SW128 slabs.
+  const int slab128 = 128 / esz;
+  if (prec != PCNN_FP32_SIMT) {
+    for (int i = 1; i < n_layers; ++i) {
+      Layer &ly = net->layers[i];
+      Layer &pv = net->layers[i - 1];
+      if (ly.d.kind != PCNN_CONV || ly.d.groups <= 1) continue;
+      const int cg = ly.in_c / ly.d.groups;
+      if ((cg % slab128) == 0 || ly.in_cs != ly.in_c) continue;
+      if (pv.d.kind != PCNN_MAXPOOL && pv.d.kind != PCNN_AVGPOOL && pv.d.kind != PCNN_LRN) continue;
+      pv.out_groups = ly.d.groups;
+      pv.out_cg_pad = round_up(cg, slab128);
+      pv.out_cs = ly.d.groups * pv.out_cg_pad;
+      ly.in_cs = pv.out_cs;
+    }
+  }
   // Space-to-depth for a strided first conv (layout transform of a1): the
   // conv S x S / st on C channels becomes ceil(S/st) x ceil(S/st) / 1 on
   // st^2 C channels over an (Ho - 1 + S') x (Wo - 1 + S') grid whose origin
@@ -942,9 +968,10 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
     const int C = desc->in_channels, Cp = st2 * st2 * C, F = l0.d.out_channels;
     net->stage_blk = st2;
     net->stage_pad = l0.d.pad;
+    net->stage_c = Cp;
     net->stage_h = l0.out_h - 1 + Sp;
     net->stage_w = l0.out_w - 1 + Sp;
-    net->in_cs = round_up(Cp, chunk_elems(prec));
+    net->in_cs = round_up(Cp, prec == PCNN_FP32_SIMT ? chunk_elems(prec) : slab128);
     s2d_w.assign((size_t)F * Cp * Sp * Sp, 0.f);
     for (int f = 0; f < F; ++f)
       for (int c = 0; c < C; ++c)
@@ -969,7 +996,7 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
       if (i == 0 && net->stage_blk > 1) {
         const int Sp = (ly.d.kernel + net->stage_blk - 1) / net->stage_blk;
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, 1, Sp, 1, 0, ly.d.relu,
-                        net->in_cs, net->stage_h, net->stage_w, net->in_cs, false,
+                        net->stage_c, net->stage_h, net->stage_w, net->in_cs, false,
                         s2d_w.data(), biases ? biases[i] : nullptr, mode);
       } else {
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, is_fc ? 1 : ly.d.groups,
