@@ -347,6 +347,8 @@ def main():
         else:
             d["gbs"] = round(f["bytes"] / (lm / 1000) / 1e9, 1) if lm > 0 else None
         per_layer.append(d)
+    per_layer.append({"layer": "staging+softmax+unstage",
+                      "ms": round(total_step_ms - sum(layer_ms) / max(nsteps, 1), 5)})
 
     res = {
         "metric": METRIC,

@@ -327,14 +327,19 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
     const int w0 = q0 * a.s, w1 = min((q1 - 1) * a.s + a.k, a.W);
     const int nr = h1 - h0, wc = w1 - w0;
     __syncthreads();
-    // stage rows [h0, h1) x cols [w0, w1): each row segment is contiguous
+    // stage rows [h0, h1) x cols [w0, w1): each row segment is contiguous;
+    // cp.async keeps every 16 B load of the tile in flight at once
     const int vec_per_row = wc * chunks;
+    const uint32_t tbase = (uint32_t)__cvta_generic_to_shared(T);
     for (int v = threadIdx.x; v < nr * vec_per_row; v += blockDim.x) {
       const int r = v / vec_per_row, rem = v - r * vec_per_row;
       const size_t src = (((size_t)n * a.H + h0 + r) * a.W + w0) * C + (size_t)rem * VN;
-      *(uint4 *)(T + ((size_t)r * wc_max * C + (size_t)rem * VN) * ESZ) =
-          __ldg((const uint4 *)((const char *)a.x + src * ESZ));
+      const uint32_t dst = tbase + (uint32_t)(((size_t)r * wc_max * C + (size_t)rem * VN) * ESZ);
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst),
+                   "l"((const char *)a.x + src * ESZ)
+                   : "memory");
     }
+    asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
     __syncthreads();
     if (LS > 0) {
       // each thread: one 16 B channel chunk of one staged pixel; the window

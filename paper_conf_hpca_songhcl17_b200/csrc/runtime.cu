@@ -514,18 +514,20 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch) {
 // ------------------------------------------------------------------ planning
 // Tile / split selection (the paper's sub-matrix choice, P:223,
 // P:267).  For every CTA grouping cg (1 CTA, M = 128 / CTA pair, M = 256) and
-// N tile bn (multiple of 16, <= 256):
+// N tile bn (multiple of 32, <= 256):
 //   tiles  = ceil(M / (128 cg)) * ceil(Nfg / bn) * groups       (eq. 4)
-//   splits = K split when the tiles cannot fill half the GPU
-//   K-block cost (cycles, per SM) = max(MMA 2.05 bn, operand bytes per SM /
-//            kOperandBytesPerCycle) + 40
+//   splits = K split when the tiles cannot fill the GPU
+//   K-block cost per SM (cycles) = max(MMA ~2.05 bn,
+//                                      TMA ~3.6 per 128-B box row x (128 + bn/cg))
 //   time   = max(waves * kblocks/splits * cost / f, weight bytes / HBM)
 //            + split-K reduction traffic
-// Small tiles raise Util (eq. 6) and rEC (eq. 9), big tiles raise the
-// computation density per operand byte -- the trade-off of P:223.  The plan
-// depends on the problem shape and the device's SM count only, never on the
-// SM budget, so every budget runs the same tiles and K order (R11).
-static constexpr double kOperandBytesPerCycle = 23.5;   // measured L2->SM feed per SM
+// (the per-row TMA cost is the measured rate of this kernel on B200; the MMA
+// figure is the tcgen05 floor).  Small tiles raise Util (eq. 6) and rEC
+// (eq. 9), big tiles raise the computation density per loaded row -- the
+// trade-off of P:223.  The plan depends on the problem shape and the device's
+// SM count only, never on the SM budget, so every budget runs the same tiles
+// and K order (bitwise-identical results, R11).
+static constexpr double kTmaCyclesPerRow = 3.6;
 
 static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
   TcPlan best{};
@@ -541,30 +543,31 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
     for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {   // epilogue drains 32 columns
       const int ntiles = (g.Nfg + bn - 1) / bn;
       const long long tiles = (long long)mtiles * ntiles * g.groups;
-      int splits = 1;
-      if (tiles * 2 < slots && kblocks >= 8) {
-        splits = (int)std::min<long long>((slots + tiles - 1) / tiles, 16);
-        splits = std::max(1, std::min(splits, kblocks / 4));
-      }
-      const int kbs = (kblocks + splits - 1) / splits;
-      splits = (kblocks + kbs - 1) / kbs;
-      const long long units = tiles * splits;
-      const long long waves = (units + slots - 1) / slots;
-      const double bytes_sm = 128.0 * 128 + (double)bn / cg * 128;   // A + B per SM per K-block
-      const double kb_cycles = std::max(2.05 * bn, bytes_sm / kOperandBytesPerCycle) + 40.0;
-      double t = (double)waves * kbs * kb_cycles / f;
-      t = std::max(t, wbytes / hbm);
-      if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
-      if (t < best_t * 0.999 || (t <= best_t * 1.001 && bn * cg > best.bn * best.cg)) {
-        best_t = t;
-        best.cg = cg;
-        best.bn = bn;
-        best.mtiles = mtiles;
-        best.ntiles = ntiles;
-        best.tiles = (int)tiles;
-        best.splits = splits;
-        best.kb_per_split = kbs;
-        best.units = (int)units;
+      const double kb_cycles =
+          std::max(2.05 * bn, kTmaCyclesPerRow * (128.0 + (double)bn / cg)) + 40.0;
+      // split-K candidates: none, or any split that keeps >= 4 K-blocks per unit
+      const int max_split = tiles >= slots ? 1 : std::min(16, std::max(1, kblocks / 4));
+      for (int want = 1; want <= max_split; ++want) {
+        const int kbs = (kblocks + want - 1) / want;
+        const int splits = (kblocks + kbs - 1) / kbs;
+        if (splits != want) continue;
+        const long long units = tiles * splits;
+        const long long waves = (units + slots - 1) / slots;
+        double t = (double)waves * kbs * kb_cycles / f + 2e-6;   // + per-tile drain
+        t = std::max(t, wbytes / hbm);
+        if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
+        if (t < best_t * 0.999 ||
+            (t <= best_t * 1.001 && (long long)bn * cg > (long long)best.bn * best.cg)) {
+          best_t = t;
+          best.cg = cg;
+          best.bn = bn;
+          best.mtiles = mtiles;
+          best.ntiles = ntiles;
+          best.tiles = (int)tiles;
+          best.splits = splits;
+          best.kb_per_split = kbs;
+          best.units = (int)units;
+        }
       }
     }
   }
@@ -673,9 +676,7 @@ static pcnn_status run_lrn_pool(pcnn_net *net, int li, int pi, int B, const void
   }
   const long long tiles = lrn_pool_tiles(net->st, B, W, C, lrn > 0, k, st, Ho, Wo);
   const bool gated = is_gated(net, ly);
-  // persistent: one wave of resident CTAs walks the tiles
-  const int grid = gated ? net->num_sms * net->occ_lp
-                         : (int)std::min<long long>(tiles, (long long)net->num_sms * net->occ_lp);
+  const int grid = gated ? net->num_sms * net->occ_lp : (int)std::min<long long>(tiles, 1 << 30);
   Budget b = make_budget(net, ly, 0, true);
   if (b.gated)
     CUDA_TRY(cudaMemsetAsync(b.ctr, 0, sizeof(unsigned long long) * (1 + kMaxSMs), s));
