@@ -109,9 +109,62 @@ stage_input_kernel(const float *__restrict__ x, void *y, int B, int C, int H, in
   }
 }
 
+// Row-staged variant: one CTA per (image, output row).  The blk input rows
+// x C channels it needs are loaded into smem with coalesced (consecutive-W)
+// reads, then every (pixel, 16 B chunk) of the output row is assembled from
+// smem and stored coalesced.  Used when those rows fit in 48 KB.
+template <int ST>
+__global__ void __launch_bounds__(256)
+stage_rows_kernel(const float *__restrict__ x, void *y, int C, int H, int W, int Hs, int Ws,
+                  int Cs, int blk, int pad, int tf32_round) {
+  extern __shared__ float rows[];                  // [blk][C][W]
+  constexpr int VN = Vec16<ST>::N;
+  const int hs = blockIdx.x % Hs;
+  const long long n = blockIdx.x / Hs;
+  const long long HW = (long long)H * W;
+  const int nrow = blk * C;
+  for (int i = threadIdx.x; i < nrow * W; i += blockDim.x) {
+    const int rc = i / W, w = i - rc * W;          // rc = dr * C + c
+    const int dr = rc / C, c = rc - dr * C;
+    const int ih = hs * blk - pad + dr;
+    rows[i] = (ih >= 0 && ih < H) ? __ldg(&x[(n * C + c) * HW + (long long)ih * W + w]) : 0.f;
+  }
+  __syncthreads();
+  const int chunks = Cs / VN;
+  const int creal = blk * blk * C;
+  char *yrow = (char *)y + ((size_t)(n * Hs + hs) * Ws) * Cs * (ST == ST_BF16 ? 2 : 4);
+  for (int i = threadIdx.x; i < Ws * chunks; i += blockDim.x) {
+    const int ws = i / chunks, ch = i - ws * chunks;
+    Vec16<ST> o;
+#pragma unroll
+    for (int j = 0; j < VN; ++j) {
+      const int cp = ch * VN + j;
+      float v = 0.f;
+      if (cp < creal) {
+        const int b = cp / C, c = cp - b * C;
+        const int dr = b / blk, iw = ws * blk - pad + b % blk;
+        if (iw >= 0 && iw < W) v = rows[(dr * C + c) * W + iw];
+      }
+      o.v[j] = v;
+    }
+    o.store(yrow + (size_t)i * 16, tf32_round);
+  }
+}
+
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
                                int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {
+  const size_t rows_bytes = (size_t)blk * C * W * sizeof(float);
+  if (rows_bytes <= 48 * 1024) {
+    const long long grid = (long long)B * Hs;
+    if (st == ST_BF16)
+      stage_rows_kernel<ST_BF16><<<(unsigned)grid, 256, rows_bytes, s>>>(x, y, C, H, W, Hs, Ws,
+                                                                          Cs, blk, pad, 0);
+    else
+      stage_rows_kernel<ST_F32><<<(unsigned)grid, 256, rows_bytes, s>>>(x, y, C, H, W, Hs, Ws,
+                                                                         Cs, blk, pad, tf32_round);
+    return cudaGetLastError();
+  }
   const int vn = st == ST_BF16 ? 8 : 4;
   const long long total = (long long)B * Hs * Ws * (Cs / vn);
   const int grid = (int)std::max<long long>(1, std::min<long long>((total + 255) / 256, 148 * 16));

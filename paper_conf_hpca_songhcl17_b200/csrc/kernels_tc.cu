@@ -286,8 +286,85 @@ struct TcArgs {
   int kblocks, kb_per_split;
   int stages;
   int slab_bytes;       // 128 / 64 / 32: A K-block = 128 / slab_bytes TMA slabs
+  int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
+  float lrn_a_over_n, lrn_beta, lrn_k;
   Budget b;
 };
+
+// Epilogue with the following LRN layer fused in (R3; Caffe size
+// 5).  The tile holds every channel of its pixels (bn == Nfg <= 128, one N
+// tile), so each thread normalises its own pixel's channel vector in
+// registers: bias, ReLU, rounding to the storage precision, then exactly the
+// stand-alone LRN kernel's arithmetic (same sum order and transcendental
+// form), so the result is bitwise identical to conv -> store -> LRN.
+template <int ST>
+__device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bool mok,
+                                             size_t orow) {
+  const ConvGeom &g = a.g;
+  constexpr int MAXC = 128;
+  float f[MAXC];
+#pragma unroll
+  for (int c0 = 0; c0 < MAXC; c0 += 32) {
+    if (c0 < a.bn) {                       // warp-uniform
+      uint32_t v[32];
+      tmem_ld32(taddr + c0, v);
+      tmem_ld_wait();
+#pragma unroll
+      for (int i = 0; i < 32; ++i) f[c0 + i] = __uint_as_float(v[i]);
+    }
+  }
+  if (!mok) return;
+  const int C = g.Nfg;
+#pragma unroll
+  for (int i = 0; i < MAXC; ++i) {
+    float x = f[i] + __ldg(&a.bias[i]);
+    if (g.relu) x = fmaxf(x, 0.f);
+    // the value the stand-alone conv would have stored
+    if constexpr (ST == ST_BF16) x = __bfloat162float(__float2bfloat16_rn(x));
+    else if (g.out_mode == OUT_F32_TF32) x = tf32_rna_tc(x);
+    f[i] = i < C ? x : 0.f;
+  }
+  float sq[MAXC + 4];
+  sq[0] = sq[1] = sq[MAXC + 2] = sq[MAXC + 3] = 0.f;
+#pragma unroll
+  for (int i = 0; i < MAXC; ++i) sq[i + 2] = f[i] * f[i];
+#pragma unroll
+  for (int c0 = 0; c0 < MAXC; c0 += 8) {
+    if (c0 < C) {
+      float o[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        float acc = 0.f;
+#pragma unroll
+        for (int w = 0; w < 5; ++w) acc += sq[c0 + j + w];
+        const float scale = a.lrn_k + a.lrn_a_over_n * acc;
+        o[j] = f[c0 + j] * exp2f(-a.lrn_beta * __log2f(scale));
+      }
+      if constexpr (ST == ST_BF16) {
+        uint4 pk;
+        uint32_t *pw = (uint32_t *)&pk;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          __nv_bfloat162 b2 = __floats2bfloat162_rn(o[2 * i], o[2 * i + 1]);
+          pw[i] = *(uint32_t *)&b2;
+        }
+        *(uint4 *)((__nv_bfloat16 *)a.y + orow + c0) = pk;
+      } else {
+        float *yp = (float *)a.y + orow + c0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          float4 q;
+          if (g.out_mode == OUT_F32_TF32)
+            q = make_float4(tf32_rna_tc(o[4 * h]), tf32_rna_tc(o[4 * h + 1]),
+                            tf32_rna_tc(o[4 * h + 2]), tf32_rna_tc(o[4 * h + 3]));
+          else
+            q = make_float4(o[4 * h], o[4 * h + 1], o[4 * h + 2], o[4 * h + 3]);
+          *(float4 *)(yp + 4 * h) = q;
+        }
+      }
+    }
+  }
+}
 
 __device__ __forceinline__ void advance(uint32_t &stage, uint32_t &phase, int stages) {
   if (++stage == (uint32_t)stages) {
@@ -470,6 +547,17 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
       const bool mok = m < g.M;
       const size_t orow = (size_t)m * g.out_cs;
+      if (a.lrn) {
+        epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX, mok,
+                         orow);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          if (CG == 2 && rank != 0) mbar_arrive_cluster(tempty_leader + 8 * buf);
+          else mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
+        }
+        continue;
+      }
       // bias is zero-padded on the device, so whole float4s can be read
       for (int c0 = 0; c0 < a.bn; c0 += 32) {
         __syncwarp();
@@ -637,8 +725,19 @@ static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias, void *y,
                            const int *ktab, const TcPlan &p, float *ws, const Budget &b,
-                           cudaStream_t s) {
+                           cudaStream_t s, const float *lrn) {
   TcArgs args;
+  args.lrn = 0;
+  args.lrn_a_over_n = args.lrn_beta = args.lrn_k = 0.f;
+  if (lrn) {   // {size, alpha, beta, k}: size 5 only, one N tile with every channel
+    if (lrn[0] != 5.f || p.ntiles != 1 || g.groups != 1 || p.splits != 1 || g.Nfg > 128 ||
+        p.bn != ((g.Nfg + 31) / 32) * 32)
+      return cudaErrorInvalidValue;
+    args.lrn = 1;
+    args.lrn_a_over_n = lrn[1] / lrn[0];
+    args.lrn_beta = lrn[2];
+    args.lrn_k = lrn[3];
+  }
   args.g = g;
   args.y = y;
   args.ws = ws;

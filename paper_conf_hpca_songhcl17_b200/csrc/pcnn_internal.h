@@ -89,7 +89,9 @@ struct TcPlan {
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias,
                            void *y, const int *ktab, const TcPlan &p, float *ws,
-                           const Budget &b, cudaStream_t s);
+                           const Budget &b, cudaStream_t s, const float *lrn = nullptr);
+// lrn (optional) = {size, alpha, beta, k} of a following LRN layer fused into
+// the epilogue (size 5, one N tile holding all channels, no split-K).
 // A-slab width in bytes (128 / 64 / 32) for Cg channels per group, 0 if the
 // group width is not a multiple of 32 bytes.
 int tc_slab_bytes(int st, int cg_channels);

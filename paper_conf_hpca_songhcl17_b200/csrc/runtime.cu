@@ -529,7 +529,8 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch) {
 // and K order (bitwise-identical results, R11).
 static constexpr double kTmaCyclesPerRow = 3.6;
 
-static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
+static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
+                      bool full_n = false) {
   TcPlan best{};
   double best_t = 1e300;
   const int nmax = std::min(256, round_up(g.Nfg, 32));
@@ -541,12 +542,14 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz) {
     const int mtiles = (g.M + 128 * cg - 1) / (128 * cg);
     const int slots = device_sms / cg;          // concurrent units
     for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {   // epilogue drains 32 columns
+      if (full_n && bn != round_up(g.Nfg, 32)) continue;      // one N tile (fused LRN)
       const int ntiles = (g.Nfg + bn - 1) / bn;
       const long long tiles = (long long)mtiles * ntiles * g.groups;
       const double kb_cycles =
           std::max(2.05 * bn, kTmaCyclesPerRow * (128.0 + (double)bn / cg)) + 40.0;
       // split-K candidates: none, or any split that keeps >= 4 K-blocks per unit
-      const int max_split = tiles >= slots ? 1 : std::min(16, std::max(1, kblocks / 4));
+      const int max_split =
+          (tiles >= slots || full_n) ? 1 : std::min(16, std::max(1, kblocks / 4));
       for (int want = 1; want <= max_split; ++want) {
         const int kbs = (kblocks + want - 1) / want;
         const int splits = (kblocks + kbs - 1) / kbs;
@@ -596,11 +599,12 @@ static Budget make_budget(const pcnn_net *net, const Layer &ly, int slot, bool g
 // ------------------------------------------------------------------ enqueue
 static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, const void *x,
                              void *y, int slot, cudaStream_t s, pcnn_layer_info *info,
-                             size_t *ws_need = nullptr) {
+                             size_t *ws_need = nullptr, const float *lrn = nullptr) {
   ConvGeom g = gs.g;
   g.M = B * g.Ho * g.Wo;
   if (gs.engine == 1) {
-    TcPlan p = plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st));
+    TcPlan p = plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st),
+                       lrn != nullptr);
     // the budget caps concurrent units; a CTA pair needs at least 2 SMs
     const int slots = std::max(1, effective_sms(net, ly) / p.cg);
     p.grid = p.cg * std::min(p.units, slots);
@@ -625,7 +629,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       return fail(PCNN_ERR_OUT_OF_MEMORY, "split-K workspace not reserved");
     g_launches += p.splits > 1 ? 1 : 0;   // the reduction kernel
     CUDA_TRY(counted(launch_conv_tc(g, gs.st, xm, tm, gs.d_bias, y, gs.d_ktab, p, net->d_ws,
-                                    b, s)));
+                                    b, s, lrn)));
   } else {
     const int tiles = conv_simt_tiles(g);
     const bool gated = is_gated(net, ly);
@@ -649,6 +653,24 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
                               (float *)y, gs.d_ktab, b, grid, s)));
   }
   return PCNN_OK;
+}
+
+// conv layer i immediately followed by a size-5 LRN that the conv epilogue can
+// apply in registers: tcgen05 engine, exact variant, one group, every output
+// channel in one N tile (<= 128).
+static bool fuse_conv_lrn(const pcnn_net *net, int i) {
+  if (!net->fuse_lrn_pool || i + 1 >= (int)net->layers.size()) return false;
+  const Layer &c = net->layers[i], &l = net->layers[i + 1];
+  return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 &&
+         c.exact.engine == 1 && c.variant == PCNN_VARIANT_EXACT && c.d.groups == 1 &&
+         c.d.out_channels <= 128 && c.out_cs == c.d.out_channels;
+}
+
+static void lrn_params(const Layer &l, float p[4]) {
+  p[0] = (float)l.d.kernel;
+  p[1] = l.d.lrn_alpha;
+  p[2] = l.d.lrn_beta;
+  p[3] = l.d.lrn_k;
 }
 
 // LRN layer `li` and / or pooling layer `pi` (-1 = absent) in one launch
@@ -733,6 +755,21 @@ static pcnn_status enqueue_all(pcnn_net *net, const float *d_images, int B, floa
   for (int i = 0; i < n; ++i) {
     const bool final_fc = (i == n - 1) && last_is_fc(net);
     void *dst = final_fc ? (void *)d_out : net->d_act[cur ^ 1];
+    if (fuse_conv_lrn(net, i)) {          // conv + LRN in one launch
+      float lp[4];
+      lrn_params(net->layers[i + 1], lp);
+      Layer &ly = net->layers[i];
+      pcnn_status r = run_stage(net, ly, ly.exact, B, net->d_act[cur], dst, 0, s, nullptr,
+                                nullptr, lp);
+      if (r != PCNN_OK) return r;
+      if (evs) {
+        CUDA_TRY(cudaEventRecord((*evs)[i + 1], s));
+        CUDA_TRY(cudaEventRecord((*evs)[i + 2], s));
+      }
+      cur ^= 1;
+      ++i;
+      continue;
+    }
     if (net->fuse_lrn_pool && net->layers[i].d.kind == PCNN_LRN && i + 1 < n &&
         (net->layers[i + 1].d.kind == PCNN_MAXPOOL || net->layers[i + 1].d.kind == PCNN_AVGPOOL)) {
       pcnn_status r = run_lrn_pool(net, i, i + 1, B, net->d_act[cur], dst, s);
@@ -1165,8 +1202,11 @@ pcnn_status pcnn_query_layer(const pcnn_net *cnet, int layer, int batch, pcnn_la
     f->gemm_n = ly.exact.g.Nfg;
     f->gemm_k = ly.d.kind == PCNN_CONV ? ly.d.kernel * ly.d.kernel * (ly.in_c / ly.d.groups)
                                        : ly.in_c * ly.in_h * ly.in_w;
+    float lp[4];
+    const bool fl = fuse_conv_lrn(net, layer);
+    if (fl) lrn_params(net->layers[layer + 1], lp);
     pcnn_status s = run_stage(net, ly, ly.variant == PCNN_VARIANT_RANK ? ly.r2 : ly.exact,
-                              batch, nullptr, nullptr, 0, nullptr, f);
+                              batch, nullptr, nullptr, 0, nullptr, f, nullptr, fl ? lp : nullptr);
     if (s != PCNN_OK) return s;
     const long long maxb = (long long)f->n_sms * std::max(f->tlp, 1);
     const long long waves = (f->tiles + maxb - 1) / maxb;

@@ -205,3 +205,23 @@ def test_space_to_depth_first_conv(orc, prec, monkeypatch):
     plain = gpu_run(net, w, b, x, prec)["out"]
     assert rel_err(s2d, ref) <= TOL[prec] / 4
     assert rel_err(plain, ref) <= TOL[prec] / 4
+
+
+@pytest.mark.parametrize("prec", ["tf32", "bf16"])
+def test_conv_lrn_epilogue_fusion(orc, prec, monkeypatch):
+    """conv -> LRN fused in the tcgen05 epilogue (AlexNet conv1 + norm1 shape,
+    smaller image): agrees with the stand-alone LRN kernel path and the oracle."""
+    net = dict(in_shape=(3, 67, 67), layers=[
+        conv_layer(96, 11, 3, 4, 0, 1, relu=True),
+        dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0),
+        dict(kind="maxpool", k=3, stride=2)])
+    w, b = params(net, seed=21)
+    x = small_inputs((3, 67, 67), 2, lo=-128, hi=128)
+    ref = orc.run_net(net, w, b, x).reshape(2, -1)
+    fused = gpu_run(net, w, b, x, prec)["out"]
+    monkeypatch.setenv("PCNN_NO_FUSE", "1")
+    plain = gpu_run(net, w, b, x, prec)["out"]
+    assert rel_err(fused, ref) <= TOL[prec] / 4
+    assert rel_err(plain, ref) <= TOL[prec] / 4
+    # same arithmetic, same roundings: at most a last-place difference
+    assert rel_err(fused, plain) <= 1e-6 if prec == "tf32" else rel_err(fused, plain) <= 8e-3
