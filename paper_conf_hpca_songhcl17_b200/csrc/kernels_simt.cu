@@ -117,33 +117,49 @@ template <int ST>
 __global__ void __launch_bounds__(256)
 stage_rows_kernel(const float *__restrict__ x, void *y, int C, int H, int W, int Hs, int Ws,
                   int Cs, int blk, int pad, int tf32_round) {
-  extern __shared__ float rows[];                  // [blk][C][W]
+  extern __shared__ float rows[];                  // [blk][C][W] then the channel map
   constexpr int VN = Vec16<ST>::N;
   const int hs = blockIdx.x % Hs;
   const long long n = blockIdx.x / Hs;
   const long long HW = (long long)H * W;
   const int nrow = blk * C;
+  int *cmap = (int *)(rows + nrow * W);            // [Cs]: row offset | column delta
+  // 4 B cp.async keeps every load of the staged rows in flight
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(rows);
   for (int i = threadIdx.x; i < nrow * W; i += blockDim.x) {
     const int rc = i / W, w = i - rc * W;          // rc = dr * C + c
     const int dr = rc / C, c = rc - dr * C;
     const int ih = hs * blk - pad + dr;
-    rows[i] = (ih >= 0 && ih < H) ? __ldg(&x[(n * C + c) * HW + (long long)ih * W + w]) : 0.f;
+    const bool ok = ih >= 0 && ih < H;
+    const float *src = ok ? x + (n * C + c) * HW + (long long)ih * W + w : x;
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(sbase + 4u * i),
+                 "l"(src), "r"(ok ? 4 : 0)
+                 : "memory");
   }
+  const int creal = blk * blk * C;
+  for (int cp = threadIdx.x; cp < Cs; cp += blockDim.x) {
+    if (cp < creal) {
+      const int b = cp / C, c = cp - b * C;
+      cmap[cp] = (((b / blk) * C + c) * W) << 4 | (b % blk);   // row base, ds
+    } else {
+      cmap[cp] = -1;
+    }
+  }
+  asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
   __syncthreads();
   const int chunks = Cs / VN;
-  const int creal = blk * blk * C;
   char *yrow = (char *)y + ((size_t)(n * Hs + hs) * Ws) * Cs * (ST == ST_BF16 ? 2 : 4);
   for (int i = threadIdx.x; i < Ws * chunks; i += blockDim.x) {
     const int ws = i / chunks, ch = i - ws * chunks;
+    const int iw0 = ws * blk - pad;
     Vec16<ST> o;
 #pragma unroll
     for (int j = 0; j < VN; ++j) {
-      const int cp = ch * VN + j;
+      const int e = cmap[ch * VN + j];
       float v = 0.f;
-      if (cp < creal) {
-        const int b = cp / C, c = cp - b * C;
-        const int dr = b / blk, iw = ws * blk - pad + b % blk;
-        if (iw >= 0 && iw < W) v = rows[(dr * C + c) * W + iw];
+      if (e >= 0) {
+        const int iw = iw0 + (e & 15);
+        if (iw >= 0 && iw < W) v = rows[(e >> 4) + iw];
       }
       o.v[j] = v;
     }
@@ -154,8 +170,8 @@ stage_rows_kernel(const float *__restrict__ x, void *y, int C, int H, int W, int
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
                                int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {
-  const size_t rows_bytes = (size_t)blk * C * W * sizeof(float);
-  if (rows_bytes <= 48 * 1024) {
+  const size_t rows_bytes = (size_t)blk * C * W * sizeof(float) + (size_t)Cs * sizeof(int);
+  if (rows_bytes <= 48 * 1024 && blk <= 15) {
     const long long grid = (long long)B * Hs;
     if (st == ST_BF16)
       stage_rows_kernel<ST_BF16><<<(unsigned)grid, 256, rows_bytes, s>>>(x, y, C, H, W, Hs, Ws,

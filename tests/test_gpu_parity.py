@@ -223,5 +223,5 @@ def test_conv_lrn_epilogue_fusion(orc, prec, monkeypatch):
     plain = gpu_run(net, w, b, x, prec)["out"]
     assert rel_err(fused, ref) <= TOL[prec] / 4
     assert rel_err(plain, ref) <= TOL[prec] / 4
-    # same arithmetic, same roundings: at most a last-place difference
-    assert rel_err(fused, plain) <= 1e-6 if prec == "tf32" else rel_err(fused, plain) <= 8e-3
+    # same arithmetic and roundings up to FMA contraction: last-place differences
+    assert rel_err(fused, plain) <= (2e-3 if prec == "tf32" else 8e-3)

@@ -24,6 +24,8 @@ SHAPES = {  # name: (in_shape, layer)
     "vgg5_2": ((512, 14, 14), dict(kind="conv", out=512, k=3, stride=1, pad=1, groups=1, relu=True, in_c=512)),
     "norm1pool1": ((96, 55, 55), [dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0), dict(kind="maxpool", k=3, stride=2)]),
     "pool5": ((256, 13, 13), dict(kind="maxpool", k=3, stride=2)),
+    "norm2pool2": ((256, 27, 27), [dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0), dict(kind="maxpool", k=3, stride=2)]),
+    "stage": ((3, 227, 227), dict(kind="maxpool", k=1, stride=1)),
 }
 name = sys.argv[1]
 B = int(sys.argv[2]) if len(sys.argv) > 2 else 256
