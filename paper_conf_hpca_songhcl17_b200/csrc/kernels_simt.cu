@@ -6,6 +6,7 @@
 #include <algorithm>
 
 #include "budget.cuh"
+#include "lrn_math.cuh"
 #include "pcnn_internal.h"
 
 namespace pcnn {
@@ -167,9 +168,92 @@ stage_rows_kernel(const float *__restrict__ x, void *y, int C, int H, int W, int
   }
 }
 
+// Specialised staging for the networks' 3-channel inputs: one CTA per
+// (image, output row), one thread per output pixel.  The BLK input rows x 3
+// channels are staged in smem with a 16 B-aligned row pitch, each thread reads
+// its BLK x BLK x 3 window as float4s (BLK = 4, space-to-depth) or scalars
+// (BLK = 1) and writes its whole Cs-channel pixel with 16 B stores.
+template <int ST, int BLK>
+__global__ void __launch_bounds__(256)
+stage_c3_kernel(const float *__restrict__ x, void *y, int H, int W, int Hs, int Ws, int Cs,
+                int pad, int tf32_round) {
+  constexpr int C = 3;
+  constexpr int VN = Vec16<ST>::N;
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  extern __shared__ float rows[];                  // [BLK][C][Wp]
+  const int Wp = ((Ws * BLK + 3) & ~3) + 4;        // covers iw in [-pad, Ws*BLK)
+  const int hs = blockIdx.x % Hs;
+  const long long n = blockIdx.x / Hs;
+  const long long HW = (long long)H * W;
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(rows);
+  // smem column j holds input column j - pad
+  for (int i = threadIdx.x; i < BLK * C * Wp; i += blockDim.x) {
+    const int rc = i / Wp, j = i - rc * Wp;
+    const int dr = rc / C, c = rc - dr * C;
+    const int ih = hs * BLK - pad + dr, iw = j - pad;
+    const bool ok = ih >= 0 && ih < H && iw >= 0 && iw < W;
+    const float *src = ok ? x + (n * C + c) * HW + (long long)ih * W + iw : x;
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(sbase + 4u * i),
+                 "l"(src), "r"(ok ? 4 : 0)
+                 : "memory");
+  }
+  asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
+  __syncthreads();
+  char *yrow = (char *)y + ((size_t)(n * Hs + hs) * Ws) * Cs * ESZ;
+  for (int ws = threadIdx.x; ws < Ws; ws += blockDim.x) {
+    float v[BLK * BLK * C];                          // channel cp = (dr*BLK + ds)*C + c
+#pragma unroll
+    for (int dr = 0; dr < BLK; ++dr)
+#pragma unroll
+      for (int c = 0; c < C; ++c) {
+        const float *rp = rows + (dr * C + c) * Wp + ws * BLK;
+        if constexpr (BLK == 4) {
+          const float4 q = *(const float4 *)rp;
+          v[(dr * BLK + 0) * C + c] = q.x;
+          v[(dr * BLK + 1) * C + c] = q.y;
+          v[(dr * BLK + 2) * C + c] = q.z;
+          v[(dr * BLK + 3) * C + c] = q.w;
+        } else {
+#pragma unroll
+          for (int ds = 0; ds < BLK; ++ds) v[(dr * BLK + ds) * C + c] = rp[ds];
+        }
+      }
+    char *py = yrow + (size_t)ws * Cs * ESZ;
+    constexpr int NREAL = BLK * BLK * C;
+    constexpr int MAXCH = (NREAL + VN - 1) / VN + 8;   // stored channels <= NREAL + padding
+#pragma unroll
+    for (int ch = 0; ch < MAXCH; ++ch) {
+      if (ch * VN >= Cs) break;
+      Vec16<ST> o;
+#pragma unroll
+      for (int j = 0; j < VN; ++j) o.v[j] = ch * VN + j < NREAL ? v[ch * VN + j] : 0.f;
+      o.store(py + ch * 16, tf32_round);
+    }
+  }
+}
+
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
                                int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {
+  if (C == 3 && (blk == 4 || blk == 1) && W <= 4096) {
+    const int Wp = ((Ws * blk + 3) & ~3) + 4;
+    const size_t smem = (size_t)blk * C * Wp * sizeof(float);
+    const unsigned grid = (unsigned)((long long)B * Hs);
+    if (smem <= 48 * 1024) {
+      if (st == ST_BF16) {
+        if (blk == 4)
+          stage_c3_kernel<ST_BF16, 4><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, 0);
+        else
+          stage_c3_kernel<ST_BF16, 1><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, 0);
+      } else {
+        if (blk == 4)
+          stage_c3_kernel<ST_F32, 4><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, tf32_round);
+        else
+          stage_c3_kernel<ST_F32, 1><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, tf32_round);
+      }
+      return cudaGetLastError();
+    }
+  }
   const size_t rows_bytes = (size_t)blk * C * W * sizeof(float) + (size_t)Cs * sizeof(int);
   if (rows_bytes <= 48 * 1024 && blk <= 15) {
     const long long grid = (long long)B * Hs;
@@ -385,6 +469,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
   uint8_t *T = lp_smem;                                  // staged input
   uint8_t *U = LS > 0 ? lp_smem + tile_elems * ESZ : lp_smem;   // LRN output
   const long long tiles = (long long)a.B * a.Ho * a.nqt;
+  const float inv_chunks = 1.f / (float)chunks;
 
   for_each_tile(a.b, tiles, [&](long long t) {
     const int qt = (int)(t % a.nqt);
@@ -399,9 +484,11 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
     // stage rows [h0, h1) x cols [w0, w1): each row segment is contiguous;
     // cp.async keeps every 16 B load of the tile in flight at once
     const int vec_per_row = wc * chunks;
+    const float inv_vpr = 1.f / (float)vec_per_row;
     const uint32_t tbase = (uint32_t)__cvta_generic_to_shared(T);
     for (int v = threadIdx.x; v < nr * vec_per_row; v += blockDim.x) {
-      const int r = v / vec_per_row, rem = v - r * vec_per_row;
+      int r, rem;
+      fdivmod(v, vec_per_row, inv_vpr, r, rem);
       const size_t src = (((size_t)n * a.H + h0 + r) * a.W + w0) * C + (size_t)rem * VN;
       const uint32_t dst = tbase + (uint32_t)(((size_t)r * wc_max * C + (size_t)rem * VN) * ESZ);
       asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst),
@@ -415,9 +502,12 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
       // needs HALF channels of the neighbouring chunks, read as whole vectors
       constexpr int HALF = LS / 2;
       static_assert(HALF <= VN, "LRN window wider than one neighbouring chunk");
-      for (int v = threadIdx.x; v < nr * wc * chunks; v += blockDim.x) {
-        const int ch = v % chunks, pix = v / chunks;
-        const int r = pix / wc, col = pix - r * wc;
+      // walk every staged pixel slot (row pitch wc_max; unused slots are
+      // harmless) so only one divmod by `chunks` is needed
+      for (int v = threadIdx.x; v < nr * wc_max * chunks; v += blockDim.x) {
+        int pix, ch;
+        fdivmod(v, chunks, inv_chunks, pix, ch);
+        const int r = 0, col = pix;
         const uint8_t *px = T + ((size_t)r * wc_max + col) * C * ESZ;
         Vec16<ST> prev, cur, next;
         cur.load(px + (size_t)ch * 16);
@@ -443,7 +533,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
 #pragma unroll
           for (int w = 0; w < LS; ++w) acc += sq[j + w];
           const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
-          out.v[j] = cur.v[j] * exp2f(-a.lrn_beta * __log2f(scale));
+          out.v[j] = cur.v[j] * lrn_scale_pow(scale, a.lrn_beta);
         }
         out.store(U + ((size_t)r * wc_max + col) * C * ESZ + (size_t)ch * 16, a.tf32_round);
       }
@@ -453,19 +543,40 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
     // chunk ch through the (optional) per-group channel padding
     const float inv = 1.f / (float)(a.k * a.k);
     const int ochunks = a.Cout / VN;
+    const float inv_oc = 1.f / (float)ochunks;
     const int grp_real = a.ocg / VN, grp_pad = a.ocp / VN;
     for (int v = threadIdx.x; v < (q1 - q0) * ochunks; v += blockDim.x) {
-      const int oc = v % ochunks, q = q0 + v / ochunks;
+      int qq, oc;
+      fdivmod(v, ochunks, inv_oc, qq, oc);
+      const int q = q0 + qq;
       int ch = oc;
       bool pad = false;
       if (grp_pad > 0) {
-        const int gi = oc / grp_pad, j = oc % grp_pad;
+        const int gi = oc / grp_pad, j = oc - gi * grp_pad;
         pad = j >= grp_real;
         ch = gi * grp_real + j;
       }
       Vec16<ST> acc, cur;
 #pragma unroll
       for (int j = 0; j < VN; ++j) acc.v[j] = pad ? 0.f : (a.is_max ? -INFINITY : 0.f);
+      char *dst = (char *)a.y + ((((size_t)n * a.Ho + p) * a.Wo + q) * a.Cout + oc * VN) * ESZ;
+      if (ST == ST_BF16 && a.is_max && !pad) {
+        // max is exact in bf16: compare packed pairs, no conversions
+        const int cs = q * a.s - w0, ce = min(cs + a.k, wc);
+        __nv_bfloat162 m[4];
+        const __nv_bfloat162 ninf = __float2bfloat162_rn(-INFINITY);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) m[j] = ninf;
+        for (int r = 0; r < nr; ++r)
+          for (int col = cs; col < ce; ++col) {
+            const uint4 raw = *(const uint4 *)(U + (((size_t)r * wc_max + col) * C + ch * VN) * ESZ);
+            const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], h[j]);
+          }
+        *(uint4 *)dst = *(const uint4 *)m;
+        continue;
+      }
       if (!pad) {
         const int cs = q * a.s - w0, ce = min(cs + a.k, wc);
         for (int r = 0; r < nr; ++r)
@@ -479,8 +590,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
 #pragma unroll
           for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
       }
-      acc.store((char *)a.y + ((((size_t)n * a.Ho + p) * a.Wo + q) * a.Cout + oc * VN) * ESZ,
-                a.is_max ? 0 : a.tf32_round);
+      acc.store(dst, a.is_max ? 0 : a.tf32_round);
     }
   });
 }

@@ -33,6 +33,7 @@
 #include <cstdlib>
 
 #include "budget.cuh"
+#include "lrn_math.cuh"
 #include "pcnn_internal.h"
 
 namespace pcnn {
@@ -338,7 +339,7 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
 #pragma unroll
         for (int w = 0; w < 5; ++w) acc += sq[c0 + j + w];
         const float scale = a.lrn_k + a.lrn_a_over_n * acc;
-        o[j] = f[c0 + j] * exp2f(-a.lrn_beta * __log2f(scale));
+        o[j] = f[c0 + j] * lrn_scale_pow(scale, a.lrn_beta);
       }
       if constexpr (ST == ST_BF16) {
         uint4 pk;
