@@ -43,8 +43,10 @@ constexpr int TC_BN_MAX = 256;          // max UMMA N
 constexpr int TC_ROW_BYTES = 128;       // one K-block row = one 128B swizzle row
 constexpr int TC_MAX_STAGES = 12;
 constexpr int TC_A_STAGE = TC_BM * TC_ROW_BYTES;          // 16 KB
-constexpr int TC_STAGE_BUDGET = 200 * 1024;               // operand stages per CTA
-constexpr int TC_MAX_KTAB = 4096;       // slab-table entries kept in smem
+constexpr int TC_STAGE_BUDGET = 176 * 1024;               // operand stages per CTA
+constexpr int TC_MAX_KTAB = 1024;       // slab-table entries kept in smem
+constexpr int EPI_PITCH = 144;          // epilogue staging row: 128 B + 16 B pad
+constexpr int EPI_WARP_BYTES = 32 * EPI_PITCH;
 constexpr int TC_THREADS = 192;
 constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 
@@ -52,6 +54,7 @@ constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 //   [0, TC_STAGE_BUDGET)   A stages, then B stages (runtime count)
 //   SM_BAR                 barriers + TMEM pointer
 //   SM_KTAB                (r, s, c) table, one entry per A slab
+//   SM_EPI                 per-epilogue-warp output staging (coalesced stores)
 constexpr int SM_BAR = TC_STAGE_BUDGET;
 constexpr int SM_FULL = SM_BAR;
 constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_STAGES;
@@ -59,7 +62,8 @@ constexpr int SM_TFULL = SM_EMPTY + 8 * TC_MAX_STAGES;
 constexpr int SM_TEMPTY = SM_TFULL + 16;
 constexpr int SM_TMEMPTR = SM_TEMPTY + 16;
 constexpr int SM_KTAB = SM_BAR + 256;
-constexpr int SM_TOTAL = SM_KTAB + 4 * TC_MAX_KTAB;
+constexpr int SM_EPI = SM_KTAB + 4 * TC_MAX_KTAB;        // 4 warps x 32 rows x 144 B
+constexpr int SM_TOTAL = SM_EPI + 4 * EPI_WARP_BYTES;
 constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
 
 size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
@@ -292,6 +296,29 @@ struct TcArgs {
   Budget b;
 };
 
+// Each lane of an epilogue warp owns one output row (pixel).  It parks the
+// row's next 128 B (8 x 16 B pieces, `np` valid) in the warp's smem staging
+// rows, then the warp writes them back row-contiguously: 8 lanes per 128 B
+// line, 4 full lines per store instruction (instead of 32 scattered 16 B
+// pieces).  `rowaddr` is each lane's destination for its piece 0 (nullptr
+// when its row is out of range).
+__device__ __forceinline__ void epi_store_rows(uint8_t *stage, const uint4 (&pc)[8], int np,
+                                               char *rowaddr, int lane) {
+  uint8_t *mine = stage + lane * EPI_PITCH;
+#pragma unroll
+  for (int j = 0; j < 8; ++j)
+    if (j < np) *(uint4 *)(mine + 16 * j) = pc[j];
+  __syncwarp();
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    const int p = it * 32 + lane, r = p >> 3, j = p & 7;
+    char *dst = (char *)__shfl_sync(0xffffffffu, (unsigned long long)rowaddr, r);
+    if (dst != nullptr && j < np)
+      *(uint4 *)(dst + 16 * j) = *(const uint4 *)(stage + r * EPI_PITCH + 16 * j);
+  }
+  __syncwarp();
+}
+
 // Epilogue with the following LRN layer fused in (R3; Caffe size
 // 5).  The tile holds every channel of its pixels (bn == Nfg <= 128, one N
 // tile), so each thread normalises its own pixel's channel vector in
@@ -300,7 +327,7 @@ struct TcArgs {
 // form), so the result is bitwise identical to conv -> store -> LRN.
 template <int ST>
 __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bool mok,
-                                             size_t orow) {
+                                             size_t orow, uint8_t *stage, int lane) {
   const ConvGeom &g = a.g;
   constexpr int MAXC = 128;
   float f[MAXC];
@@ -314,7 +341,6 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
       for (int i = 0; i < 32; ++i) f[c0 + i] = __uint_as_float(v[i]);
     }
   }
-  if (!mok) return;
   const int C = g.Nfg;
 #pragma unroll
   for (int i = 0; i < MAXC; ++i) {
@@ -329,41 +355,45 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
   sq[0] = sq[1] = sq[MAXC + 2] = sq[MAXC + 3] = 0.f;
 #pragma unroll
   for (int i = 0; i < MAXC; ++i) sq[i + 2] = f[i] * f[i];
+  // normalised outputs, 8 channels = one 16 B piece (bf16) / two (fp32)
+  constexpr int EB = ST == ST_BF16 ? 2 : 4;
+  const int row_bytes = C * EB;
+  char *rowp = mok ? (char *)a.y + orow * EB : nullptr;
 #pragma unroll
-  for (int c0 = 0; c0 < MAXC; c0 += 8) {
-    if (c0 < C) {
-      float o[8];
+  for (int pass = 0; pass < MAXC * EB / 128; ++pass) {   // 128 B of the row per pass
+    if (pass * 128 >= row_bytes) break;                  // warp-uniform
+    uint4 pc[8];
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
+    for (int q = 0; q < 8; ++q) {
+      constexpr int PER = 16 / EB;                       // channels per piece
+      const int c0 = (pass * 128 + q * 16) / EB;
+      float o[PER];
+#pragma unroll
+      for (int j = 0; j < PER; ++j) {
+        const int c = c0 + j;
         float acc = 0.f;
 #pragma unroll
-        for (int w = 0; w < 5; ++w) acc += sq[c0 + j + w];
+        for (int w = 0; w < 5; ++w) acc += sq[(c + w) < MAXC + 4 ? c + w : MAXC + 3];
         const float scale = a.lrn_k + a.lrn_a_over_n * acc;
-        o[j] = f[c0 + j] * lrn_scale_pow(scale, a.lrn_beta);
+        o[j] = (c < MAXC ? f[c < MAXC ? c : 0] : 0.f) * lrn_scale_pow(scale, a.lrn_beta);
       }
       if constexpr (ST == ST_BF16) {
-        uint4 pk;
-        uint32_t *pw = (uint32_t *)&pk;
+        uint32_t *pw = (uint32_t *)&pc[q];
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           __nv_bfloat162 b2 = __floats2bfloat162_rn(o[2 * i], o[2 * i + 1]);
           pw[i] = *(uint32_t *)&b2;
         }
-        *(uint4 *)((__nv_bfloat16 *)a.y + orow + c0) = pk;
       } else {
-        float *yp = (float *)a.y + orow + c0;
+        float t[4];
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          float4 q;
-          if (g.out_mode == OUT_F32_TF32)
-            q = make_float4(tf32_rna_tc(o[4 * h]), tf32_rna_tc(o[4 * h + 1]),
-                            tf32_rna_tc(o[4 * h + 2]), tf32_rna_tc(o[4 * h + 3]));
-          else
-            q = make_float4(o[4 * h], o[4 * h + 1], o[4 * h + 2], o[4 * h + 3]);
-          *(float4 *)(yp + 4 * h) = q;
-        }
+        for (int i = 0; i < 4; ++i) t[i] = g.out_mode == OUT_F32_TF32 ? tf32_rna_tc(o[i]) : o[i];
+        pc[q] = make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]), __float_as_uint(t[2]),
+                           __float_as_uint(t[3]));
       }
     }
+    const int np = min(8, (row_bytes - pass * 128) / 16);
+    epi_store_rows(stage, pc, np, rowp ? rowp + pass * 128 : nullptr, lane);
   }
 }
 
@@ -536,6 +566,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     const int quarter = warp & 3;
     const int row = quarter * 32 + lane;
     const bool partial = a.splits > 1;
+    uint8_t *stage = smem + SM_EPI + (warp - 2) * EPI_WARP_BYTES;
     const uint32_t tempty_leader =
         CG == 2 ? mapa(sbase + SM_TEMPTY, 0) : sbase + SM_TEMPTY;
     uint32_t lt = 0;
@@ -550,7 +581,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       const size_t orow = (size_t)m * g.out_cs;
       if (a.lrn) {
         epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX, mok,
-                         orow);
+                         orow, stage, lane);
         tc_fence_before();
         __syncwarp();
         if (lane == 0) {
@@ -559,72 +590,70 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         }
         continue;
       }
-      // bias is zero-padded on the device, so whole float4s can be read
-      for (int c0 = 0; c0 < a.bn; c0 += 32) {
-        __syncwarp();
-        uint32_t v[32];
-        tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0, v);
-        tmem_ld_wait();
+      // bias is zero-padded on the device, so whole float4s can be read.
+      // Each pass drains 128 B of every row: 64 bf16 or 32 fp32 columns.
+      const bool out16 = !partial && g.out_mode == OUT_BF16;
+      const int pass_cols = out16 ? 64 : 32;
+      const int ocs = partial ? g.out_cs : g.out_cs;
+      char *obase = partial ? (char *)(a.ws + (size_t)sp * g.M * g.out_cs)
+                            : (char *)a.y;
+      const int eb = out16 ? 2 : 4;
+      for (int c0 = 0; c0 < a.bn; c0 += pass_cols) {
         const int n = nt * a.bn + c0;          // column within the group
-        if (mok && n < g.Nfg) {
-          const int col = grp * g.Nfg + n;
-          float f[32];
+        if (n >= g.Nfg) break;                 // warp-uniform
+        const int col = grp * g.Nfg + n;
+        float f[64];
 #pragma unroll
-          for (int i = 0; i < 32; ++i) f[i] = __uint_as_float(v[i]);
-          if (!partial) {
-            const float4 *bp = (const float4 *)(a.bias + col);
+        for (int h = 0; h < 2; ++h) {
+          if (h == 0 || out16) {
+            uint32_t v[32];
+            tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0 + 32 * h, v);
+            tmem_ld_wait();
 #pragma unroll
-            for (int q = 0; q < 8; ++q) {
+            for (int i = 0; i < 32; ++i) f[32 * h + i] = __uint_as_float(v[i]);
+          }
+        }
+        if (!partial) {
+          const float4 *bp = (const float4 *)(a.bias + col);
+#pragma unroll
+          for (int q = 0; q < 16; ++q) {
+            if (q < 8 || out16) {
               const float4 bb = __ldg(bp + q);
               f[4 * q] += bb.x;
               f[4 * q + 1] += bb.y;
               f[4 * q + 2] += bb.z;
               f[4 * q + 3] += bb.w;
             }
-            if (g.relu)
-#pragma unroll
-              for (int i = 0; i < 32; ++i) f[i] = fmaxf(f[i], 0.f);
           }
-          if (partial) {
-            float *yp = a.ws + (size_t)sp * g.M * g.out_cs + orow + col;
+          if (g.relu)
 #pragma unroll
-            for (int h = 0; h < 8; ++h)
-              if (n + 4 * h < g.Nfg)
-                *(float4 *)(yp + 4 * h) =
-                    make_float4(f[4 * h], f[4 * h + 1], f[4 * h + 2], f[4 * h + 3]);
-          } else if (g.out_mode == OUT_BF16) {
-            __nv_bfloat16 *yp = (__nv_bfloat16 *)a.y + orow + col;
+            for (int i = 0; i < 64; ++i) f[i] = fmaxf(f[i], 0.f);
+        }
+        uint4 pc[8];
+        if (out16) {
 #pragma unroll
-            for (int h = 0; h < 4; ++h) {
-              if (n + 8 * h < g.Nfg) {
-                uint4 pk;
-                uint32_t *pw = (uint32_t *)&pk;
+          for (int q = 0; q < 8; ++q) {
+            uint32_t *pw = (uint32_t *)&pc[q];
 #pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                  __nv_bfloat162 b2 =
-                      __floats2bfloat162_rn(f[8 * h + 2 * i], f[8 * h + 2 * i + 1]);
-                  pw[i] = *(uint32_t *)&b2;
-                }
-                *(uint4 *)(yp + 8 * h) = pk;
-              }
+            for (int i = 0; i < 4; ++i) {
+              __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * q + 2 * i], f[8 * q + 2 * i + 1]);
+              pw[i] = *(uint32_t *)&b2;
             }
-          } else {
-            float *yp = (float *)a.y + orow + col;
+          }
+        } else {
+          const bool rnd = !partial && g.out_mode == OUT_F32_TF32;
 #pragma unroll
-            for (int h = 0; h < 8; ++h) {
-              if (n + 4 * h < g.Nfg) {
-                float4 q;
-                if (g.out_mode == OUT_F32_TF32) {
-                  q = make_float4(tf32_rna_tc(f[4 * h]), tf32_rna_tc(f[4 * h + 1]),
-                                  tf32_rna_tc(f[4 * h + 2]), tf32_rna_tc(f[4 * h + 3]));
-                } else {
-                  q = make_float4(f[4 * h], f[4 * h + 1], f[4 * h + 2], f[4 * h + 3]);
-                }
-                *(float4 *)(yp + 4 * h) = q;
-              }
-            }
+          for (int q = 0; q < 8; ++q) {
+            float t[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) t[i] = rnd ? tf32_rna_tc(f[4 * q + i]) : f[4 * q + i];
+            pc[q] = make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]),
+                               __float_as_uint(t[2]), __float_as_uint(t[3]));
           }
         }
+        const int np = min(8, ((min(g.Nfg - n, pass_cols)) * eb) / 16);
+        char *rowp = mok ? obase + ((size_t)m * ocs + col) * eb : nullptr;
+        epi_store_rows(stage, pc, np, rowp, lane);
       }
       tc_fence_before();
       __syncwarp();
