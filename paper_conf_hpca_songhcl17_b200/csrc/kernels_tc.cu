@@ -651,7 +651,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
                                __float_as_uint(t[2]), __float_as_uint(t[3]));
           }
         }
-        const int np = min(8, ((min(g.Nfg - n, pass_cols)) * eb) / 16);
+        // pieces of this pass inside both the group (Nfg) and this N tile (bn)
+        const int np = min(8, (min(min(g.Nfg - n, a.bn - c0), pass_cols) * eb) / 16);
         char *rowp = mok ? obase + ((size_t)m * ocs + col) * eb : nullptr;
         epi_store_rows(stage, pc, np, rowp, lane);
       }
