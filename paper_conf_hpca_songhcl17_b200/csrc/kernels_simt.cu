@@ -232,6 +232,76 @@ stage_c3_kernel(const float *__restrict__ x, void *y, int H, int W, int Hs, int 
   }
 }
 
+// First-layer im2col staging (3-channel inputs, S x S taps, stride st, pad):
+// output pixel (n, p, q) gets the K = S*S*3 values of its receptive field in
+// (r, s, c) order, zero-padded to Kp channels, so the first conv runs as a
+// 1x1 conv with one full 128 B TMA slab per pixel.  One CTA per output row;
+// the S input rows x 3 channels are staged in smem with cp.async.
+template <int ST, int S>
+__global__ void __launch_bounds__(256)
+stage_im2col_kernel(const float *__restrict__ x, void *y, int H, int W, int Ho, int Wo, int Kp,
+                    int st, int pad, int tf32_round) {
+  constexpr int C = 3, K = S * S * C;
+  constexpr int VN = Vec16<ST>::N;
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  extern __shared__ float rows[];                  // [S][C][Wp], column j = input col j - pad
+  const int Wp = (Wo - 1) * st + S;
+  const int p = blockIdx.x % Ho;
+  const long long n = blockIdx.x / Ho;
+  const long long HW = (long long)H * W;
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(rows);
+  for (int i = threadIdx.x; i < S * C * Wp; i += blockDim.x) {
+    const int rc = i / Wp, j = i - rc * Wp;
+    const int r = rc / C, c = rc - r * C;
+    const int ih = p * st - pad + r, iw = j - pad;
+    const bool ok = ih >= 0 && ih < H && iw >= 0 && iw < W;
+    const float *src = ok ? x + (n * C + c) * HW + (long long)ih * W + iw : x;
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(sbase + 4u * i),
+                 "l"(src), "r"(ok ? 4 : 0)
+                 : "memory");
+  }
+  asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
+  __syncthreads();
+  char *yrow = (char *)y + ((size_t)(n * Ho + p) * Wo) * Kp * ESZ;
+  for (int q = threadIdx.x; q < Wo; q += blockDim.x) {
+    float v[K];
+#pragma unroll
+    for (int r = 0; r < S; ++r)
+#pragma unroll
+      for (int s2 = 0; s2 < S; ++s2)
+#pragma unroll
+        for (int c = 0; c < C; ++c) v[(r * S + s2) * C + c] = rows[(r * C + c) * Wp + q * st + s2];
+    char *py = yrow + (size_t)q * Kp * ESZ;
+    constexpr int MAXCH = (K + VN - 1) / VN + 16;
+#pragma unroll
+    for (int ch = 0; ch < MAXCH; ++ch) {
+      if (ch * VN >= Kp) break;
+      Vec16<ST> o;
+#pragma unroll
+      for (int j = 0; j < VN; ++j) o.v[j] = ch * VN + j < K ? v[ch * VN + j] : 0.f;
+      o.store(py + ch * 16, tf32_round);
+    }
+  }
+}
+
+cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, int H, int W,
+                                int S, int stride, int pad, int Ho, int Wo, int Kp,
+                                int tf32_round, cudaStream_t s) {
+  if (C != 3 || (S != 3 && S != 5)) return cudaErrorInvalidValue;
+  const size_t smem = (size_t)S * C * ((Wo - 1) * stride + S) * sizeof(float);
+  if (smem > 48 * 1024) return cudaErrorInvalidValue;
+  const unsigned grid = (unsigned)((long long)B * Ho);
+#define PCNN_IM2COL(STT, SS) \
+  stage_im2col_kernel<STT, SS><<<grid, 256, smem, s>>>(x, y, H, W, Ho, Wo, Kp, stride, pad, tf32_round)
+  if (st == ST_BF16) {
+    if (S == 3) PCNN_IM2COL(ST_BF16, 3); else PCNN_IM2COL(ST_BF16, 5);
+  } else {
+    if (S == 3) PCNN_IM2COL(ST_F32, 3); else PCNN_IM2COL(ST_F32, 5);
+  }
+#undef PCNN_IM2COL
+  return cudaGetLastError();
+}
+
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
                                int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {

@@ -58,6 +58,11 @@ struct ConvGeom {
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C,
                                int H, int W, int Hs, int Ws, int Cs, int blk,
                                int pad, int tf32_round, cudaStream_t s);
+// a1 for a first conv with 3 input channels and S*S*3 <= 128: writes the
+// conv's im2col rows [B][Ho][Wo][Kp] so the conv runs as a 1x1 conv.
+cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, int H,
+                                int W, int S, int stride, int pad, int Ho, int Wo,
+                                int Kp, int tf32_round, cudaStream_t s);
 // final NHWC storage -> NCHW fp32 flatten
 cudaError_t launch_unstage_output(const void *x, int st, float *y, int B,
                                   int C, int H, int W, int Cs, cudaStream_t s);

@@ -155,6 +155,7 @@ struct pcnn_net {
   int occ_simt = 1, occ_lp = 1;
   // input staging geometry (space-to-depth by `blk` for a strided first conv)
   int stage_h = 0, stage_w = 0, stage_blk = 1, stage_pad = 0, stage_c = 0;
+  int stage_im2col = 0;     // 1: layer 0 input staged as im2col rows (1x1 conv)
   bool fuse_lrn_pool = true;
   bool census = false;
   // CUDA graph cache
@@ -745,10 +746,18 @@ static pcnn_status enqueue_all(pcnn_net *net, const float *d_images, int B, floa
   g_launches = 0;
   if (net->census)
     for (auto &ly : net->layers) CUDA_TRY(cudaMemsetAsync(ly.d_census, 0, 32, s));
-  CUDA_TRY(counted(launch_stage_input(d_images, net->d_act[0], st, B, net->desc.in_channels,
-                                      net->desc.in_height, net->desc.in_width, net->stage_h,
-                                      net->stage_w, net->in_cs, net->stage_blk, net->stage_pad,
-                                      tf32, s)));
+  if (net->stage_im2col) {
+    const Layer &l0 = net->layers[0];
+    CUDA_TRY(counted(launch_stage_im2col(d_images, net->d_act[0], st, B, net->desc.in_channels,
+                                         net->desc.in_height, net->desc.in_width, l0.d.kernel,
+                                         l0.d.stride, l0.d.pad, l0.out_h, l0.out_w, net->in_cs,
+                                         tf32, s)));
+  } else {
+    CUDA_TRY(counted(launch_stage_input(d_images, net->d_act[0], st, B, net->desc.in_channels,
+                                        net->desc.in_height, net->desc.in_width, net->stage_h,
+                                        net->stage_w, net->in_cs, net->stage_blk,
+                                        net->stage_pad, tf32, s)));
+  }
   if (evs) CUDA_TRY(cudaEventRecord((*evs)[0], s));
   int cur = 0;
   const int n = (int)net->layers.size();
@@ -1000,7 +1009,25 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   std::vector<float> s2d_w;
   const Layer &l0 = net->layers[0];
   const char *no_s2d = getenv("PCNN_NO_S2D");
-  if (l0.d.kind == PCNN_CONV && l0.d.groups == 1 && l0.d.stride >= 2 && l0.d.stride <= 8 &&
+  const int k0 = l0.d.kernel;
+  if (prec != PCNN_FP32_SIMT && l0.d.kind == PCNN_CONV && l0.d.groups == 1 &&
+      desc->in_channels == 3 && (k0 == 3 || k0 == 5) && 3 * k0 * k0 <= 128 &&
+      !(no_s2d && no_s2d[0] == '1')) {
+    // im2col staging: W'[f][(r*S + s)*3 + c] = W[f][c][r][s], a 1x1 conv on Kp channels
+    const int K = 3 * k0 * k0, F = l0.d.out_channels;
+    const int Kp = K <= 64 / esz * 2 ? round_up(K, 64 / esz) : round_up(K, 128 / esz);
+    net->stage_im2col = 1;
+    net->stage_c = K;
+    net->stage_h = l0.out_h;
+    net->stage_w = l0.out_w;
+    net->in_cs = Kp;
+    s2d_w.assign((size_t)F * K, 0.f);
+    for (int f = 0; f < F; ++f)
+      for (int c = 0; c < 3; ++c)
+        for (int r = 0; r < k0; ++r)
+          for (int q = 0; q < k0; ++q)
+            s2d_w[(size_t)f * K + (r * k0 + q) * 3 + c] = weights[0][(((size_t)f * 3 + c) * k0 + r) * k0 + q];
+  } else if (l0.d.kind == PCNN_CONV && l0.d.groups == 1 && l0.d.stride >= 2 && l0.d.stride <= 8 &&
       !(no_s2d && no_s2d[0] == '1')) {
     const int st2 = l0.d.stride, S = l0.d.kernel, Sp = (S + st2 - 1) / st2;
     const int C = desc->in_channels, Cp = st2 * st2 * C, F = l0.d.out_channels;
@@ -1031,7 +1058,11 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
                                 : (net->st == ST_BF16 ? OUT_BF16
                                                       : (prec == PCNN_TF32 ? OUT_F32_TF32 : OUT_F32));
       const bool is_fc = ly.d.kind == PCNN_FC;
-      if (i == 0 && net->stage_blk > 1) {
+      if (i == 0 && net->stage_im2col) {
+        s = build_stage(ly.exact, ly, prec, ly.d.out_channels, 1, 1, 1, 0, ly.d.relu,
+                        net->stage_c, net->stage_h, net->stage_w, net->in_cs, false,
+                        s2d_w.data(), biases ? biases[i] : nullptr, mode);
+      } else if (i == 0 && net->stage_blk > 1) {
         const int Sp = (ly.d.kernel + net->stage_blk - 1) / net->stage_blk;
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, 1, Sp, 1, 0, ly.d.relu,
                         net->stage_c, net->stage_h, net->stage_w, net->in_cs, false,
