@@ -47,14 +47,18 @@ constexpr int TC_STAGE_BUDGET = 176 * 1024;               // operand stages per 
 constexpr int TC_MAX_KTAB = 1024;       // slab-table entries kept in smem
 constexpr int EPI_PITCH = 144;          // epilogue staging row: 128 B + 16 B pad
 constexpr int EPI_WARP_BYTES = 32 * EPI_PITCH;
-constexpr int TC_THREADS = 192;
+// warps: 0 TMA producer, 1 MMA issuer, then NEPI epilogue warps (8, two per
+// TMEM lane quarter splitting the columns; 4 for the LRN-fused variant, whose
+// per-row channel vector needs ~255 registers)
+template <bool LRN> __host__ __device__ constexpr int tc_nepi() { return LRN ? 4 : 8; }
+template <bool LRN> __host__ __device__ constexpr int tc_threads() { return 64 + 32 * tc_nepi<LRN>(); }
 constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 
 // smem layout (bytes from the 1024-aligned base):
 //   [0, TC_STAGE_BUDGET)   A stages, then B stages (runtime count)
 //   SM_BAR                 barriers + TMEM pointer
 //   SM_KTAB                (r, s, c) table, one entry per A slab
-//   SM_EPI                 per-epilogue-warp output staging (coalesced stores)
+//   SM_EPI                 per-epilogue-warp output staging (coalesced stores, 8 warps)
 constexpr int SM_BAR = TC_STAGE_BUDGET;
 constexpr int SM_FULL = SM_BAR;
 constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_STAGES;
@@ -63,7 +67,7 @@ constexpr int SM_TEMPTY = SM_TFULL + 16;
 constexpr int SM_TMEMPTR = SM_TEMPTY + 16;
 constexpr int SM_KTAB = SM_BAR + 256;
 constexpr int SM_EPI = SM_KTAB + 4 * TC_MAX_KTAB;        // 4 warps x 32 rows x 144 B
-constexpr int SM_TOTAL = SM_EPI + 4 * EPI_WARP_BYTES;
+constexpr int SM_TOTAL = SM_EPI + 8 * EPI_WARP_BYTES;
 constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
 
 size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
@@ -404,8 +408,8 @@ __device__ __forceinline__ void advance(uint32_t &stage, uint32_t &phase, int st
   }
 }
 
-template <int ST, int CG>
-__global__ void __launch_bounds__(TC_THREADS, 1)
+template <int ST, int CG, bool LRN>
+__global__ void __launch_bounds__(tc_threads<LRN>(), 1)
 conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
                const __grid_constant__ CUtensorMap tmap_x, const TcArgs a) {
   extern __shared__ uint8_t smem_raw[];
@@ -430,7 +434,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   const bool use_tab = a.ktab != nullptr;
   const int nent = g.Kpad / slab_elems;
   if (use_tab) {
-    for (int i = tid; i < nent && i < TC_MAX_KTAB; i += TC_THREADS) {
+    for (int i = tid; i < nent && i < TC_MAX_KTAB; i += tc_threads<LRN>()) {
       const int k = i * slab_elems;
       ktab_s[i] = k < g.K ? (uint32_t)__ldg(&a.ktab[k]) : 0xFF000000u;
     }
@@ -442,7 +446,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(sbase + SM_TFULL + 8 * i, 1);
-      mbar_init(sbase + SM_TEMPTY + 8 * i, 4 * CG);   // one arrive per epilogue warp
+      mbar_init(sbase + SM_TEMPTY + 8 * i, tc_nepi<LRN>() * CG);   // one arrive per epilogue warp
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     census_mark(a.b);
@@ -562,8 +566,9 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       }
     }
   } else {
-    // ------------------------------------------------ epilogue (warps 2..5)
-    const int quarter = warp & 3;
+    // ------------------------------------------------ epilogue (warps 2..)
+    const int quarter = warp & 3;               // TMEM lanes 32*quarter..
+    const int half = (warp - 2) >> 2;           // column half (8-warp epilogue)
     const int row = quarter * 32 + lane;
     const bool partial = a.splits > 1;
     uint8_t *stage = smem + SM_EPI + (warp - 2) * EPI_WARP_BYTES;
@@ -579,7 +584,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
       const bool mok = m < g.M;
       const size_t orow = (size_t)m * g.out_cs;
-      if (a.lrn) {
+      if constexpr (LRN) {
         epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX, mok,
                          orow, stage, lane);
         tc_fence_before();
@@ -598,14 +603,17 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       char *obase = partial ? (char *)(a.ws + (size_t)sp * g.M * g.out_cs)
                             : (char *)a.y;
       const int eb = out16 ? 2 : 4;
-      for (int c0 = 0; c0 < a.bn; c0 += pass_cols) {
+      // the two warps of a lane quarter split the tile's columns at a 32 boundary
+      const int split = ((a.bn / 2 + 31) / 32) * 32;
+      const int cbeg = half == 0 ? 0 : split, cend = half == 0 ? split : a.bn;
+      for (int c0 = cbeg; c0 < cend; c0 += pass_cols) {
         const int n = nt * a.bn + c0;          // column within the group
         if (n >= g.Nfg) break;                 // warp-uniform
         const int col = grp * g.Nfg + n;
         float f[64];
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
-          if (h == 0 || out16) {
+          if (h == 0 || (out16 && c0 + 32 < cend)) {
             uint32_t v[32];
             tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0 + 32 * h, v);
             tmem_ld_wait();
@@ -652,7 +660,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           }
         }
         // pieces of this pass inside both the group (Nfg) and this N tile (bn)
-        const int np = min(8, (min(min(g.Nfg - n, a.bn - c0), pass_cols) * eb) / 16);
+        const int np = min(8, (min(min(g.Nfg - n, cend - c0), pass_cols) * eb) / 16);
         char *rowp = mok ? obase + ((size_t)m * ocs + col) * eb : nullptr;
         epi_store_rows(stage, pc, np, rowp, lane);
       }
@@ -714,18 +722,22 @@ __global__ void splitk_reduce_kernel(const float *__restrict__ ws, void *y,
   }
 }
 
-template <int ST, int CG>
+template <int ST, int CG, bool LRN>
 static cudaError_t set_smem_attr() {
-  return cudaFuncSetAttribute(conv_tc_kernel<ST, CG>,
+  return cudaFuncSetAttribute(conv_tc_kernel<ST, CG, LRN>,
                               cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TC_SMEM_BYTES);
 }
 
 cudaError_t tc_init() {
   cudaError_t e;
-  if ((e = set_smem_attr<ST_BF16, 1>()) != cudaSuccess) return e;
-  if ((e = set_smem_attr<ST_BF16, 2>()) != cudaSuccess) return e;
-  if ((e = set_smem_attr<ST_F32, 1>()) != cudaSuccess) return e;
-  return set_smem_attr<ST_F32, 2>();
+  if ((e = set_smem_attr<ST_BF16, 1, false>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_BF16, 2, false>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_F32, 1, false>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_F32, 2, false>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_BF16, 1, true>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_BF16, 2, true>()) != cudaSuccess) return e;
+  if ((e = set_smem_attr<ST_F32, 1, true>()) != cudaSuccess) return e;
+  return set_smem_attr<ST_F32, 2, true>();
 }
 
 int tc_slab_bytes(int st, int cg_channels) {
@@ -735,12 +747,12 @@ int tc_slab_bytes(int st, int cg_channels) {
   return 0;   // channels per group must be a multiple of 32 bytes
 }
 
-template <int ST, int CG>
+template <int ST, int CG, bool LRN>
 static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_x,
                              const TcArgs &args, int grid, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
-  cfg.blockDim = dim3(TC_THREADS);
+  cfg.blockDim = dim3(tc_threads<LRN>());
   cfg.dynamicSmemBytes = TC_SMEM_BYTES;
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
@@ -750,7 +762,7 @@ static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG>, *tmap_w, *tmap_x, args);
+  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG, LRN>, *tmap_w, *tmap_x, args);
 }
 
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
@@ -786,12 +798,17 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
   cudaError_t e;
+  const bool L = args.lrn != 0;
   if (st == ST_BF16)
-    e = p.cg == 2 ? launch_tc<ST_BF16, 2>(tmap_w, tmap_x, args, p.grid, s)
-                  : launch_tc<ST_BF16, 1>(tmap_w, tmap_x, args, p.grid, s);
+    e = p.cg == 2 ? (L ? launch_tc<ST_BF16, 2, true>(tmap_w, tmap_x, args, p.grid, s)
+                       : launch_tc<ST_BF16, 2, false>(tmap_w, tmap_x, args, p.grid, s))
+                  : (L ? launch_tc<ST_BF16, 1, true>(tmap_w, tmap_x, args, p.grid, s)
+                       : launch_tc<ST_BF16, 1, false>(tmap_w, tmap_x, args, p.grid, s));
   else
-    e = p.cg == 2 ? launch_tc<ST_F32, 2>(tmap_w, tmap_x, args, p.grid, s)
-                  : launch_tc<ST_F32, 1>(tmap_w, tmap_x, args, p.grid, s);
+    e = p.cg == 2 ? (L ? launch_tc<ST_F32, 2, true>(tmap_w, tmap_x, args, p.grid, s)
+                       : launch_tc<ST_F32, 2, false>(tmap_w, tmap_x, args, p.grid, s))
+                  : (L ? launch_tc<ST_F32, 1, true>(tmap_w, tmap_x, args, p.grid, s)
+                       : launch_tc<ST_F32, 1, false>(tmap_w, tmap_x, args, p.grid, s));
   if (e != cudaSuccess) return e;
   e = cudaGetLastError();
   if (e != cudaSuccess || p.splits <= 1) return e;
