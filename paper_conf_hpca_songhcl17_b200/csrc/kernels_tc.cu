@@ -295,6 +295,8 @@ struct TcArgs {
   int kblocks, kb_per_split;
   int stages;
   int slab_bytes;       // 128 / 64 / 32: A K-block = 128 / slab_bytes TMA slabs
+  int prof;             // 1: accumulate per-role barrier-wait cycles (debug)
+  int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
   float lrn_a_over_n, lrn_beta, lrn_k;
   Budget b;
@@ -401,6 +403,26 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
   }
 }
 
+// Debug counters (PCNN_TC_PROFILE=1): summed clock64 cycles per role.
+//  0 producer waits on EMPTY   1 MMA waits on FULL   2 MMA waits on TEMPTY
+//  3 epilogue waits on TFULL   4 CTA lifetime        5 K-blocks issued
+//  6 epilogue busy cycles      7 CTAs
+__device__ unsigned long long g_tc_prof[8];
+
+struct WaitClock {
+  bool on;
+  unsigned long long acc = 0;
+  __device__ __forceinline__ void wait(uint32_t bar, uint32_t parity) {
+    if (on) {
+      const long long t0 = clock64();
+      mbar_wait(bar, parity);
+      acc += (unsigned long long)(clock64() - t0);
+    } else {
+      mbar_wait(bar, parity);
+    }
+  }
+};
+
 __device__ __forceinline__ void advance(uint32_t &stage, uint32_t &phase, int stages) {
   if (++stage == (uint32_t)stages) {
     stage = 0;
@@ -470,6 +492,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *(volatile uint32_t *)(smem + SM_TMEMPTR);
+  const long long t_start = a.prof ? clock64() : 0;
+  unsigned long long wtf_acc_out = 0, busy_out = 0;   // epilogue profile (warp 2)
 
   const int HoWo = g.Ho * g.Wo;
   // work unit u -> (m tile, n tile, group, split); m fastest so CTAs running
@@ -493,21 +517,26 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
       uint32_t stage = 0, phase = 0;
+      WaitClock wc{a.prof != 0};
+      unsigned long long nkb = 0;
       for (int u = pair; u < a.units; u += npairs) {
         int mt, nt, grp, sp, k0, k1;
         decode(u, mt, nt, grp, sp);
         kb_range(sp, k0, k1);
+        nkb += k1 - k0;
         const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
         // input-space corner of this CTA's first output pixel
         const int m0 = mt * (TC_BM * CG) + (int)rank * TC_BM;
         const int n0 = m0 / HoWo, pq = m0 % HoWo;
         const int w0 = (pq % g.Wo) * g.stride - g.pad, h0 = (pq / g.Wo) * g.stride - g.pad;
         for (int kb = k0; kb < k1; ++kb) {
-          mbar_wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
+          wc.wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
           const uint32_t fb = sbase + SM_FULL + 8 * stage;
-          if (rank == 0) mbar_arrive_expect_tx(fb, CG * (TC_A_STAGE + b_stage));
+          if (rank == 0)
+            mbar_arrive_expect_tx(fb, CG * (((a.skip & 1) ? 0 : TC_A_STAGE) +
+                                            ((a.skip & 2) ? 0 : b_stage)));
           const uint32_t dA = sA + stage * TC_A_STAGE;
-          for (int sl = 0; sl < nslab; ++sl) {
+          for (int sl = 0; sl < ((a.skip & 1) ? 0 : nslab); ++sl) {
             const int ke = kb * (TC_ROW_BYTES / ESZ) + sl * slab_elems;   // K element
             int r = 0, s = 0, c = ke;
             if (use_tab) {
@@ -526,12 +555,18 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
             else
               tma_im2col_2sm(dst, &tmap_x, fb, cc, w0, h0, n0, (uint16_t)s, (uint16_t)r);
           }
-          if constexpr (CG == 1)
-            tma_load_2d(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
-          else
-            tma_load_2d_2sm(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
+          if (!(a.skip & 2)) {
+            if constexpr (CG == 1)
+              tma_load_2d(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
+            else
+              tma_load_2d_2sm(sB + stage * b_stage, &tmap_w, fb, kb * (TC_ROW_BYTES / ESZ), nrow);
+          }
           advance(stage, phase, stages);
         }
+      }
+      if (a.prof) {
+        atomicAdd(&g_tc_prof[0], wc.acc);
+        atomicAdd(&g_tc_prof[5], nkb);
       }
     }
   } else if (warp == 1) {
@@ -540,21 +575,23 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
       const int mma_per_slab = slab_bytes / 32;      // K = 32 B per UMMA
       uint32_t stage = 0, phase = 0, lt = 0;
+      WaitClock wfull{a.prof != 0}, wtemp{a.prof != 0};
       for (int u = pair; u < a.units; u += npairs, ++lt) {
         int mt, nt, grp, sp, k0, k1;
         decode(u, mt, nt, grp, sp);
         kb_range(sp, k0, k1);
         const uint32_t buf = lt & 1, use = lt >> 1;
-        mbar_wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
+        wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
         tc_fence_after();
         const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
         for (int kb = k0; kb < k1; ++kb) {
-          mbar_wait(sbase + SM_FULL + 8 * stage, phase);
+          wfull.wait(sbase + SM_FULL + 8 * stage, phase);
           tc_fence_after();
           const uint32_t aS = sA + stage * TC_A_STAGE;
           const uint64_t bd = umma_desc_sw128(sB + stage * b_stage);
 #pragma unroll
           for (int k = 0; k < 4; ++k) {   // 4 x 32 B of K per 128 B K-block
+            if (a.skip & 4) break;
             const int sl = k / mma_per_slab, kin = k % mma_per_slab;
             const uint64_t ad = umma_desc(aS + sl * (TC_BM * slab_bytes), slab_bytes) + 2 * kin;
             tc_mma<ST, CG>(dcol, ad, bd + 2 * k, idesc, (kb > k0) || (k > 0));
@@ -563,6 +600,10 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           advance(stage, phase, stages);
         }
         tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
+      }
+      if (a.prof) {
+        atomicAdd(&g_tc_prof[1], wfull.acc);
+        atomicAdd(&g_tc_prof[2], wtemp.acc);
       }
     }
   } else {
@@ -575,11 +616,16 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     const uint32_t tempty_leader =
         CG == 2 ? mapa(sbase + SM_TEMPTY, 0) : sbase + SM_TEMPTY;
     uint32_t lt = 0;
+    WaitClock wtf{a.prof != 0 && lane == 0 && warp == 2};
+    unsigned long long busy = 0;
+    long long tb = 0;
     for (int u = pair; u < a.units; u += npairs, ++lt) {
       int mt, nt, grp, sp;
       decode(u, mt, nt, grp, sp);
       const uint32_t buf = lt & 1, use = lt >> 1;
-      mbar_wait(sbase + SM_TFULL + 8 * buf, use & 1);
+      if (wtf.on && tb) busy += clock64() - tb;
+      wtf.wait(sbase + SM_TFULL + 8 * buf, use & 1);
+      if (wtf.on) tb = clock64();
       tc_fence_after();
       const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
       const bool mok = m < g.M;
@@ -671,11 +717,22 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         else mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
       }
     }
+    if (wtf.on && tb) busy += clock64() - tb;
+    wtf_acc_out = wtf.acc;
+    busy_out = busy;
   }
 
+  if (a.prof && warp == 2 && lane == 0) {
+    atomicAdd(&g_tc_prof[3], wtf_acc_out);
+    atomicAdd(&g_tc_prof[6], busy_out);
+  }
   tc_fence_before();
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
+  if (a.prof && tid == 0) {
+    atomicAdd(&g_tc_prof[4], (unsigned long long)(clock64() - t_start));
+    atomicAdd(&g_tc_prof[7], 1ULL);
+  }
   if (warp == 1) {
     if constexpr (CG == 1)
       asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
@@ -765,11 +822,33 @@ static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_
   return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG, LRN>, *tmap_w, *tmap_x, args);
 }
 
+cudaError_t tc_profile(int reset, unsigned long long out[8]) {
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return e;
+  if (out) e = cudaMemcpyFromSymbol(out, g_tc_prof, sizeof(unsigned long long) * 8);
+  if (e != cudaSuccess) return e;
+  if (reset) {
+    unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    e = cudaMemcpyToSymbol(g_tc_prof, z, sizeof(z));
+  }
+  return e;
+}
+
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias, void *y,
                            const int *ktab, const TcPlan &p, float *ws, const Budget &b,
                            cudaStream_t s, const float *lrn) {
   TcArgs args;
+  static const int prof_env = [] {
+    const char *e = getenv("PCNN_TC_PROFILE");
+    return e && e[0] == '1' ? 1 : 0;
+  }();
+  static const int skip_env = [] {
+    const char *e = getenv("PCNN_TC_SKIP");
+    return e ? atoi(e) : 0;
+  }();
+  args.prof = prof_env;
+  args.skip = skip_env;
   args.lrn = 0;
   args.lrn_a_over_n = args.lrn_beta = args.lrn_k = 0.f;
   if (lrn) {   // {size, alpha, beta, k}: size 5 only, one N tile with every channel

@@ -101,6 +101,8 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
 // group width is not a multiple of 32 bytes.
 int tc_slab_bytes(int st, int cg_channels);
 int tc_stages_for(int bn, int cg);
+// debug: per-role barrier-wait cycle totals accumulated while PCNN_TC_PROFILE=1
+cudaError_t tc_profile(int reset, unsigned long long out[8]);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)
 cudaError_t tc_init();                 // sets the kernels' smem attributes
 size_t tc_smem_bytes();

@@ -1405,6 +1405,12 @@ pcnn_status pcnn_last_launch_count(const pcnn_net *net, int *launches) {
   return PCNN_OK;
 }
 
+// Debug export (not part of include/pcnn.h): tcgen05 kernel role-wait counters.
+pcnn_status pcnn_debug_tc_profile(int reset, unsigned long long out[8]) {
+  CUDA_TRY(tc_profile(reset, out));
+  return PCNN_OK;
+}
+
 pcnn_status pcnn_enable_sm_census(pcnn_net *net, int enable) {
   if (!net) return fail(PCNN_ERR_INVALID_ARGUMENT, "null net");
   net->census = enable != 0;

@@ -27,23 +27,28 @@ SHAPES = {  # name: (in_shape, layer)
     "norm2pool2": ((256, 27, 27), [dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0), dict(kind="maxpool", k=3, stride=2)]),
     "stage": ((3, 227, 227), dict(kind="maxpool", k=1, stride=1)),
 }
-name = sys.argv[1]
-B = int(sys.argv[2]) if len(sys.argv) > 2 else 256
-reps = int(sys.argv[3]) if len(sys.argv) > 3 else 20
-prec = sys.argv[4] if len(sys.argv) > 4 else "bf16"
-shape, L = SHAPES[name]
-net = dict(in_shape=shape, layers=L if isinstance(L, list) else [L])
-w, b = synth.net_params(net)
-n = pcnn.Net(net, w, b, B, prec)
-x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
-n.set_layer_timing(True)
-for _ in range(reps):
-    n.infer(x)
-torch.cuda.synchronize()
-ms, k = n.read_layer_timing()
-info = n.query_layer(0, B)
-t = sum(ms) / k
-byt = sum(n.query_layer(i, B)["bytes"] for i in range(len(net["layers"])))
-print("%s B=%d %s: %.4f ms  %.1f TFLOP/s  %.0f GB/s  tile %dx%d grid %d splits %d" % (
-    name, B, prec, t, info["flops"] / t / 1e9, byt / t / 1e6, info["tile_m"], info["tile_n"],
-    info["grid"], info["splits"]))
+def main():
+    name = sys.argv[1]
+    B = int(sys.argv[2]) if len(sys.argv) > 2 else 256
+    reps = int(sys.argv[3]) if len(sys.argv) > 3 else 20
+    prec = sys.argv[4] if len(sys.argv) > 4 else "bf16"
+    shape, L = SHAPES[name]
+    net = dict(in_shape=shape, layers=L if isinstance(L, list) else [L])
+    w, b = synth.net_params(net)
+    n = pcnn.Net(net, w, b, B, prec)
+    x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
+    n.set_layer_timing(True)
+    for _ in range(reps):
+        n.infer(x)
+    torch.cuda.synchronize()
+    ms, k = n.read_layer_timing()
+    info = n.query_layer(0, B)
+    t = sum(ms) / k
+    byt = sum(n.query_layer(i, B)["bytes"] for i in range(len(net["layers"])))
+    print("%s B=%d %s: %.4f ms  %.1f TFLOP/s  %.0f GB/s  tile %dx%d grid %d splits %d" % (
+        name, B, prec, t, info["flops"] / t / 1e9, byt / t / 1e6, info["tile_m"], info["tile_n"],
+        info["grid"], info["splits"]))
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,34 @@
+"""Per-role barrier-wait breakdown of the tcgen05 kernel for one layer shape.
+    python tools/tc_roles.py conv3 [batch]      (sets PCNN_TC_PROFILE=1)
+Counters are summed over CTAs; divided by CTAs they give the average cycles
+per CTA each role spent blocked."""
+import ctypes, os, sys
+os.environ["PCNN_TC_PROFILE"] = "1"
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import synth
+from paper_conf_hpca_songhcl17_b200 import pcnn
+from tools.one_layer import SHAPES
+
+name = sys.argv[1]
+B = int(sys.argv[2]) if len(sys.argv) > 2 else 256
+shape, L = SHAPES[name]
+net = dict(in_shape=shape, layers=L if isinstance(L, list) else [L])
+w, b = synth.net_params(net)
+n = pcnn.Net(net, w, b, B, "bf16")
+x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
+lib = pcnn.library()
+lib.pcnn_debug_tc_profile.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_ulonglong)]
+out = (ctypes.c_ulonglong * 8)()
+n.infer(x); torch.cuda.synchronize()
+lib.pcnn_debug_tc_profile(1, out)
+for _ in range(3):
+    n.infer(x)
+lib.pcnn_debug_tc_profile(1, out)
+c = list(out)
+ctas = max(c[7], 1)
+life = c[4] / ctas
+print("%s B=%d plan %s" % (name, B, {k: v for k, v in n.query_layer(0, B).items() if k in ("tile_m", "tile_n", "grid", "splits", "tiles")}))
+print("  per CTA: lifetime %.0f cyc, K-blocks %.1f (%.0f cyc/kb)" % (life, c[5] / ctas, life / max(c[5] / ctas, 1)))
+for i, lab in [(0, "producer wait EMPTY"), (1, "MMA wait FULL"), (2, "MMA wait TEMPTY"), (3, "epi wait TFULL"), (6, "epi busy")]:
+    print("  %-22s %5.1f%%" % (lab, 100.0 * c[i] / ctas / life))
