@@ -131,6 +131,25 @@ __device__ __forceinline__ void tma_im2col(uint32_t dst, const CUtensorMap *map,
       "l"((uint64_t)map), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ow), "h"(oh)
       : "memory");
 }
+// tiled 4-D TMA load (A slab of a rectangle tile: channels x W x H x N box)
+template <int CG>
+__device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap *map, uint32_t bar,
+                                            int c0, int c1, int c2, int c3) {
+  if constexpr (CG == 1) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(dst),
+        "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+        : "memory");
+  } else {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(dst),
+        "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+        : "memory");
+  }
+}
+
 // 2-SM form: lands in this CTA's smem, bytes counted on the leader's barrier.
 __device__ __forceinline__ void tma_im2col_2sm(uint32_t dst, const CUtensorMap *map,
                                                uint32_t bar, int c, int w, int h, int n,
@@ -144,6 +163,16 @@ __device__ __forceinline__ void tma_im2col_2sm(uint32_t dst, const CUtensorMap *
 }
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// one lane of a converged warp (the tcgen05 / TMA issue idiom): the loop
+// around it stays warp-uniform, so its values live in uniform registers
+__device__ __forceinline__ bool elect_one() {
+  uint32_t pred = 0;
+  asm volatile(
+      "{\n.reg .pred P;\nelect.sync _|P, 0xffffffff;\nselp.u32 %0, 1, 0, P;\n}"
+      : "=r"(pred));
+  return pred != 0;
 }
 
 __device__ __forceinline__ void tc_fence_before() {
@@ -295,6 +324,12 @@ struct TcArgs {
   int kblocks, kb_per_split;
   int stages;
   int slab_bytes;       // 128 / 64 / 32: A K-block = 128 / slab_bytes TMA slabs
+  // A addressing: rect_w == 0 -> TMA im2col over 128 consecutive output pixels;
+  // rect_w > 0 -> the M tile is a rect_n x rect_h x rect_w block of output
+  // pixels (<= 128) and each tap's A slab is one tiled 4-D TMA box at the
+  // tap-shifted input corner (stride 1; padding = OOB zero fill)
+  int rect_w, rect_h, rect_n;
+  int rects_w, rects_h;  // rect grid per image: ceil(Wo / rect_w), ceil(Ho / rect_h)
   int prof;             // 1: accumulate per-role barrier-wait cycles (debug)
   int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
@@ -451,6 +486,9 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   const int slab_bytes = a.slab_bytes;
   const int nslab = TC_ROW_BYTES / slab_bytes;
   const int slab_elems = slab_bytes / ESZ;
+  const bool rect = a.rect_w > 0;
+  const int rect_rows = rect ? a.rect_w * a.rect_h * a.rect_n : TC_BM;   // A rows loaded
+  const uint32_t a_bytes = (uint32_t)rect_rows * TC_ROW_BYTES;         // per stage
 
   uint32_t *ktab_s = (uint32_t *)(smem + SM_KTAB);
   const bool use_tab = a.ktab != nullptr;
@@ -525,15 +563,27 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         kb_range(sp, k0, k1);
         nkb += k1 - k0;
         const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
-        // input-space corner of this CTA's first output pixel
-        const int m0 = mt * (TC_BM * CG) + (int)rank * TC_BM;
-        const int n0 = m0 / HoWo, pq = m0 % HoWo;
-        const int w0 = (pq % g.Wo) * g.stride - g.pad, h0 = (pq / g.Wo) * g.stride - g.pad;
+        // input-space corner of this CTA's first output pixel (im2col) or of
+        // its output rectangle (rect mode)
+        int n0, w0, h0;
+        if (rect) {
+          const int ri = mt * CG + (int)rank;
+          const int rw = ri % a.rects_w, rt = ri / a.rects_w;
+          n0 = (rt / a.rects_h) * a.rect_n;
+          h0 = (rt % a.rects_h) * a.rect_h - g.pad;
+          w0 = rw * a.rect_w - g.pad;
+        } else {
+          const int m0 = mt * (TC_BM * CG) + (int)rank * TC_BM;
+          n0 = m0 / HoWo;
+          const int pq = m0 % HoWo;
+          w0 = (pq % g.Wo) * g.stride - g.pad;
+          h0 = (pq / g.Wo) * g.stride - g.pad;
+        }
         for (int kb = k0; kb < k1; ++kb) {
           wc.wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
           const uint32_t fb = sbase + SM_FULL + 8 * stage;
           if (rank == 0)
-            mbar_arrive_expect_tx(fb, CG * (((a.skip & 1) ? 0 : TC_A_STAGE) +
+            mbar_arrive_expect_tx(fb, CG * (((a.skip & 1) ? 0 : a_bytes) +
                                             ((a.skip & 2) ? 0 : b_stage)));
           const uint32_t dA = sA + stage * TC_A_STAGE;
           for (int sl = 0; sl < ((a.skip & 1) ? 0 : nslab); ++sl) {
@@ -550,7 +600,9 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
             }
             const int cc = c >= g.Cs ? g.Cs : grp * g.Cg + c;
             const uint32_t dst = dA + sl * (TC_BM * slab_bytes);
-            if constexpr (CG == 1)
+            if (rect)
+              tma_load_4d<CG>(dst, &tmap_x, fb, cc, w0 + s, h0 + r, n0);
+            else if constexpr (CG == 1)
               tma_im2col(dst, &tmap_x, fb, cc, w0, h0, n0, (uint16_t)s, (uint16_t)r);
             else
               tma_im2col_2sm(dst, &tmap_x, fb, cc, w0, h0, n0, (uint16_t)s, (uint16_t)r);
@@ -570,12 +622,24 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       }
     }
   } else if (warp == 1) {
-    if (lane == 0 && rank == 0) {
-      // ---------------------------------------------- MMA issuer (leader)
+    if (rank == 0) {
+      // ---------------------------------------------- MMA issuer (leader):
+      // the warp walks the schedule; one elected lane issues.  All descriptor
+      // arithmetic is hoisted: per K-block only stage offsets are added.
       const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
-      const int mma_per_slab = slab_bytes / 32;      // K = 32 B per UMMA
+      const uint64_t a_desc0 = umma_desc(sA, slab_bytes);
+      const uint64_t b_desc0 = umma_desc_sw128(sB);
+      uint32_t a_koff[4];              // 16 B units: slab base + K offset inside the slab
+      {
+        const int mma_per_slab = slab_bytes / 32;   // K = 32 B per UMMA
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          a_koff[k] = (uint32_t)((k / mma_per_slab) * (TC_BM * slab_bytes) / 16 +
+                                 2 * (k % mma_per_slab));
+      }
+      const uint32_t a_stage16 = TC_A_STAGE / 16, b_stage16 = b_stage / 16;
       uint32_t stage = 0, phase = 0, lt = 0;
-      WaitClock wfull{a.prof != 0}, wtemp{a.prof != 0};
+      WaitClock wfull{a.prof != 0 && lane == 0}, wtemp{a.prof != 0 && lane == 0};
       for (int u = pair; u < a.units; u += npairs, ++lt) {
         int mt, nt, grp, sp, k0, k1;
         decode(u, mt, nt, grp, sp);
@@ -587,21 +651,23 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         for (int kb = k0; kb < k1; ++kb) {
           wfull.wait(sbase + SM_FULL + 8 * stage, phase);
           tc_fence_after();
-          const uint32_t aS = sA + stage * TC_A_STAGE;
-          const uint64_t bd = umma_desc_sw128(sB + stage * b_stage);
+          const uint64_t ad = a_desc0 + stage * a_stage16;
+          const uint64_t bd = b_desc0 + stage * b_stage16;
+          if (elect_one()) {
+            if (!(a.skip & 4)) {
 #pragma unroll
-          for (int k = 0; k < 4; ++k) {   // 4 x 32 B of K per 128 B K-block
-            if (a.skip & 4) break;
-            const int sl = k / mma_per_slab, kin = k % mma_per_slab;
-            const uint64_t ad = umma_desc(aS + sl * (TC_BM * slab_bytes), slab_bytes) + 2 * kin;
-            tc_mma<ST, CG>(dcol, ad, bd + 2 * k, idesc, (kb > k0) || (k > 0));
+              for (int k = 0; k < 4; ++k)   // 4 x 32 B of K per 128 B K-block
+                tc_mma<ST, CG>(dcol, ad + a_koff[k], bd + 2 * k, idesc, (kb > k0) || (k > 0));
+            }
+            tc_commit<CG>(sbase + SM_EMPTY + 8 * stage);
           }
-          tc_commit<CG>(sbase + SM_EMPTY + 8 * stage);
+          __syncwarp();
           advance(stage, phase, stages);
         }
-        tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
+        if (elect_one()) tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
+        __syncwarp();
       }
-      if (a.prof) {
+      if (a.prof && lane == 0) {
         atomicAdd(&g_tc_prof[1], wfull.acc);
         atomicAdd(&g_tc_prof[2], wtemp.acc);
       }
@@ -627,8 +693,21 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       wtf.wait(sbase + SM_TFULL + 8 * buf, use & 1);
       if (wtf.on) tb = clock64();
       tc_fence_after();
-      const int m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
-      const bool mok = m < g.M;
+      int m;
+      bool mok;
+      if (rect) {
+        const int ri = mt * CG + (int)rank;
+        const int rw = ri % a.rects_w, rt = ri / a.rects_w;
+        const int wi = row % a.rect_w, hr = row / a.rect_w;
+        const int hi = hr % a.rect_h, ni = hr / a.rect_h;
+        const int n = (rt / a.rects_h) * a.rect_n + ni;
+        const int p = (rt % a.rects_h) * a.rect_h + hi, q = rw * a.rect_w + wi;
+        mok = row < rect_rows && q < g.Wo && p < g.Ho && n * HoWo < g.M;
+        m = (n * g.Ho + p) * g.Wo + q;
+      } else {
+        m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
+        mok = m < g.M;
+      }
       const size_t orow = (size_t)m * g.out_cs;
       if constexpr (LRN) {
         epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX, mok,
@@ -874,6 +953,11 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.kb_per_split = p.kb_per_split;
   args.stages = tc_stages_for(p.bn, p.cg);
   args.slab_bytes = tc_slab_bytes(st, g.Cg);
+  args.rect_w = p.rect_w;
+  args.rect_h = p.rect_h;
+  args.rect_n = p.rect_n;
+  args.rects_w = p.rect_w ? (g.Wo + p.rect_w - 1) / p.rect_w : 0;
+  args.rects_h = p.rect_w ? (g.Ho + p.rect_h - 1) / p.rect_h : 0;
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
   cudaError_t e;

@@ -84,6 +84,7 @@ struct TcPlan {
   int kb_per_split;
   int units;       // tiles * splits work units
   int grid;        // CTAs = cg * min(units, SM budget / cg)
+  int rect_w, rect_h, rect_n;  // 0 = im2col A tiles; else rectangle tiles (tiled TMA)
 };
 // Launches the GEMM and, when p.splits > 1, the deterministic split-K
 // reduction (ws must hold splits * M * out_cs floats; a split-K output must

@@ -15,6 +15,7 @@
 #include <memory>
 #include <mutex>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "../../include/pcnn.h"
@@ -106,7 +107,8 @@ struct GemmStage {           // one implicit-GEMM launch
   float *d_bias = nullptr;
   int *d_ktab = nullptr;     // per-element (r,s,c) table
   std::map<int, CUtensorMap> tmaps;  // weight maps by box rows
-  std::map<std::pair<const void *, int>, CUtensorMap> xmaps;   // im2col maps by (input, batch)
+  std::map<std::tuple<const void *, int, int, int, int>, CUtensorMap> xmaps;   // A maps by
+                                                 // (input, batch, rect w, h, n)
   size_t w_bytes = 0;
   void release() {
     if (d_w) cudaFree(d_w);
@@ -481,12 +483,10 @@ static const CUtensorMap *stage_tmap(GemmStage &gs, int rows) {
 }
 
 // TMA im2col map of a stage's NHWC input for `batch` images.
-static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch) {
-  const auto key = std::make_pair(x, batch);
+static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, const TcPlan &p) {
+  const auto key = std::make_tuple(x, batch, p.rect_w, p.rect_h, p.rect_n);
   auto it = gs.xmaps.find(key);
   if (it != gs.xmaps.end()) return &it->second;
-  auto enc = get_encode_im2col();
-  if (!enc) return nullptr;
   const ConvGeom &g = gs.g;
   const int esz = esz_of(gs.st);
   const int slab = tc_slab_bytes(gs.st, g.Cg);
@@ -495,6 +495,28 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch) {
                               (cuuint64_t)batch};
   const cuuint64_t strides[3] = {(cuuint64_t)g.Cs * esz, (cuuint64_t)g.W * g.Cs * esz,
                                  (cuuint64_t)g.H * g.W * g.Cs * esz};
+  if (p.rect_w > 0) {
+    // rectangle tiles: a plain tiled box per tap; OOB (padding, ragged rects,
+    // images past the batch) is zero-filled
+    auto enct = get_encode_tiled();
+    if (!enct) return nullptr;
+    const cuuint32_t box[4] = {(cuuint32_t)(slab / esz), (cuuint32_t)p.rect_w,
+                               (cuuint32_t)p.rect_h, (cuuint32_t)p.rect_n};
+    const cuuint32_t estr[4] = {1, 1, 1, 1};
+    const CUtensorMapSwizzle sw = slab == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                  : slab == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                               : CU_TENSOR_MAP_SWIZZLE_32B;
+    CUresult r = enct(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                           : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                      4, const_cast<void *>(x), dims, strides, box, estr,
+                      CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return nullptr;
+    if (gs.xmaps.size() > 64) gs.xmaps.clear();
+    return &(gs.xmaps[key] = m);
+  }
+  auto enc = get_encode_im2col();
+  if (!enc) return nullptr;
   // bounding box of the conv's input corners (square kernels: W and H equal)
   const int lower[2] = {-g.pad, -g.pad};
   const int upper[2] = {g.pad - (g.S - 1), g.pad - (g.S - 1)};
@@ -528,7 +550,35 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch) {
 // trade-off of P:223.  The plan depends on the problem shape and the device's
 // SM count only, never on the SM budget, so every budget runs the same tiles
 // and K order (bitwise-identical results, R11).
-static constexpr double kTmaCyclesPerRow = 3.6;
+// Measured on B200 (tools/tc_roles.py, PCNN_TC_SKIP / PCNN_AMODE experiments):
+// operand delivery is bound by L2->SM bandwidth (~10 TB/s chip, ~36 B/cycle
+// per SM) whether A comes by im2col or by tiled boxes, so one K-block costs
+// its operand bytes / 36 B per cycle; rectangle tiles only add padded MMA
+// rows and are therefore opt-in (PCNN_AMODE=rect).  The tcgen05 pipe sustains
+// ~80% of its nominal rate in this kernel.
+static constexpr double kOperandBytesPerCycle = 36.0;
+static constexpr double kMmaEfficiency = 0.8;
+
+// Best rectangle tile (w x h x n <= 128 output pixels) for rect-mode A loads,
+// maximising the fraction of useful MMA rows; {0,0,0} when not applicable.
+struct Rect { int w, h, n; double util; };
+static Rect best_rect(const ConvGeom &g) {
+  Rect best{0, 0, 0, 0.0};
+  if (g.stride != 1) return best;
+  const long long B = g.M / ((long long)g.Ho * g.Wo);
+  const int ws[] = {g.Wo, 8, 16, 32, 64, 128};
+  for (int w : ws) {
+    if (w < 1 || w > 128 || w > g.Wo) continue;
+    for (int h = std::min(128 / w, g.Ho); h >= 1; --h) {
+      // FC (1 x 1 "images"): the rectangle spans up to 128 images
+      const int n = (g.Ho == 1 && g.Wo == 1) ? (int)std::min<long long>(128, B) : 1;
+      const long long rects = ((B + n - 1) / n) * ((g.Ho + h - 1) / h) * ((g.Wo + w - 1) / w);
+      const double util = (double)g.M / ((double)rects * 128.0);
+      if (util > best.util + 1e-9) best = Rect{w, h, n, util};
+    }
+  }
+  return best;
+}
 
 static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
                       bool full_n = false) {
@@ -538,39 +588,53 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
   const double f = 1.9e9, hbm = 6.0e12;
   const double wbytes = (double)g.Nfg * g.groups * g.Kpad * esz;
   const char *force_cg = getenv("PCNN_FORCE_CG");
-  for (int cg = 1; cg <= 2; ++cg) {
-    if (force_cg && atoi(force_cg) != cg) continue;
-    const int mtiles = (g.M + 128 * cg - 1) / (128 * cg);
-    const int slots = device_sms / cg;          // concurrent units
-    for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {   // epilogue drains 32 columns
-      if (full_n && bn != round_up(g.Nfg, 32)) continue;      // one N tile (fused LRN)
-      const int ntiles = (g.Nfg + bn - 1) / bn;
-      const long long tiles = (long long)mtiles * ntiles * g.groups;
-      const double kb_cycles =
-          std::max(2.05 * bn, kTmaCyclesPerRow * (128.0 + (double)bn / cg)) + 40.0;
-      // split-K candidates: none, or any split that keeps >= 4 K-blocks per unit
-      const int max_split =
-          (tiles >= slots || full_n) ? 1 : std::min(16, std::max(1, kblocks / 4));
-      for (int want = 1; want <= max_split; ++want) {
-        const int kbs = (kblocks + want - 1) / want;
-        const int splits = (kblocks + kbs - 1) / kbs;
-        if (splits != want) continue;
-        const long long units = tiles * splits;
-        const long long waves = (units + slots - 1) / slots;
-        double t = (double)waves * kbs * kb_cycles / f + 2e-6;   // + per-tile drain
-        t = std::max(t, wbytes / hbm);
-        if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
-        if (t < best_t * 0.999 ||
-            (t <= best_t * 1.001 && (long long)bn * cg > (long long)best.bn * best.cg)) {
-          best_t = t;
-          best.cg = cg;
-          best.bn = bn;
-          best.mtiles = mtiles;
-          best.ntiles = ntiles;
-          best.tiles = (int)tiles;
-          best.splits = splits;
-          best.kb_per_split = kbs;
-          best.units = (int)units;
+  const char *force_bn = getenv("PCNN_FORCE_BN");          // tuning experiments
+  const char *force_am = getenv("PCNN_AMODE");             // "im2col" | "rect"
+  const Rect rc = best_rect(g);
+  for (int am = 0; am < 2; ++am) {            // 0 im2col, 1 rectangle tiles (opt-in)
+    if (am == 1 && (rc.w == 0 || !force_am || std::string(force_am) != "rect")) continue;
+    if (am == 0 && force_am && std::string(force_am) == "rect" && rc.w != 0) continue;
+    const long long rows_total = am ? (long long)std::llround(g.M / rc.util) : g.M;
+    const double a_bytes = 128.0 * (am ? rc.w * rc.h * rc.n : 128);
+    for (int cg = 1; cg <= 2; ++cg) {
+      if (force_cg && atoi(force_cg) != cg) continue;
+      const int mtiles = (int)((rows_total + 128LL * cg - 1) / (128LL * cg));
+      const int slots = device_sms / cg;          // concurrent units
+      for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {   // epilogue drains 32 columns
+        if (full_n && bn != round_up(g.Nfg, 32)) continue;      // one N tile (fused LRN)
+        if (force_bn && !full_n && atoi(force_bn) != bn) continue;
+        const int ntiles = (g.Nfg + bn - 1) / bn;
+        const long long tiles = (long long)mtiles * ntiles * g.groups;
+        const double load = (a_bytes + 128.0 * bn / cg) / kOperandBytesPerCycle;
+        const double mma = 2.05 * bn / kMmaEfficiency;
+        const double kb_cycles = std::max(load, mma) + 40.0;
+        // split-K candidates: none, or any split that keeps >= 4 K-blocks per unit
+        const int max_split =
+            (tiles >= slots || full_n) ? 1 : std::min(16, std::max(1, kblocks / 4));
+        for (int want = 1; want <= max_split; ++want) {
+          const int kbs = (kblocks + want - 1) / want;
+          const int splits = (kblocks + kbs - 1) / kbs;
+          if (splits != want) continue;
+          const long long units = tiles * splits;
+          const long long waves = (units + slots - 1) / slots;
+          double t = (double)waves * kbs * kb_cycles / f + 2e-6;   // + per-tile drain
+          t = std::max(t, wbytes / hbm);
+          if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
+          if (t < best_t * 0.999 ||
+              (t <= best_t * 1.001 && (long long)bn * cg > (long long)best.bn * best.cg)) {
+            best_t = t;
+            best.cg = cg;
+            best.bn = bn;
+            best.mtiles = mtiles;
+            best.ntiles = ntiles;
+            best.tiles = (int)tiles;
+            best.splits = splits;
+            best.kb_per_split = kbs;
+            best.units = (int)units;
+            best.rect_w = am ? rc.w : 0;
+            best.rect_h = am ? rc.h : 0;
+            best.rect_n = am ? rc.n : 0;
+          }
         }
       }
     }
@@ -623,7 +687,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
     }
     if (ws_need) *ws_need = std::max(*ws_need, p.splits > 1 ? (size_t)p.splits * g.M * g.out_cs * 4 : 0);
     if (!x) return PCNN_OK;   // planning only
-    const CUtensorMap *xm = stage_xmap(gs, x, B);
+    const CUtensorMap *xm = stage_xmap(gs, x, B, p);
     if (!xm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeIm2col failed");
     Budget b = make_budget(net, ly, slot, false);
     if (p.splits > 1 && (size_t)p.splits * g.M * g.out_cs * 4 > net->ws_bytes)
