@@ -121,6 +121,12 @@ typedef struct {
     double util;        /* eq. 6 with maxBlocks = n_sms * tlp                */
     double rec;         /* eq. 9 (tile-padding efficiency)                   */
     int splits;         /* split-K factor of the GEMM (1 = none)             */
+    int a_mode;         /* tcgen05 A-operand addressing: 0 = TMA im2col over
+                           output pixels, 1 = rectangle tiles (opt-in),
+                           2 = padded-layout shifted window (one TMA row
+                           window per filter row feeds all S taps)           */
+    int halo_in, halo_out; /* zero border of the stored input / output
+                           activation layouts ([B][H+2h][W+2h][C])           */
 } pcnn_layer_info;
 
 typedef struct pcnn_net pcnn_net;

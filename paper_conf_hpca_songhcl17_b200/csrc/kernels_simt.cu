@@ -240,7 +240,7 @@ stage_c3_kernel(const float *__restrict__ x, void *y, int H, int W, int Hs, int 
 template <int ST, int S>
 __global__ void __launch_bounds__(256)
 stage_im2col_kernel(const float *__restrict__ x, void *y, int H, int W, int Ho, int Wo, int Kp,
-                    int st, int pad, int tf32_round) {
+                    int st, int pad, int halo, int tf32_round) {
   constexpr int C = 3, K = S * S * C;
   constexpr int VN = Vec16<ST>::N;
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
@@ -262,7 +262,10 @@ stage_im2col_kernel(const float *__restrict__ x, void *y, int H, int W, int Ho, 
   }
   asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
   __syncthreads();
-  char *yrow = (char *)y + ((size_t)(n * Ho + p) * Wo) * Kp * ESZ;
+  // rows of a zero-haloed output grid (Ho + 2 halo) x (Wo + 2 halo): the
+  // interior only (the consumer never reads the halo rows of a 1x1 conv)
+  const int Wop = Wo + 2 * halo;
+  char *yrow = (char *)y + ((size_t)(n * (Ho + 2 * halo) + p + halo) * Wop + halo) * Kp * ESZ;
   for (int q = threadIdx.x; q < Wo; q += blockDim.x) {
     float v[K];
 #pragma unroll
@@ -286,13 +289,13 @@ stage_im2col_kernel(const float *__restrict__ x, void *y, int H, int W, int Ho, 
 
 cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, int H, int W,
                                 int S, int stride, int pad, int Ho, int Wo, int Kp,
-                                int tf32_round, cudaStream_t s) {
+                                int halo, int tf32_round, cudaStream_t s) {
   if (C != 3 || (S != 3 && S != 5)) return cudaErrorInvalidValue;
   const size_t smem = (size_t)S * C * ((Wo - 1) * stride + S) * sizeof(float);
   if (smem > 48 * 1024) return cudaErrorInvalidValue;
   const unsigned grid = (unsigned)((long long)B * Ho);
 #define PCNN_IM2COL(STT, SS) \
-  stage_im2col_kernel<STT, SS><<<grid, 256, smem, s>>>(x, y, H, W, Ho, Wo, Kp, stride, pad, tf32_round)
+  stage_im2col_kernel<STT, SS><<<grid, 256, smem, s>>>(x, y, H, W, Ho, Wo, Kp, stride, pad, halo, tf32_round)
   if (st == ST_BF16) {
     if (S == 3) PCNN_IM2COL(ST_BF16, 3); else PCNN_IM2COL(ST_BF16, 5);
   } else {
@@ -525,6 +528,7 @@ struct LrnPoolArgs {
   int Cout;                // stored output channels
   int ocg, ocp;            // output group layout: ocg real channels padded to
                            // ocp per group (0 = compact, Cout == C)
+  int hi, ho;              // zero halo of the input / output layout (pixels per side)
   Budget b;
 };
 
@@ -550,6 +554,28 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
     const int h0 = p * a.s, h1 = min(h0 + a.k, a.H);
     const int w0 = q0 * a.s, w1 = min((q1 - 1) * a.s + a.k, a.W);
     const int nr = h1 - h0, wc = w1 - w0;
+    const int Hp = a.H + 2 * a.hi, Wp = a.W + 2 * a.hi;          // stored input grid
+    const int Hop = a.Ho + 2 * a.ho, Wop = a.Wo + 2 * a.ho;      // stored output grid
+    if (a.ho > 0) {
+      // halo output: the edge tiles zero the border cells of their image
+      // (top rows with row 0, bottom rows with the last row, the left / right
+      // columns of this output row with the first / last column tile)
+      const int oc16 = a.Cout * ESZ / 16;
+      const uint4 z = make_uint4(0, 0, 0, 0);
+      uint4 *yb = (uint4 *)a.y;
+      for (int e = 0; e < 2; ++e)
+        if (qt == 0 && p == (e == 0 ? 0 : a.Ho - 1)) {
+          const int r0 = e == 0 ? 0 : a.Ho + a.ho;
+          const size_t base = ((size_t)n * Hop + r0) * Wop * oc16;
+          for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x) yb[base + v] = z;
+        }
+      const size_t rowb = ((size_t)n * Hop + p + a.ho) * Wop * oc16;
+      if (qt == 0)
+        for (int v = threadIdx.x; v < a.ho * oc16; v += blockDim.x) yb[rowb + v] = z;
+      if (qt == a.nqt - 1)
+        for (int v = threadIdx.x; v < a.ho * oc16; v += blockDim.x)
+          yb[rowb + (size_t)(a.Wo + a.ho) * oc16 + v] = z;
+    }
     __syncthreads();
     // stage rows [h0, h1) x cols [w0, w1): each row segment is contiguous;
     // cp.async keeps every 16 B load of the tile in flight at once
@@ -559,7 +585,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
     for (int v = threadIdx.x; v < nr * vec_per_row; v += blockDim.x) {
       int r, rem;
       fdivmod(v, vec_per_row, inv_vpr, r, rem);
-      const size_t src = (((size_t)n * a.H + h0 + r) * a.W + w0) * C + (size_t)rem * VN;
+      const size_t src = (((size_t)n * Hp + h0 + r + a.hi) * Wp + w0 + a.hi) * C + (size_t)rem * VN;
       const uint32_t dst = tbase + (uint32_t)(((size_t)r * wc_max * C + (size_t)rem * VN) * ESZ);
       asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst),
                    "l"((const char *)a.x + src * ESZ)
@@ -629,7 +655,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
       Vec16<ST> acc, cur;
 #pragma unroll
       for (int j = 0; j < VN; ++j) acc.v[j] = pad ? 0.f : (a.is_max ? -INFINITY : 0.f);
-      char *dst = (char *)a.y + ((((size_t)n * a.Ho + p) * a.Wo + q) * a.Cout + oc * VN) * ESZ;
+      char *dst = (char *)a.y + ((((size_t)n * Hop + p + a.ho) * Wop + q + a.ho) * a.Cout + oc * VN) * ESZ;
       if (ST == ST_BF16 && a.is_max && !pad) {
         // max is exact in bf16: compare packed pairs, no conversions
         const int cs = q * a.s - w0, ce = min(cs + a.k, wc);
@@ -716,7 +742,8 @@ long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int
 cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int B, int H, int W,
                             int C, int lrn_size, float alpha, float beta, float kk, int k,
                             int s, int is_max, int Ho, int Wo, int out_groups, int out_cg_pad,
-                            const Budget &b, int grid, cudaStream_t stream) {
+                            int in_halo, int out_halo, const Budget &b, int grid,
+                            cudaStream_t stream) {
   const int vn = st == ST_BF16 ? 8 : 4;
   if (C % vn) return cudaErrorInvalidValue;
   const int ocg = out_groups > 0 ? C / out_groups : 0;
@@ -745,6 +772,8 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.ocg = ocg;
   a.ocp = ocp;
   a.Cout = out_groups > 0 ? out_groups * ocp : C;
+  a.hi = in_halo;
+  a.ho = out_halo;
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
   const size_t smem = (size_t)k * ((a.Q - 1) * s + k) * C * esz * (lrn_size > 0 ? 2 : 1);

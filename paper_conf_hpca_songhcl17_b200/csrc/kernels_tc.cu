@@ -65,7 +65,10 @@ constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_STAGES;
 constexpr int SM_TFULL = SM_EMPTY + 8 * TC_MAX_STAGES;
 constexpr int SM_TEMPTY = SM_TFULL + 16;
 constexpr int SM_TMEMPTR = SM_TEMPTY + 16;
-constexpr int SM_KTAB = SM_BAR + 256;
+constexpr int TC_MAX_ASTAGES = 4;       // padded mode: A row-window ring
+constexpr int SM_AFULL = SM_TMEMPTR + 16;
+constexpr int SM_AEMPTY = SM_AFULL + 8 * TC_MAX_ASTAGES;
+constexpr int SM_KTAB = SM_BAR + 512;
 constexpr int SM_EPI = SM_KTAB + 4 * TC_MAX_KTAB;        // 4 warps x 32 rows x 144 B
 constexpr int SM_TOTAL = SM_EPI + 8 * EPI_WARP_BYTES;
 constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
@@ -73,6 +76,22 @@ constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
 size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
 int tc_max_ktab() { return TC_MAX_KTAB; }
 int tc_block_k_elems(int st) { return st == ST_BF16 ? 64 : 32; }
+// Padded mode: one A stage is the (128 + 2 pad)-row window of one filter row
+// r and channel slab; one B stage is the weight slab of one tap (r, s).
+static int pm_a_stage_bytes(int slab_bytes, int S) {
+  return ((TC_BM + (S - 1)) * slab_bytes + 1023) / 1024 * 1024;
+}
+void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int *a_stages, int *b_stages) {
+  const int as_bytes = pm_a_stage_bytes(slab_bytes, S);
+  const int bs_bytes = bn / cg * slab_bytes;
+  int na = TC_MAX_ASTAGES;
+  while (na > 2 && na * as_bytes + 2 * S * bs_bytes > TC_STAGE_BUDGET) --na;
+  int nb = (TC_STAGE_BUDGET - na * as_bytes) / bs_bytes;
+  if (nb > TC_MAX_STAGES) nb = TC_MAX_STAGES;
+  *a_stages = na;
+  *b_stages = nb;
+}
+
 int tc_stages_for(int bn, int cg) {
   const int per = TC_A_STAGE + bn / cg * TC_ROW_BYTES;
   int n = TC_STAGE_BUDGET / per;
@@ -332,6 +351,7 @@ struct TcArgs {
   int rects_w, rects_h;  // rect grid per image: ceil(Wo / rect_w), ceil(Ho / rect_h)
   int prof;             // 1: accumulate per-role barrier-wait cycles (debug)
   int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
+  int a_stages, b_stages, pm_a_stage;   // padded mode rings (g.pm)
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
   float lrn_a_over_n, lrn_beta, lrn_k;
   Budget b;
@@ -500,9 +520,13 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     }
   }
   if (tid == 0) {
-    for (int s = 0; s < stages; ++s) {
+    for (int s = 0; s < (g.pm ? a.b_stages : stages); ++s) {
       mbar_init(sbase + SM_FULL + 8 * s, 1);
       mbar_init(sbase + SM_EMPTY + 8 * s, 1);
+    }
+    for (int s = 0; s < (g.pm ? a.a_stages : 0); ++s) {
+      mbar_init(sbase + SM_AFULL + 8 * s, 1);
+      mbar_init(sbase + SM_AEMPTY + 8 * s, 1);
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(sbase + SM_TFULL + 8 * i, 1);
@@ -549,7 +573,108 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     k1 = min(a.kblocks, k0 + a.kb_per_split);
   };
 
-  if (warp == 0) {
+  // padded mode: K runs over (channel slab cb, filter row r) windows, each
+  // feeding the S taps (r, s) of that row by shifting the A descriptor s rows
+  const int pm_se = slab_bytes / ESZ;                  // channels per slab
+  const int pm_nj = g.pm ? (g.Cg / pm_se) * g.S : 0;   // A windows per tile
+  const uint32_t sBp = sbase + (uint32_t)a.a_stages * (uint32_t)a.pm_a_stage;
+  const uint32_t pm_b_bytes = (uint32_t)b_rows * slab_bytes;
+  if (warp == 0 && g.pm) {
+    // ------------------------------------------------ TMA producer, padded mode
+    if (lane == 0) {
+      asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
+      asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
+      const uint32_t pm_a_bytes = (uint32_t)(TC_BM + 2 * g.pad) * slab_bytes;
+      uint32_t as = 0, aph = 0, bs = 0, bph = 0;
+      WaitClock wc{a.prof != 0};
+      unsigned long long nkb = 0;
+      for (int u = pair; u < a.units; u += npairs) {
+        int mt, nt, grp, sp;
+        decode(u, mt, nt, grp, sp);
+        nkb += pm_nj;
+        const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
+        const int i0 = mt * (TC_BM * CG) + (int)rank * TC_BM;
+        int cb = 0, r = 0;
+        for (int j = 0; j < pm_nj; ++j) {
+          wc.wait(sbase + SM_AEMPTY + 8 * as, aph ^ 1);
+          const uint32_t fa = sbase + SM_AFULL + 8 * as;
+          if (rank == 0) mbar_arrive_expect_tx(fa, (a.skip & 1) ? 0 : CG * pm_a_bytes);
+          if (!(a.skip & 1)) {
+            const uint32_t dA = sA + as * (uint32_t)a.pm_a_stage;
+            const int cc = grp * g.Cg + cb * pm_se, row = i0 + (r - g.pad) * g.wv - g.pad;
+            if constexpr (CG == 1) tma_load_2d(dA, &tmap_x, fa, cc, row);
+            else tma_load_2d_2sm(dA, &tmap_x, fa, cc, row);
+          }
+          advance(as, aph, a.a_stages);
+          for (int s2 = 0; s2 < g.S; ++s2) {
+            wc.wait(sbase + SM_EMPTY + 8 * bs, bph ^ 1);
+            const uint32_t fb = sbase + SM_FULL + 8 * bs;
+            if (rank == 0) mbar_arrive_expect_tx(fb, (a.skip & 2) ? 0 : CG * pm_b_bytes);
+            if (!(a.skip & 2)) {
+              const int kk = (r * g.S + s2) * g.Cg + cb * pm_se;
+              if constexpr (CG == 1) tma_load_2d(sBp + bs * pm_b_bytes, &tmap_w, fb, kk, nrow);
+              else tma_load_2d_2sm(sBp + bs * pm_b_bytes, &tmap_w, fb, kk, nrow);
+            }
+            advance(bs, bph, a.b_stages);
+          }
+          if (++r == g.S) { r = 0; ++cb; }
+        }
+      }
+      if (a.prof) {
+        atomicAdd(&g_tc_prof[0], wc.acc);
+        atomicAdd(&g_tc_prof[5], nkb);
+      }
+    }
+  } else if (warp == 1 && g.pm) {
+    if (rank == 0) {
+      // ---------------------------------------------- MMA issuer, padded mode
+      const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
+      const uint64_t a_desc0 = umma_desc(sA, slab_bytes);
+      const uint64_t b_desc0 = umma_desc(sBp, slab_bytes);
+      const uint32_t a_st16 = (uint32_t)a.pm_a_stage / 16, b_st16 = pm_b_bytes / 16;
+      const uint32_t row16 = (uint32_t)slab_bytes / 16;   // one A row = one tap shift
+      const int kmma = slab_bytes / 32;                     // UMMAs per slab row (K = 32 B)
+      uint32_t as = 0, aph = 0, bs = 0, bph = 0, lt = 0;
+      WaitClock wfull{a.prof != 0 && lane == 0}, wtemp{a.prof != 0 && lane == 0};
+      for (int u = pair; u < a.units; u += npairs, ++lt) {
+        const uint32_t buf = lt & 1, use = lt >> 1;
+        wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
+        for (int j = 0; j < pm_nj; ++j) {
+          wfull.wait(sbase + SM_AFULL + 8 * as, aph);
+          tc_fence_after();
+          const uint64_t ad = a_desc0 + as * a_st16;
+          for (int s2 = 0; s2 < g.S; ++s2) {
+            wfull.wait(sbase + SM_FULL + 8 * bs, bph);
+            tc_fence_after();
+            const uint64_t bd = b_desc0 + bs * b_st16;
+            if (elect_one()) {
+              if (!(a.skip & 4)) {
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+                  if (k < kmma)
+                    tc_mma<ST, CG>(dcol, ad + s2 * row16 + 2 * k, bd + 2 * k, idesc,
+                                   (j > 0) || (s2 > 0) || (k > 0));
+              }
+              tc_commit<CG>(sbase + SM_EMPTY + 8 * bs);
+            }
+            __syncwarp();
+            advance(bs, bph, a.b_stages);
+          }
+          if (elect_one()) tc_commit<CG>(sbase + SM_AEMPTY + 8 * as);
+          __syncwarp();
+          advance(as, aph, a.a_stages);
+        }
+        if (elect_one()) tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
+        __syncwarp();
+      }
+      if (a.prof && lane == 0) {
+        atomicAdd(&g_tc_prof[1], wfull.acc);
+        atomicAdd(&g_tc_prof[2], wtemp.acc);
+      }
+    }
+  } else if (warp == 0) {
     // ------------------------------------------------ TMA producer (A im2col + B)
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
@@ -708,6 +833,13 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
         mok = m < g.M;
       }
+      bool valid = true;      // padded mode: halo rows are stored as zeros
+      if (g.pm) {
+        const int hvwv = g.hv * g.wv;
+        const int ni = m / hvwv, rem = m - ni * hvwv;
+        const int pv = rem / g.wv, qv = rem - pv * g.wv;
+        valid = pv >= g.vh && pv < g.vh + g.Ho && qv >= g.vh && qv < g.vh + g.Wo;
+      }
       const size_t orow = (size_t)m * g.out_cs;
       if constexpr (LRN) {
         epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX, mok,
@@ -761,6 +893,9 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           if (g.relu)
 #pragma unroll
             for (int i = 0; i < 64; ++i) f[i] = fmaxf(f[i], 0.f);
+          if (!valid)
+#pragma unroll
+            for (int i = 0; i < 64; ++i) f[i] = 0.f;
         }
         uint4 pc[8];
         if (out16) {
@@ -958,8 +1093,15 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.rect_n = p.rect_n;
   args.rects_w = p.rect_w ? (g.Wo + p.rect_w - 1) / p.rect_w : 0;
   args.rects_h = p.rect_w ? (g.Ho + p.rect_h - 1) / p.rect_h : 0;
+  args.a_stages = p.a_stages;
+  args.b_stages = p.b_stages;
+  args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, g.S) : 0;
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
+  if (g.pm && (p.splits != 1 || lrn || p.rect_w || g.stride != 1 || g.S != 2 * g.pad + 1 ||
+               g.Cg % (args.slab_bytes / (st == ST_BF16 ? 2 : 4)) || p.a_stages < 2 ||
+               p.b_stages < 2 || p.a_stages > TC_MAX_ASTAGES || p.b_stages > TC_MAX_STAGES))
+    return cudaErrorInvalidValue;
   cudaError_t e;
   const bool L = args.lrn != 0;
   if (st == ST_BF16)

@@ -48,6 +48,14 @@ struct ConvGeom {
   int Kpad;         // K rounded up to the kernel's K-block
   int relu;
   int out_mode;     // OutMode
+  // padded-layout ("shifted window") mode, tcgen05 only (pm = 1): input and
+  // output share one zero-haloed grid hv x wv = (H + 2 vh) x (W + 2 vh) per
+  // image, M = B*hv*wv virtual rows, and the A rows of tap (r, s) for output
+  // row i are input rows i + (r - pad)*wv + (s - pad).  Rows outside the
+  // valid window [vh, vh + Ho) x [vh, vh + Wo) are written as zeros (they are
+  // the next layer's padding).  Requires stride 1 and S == 2*pad + 1.
+  int pm;
+  int hv, wv, vh;
 };
 
 // ---------------------------------------------------------------- launchers
@@ -59,10 +67,11 @@ cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C,
                                int H, int W, int Hs, int Ws, int Cs, int blk,
                                int pad, int tf32_round, cudaStream_t s);
 // a1 for a first conv with 3 input channels and S*S*3 <= 128: writes the
-// conv's im2col rows [B][Ho][Wo][Kp] so the conv runs as a 1x1 conv.
+// conv's im2col rows [B][Ho + 2h][Wo + 2h][Kp] (interior of a halo-h grid;
+// h = 0: compact) so the conv runs as a 1x1 conv.
 cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, int H,
                                 int W, int S, int stride, int pad, int Ho, int Wo,
-                                int Kp, int tf32_round, cudaStream_t s);
+                                int Kp, int halo, int tf32_round, cudaStream_t s);
 // final NHWC storage -> NCHW fp32 flatten
 cudaError_t launch_unstage_output(const void *x, int st, float *y, int B,
                                   int C, int H, int W, int Cs, cudaStream_t s);
@@ -85,6 +94,7 @@ struct TcPlan {
   int units;       // tiles * splits work units
   int grid;        // CTAs = cg * min(units, SM budget / cg)
   int rect_w, rect_h, rect_n;  // 0 = im2col A tiles; else rectangle tiles (tiled TMA)
+  int a_stages, b_stages;      // padded mode: A (row-window) and B (tap slab) ring depths
 };
 // Launches the GEMM and, when p.splits > 1, the deterministic split-K
 // reduction (ws must hold splits * M * out_cs floats; a split-K output must
@@ -102,6 +112,8 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
 // group width is not a multiple of 32 bytes.
 int tc_slab_bytes(int st, int cg_channels);
 int tc_stages_for(int bn, int cg);
+// padded mode: ring depths for an N tile, CTA grouping, slab width and kernel size
+void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int *a_stages, int *b_stages);
 // debug: per-role barrier-wait cycle totals accumulated while PCNN_TC_PROFILE=1
 cudaError_t tc_profile(int reset, unsigned long long out[8]);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)
@@ -113,12 +125,15 @@ int tc_max_ktab();
 // 1 for no pooling), NHWC with C stored input channels.  out_groups > 0
 // writes the output with each of the out_groups channel groups padded to
 // out_cg_pad channels (zeros), the layout a following grouped conv loads
-// with full 128-byte TMA slabs.
+// with full 128-byte TMA slabs.  in_halo / out_halo: zero border width of
+// the input / output layouts ([B][H + 2h][W + 2h][C]); the kernel writes the
+// output border zeros itself.
 cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int B,
                             int H, int W, int C, int lrn_size, float alpha,
                             float beta, float kk, int k, int s, int is_max,
                             int Ho, int Wo, int out_groups, int out_cg_pad,
-                            const Budget &b, int grid, cudaStream_t stream);
+                            int in_halo, int out_halo, const Budget &b, int grid,
+                            cudaStream_t stream);
 long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s,
                          int Ho, int Wo);
 int lrn_pool_occupancy(int st);

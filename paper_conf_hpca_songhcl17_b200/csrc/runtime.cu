@@ -136,6 +136,9 @@ struct Layer {
   // budget
   int n_sms = 0, tlp = 0;
   int out_groups = 0, out_cg_pad = 0;    // padded-group output layout (lrn/pool)
+  // zero border (halo) of the stored input / output activation; pm_halo > 0:
+  // this conv runs in padded-layout mode (ConvGeom::pm) with that halo
+  int in_halo = 0, out_halo = 0, pm_halo = 0;
   unsigned long long *d_ctr = nullptr;   // 3 launch slots x (1 + kMaxSMs)
   unsigned int *d_census = nullptr;      // 8 words
 };
@@ -386,7 +389,8 @@ static int k_align(int precision) {
 static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, int Nf,
                                int groups, int S, int stride, int pad, int relu,
                                int in_c, int in_h, int in_w, int in_cs, bool is_fc,
-                               const float *w, const float *bias, int out_mode) {
+                               const float *w, const float *bias, int out_mode,
+                               int pm_halo = 0) {
   gs.release();
   gs.st = storage_of(precision);
   gs.engine = precision == PCNN_FP32_SIMT ? 0 : 1;
@@ -429,6 +433,14 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
     g.Nfg = Nf / groups;
     g.K = S * S * Cg_st;
     g.Kpad = round_up(g.K, k_align(precision));
+    if (pm_halo > 0) {
+      if (gs.engine != 1 || stride != 1 || S != 2 * pad + 1 || pad > pm_halo)
+        return fail(PCNN_ERR_UNSUPPORTED, "padded-layout mode needs a stride-1 'same' conv");
+      g.pm = 1;
+      g.vh = pm_halo;
+      g.hv = in_h + 2 * pm_halo;
+      g.wv = in_w + 2 * pm_halo;
+    }
     packed = pack_conv(w, Nf, Cg_log, Cg_st, S, g.Kpad);
     if (S > 1) {
       if (gs.engine == 1 && g.Kpad / ch > tc_max_ktab())
@@ -462,9 +474,11 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
   return PCNN_OK;
 }
 
-static const CUtensorMap *stage_tmap(GemmStage &gs, int rows) {
+// Weight (B operand) map: boxes of `rows` filters x `slab` bytes of K.
+static const CUtensorMap *stage_tmap(GemmStage &gs, int rows, int slab = 128) {
   const int bn = rows;
-  auto it = gs.tmaps.find(bn);
+  const int key = rows * 1024 + slab;
+  auto it = gs.tmaps.find(key);
   if (it != gs.tmaps.end()) return &it->second;
   auto enc = get_encode_tiled();
   if (!enc) return nullptr;
@@ -472,14 +486,16 @@ static const CUtensorMap *stage_tmap(GemmStage &gs, int rows) {
   const int esz = esz_of(gs.st);
   const cuuint64_t dims[2] = {(cuuint64_t)gs.g.Kpad, (cuuint64_t)gs.g.Nfg * gs.g.groups};
   const cuuint64_t strides[1] = {(cuuint64_t)gs.g.Kpad * esz};
-  const cuuint32_t box[2] = {(cuuint32_t)(128 / esz), (cuuint32_t)bn};
+  const cuuint32_t box[2] = {(cuuint32_t)(slab / esz), (cuuint32_t)bn};
   const cuuint32_t estr[2] = {1, 1};
+  const CUtensorMapSwizzle sw = slab == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                : slab == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                             : CU_TENSOR_MAP_SWIZZLE_32B;
   CUresult r = enc(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
                    2, gs.d_w, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return nullptr;
-  return &(gs.tmaps[bn] = m);
+  return &(gs.tmaps[key] = m);
 }
 
 // TMA im2col map of a stage's NHWC input for `batch` images.
@@ -491,6 +507,27 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, co
   const int esz = esz_of(gs.st);
   const int slab = tc_slab_bytes(gs.st, g.Cg);
   CUtensorMap m;
+  if (g.pm) {
+    // padded layout: the input is a plain [B*hv*wv][Cs] matrix; a box is the
+    // (128 + S - 1)-row window of one filter row (rows outside the tensor --
+    // the first / last window of the batch -- are zero-filled)
+    auto enct = get_encode_tiled();
+    if (!enct) return nullptr;
+    const cuuint64_t d2[2] = {(cuuint64_t)g.Cs, (cuuint64_t)batch * g.hv * g.wv};
+    const cuuint64_t s2[1] = {(cuuint64_t)g.Cs * esz};
+    const cuuint32_t box[2] = {(cuuint32_t)(slab / esz), (cuuint32_t)(128 + g.S - 1)};
+    const cuuint32_t estr[2] = {1, 1};
+    const CUtensorMapSwizzle sw = slab == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                  : slab == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                               : CU_TENSOR_MAP_SWIZZLE_32B;
+    CUresult r = enct(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                           : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                      2, const_cast<void *>(x), d2, s2, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                      sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return nullptr;
+    if (gs.xmaps.size() > 64) gs.xmaps.clear();
+    return &(gs.xmaps[key] = m);
+  }
   const cuuint64_t dims[4] = {(cuuint64_t)g.Cs, (cuuint64_t)g.W, (cuuint64_t)g.H,
                               (cuuint64_t)batch};
   const cuuint64_t strides[3] = {(cuuint64_t)g.Cs * esz, (cuuint64_t)g.W * g.Cs * esz,
@@ -642,6 +679,50 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
   return best;
 }
 
+// Padded-layout plan: per (slab, filter row) window the SM loads
+// (128 + S - 1) A rows once plus S weight slabs and issues S x slab/32 UMMAs;
+// no split-K (a split would need the halo zeroing in the reduction).
+static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz) {
+  TcPlan best{};
+  double best_t = 1e300;
+  const int nmax = std::min(256, round_up(g.Nfg, 32));
+  const double f = 1.9e9;
+  const int slab = tc_slab_bytes(esz == 2 ? ST_BF16 : ST_F32, g.Cg);
+  const int nj = g.Cg * esz / slab * g.S;
+  const char *force_cg = getenv("PCNN_FORCE_CG");
+  const char *force_bn = getenv("PCNN_FORCE_BN");
+  for (int cg = 1; cg <= 2; ++cg) {
+    if (force_cg && atoi(force_cg) != cg) continue;
+    const int mtiles = (int)(((long long)g.M + 128LL * cg - 1) / (128LL * cg));
+    const int slots = device_sms / cg;
+    for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {
+      if (force_bn && atoi(force_bn) != bn) continue;
+      const int ntiles = (g.Nfg + bn - 1) / bn;
+      const long long tiles = (long long)mtiles * ntiles * g.groups;
+      const double load = ((128.0 + g.S - 1) * slab + (double)g.S * slab * bn / cg) /
+                          kOperandBytesPerCycle;
+      const double mma = g.S * (slab / 128.0) * 2.05 * bn / kMmaEfficiency;
+      const double j_cycles = std::max(load, mma) + 40.0;
+      const long long waves = (tiles + slots - 1) / slots;
+      const double t = (double)waves * nj * j_cycles / f + 2e-6;
+      if (t < best_t * 0.999 ||
+          (t <= best_t * 1.001 && (long long)bn * cg > (long long)best.bn * best.cg)) {
+        best_t = t;
+        best.cg = cg;
+        best.bn = bn;
+        best.mtiles = mtiles;
+        best.ntiles = ntiles;
+        best.tiles = (int)tiles;
+        best.splits = 1;
+        best.kb_per_split = nj;
+        best.units = (int)tiles;
+      }
+    }
+  }
+  tc_pm_stages(best.bn, best.cg, slab, g.S, &best.a_stages, &best.b_stages);
+  return best;
+}
+
 static int effective_sms(const pcnn_net *net, const Layer &ly) {
   int n = ly.n_sms <= 0 ? net->num_sms : std::min(ly.n_sms, net->num_sms);
   return std::max(n, 1);
@@ -666,14 +747,18 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
                              void *y, int slot, cudaStream_t s, pcnn_layer_info *info,
                              size_t *ws_need = nullptr, const float *lrn = nullptr) {
   ConvGeom g = gs.g;
-  g.M = B * g.Ho * g.Wo;
+  g.M = g.pm ? B * g.hv * g.wv : B * g.Ho * g.Wo;
   if (gs.engine == 1) {
-    TcPlan p = plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st),
-                       lrn != nullptr);
+    if (g.pm && lrn) return fail(PCNN_ERR_UNSUPPORTED, "LRN fusion in padded-layout mode");
+    TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st))
+                    : plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st),
+                              lrn != nullptr);
     // the budget caps concurrent units; a CTA pair needs at least 2 SMs
     const int slots = std::max(1, effective_sms(net, ly) / p.cg);
     p.grid = p.cg * std::min(p.units, slots);
-    const CUtensorMap *tm = stage_tmap(gs, p.bn / p.cg);   // weight rows per CTA
+    // weight rows per CTA; padded mode loads one tap's slab per stage
+    const CUtensorMap *tm =
+        stage_tmap(gs, p.bn / p.cg, g.pm ? tc_slab_bytes(gs.st, g.Cg) : 128);
     if (!tm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeTiled failed");
     if (info) {
       info->tile_m = 128 * p.cg;
@@ -683,6 +768,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->tlp = 1;
       info->engine = 1;
       info->splits = p.splits;
+      info->a_mode = g.pm ? 2 : (p.rect_w ? 1 : 0);
       info->n_sms = std::max(info->n_sms, p.grid);   // pair granularity
     }
     if (ws_need) *ws_need = std::max(*ws_need, p.splits > 1 ? (size_t)p.splits * g.M * g.out_cs * 4 : 0);
@@ -770,7 +856,7 @@ static pcnn_status run_lrn_pool(pcnn_net *net, int li, int pi, int B, const void
   const Layer &last = net->layers[pi >= 0 ? pi : li];
   CUDA_TRY(counted(launch_lrn_pool(x, y, net->st, net->desc.precision == PCNN_TF32, B, H, W, C,
                                    lrn, alpha, beta, kk, k, st, is_max, Ho, Wo, last.out_groups,
-                                   last.out_cg_pad, b, grid, s)));
+                                   last.out_cg_pad, ly.in_halo, last.out_halo, b, grid, s)));
   return PCNN_OK;
 }
 
@@ -815,7 +901,7 @@ static pcnn_status enqueue_all(pcnn_net *net, const float *d_images, int B, floa
     CUDA_TRY(counted(launch_stage_im2col(d_images, net->d_act[0], st, B, net->desc.in_channels,
                                          net->desc.in_height, net->desc.in_width, l0.d.kernel,
                                          l0.d.stride, l0.d.pad, l0.out_h, l0.out_w, net->in_cs,
-                                         tf32, s)));
+                                         l0.in_halo, tf32, s)));
   } else {
     CUDA_TRY(counted(launch_stage_input(d_images, net->d_act[0], st, B, net->desc.in_channels,
                                         net->desc.in_height, net->desc.in_width, net->stage_h,
@@ -893,13 +979,15 @@ static pcnn_status build_rank_stages(pcnn_net *net, Layer &ly, int r, const floa
       for (int a = 0; a < r; ++a)
         w2[((size_t)gi * Nfg + f) * rs + a] = A[((size_t)gi * Nfg + f) * r + a];
   const int mode1 = st == ST_BF16 ? OUT_BF16 : (prec == PCNN_TF32 ? OUT_F32_TF32 : OUT_F32);
+  // a padded-layout layer keeps its halo grid through both stages
   pcnn_status s1 = build_stage(ly.r1, ly, prec, g * rs, g, S, d.stride, d.pad, 0, ly.in_c,
-                               ly.in_h, ly.in_w, ly.in_cs, false, w1.data(), nullptr, mode1);
+                               ly.in_h, ly.in_w, ly.in_cs, false, w1.data(), nullptr, mode1,
+                               ly.pm_halo);
   if (s1 != PCNN_OK) return s1;
   const int ho = ly.out_h, wo = ly.out_w;
   const GemmStage &ex = ly.exact;
   pcnn_status s2 = build_stage(ly.r2, ly, prec, d.out_channels, g, 1, 1, 0, d.relu, g * rs, ho,
-                               wo, g * rs, false, w2.data(), nullptr, ex.g.out_mode);
+                               wo, g * rs, false, w2.data(), nullptr, ex.g.out_mode, ly.pm_halo);
   if (s2 != PCNN_OK) return s2;
   // stage 2 carries the layer's bias: copy it from the exact stage.
   CUDA_TRY(cudaMemcpy(ly.r2.d_bias, ex.d_bias, sizeof(float) * d.out_channels,
@@ -1111,11 +1199,66 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
                 weights[0][(((size_t)f * C + c) * S + r) * S + q];
           }
   }
-  size_t act = (size_t)B * net->stage_h * net->stage_w * net->in_cs * esz;
+  // Padded-layout ("shifted window") convs, ConvGeom::pm: a stride-1 'same'
+  // conv whose input and output share one zero-haloed grid loads, per filter
+  // row, one TMA window of 128 + S - 1 rows that feeds all S taps -- S times
+  // fewer A bytes than im2col boxes.  Chosen per net: the conv's producer and
+  // consumer must read / write the halo layout (pools and pm convs of the same
+  // halo do; a staged-im2col first layer joins as a 1 x 1 pm conv), channels
+  // per group must fill 128 B slabs, and the halo may add at most 25% rows.
   const int n = n_layers;
+  {
+    const char *e = getenv("PCNN_NO_PM");
+    const bool allow = prec != PCNN_FP32_SIMT && !(e && e[0] == '1');
+    auto kind = [&](int j) { return net->layers[j].d.kind; };
+    auto is_pool = [&](int j) { return kind(j) == PCNN_MAXPOOL || kind(j) == PCNN_AVGPOOL; };
+    std::vector<int> pmh(n, 0);
+    if (allow) {
+      for (int i = 1; i < n; ++i) {
+        const Layer &ly = net->layers[i];
+        if (ly.d.kind != PCNN_CONV) continue;
+        const int S = ly.d.kernel, P = ly.d.pad, g = ly.d.groups;
+        if (ly.d.stride != 1 || S != 2 * P + 1 || P < 1 || P > 3 || ly.in_cs % g) continue;
+        if (tc_slab_bytes(net->st, ly.in_cs / g) != 128) continue;
+        if ((double)(ly.in_h + 2 * P) * (ly.in_w + 2 * P) > 1.25 * ly.in_h * ly.in_w) continue;
+        pmh[i] = P;
+      }
+      for (bool changed = true; changed;) {
+        changed = false;
+        if (net->stage_im2col && n > 1) {
+          const int h = kind(1) == PCNN_CONV && tc_slab_bytes(net->st, net->in_cs) ? pmh[1] : 0;
+          if (pmh[0] != h) {
+            pmh[0] = h;
+            changed = true;
+          }
+        }
+        for (int i = 1; i < n; ++i) {
+          if (!pmh[i]) continue;
+          auto nb_ok = [&](int j) {
+            return j >= 0 && j < n && (is_pool(j) || (kind(j) == PCNN_CONV && pmh[j] == pmh[i]));
+          };
+          if (!nb_ok(i - 1) || !nb_ok(i + 1)) {
+            pmh[i] = 0;
+            changed = true;
+          }
+        }
+      }
+    }
+    for (int i = 0; i < n; ++i) {
+      Layer &ly = net->layers[i];
+      ly.in_halo = i > 0 ? net->layers[i - 1].out_halo : pmh[0];
+      ly.pm_halo = pmh[i];
+      if (pmh[i]) ly.out_halo = pmh[i];
+      else if (is_pool(i) && i + 1 < n && kind(i + 1) == PCNN_CONV) ly.out_halo = pmh[i + 1];
+      else ly.out_halo = 0;
+    }
+  }
+  const int h0 = net->layers[0].in_halo;
+  size_t act = (size_t)B * (net->stage_h + 2 * h0) * (net->stage_w + 2 * h0) * net->in_cs * esz;
   for (int i = 0; i < n; ++i) {
     Layer &ly = net->layers[i];
-    act = std::max(act, (size_t)B * ly.out_h * ly.out_w * ly.out_cs * esz);
+    act = std::max(act, (size_t)B * (ly.out_h + 2 * ly.out_halo) * (ly.out_w + 2 * ly.out_halo) *
+                            ly.out_cs * esz);
     if (ly.gemm) {
       const bool final_fc = (i == n - 1) && ly.d.kind == PCNN_FC;
       const int mode = final_fc ? OUT_F32
@@ -1125,7 +1268,7 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
       if (i == 0 && net->stage_im2col) {
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, 1, 1, 1, 0, ly.d.relu,
                         net->stage_c, net->stage_h, net->stage_w, net->in_cs, false,
-                        s2d_w.data(), biases ? biases[i] : nullptr, mode);
+                        s2d_w.data(), biases ? biases[i] : nullptr, mode, ly.pm_halo);
       } else if (i == 0 && net->stage_blk > 1) {
         const int Sp = (ly.d.kernel + net->stage_blk - 1) / net->stage_blk;
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, 1, Sp, 1, 0, ly.d.relu,
@@ -1135,7 +1278,8 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, is_fc ? 1 : ly.d.groups,
                         is_fc ? 1 : ly.d.kernel, is_fc ? 1 : ly.d.stride,
                         is_fc ? 0 : ly.d.pad, ly.d.relu, ly.in_c, ly.in_h, ly.in_w,
-                        ly.in_cs, is_fc, weights[i], biases ? biases[i] : nullptr, mode);
+                        ly.in_cs, is_fc, weights[i], biases ? biases[i] : nullptr, mode,
+                        ly.pm_halo);
       }
       if (s != PCNN_OK) {
         for (auto &l2 : net->layers) l2.exact.release();
@@ -1220,6 +1364,9 @@ pcnn_status pcnn_set_variant(pcnn_net *net, int layer, int variant, int rank) {
   if (variant != PCNN_VARIANT_RANK) return fail(PCNN_ERR_INVALID_ARGUMENT, "bad variant");
   if (ly.d.kind != PCNN_CONV)
     return fail(PCNN_ERR_UNSUPPORTED, "rank variant is implemented for conv layers");
+  if (layer == 0 && (net->stage_im2col || net->stage_blk > 1))
+    return fail(PCNN_ERR_UNSUPPORTED,
+                "rank variant of a first conv whose input is staged (im2col / space-to-depth)");
   const int g = ly.d.groups, Nfg = ly.d.out_channels / g, Cg = ly.in_c / g,
             S = ly.d.kernel, K = Cg * S * S;
   const int rmax = std::min(Nfg, K);
@@ -1291,6 +1438,8 @@ pcnn_status pcnn_query_layer(const pcnn_net *cnet, int layer, int batch, pcnn_la
   f->n_sms = effective_sms(net, ly);
   f->tlp = ly.tlp;
   f->engine = 2;
+  f->halo_in = ly.in_halo;
+  f->halo_out = ly.out_halo;
   if (ly.gemm) {
     GemmStage &gs = ly.variant == PCNN_VARIANT_RANK ? ly.r1 : ly.exact;
     f->gemm_m = (long long)batch * gs.g.Ho * gs.g.Wo;

@@ -52,7 +52,8 @@ class LayerInfo(ctypes.Structure):
                 ("variant", ctypes.c_int), ("rank", ctypes.c_int), ("n_sms", ctypes.c_int),
                 ("tlp", ctypes.c_int), ("engine", ctypes.c_int), ("tile_m", ctypes.c_int),
                 ("tile_n", ctypes.c_int), ("tiles", ctypes.c_longlong), ("grid", ctypes.c_int),
-                ("util", ctypes.c_double), ("rec", ctypes.c_double), ("splits", ctypes.c_int)]
+                ("util", ctypes.c_double), ("rec", ctypes.c_double), ("splits", ctypes.c_int),
+                ("a_mode", ctypes.c_int), ("halo_in", ctypes.c_int), ("halo_out", ctypes.c_int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

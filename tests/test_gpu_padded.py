@@ -1,0 +1,109 @@
+"""Padded-layout ("shifted window") conv mode (kernel K1 a_mode 2):
+activations live on zero-haloed grids, one TMA row window per filter row
+feeds all S taps.  Parity with the FP64 oracle, agreement with the im2col
+mode, ragged tails, the rank-r variant and the SM budget on pm layers."""
+import numpy as np
+import pytest
+
+from tests.helpers import TOL, conv_layer, gpu_run, params, rel_err, small_inputs
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+
+
+def vgg_like(hw=40, c1=64, c2=128, groups=1):
+    """VGG-shaped blocks (3x3 / 1 / pad 1 convs + 2x2 pools) at a size whose
+    halo overhead passes the 25% rule and whose M = B*(H+2)*(W+2) rows end
+    in a ragged tile."""
+    q = hw // 4
+    return dict(in_shape=(3, hw, hw), layers=[
+        conv_layer(c1, 3, 3, 1, 1), conv_layer(c1, 3, c1, 1, 1, groups),
+        dict(kind="maxpool", k=2, stride=2),
+        conv_layer(c2, 3, c1, 1, 1), conv_layer(c2, 3, c2, 1, 1, groups),
+        dict(kind="maxpool", k=2, stride=2),
+        dict(kind="fc", out=16, in_f=c2 * q * q, relu=False)])
+
+
+PM_LAYERS = [0, 1, 3, 4]
+
+
+@pytest.mark.parametrize("prec", ["tf32", "bf16"])
+def test_padded_mode_matches_oracle(orc, prec):
+    net = vgg_like()
+    w, b = params(net, seed=21)
+    x = small_inputs((3, 40, 40), 3, lo=-128, hi=128)
+    ref = orc.run_net(net, w, b, x).reshape(3, -1)
+    r = gpu_run(net, w, b, x, prec)
+    infos = [r["net"].query_layer(i, 3) for i in range(len(net["layers"]))]
+    assert [i for i, f in enumerate(infos) if f["a_mode"] == 2] == PM_LAYERS
+    assert [(f["halo_in"], f["halo_out"]) for f in infos] == \
+        [(1, 1), (1, 1), (1, 1), (1, 1), (1, 1), (1, 0), (0, 0)]
+    assert rel_err(r["out"], ref) <= TOL[prec] / 2
+
+
+@pytest.mark.parametrize("prec", ["tf32", "bf16"])
+def test_padded_mode_agrees_with_im2col_mode(orc, prec, monkeypatch):
+    """Same products, different K order: the two A-addressing modes agree far
+    inside the tolerance (and the zero halos never leak into the result)."""
+    net = vgg_like(hw=36, c1=64, c2=64)
+    w, b = params(net, seed=5)
+    x = small_inputs((3, 36, 36), 5, lo=-128, hi=128)
+    pm = gpu_run(net, w, b, x, prec)
+    assert pm["net"].query_layer(1, 5)["a_mode"] == 2
+    monkeypatch.setenv("PCNN_NO_PM", "1")
+    im = gpu_run(net, w, b, x, prec)
+    assert im["net"].query_layer(1, 5)["a_mode"] == 0
+    assert rel_err(pm["out"], im["out"]) <= TOL[prec] / 4
+
+
+def test_padded_mode_grouped_conv(orc):
+    net = vgg_like(hw=40, c1=128, c2=128, groups=2)
+    w, b = params(net, seed=8)
+    x = small_inputs((3, 40, 40), 2, lo=-128, hi=128)
+    ref = orc.run_net(net, w, b, x).reshape(2, -1)
+    r = gpu_run(net, w, b, x, "bf16")
+    assert r["net"].query_layer(1, 2)["a_mode"] == 2
+    assert rel_err(r["out"], ref) <= TOL["bf16"] / 2
+
+
+@pytest.mark.parametrize("prec", ["tf32", "bf16"])
+def test_padded_mode_rank_variant(orc, prec):
+    """Rank-r on a pm layer: both stages stay on the halo grid."""
+    net = vgg_like()
+    w, b = params(net, seed=21)
+    x = small_inputs((3, 40, 40), 2, lo=-128, hi=128)
+    for i, r in [(1, 24), (4, 48)]:
+        ref = orc.run_net(net, w, b, x, ranks={i: r}).reshape(2, -1)
+        res = gpu_run(net, w, b, x, prec, variants={i: ("rank", r)})
+        assert res["net"].query_layer(i, 2)["a_mode"] == 2
+        assert rel_err(res["out"], ref) <= TOL[prec] / 2, (prec, i, r)
+
+
+def test_padded_mode_budget_bitwise():
+    net = vgg_like()
+    w, b = params(net, seed=21)
+    x = small_inputs((3, 40, 40), 3, lo=-128, hi=128)
+    base = gpu_run(net, w, b, x, "bf16")["out"]
+    for n_sms in (2, 16, 74):
+        r = gpu_run(net, w, b, x, "bf16", budgets={i: (n_sms, 0) for i in PM_LAYERS}, census=True)
+        np.testing.assert_array_equal(r["out"], base)
+        for i in PM_LAYERS:
+            assert 0 < len(r["census"][i]) <= n_sms
+
+
+def test_padded_mode_batch_one_and_max_batch(orc):
+    """B = 1 (M smaller than one CTA pair's rows) and a net created for a
+    larger max batch run at a smaller batch."""
+    net = vgg_like(hw=24, c1=64, c2=64)
+    w, b = params(net, seed=3)
+    x = small_inputs((3, 24, 24), 1, lo=-128, hi=128)
+    ref = orc.run_net(net, w, b, x).reshape(1, -1)
+    r = gpu_run(net, w, b, x, "bf16", max_batch=7)
+    assert r["net"].query_layer(1, 1)["a_mode"] == 2
+    assert rel_err(r["out"], ref) <= TOL["bf16"] / 2
