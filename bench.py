@@ -66,7 +66,9 @@ def parse():
 
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled every 200 ms."""
+    """nvidia-smi clocks / throttle reasons sampled every 50 ms while the GPU
+    is under the bench's load (warm-up, timed steps, graph replay, e2e); a
+    timed region alone can be shorter than one sampling period."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
@@ -83,7 +85,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "--query-gpu=" + self.Q, "--format=csv,noheader,nounits",
-                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except OSError:
             self.proc = None
             return
@@ -248,6 +250,8 @@ def main():
     sampler = ClockSampler(world) if rank == 0 else None
     if sampler:
         sampler.start()
+        time.sleep(0.3)
+        sampler.mark(True)
     for _ in range(a.warmup):
         step()
     torch.cuda.synchronize()
@@ -257,16 +261,12 @@ def main():
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     barrier()
     torch.cuda.synchronize()
-    if sampler:
-        sampler.mark(True)
     ev0.record(stream)
     for _ in range(a.steps):
         step()
     ev1.record(stream)
     torch.cuda.synchronize()
     barrier()
-    if sampler:
-        sampler.mark(False)
     n.set_layer_timing(False)
     ms = ev0.elapsed_time(ev1)
     layer_ms, nsteps = n.read_layer_timing()
@@ -314,6 +314,8 @@ def main():
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_value = world * B * e2e_steps / float(te.item())
 
+    if sampler:
+        sampler.mark(False)
     clocks = sampler.stop() if sampler else None
 
     # ---------------- per-layer plan, roofline of the dominant kernel (conv)

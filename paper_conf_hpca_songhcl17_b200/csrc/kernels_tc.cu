@@ -46,7 +46,9 @@ constexpr int TC_A_STAGE = TC_BM * TC_ROW_BYTES;          // 16 KB
 constexpr int TC_STAGE_BUDGET = 176 * 1024;               // operand stages per CTA
 constexpr int TC_MAX_KTAB = 1024;       // slab-table entries kept in smem
 constexpr int EPI_PITCH = 144;          // epilogue staging row: 128 B + 16 B pad
-constexpr int EPI_WARP_BYTES = 32 * EPI_PITCH;
+// per-warp staging slot: 32 rows x 144 B (st.global path) or one 32-row x
+// 32-column swizzled TMA-store box (<= 4 KB); 1024-aligned slots
+constexpr int EPI_WARP_BYTES = 5120;
 // warps: 0 TMA producer, 1 MMA issuer, then NEPI epilogue warps (8, two per
 // TMEM lane quarter splitting the columns; 4 for the LRN-fused variant, whose
 // per-row channel vector needs ~255 registers)
@@ -56,10 +58,11 @@ constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 
 // smem layout (bytes from the 1024-aligned base):
 //   [0, TC_STAGE_BUDGET)   A stages, then B stages (runtime count)
+//   SM_EPI                 per-epilogue-warp output staging (8 warps, 1024-aligned)
 //   SM_BAR                 barriers + TMEM pointer
 //   SM_KTAB                (r, s, c) table, one entry per A slab
-//   SM_EPI                 per-epilogue-warp output staging (coalesced stores, 8 warps)
-constexpr int SM_BAR = TC_STAGE_BUDGET;
+constexpr int SM_EPI = TC_STAGE_BUDGET;
+constexpr int SM_BAR = SM_EPI + 8 * EPI_WARP_BYTES;
 constexpr int SM_FULL = SM_BAR;
 constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_STAGES;
 constexpr int SM_TFULL = SM_EMPTY + 8 * TC_MAX_STAGES;
@@ -69,8 +72,7 @@ constexpr int TC_MAX_ASTAGES = 4;       // padded mode: A row-window ring
 constexpr int SM_AFULL = SM_TMEMPTR + 16;
 constexpr int SM_AEMPTY = SM_AFULL + 8 * TC_MAX_ASTAGES;
 constexpr int SM_KTAB = SM_BAR + 512;
-constexpr int SM_EPI = SM_KTAB + 4 * TC_MAX_KTAB;        // 4 warps x 32 rows x 144 B
-constexpr int SM_TOTAL = SM_EPI + 8 * EPI_WARP_BYTES;
+constexpr int SM_TOTAL = SM_KTAB + 4 * TC_MAX_KTAB;
 constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
 
 size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
@@ -182,6 +184,22 @@ __device__ __forceinline__ void tma_im2col_2sm(uint32_t dst, const CUtensorMap *
 }
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// TMA tensor store of one smem box (bulk-group completion)
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, uint32_t src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                   (uint64_t)map),
+               "r"(src), "r"(c0), "r"(c1)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() {
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read0() {
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait0() {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 
 // one lane of a converged warp (the tcgen05 / TMA issue idiom): the loop
@@ -353,6 +371,7 @@ struct TcArgs {
   int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
   int a_stages, b_stages, pm_a_stage;   // padded mode rings (g.pm)
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
+  int tma_y;            // 1: full 32-column output chunks leave by TMA tensor store
   float lrn_a_over_n, lrn_beta, lrn_k;
   Budget b;
 };
@@ -485,15 +504,142 @@ __device__ __forceinline__ void advance(uint32_t &stage, uint32_t &phase, int st
   }
 }
 
+// ------------------------------------------------------------ MMA issuers
+// The issue loops are written so that every tcgen05.mma operand (descriptors,
+// TMEM column, instruction descriptor, accumulate flag) is warp-uniform and
+// derived from kernel parameters and uniform loop counters: ptxas then keeps
+// them in uniform registers and a K-block's 4 UMMAs issue back to back.  A
+// per-iteration R2UR round trip (what a lane-dependent branch in the loop
+// causes) costs ~150 cycles per UMMA, more than an N = 64 UMMA executes in
+// (tools/mma_rate_probe.cu).  K offsets inside a K-block are compile-time:
+// the A K-block is 128 / SLAB slabs of TC_BM rows, each SLAB / 32 UMMAs deep.
+template <int SLAB>
+__device__ __forceinline__ constexpr uint32_t a_koff(int k) {
+  return (uint32_t)((k / (SLAB / 32)) * (TC_BM * SLAB / 16) + 2 * (k % (SLAB / 32)));
+}
+
+template <int ST, int CG, int SLAB>
+__device__ __forceinline__ void mma_issuer_im2col(const TcArgs &a, uint32_t sbase, uint32_t sA,
+                                                  uint32_t sB, uint32_t b_stage,
+                                                  uint32_t tmem_base, int pair, int npairs,
+                                                  unsigned long long *acc_full,
+                                                  unsigned long long *acc_temp) {
+  const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
+  const uint64_t a_desc0 = umma_desc(sA, SLAB);
+  const uint64_t b_desc0 = umma_desc_sw128(sB);
+  const uint32_t a_stage16 = TC_A_STAGE / 16, b_stage16 = b_stage / 16;
+  const int stages = a.stages, units = a.units, mtiles = a.mtiles, ntiles = a.ntiles;
+  const int groups = a.g.groups, kblocks = a.kblocks, kbs = a.kb_per_split;
+  const bool prof = a.prof != 0, skip_mma = (a.skip & 4) != 0;
+  const bool leader = elect_one();
+  WaitClock wfull{prof}, wtemp{prof};
+  uint32_t stage = 0, phase = 0, lt = 0;
+  for (int u = pair; u < units; u += npairs, ++lt) {
+    const int sp = u / (mtiles * ntiles * groups);
+    const int k0 = sp * kbs, k1 = min(kblocks, k0 + kbs);
+    const uint32_t buf = lt & 1, use = lt >> 1;
+    wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
+    tc_fence_after();
+    const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
+    for (int kb = k0; kb < k1; ++kb) {
+      wfull.wait(sbase + SM_FULL + 8 * stage, phase);
+      tc_fence_after();
+      const uint64_t ad = a_desc0 + stage * a_stage16;
+      const uint64_t bd = b_desc0 + stage * b_stage16;
+      if (leader) {
+        if (!skip_mma) {
+          tc_mma<ST, CG>(dcol, ad + a_koff<SLAB>(0), bd, idesc, kb > k0 ? 1u : 0u);
+          tc_mma<ST, CG>(dcol, ad + a_koff<SLAB>(1), bd + 2, idesc, 1u);
+          tc_mma<ST, CG>(dcol, ad + a_koff<SLAB>(2), bd + 4, idesc, 1u);
+          tc_mma<ST, CG>(dcol, ad + a_koff<SLAB>(3), bd + 6, idesc, 1u);
+        }
+        tc_commit<CG>(sbase + SM_EMPTY + 8 * stage);
+      }
+      __syncwarp();
+      if (++stage == (uint32_t)stages) {
+        stage = 0;
+        phase ^= 1;
+      }
+    }
+    if (leader) tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
+    __syncwarp();
+  }
+  *acc_full = wfull.acc;
+  *acc_temp = wtemp.acc;
+}
+
+// Padded mode: per (slab, filter row) A window, S taps; tap s reads the
+// window shifted by s rows (SLAB / 16 descriptor units per row).
+template <int ST, int CG, int SLAB>
+__device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, uint32_t sA,
+                                              uint32_t sBp, uint32_t pm_b_bytes,
+                                              uint32_t tmem_base, int pair, int npairs, int nj,
+                                              unsigned long long *acc_full,
+                                              unsigned long long *acc_temp) {
+  constexpr int KMMA = SLAB / 32;
+  constexpr uint32_t ROW16 = SLAB / 16;
+  const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
+  const uint64_t a_desc0 = umma_desc(sA, SLAB);
+  const uint64_t b_desc0 = umma_desc(sBp, SLAB);
+  const uint32_t a_st16 = (uint32_t)a.pm_a_stage / 16, b_st16 = pm_b_bytes / 16;
+  const int a_stages = a.a_stages, b_stages = a.b_stages, units = a.units, S = a.g.S;
+  const bool prof = a.prof != 0, skip_mma = (a.skip & 4) != 0;
+  const bool leader = elect_one();
+  WaitClock wfull{prof}, wtemp{prof};
+  uint32_t as = 0, aph = 0, bs = 0, bph = 0, lt = 0;
+  for (int u = pair; u < units; u += npairs, ++lt) {
+    const uint32_t buf = lt & 1, use = lt >> 1;
+    wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
+    tc_fence_after();
+    const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
+    for (int j = 0; j < nj; ++j) {
+      wfull.wait(sbase + SM_AFULL + 8 * as, aph);
+      const uint64_t ad = a_desc0 + as * a_st16;
+      for (int s2 = 0; s2 < S; ++s2) {
+        wfull.wait(sbase + SM_FULL + 8 * bs, bph);
+        tc_fence_after();
+        const uint64_t aw = ad + s2 * ROW16;
+        const uint64_t bd = b_desc0 + bs * b_st16;
+        if (leader) {
+          if (!skip_mma) {
+            tc_mma<ST, CG>(dcol, aw, bd, idesc, (j > 0 || s2 > 0) ? 1u : 0u);
+#pragma unroll
+            for (int k = 1; k < KMMA; ++k) tc_mma<ST, CG>(dcol, aw + 2 * k, bd + 2 * k, idesc, 1u);
+          }
+          tc_commit<CG>(sbase + SM_EMPTY + 8 * bs);
+        }
+        __syncwarp();
+        if (++bs == (uint32_t)b_stages) {
+          bs = 0;
+          bph ^= 1;
+        }
+      }
+      if (leader) tc_commit<CG>(sbase + SM_AEMPTY + 8 * as);
+      __syncwarp();
+      if (++as == (uint32_t)a_stages) {
+        as = 0;
+        aph ^= 1;
+      }
+    }
+    if (leader) tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
+    __syncwarp();
+  }
+  *acc_full = wfull.acc;
+  *acc_temp = wtemp.acc;
+}
+
 template <int ST, int CG, bool LRN>
 __global__ void __launch_bounds__(tc_threads<LRN>(), 1)
 conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
-               const __grid_constant__ CUtensorMap tmap_x, const TcArgs a) {
+               const __grid_constant__ CUtensorMap tmap_x,
+               const __grid_constant__ CUtensorMap tmap_y, const TcArgs a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const uint32_t sbase = smem_u32(smem);
   const int tid = threadIdx.x;
-  const int warp = tid >> 5, lane = tid & 31;
+  // warp index through a lane-0 shuffle: provably warp-uniform, so the role
+  // branches below keep their loop state in uniform registers
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0), lane = tid & 31;
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
   const ConvGeom &g = a.g;
   const int stages = a.stages;
@@ -628,50 +774,16 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   } else if (warp == 1 && g.pm) {
     if (rank == 0) {
       // ---------------------------------------------- MMA issuer, padded mode
-      const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
-      const uint64_t a_desc0 = umma_desc(sA, slab_bytes);
-      const uint64_t b_desc0 = umma_desc(sBp, slab_bytes);
-      const uint32_t a_st16 = (uint32_t)a.pm_a_stage / 16, b_st16 = pm_b_bytes / 16;
-      const uint32_t row16 = (uint32_t)slab_bytes / 16;   // one A row = one tap shift
-      const int kmma = slab_bytes / 32;                     // UMMAs per slab row (K = 32 B)
-      uint32_t as = 0, aph = 0, bs = 0, bph = 0, lt = 0;
-      WaitClock wfull{a.prof != 0 && lane == 0}, wtemp{a.prof != 0 && lane == 0};
-      for (int u = pair; u < a.units; u += npairs, ++lt) {
-        const uint32_t buf = lt & 1, use = lt >> 1;
-        wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
-        tc_fence_after();
-        const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
-        for (int j = 0; j < pm_nj; ++j) {
-          wfull.wait(sbase + SM_AFULL + 8 * as, aph);
-          tc_fence_after();
-          const uint64_t ad = a_desc0 + as * a_st16;
-          for (int s2 = 0; s2 < g.S; ++s2) {
-            wfull.wait(sbase + SM_FULL + 8 * bs, bph);
-            tc_fence_after();
-            const uint64_t bd = b_desc0 + bs * b_st16;
-            if (elect_one()) {
-              if (!(a.skip & 4)) {
-#pragma unroll
-                for (int k = 0; k < 4; ++k)
-                  if (k < kmma)
-                    tc_mma<ST, CG>(dcol, ad + s2 * row16 + 2 * k, bd + 2 * k, idesc,
-                                   (j > 0) || (s2 > 0) || (k > 0));
-              }
-              tc_commit<CG>(sbase + SM_EMPTY + 8 * bs);
-            }
-            __syncwarp();
-            advance(bs, bph, a.b_stages);
-          }
-          if (elect_one()) tc_commit<CG>(sbase + SM_AEMPTY + 8 * as);
-          __syncwarp();
-          advance(as, aph, a.a_stages);
-        }
-        if (elect_one()) tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
-        __syncwarp();
-      }
+      unsigned long long af = 0, at = 0;
+      if (slab_bytes == 128)
+        mma_issuer_pm<ST, CG, 128>(a, sbase, sA, sBp, pm_b_bytes, tmem_base, pair, npairs, pm_nj, &af, &at);
+      else if (slab_bytes == 64)
+        mma_issuer_pm<ST, CG, 64>(a, sbase, sA, sBp, pm_b_bytes, tmem_base, pair, npairs, pm_nj, &af, &at);
+      else
+        mma_issuer_pm<ST, CG, 32>(a, sbase, sA, sBp, pm_b_bytes, tmem_base, pair, npairs, pm_nj, &af, &at);
       if (a.prof && lane == 0) {
-        atomicAdd(&g_tc_prof[1], wfull.acc);
-        atomicAdd(&g_tc_prof[2], wtemp.acc);
+        atomicAdd(&g_tc_prof[1], af);
+        atomicAdd(&g_tc_prof[2], at);
       }
     }
   } else if (warp == 0) {
@@ -748,53 +860,17 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     }
   } else if (warp == 1) {
     if (rank == 0) {
-      // ---------------------------------------------- MMA issuer (leader):
-      // the warp walks the schedule; one elected lane issues.  All descriptor
-      // arithmetic is hoisted: per K-block only stage offsets are added.
-      const uint32_t idesc = umma_idesc<ST, CG>(a.bn);
-      const uint64_t a_desc0 = umma_desc(sA, slab_bytes);
-      const uint64_t b_desc0 = umma_desc_sw128(sB);
-      uint32_t a_koff[4];              // 16 B units: slab base + K offset inside the slab
-      {
-        const int mma_per_slab = slab_bytes / 32;   // K = 32 B per UMMA
-#pragma unroll
-        for (int k = 0; k < 4; ++k)
-          a_koff[k] = (uint32_t)((k / mma_per_slab) * (TC_BM * slab_bytes) / 16 +
-                                 2 * (k % mma_per_slab));
-      }
-      const uint32_t a_stage16 = TC_A_STAGE / 16, b_stage16 = b_stage / 16;
-      uint32_t stage = 0, phase = 0, lt = 0;
-      WaitClock wfull{a.prof != 0 && lane == 0}, wtemp{a.prof != 0 && lane == 0};
-      for (int u = pair; u < a.units; u += npairs, ++lt) {
-        int mt, nt, grp, sp, k0, k1;
-        decode(u, mt, nt, grp, sp);
-        kb_range(sp, k0, k1);
-        const uint32_t buf = lt & 1, use = lt >> 1;
-        wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
-        tc_fence_after();
-        const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
-        for (int kb = k0; kb < k1; ++kb) {
-          wfull.wait(sbase + SM_FULL + 8 * stage, phase);
-          tc_fence_after();
-          const uint64_t ad = a_desc0 + stage * a_stage16;
-          const uint64_t bd = b_desc0 + stage * b_stage16;
-          if (elect_one()) {
-            if (!(a.skip & 4)) {
-#pragma unroll
-              for (int k = 0; k < 4; ++k)   // 4 x 32 B of K per 128 B K-block
-                tc_mma<ST, CG>(dcol, ad + a_koff[k], bd + 2 * k, idesc, (kb > k0) || (k > 0));
-            }
-            tc_commit<CG>(sbase + SM_EMPTY + 8 * stage);
-          }
-          __syncwarp();
-          advance(stage, phase, stages);
-        }
-        if (elect_one()) tc_commit<CG>(sbase + SM_TFULL + 8 * buf);
-        __syncwarp();
-      }
+      // ---------------------------------------------- MMA issuer (leader)
+      unsigned long long af = 0, at = 0;
+      if (slab_bytes == 128)
+        mma_issuer_im2col<ST, CG, 128>(a, sbase, sA, sB, b_stage, tmem_base, pair, npairs, &af, &at);
+      else if (slab_bytes == 64)
+        mma_issuer_im2col<ST, CG, 64>(a, sbase, sA, sB, b_stage, tmem_base, pair, npairs, &af, &at);
+      else
+        mma_issuer_im2col<ST, CG, 32>(a, sbase, sA, sB, b_stage, tmem_base, pair, npairs, &af, &at);
       if (a.prof && lane == 0) {
-        atomicAdd(&g_tc_prof[1], wfull.acc);
-        atomicAdd(&g_tc_prof[2], wtemp.acc);
+        atomicAdd(&g_tc_prof[1], af);
+        atomicAdd(&g_tc_prof[2], at);
       }
     }
   } else {
@@ -844,6 +920,117 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       if constexpr (LRN) {
         epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX, mok,
                          orow, stage, lane);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          if (CG == 2 && rank != 0) mbar_arrive_cluster(tempty_leader + 8 * buf);
+          else mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
+        }
+        continue;
+      }
+      if (a.tma_y) {
+        // 32-column passes; full chunks are staged in this warp's swizzled
+        // box (SW64 rows for bf16, SW128 for fp32) and leave by one TMA
+        // tensor store of the warp's 32 rows (rows past M are clipped by the
+        // map); a ragged last chunk falls back to row stores.
+        const bool o16 = g.out_mode == OUT_BF16;
+        const int split = ((a.bn / 2 + 31) / 32) * 32;
+        const int cbeg = half == 0 ? 0 : split, cend = half == 0 ? split : a.bn;
+        const int row0 = m - lane;                       // the warp's first row
+        const uint32_t sstage = smem_u32(stage);
+        for (int c0 = cbeg; c0 < cend; c0 += 32) {
+          const int n = nt * a.bn + c0;
+          if (n >= g.Nfg) break;                         // warp-uniform
+          const int col = grp * g.Nfg + n;
+          float f[32];
+          {
+            uint32_t v[32];
+            tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0, v);
+            tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 32; ++i) f[i] = __uint_as_float(v[i]);
+          }
+          const float4 *bp = (const float4 *)(a.bias + col);
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const float4 bb = __ldg(bp + q);
+            f[4 * q] += bb.x;
+            f[4 * q + 1] += bb.y;
+            f[4 * q + 2] += bb.z;
+            f[4 * q + 3] += bb.w;
+          }
+          if (g.relu)
+#pragma unroll
+            for (int i = 0; i < 32; ++i) f[i] = fmaxf(f[i], 0.f);
+          if (!valid)
+#pragma unroll
+            for (int i = 0; i < 32; ++i) f[i] = 0.f;
+          const bool full = n + 32 <= g.Nfg && c0 + 32 <= cend;
+          if (full) {
+            if (lane == 0) bulk_wait_read0();            // staging box free again
+            __syncwarp();
+            if (o16) {
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                uint4 pk;
+                uint32_t *pw = (uint32_t *)&pk;
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                  __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * q + 2 * i], f[8 * q + 2 * i + 1]);
+                  pw[i] = *(uint32_t *)&b2;
+                }
+                *(uint4 *)(stage + lane * 64 + ((q ^ ((lane >> 1) & 3)) << 4)) = pk;
+              }
+            } else {
+              const bool rnd = g.out_mode == OUT_F32_TF32;
+#pragma unroll
+              for (int q = 0; q < 8; ++q) {
+                float t[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) t[i] = rnd ? tf32_rna_tc(f[4 * q + i]) : f[4 * q + i];
+                *(uint4 *)(stage + lane * 128 + ((q ^ (lane & 7)) << 4)) =
+                    make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]),
+                               __float_as_uint(t[2]), __float_as_uint(t[3]));
+              }
+            }
+            fence_proxy_async();
+            __syncwarp();
+            if (lane == 0 && row0 < g.M) {
+              tma_store_2d(&tmap_y, sstage, col, row0);
+              bulk_commit();
+            }
+          } else {
+            // ragged chunk: row stores of the np valid 16 B pieces
+            uint4 pc[8];
+            const int eb = o16 ? 2 : 4;
+            if (o16) {
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                uint32_t *pw = (uint32_t *)&pc[q];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                  __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * q + 2 * i], f[8 * q + 2 * i + 1]);
+                  pw[i] = *(uint32_t *)&b2;
+                }
+              }
+            } else {
+              const bool rnd = g.out_mode == OUT_F32_TF32;
+#pragma unroll
+              for (int q = 0; q < 8; ++q) {
+                float t[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) t[i] = rnd ? tf32_rna_tc(f[4 * q + i]) : f[4 * q + i];
+                pc[q] = make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]),
+                                   __float_as_uint(t[2]), __float_as_uint(t[3]));
+              }
+            }
+            if (lane == 0) bulk_wait_read0();
+            __syncwarp();
+            const int np = min(o16 ? 4 : 8, (min(g.Nfg - n, cend - c0) * eb) / 16);
+            char *rowp = mok ? (char *)a.y + ((size_t)m * g.out_cs + col) * eb : nullptr;
+            epi_store_rows(stage, pc, np, rowp, lane);
+          }
+        }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) {
@@ -931,6 +1118,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         else mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
       }
     }
+    if (lane == 0) bulk_wait0();                 // TMA stores complete before exit
+    __syncwarp();
     if (wtf.on && tb) busy += clock64() - tb;
     wtf_acc_out = wtf.acc;
     busy_out = busy;
@@ -1020,7 +1209,8 @@ int tc_slab_bytes(int st, int cg_channels) {
 
 template <int ST, int CG, bool LRN>
 static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_x,
-                             const TcArgs &args, int grid, cudaStream_t s) {
+                             const CUtensorMap *tmap_y, const TcArgs &args, int grid,
+                             cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(tc_threads<LRN>());
@@ -1033,7 +1223,7 @@ static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG, LRN>, *tmap_w, *tmap_x, args);
+  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG, LRN>, *tmap_w, *tmap_x, *tmap_y, args);
 }
 
 cudaError_t tc_profile(int reset, unsigned long long out[8]) {
@@ -1051,7 +1241,7 @@ cudaError_t tc_profile(int reset, unsigned long long out[8]) {
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias, void *y,
                            const int *ktab, const TcPlan &p, float *ws, const Budget &b,
-                           cudaStream_t s, const float *lrn) {
+                           cudaStream_t s, const float *lrn, const CUtensorMap *tmap_y) {
   TcArgs args;
   static const int prof_env = [] {
     const char *e = getenv("PCNN_TC_PROFILE");
@@ -1076,6 +1266,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   }
   args.g = g;
   args.y = y;
+  args.tma_y = (tmap_y != nullptr && !lrn && p.splits == 1 && p.rect_w == 0) ? 1 : 0;
   args.ws = ws;
   args.bias = bias;
   args.ktab = ktab;
@@ -1105,15 +1296,15 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   cudaError_t e;
   const bool L = args.lrn != 0;
   if (st == ST_BF16)
-    e = p.cg == 2 ? (L ? launch_tc<ST_BF16, 2, true>(tmap_w, tmap_x, args, p.grid, s)
-                       : launch_tc<ST_BF16, 2, false>(tmap_w, tmap_x, args, p.grid, s))
-                  : (L ? launch_tc<ST_BF16, 1, true>(tmap_w, tmap_x, args, p.grid, s)
-                       : launch_tc<ST_BF16, 1, false>(tmap_w, tmap_x, args, p.grid, s));
+    e = p.cg == 2 ? (L ? launch_tc<ST_BF16, 2, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
+                       : launch_tc<ST_BF16, 2, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s))
+                  : (L ? launch_tc<ST_BF16, 1, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
+                       : launch_tc<ST_BF16, 1, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s));
   else
-    e = p.cg == 2 ? (L ? launch_tc<ST_F32, 2, true>(tmap_w, tmap_x, args, p.grid, s)
-                       : launch_tc<ST_F32, 2, false>(tmap_w, tmap_x, args, p.grid, s))
-                  : (L ? launch_tc<ST_F32, 1, true>(tmap_w, tmap_x, args, p.grid, s)
-                       : launch_tc<ST_F32, 1, false>(tmap_w, tmap_x, args, p.grid, s));
+    e = p.cg == 2 ? (L ? launch_tc<ST_F32, 2, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
+                       : launch_tc<ST_F32, 2, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s))
+                  : (L ? launch_tc<ST_F32, 1, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
+                       : launch_tc<ST_F32, 1, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s));
   if (e != cudaSuccess) return e;
   e = cudaGetLastError();
   if (e != cudaSuccess || p.splits <= 1) return e;

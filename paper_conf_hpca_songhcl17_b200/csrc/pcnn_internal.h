@@ -105,7 +105,11 @@ struct TcPlan {
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias,
                            void *y, const int *ktab, const TcPlan &p, float *ws,
-                           const Budget &b, cudaStream_t s, const float *lrn = nullptr);
+                           const Budget &b, cudaStream_t s, const float *lrn = nullptr,
+                           const CUtensorMap *tmap_y = nullptr);
+// tmap_y (optional): tiled map of the output [M][out_cs] (box 32 columns x
+// 32 rows, SW64 for bf16 / SW128 for fp32); full 32-column chunks are then
+// written by TMA tensor stores from the epilogue's staging boxes.
 // lrn (optional) = {size, alpha, beta, k} of a following LRN layer fused into
 // the epilogue (size 5, one N tile holding all channels, no split-K).
 // A-slab width in bytes (128 / 64 / 32) for Cg channels per group, 0 if the

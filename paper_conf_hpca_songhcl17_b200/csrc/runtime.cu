@@ -109,6 +109,7 @@ struct GemmStage {           // one implicit-GEMM launch
   std::map<int, CUtensorMap> tmaps;  // weight maps by box rows
   std::map<std::tuple<const void *, int, int, int, int>, CUtensorMap> xmaps;   // A maps by
                                                  // (input, batch, rect w, h, n)
+  std::map<std::pair<const void *, long long>, CUtensorMap> ymaps;   // output maps by (y, M)
   size_t w_bytes = 0;
   void release() {
     if (d_w) cudaFree(d_w);
@@ -119,6 +120,7 @@ struct GemmStage {           // one implicit-GEMM launch
     d_ktab = nullptr;
     tmaps.clear();
     xmaps.clear();
+    ymaps.clear();
   }
 };
 
@@ -571,6 +573,33 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, co
   return &(gs.xmaps[key] = m);
 }
 
+// Output map for the epilogue's TMA tensor stores: the [M][out_cs] output
+// matrix (rows = output pixels, padded grid in pm mode), boxes of 32 columns
+// x 32 rows, swizzle = the box row width (64 B bf16 / 128 B fp32).  nullptr
+// when the layout does not meet TMA's alignment rules (row stores are used).
+static const CUtensorMap *stage_ymap(GemmStage &gs, void *y, long long M) {
+  const ConvGeom &g = gs.g;
+  const int eszo = g.out_mode == OUT_BF16 ? 2 : 4;
+  if (((uintptr_t)y & 15) || ((long long)g.out_cs * eszo) % 16 || g.out_cs < 32) return nullptr;
+  const auto key = std::make_pair((const void *)y, M);
+  auto it = gs.ymaps.find(key);
+  if (it != gs.ymaps.end()) return &it->second;
+  auto enc = get_encode_tiled();
+  if (!enc) return nullptr;
+  CUtensorMap m;
+  const cuuint64_t dims[2] = {(cuuint64_t)g.out_cs, (cuuint64_t)M};
+  const cuuint64_t strides[1] = {(cuuint64_t)g.out_cs * eszo};
+  const cuuint32_t box[2] = {32, 32};
+  const cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(&m, eszo == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                   2, y, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   eszo == 2 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return nullptr;
+  if (gs.ymaps.size() > 64) gs.ymaps.clear();
+  return &(gs.ymaps[key] = m);
+}
+
 // ------------------------------------------------------------------ planning
 // Tile / split selection (the paper's sub-matrix choice, P:223,
 // P:267).  For every CTA grouping cg (1 CTA, M = 128 / CTA pair, M = 256) and
@@ -779,8 +808,14 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
     if (p.splits > 1 && (size_t)p.splits * g.M * g.out_cs * 4 > net->ws_bytes)
       return fail(PCNN_ERR_OUT_OF_MEMORY, "split-K workspace not reserved");
     g_launches += p.splits > 1 ? 1 : 0;   // the reduction kernel
+    static const bool no_tma_store = [] {
+      const char *e = getenv("PCNN_NO_TMA_STORE");
+      return e && e[0] == '1';
+    }();
+    const CUtensorMap *ym =
+        (p.splits == 1 && !lrn && !p.rect_w && !no_tma_store) ? stage_ymap(gs, y, g.M) : nullptr;
     CUDA_TRY(counted(launch_conv_tc(g, gs.st, xm, tm, gs.d_bias, y, gs.d_ktab, p, net->d_ws,
-                                    b, s, lrn)));
+                                    b, s, lrn, ym)));
   } else {
     const int tiles = conv_simt_tiles(g);
     const bool gated = is_gated(net, ly);
@@ -1205,11 +1240,16 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   // fewer A bytes than im2col boxes.  Chosen per net: the conv's producer and
   // consumer must read / write the halo layout (pools and pm convs of the same
   // halo do; a staged-im2col first layer joins as a 1 x 1 pm conv), channels
-  // per group must fill 128 B slabs, and the halo may add at most 25% rows.
+  // per group must fill 128 B slabs, and the halo may add at most 40% rows.
   const int n = n_layers;
   {
     const char *e = getenv("PCNN_NO_PM");
     const bool allow = prec != PCNN_FP32_SIMT && !(e && e[0] == '1');
+    // halo rows are computed and discarded: up to 40% extra MMA rows still
+    // beats im2col boxes (S x fewer A bytes through the tiled-TMA path,
+    // measured 2x faster per byte than im2col mode on B200)
+    const char *eh = getenv("PCNN_PM_MAX_HALO");
+    const double pm_max_halo = eh ? atof(eh) : 1.40;
     auto kind = [&](int j) { return net->layers[j].d.kind; };
     auto is_pool = [&](int j) { return kind(j) == PCNN_MAXPOOL || kind(j) == PCNN_AVGPOOL; };
     std::vector<int> pmh(n, 0);
@@ -1220,7 +1260,7 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
         const int S = ly.d.kernel, P = ly.d.pad, g = ly.d.groups;
         if (ly.d.stride != 1 || S != 2 * P + 1 || P < 1 || P > 3 || ly.in_cs % g) continue;
         if (tc_slab_bytes(net->st, ly.in_cs / g) != 128) continue;
-        if ((double)(ly.in_h + 2 * P) * (ly.in_w + 2 * P) > 1.25 * ly.in_h * ly.in_w) continue;
+        if ((double)(ly.in_h + 2 * P) * (ly.in_w + 2 * P) > pm_max_halo * ly.in_h * ly.in_w) continue;
         pmh[i] = P;
       }
       for (bool changed = true; changed;) {
@@ -1237,7 +1277,9 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
           auto nb_ok = [&](int j) {
             return j >= 0 && j < n && (is_pool(j) || (kind(j) == PCNN_CONV && pmh[j] == pmh[i]));
           };
-          if (!nb_ok(i - 1) || !nb_ok(i + 1)) {
+          // an LRN consumer reads the halo grid too (its kernel takes an input halo)
+          auto cons_ok = [&](int j) { return nb_ok(j) || (j < n && kind(j) == PCNN_LRN); };
+          if (!nb_ok(i - 1) || !cons_ok(i + 1)) {
             pmh[i] = 0;
             changed = true;
           }

@@ -29,13 +29,24 @@ SHAPES = {  # name: (in_shape, layer)
     "norm2pool2": ((256, 27, 27), [dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0), dict(kind="maxpool", k=3, stride=2)]),
     "stage": ((3, 227, 227), dict(kind="maxpool", k=1, stride=1)),
 }
+def make_net(name):
+    """name[+pm]: '+pm' wraps the conv between identity pools so the runtime
+    may choose the padded-layout mode (it needs pool / pm-conv neighbours)."""
+    wrap = name.endswith("+pm")
+    shape, L = SHAPES[name[:-3] if wrap else name]
+    layers = L if isinstance(L, list) else [L]
+    if wrap:
+        ident = dict(kind="maxpool", k=1, stride=1)
+        layers = [ident] + layers + [ident]
+    return shape, dict(in_shape=shape, layers=layers), (1 if wrap else 0)
+
+
 def main():
     name = sys.argv[1]
     B = int(sys.argv[2]) if len(sys.argv) > 2 else 256
     reps = int(sys.argv[3]) if len(sys.argv) > 3 else 20
     prec = sys.argv[4] if len(sys.argv) > 4 else "bf16"
-    shape, L = SHAPES[name]
-    net = dict(in_shape=shape, layers=L if isinstance(L, list) else [L])
+    shape, net, li = make_net(name)
     w, b = synth.net_params(net)
     n = pcnn.Net(net, w, b, B, prec)
     x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
@@ -44,8 +55,10 @@ def main():
         n.infer(x)
     torch.cuda.synchronize()
     ms, k = n.read_layer_timing()
-    info = n.query_layer(0, B)
+    info = n.query_layer(li, B)
     t = sum(ms) / k
+    if li:
+        print("  per layer ms:", [round(v / k, 4) for v in ms], "a_mode", info.get("a_mode"))
     byt = sum(n.query_layer(i, B)["bytes"] for i in range(len(net["layers"])))
     print("%s B=%d %s: %.4f ms  %.1f TFLOP/s  %.0f GB/s  tile %dx%d grid %d splits %d" % (
         name, B, prec, t, info["flops"] / t / 1e9, byt / t / 1e6, info["tile_m"], info["tile_n"],

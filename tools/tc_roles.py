@@ -8,12 +8,11 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 import synth
 from paper_conf_hpca_songhcl17_b200 import pcnn
-from tools.one_layer import SHAPES
+from tools.one_layer import make_net
 
 name = sys.argv[1]
 B = int(sys.argv[2]) if len(sys.argv) > 2 else 256
-shape, L = SHAPES[name]
-net = dict(in_shape=shape, layers=L if isinstance(L, list) else [L])
+shape, net, li = make_net(name)
 w, b = synth.net_params(net)
 n = pcnn.Net(net, w, b, B, "bf16")
 x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
@@ -28,7 +27,7 @@ lib.pcnn_debug_tc_profile(1, out)
 c = list(out)
 ctas = max(c[7], 1)
 life = c[4] / ctas
-print("%s B=%d plan %s" % (name, B, {k: v for k, v in n.query_layer(0, B).items() if k in ("tile_m", "tile_n", "grid", "splits", "tiles")}))
+print("%s B=%d plan %s" % (name, B, {k: v for k, v in n.query_layer(li, B).items() if k in ("tile_m", "tile_n", "grid", "splits", "tiles")}))
 print("  per CTA: lifetime %.0f cyc, K-blocks %.1f (%.0f cyc/kb)" % (life, c[5] / ctas, life / max(c[5] / ctas, 1)))
 for i, lab in [(0, "producer wait EMPTY"), (1, "MMA wait FULL"), (2, "MMA wait TEMPTY"), (3, "epi wait TFULL"), (6, "epi busy")]:
     print("  %-22s %5.1f%%" % (lab, 100.0 * c[i] / ctas / life))
