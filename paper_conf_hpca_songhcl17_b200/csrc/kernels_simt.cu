@@ -3,6 +3,7 @@
 //   conv/FC check path
 //   (the paper's SGEMM), a4/a5 LRN + pooling (fused), a7 softmax + entropy.
 // Activations are NHWC; all arithmetic is fp32; storage is bf16 or fp32.
+#include <cstdlib>
 #include <algorithm>
 
 #include "budget.cuh"
@@ -287,10 +288,165 @@ stage_im2col_kernel(const float *__restrict__ x, void *y, int H, int W, int Ho, 
   }
 }
 
+// 3-channel first-layer staging, both layouts (a1): output pixel (h, w) of
+// an output row, channel k < K = D*D*3 is input (c, h*step - pad + a,
+// w*step - pad + b) with k = (a*D + b)*3 + c -- the (dr, ds, c) order of
+// space-to-depth (D = step = blk) and the (r, s, c) order of first-layer
+// im2col (D = S, step = conv stride) -- and 0 for K <= k < Kp.  One CTA per
+// (image, band of output rows): the band's input rows x 3 channels are copied
+// to smem as aligned 16 B chunks (the fp32 rows are not 16 B aligned: each
+// keeps its 0..3-float shift), then each thread assembles one 16 B output
+// chunk of a pixel -- its chunk's channel map is fixed and lives in registers.
+template <int ST>
+__global__ void __launch_bounds__(256)
+stage_gather3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Ho, int Wo,
+                     int Kp, int D, int step, int pad, int halo, int rows_per_cta, int tf32_round) {
+  constexpr int C = 3;
+  constexpr int VN = Vec16<ST>::N;
+  extern __shared__ __align__(16) float g3_rows[];   // [span*C][Wrow] input rows, 16 B-aligned copies
+  const int Wrow = (W + 3) / 4 * 4 + 4;              // room for the 0..3 float alignment shift
+  const int cpr = Wrow / 4;                          // 16 B chunks loaded per row
+  const int K = D * D * C;
+  const int bands = (Ho + rows_per_cta - 1) / rows_per_cta;
+  const int h0 = (blockIdx.x % bands) * rows_per_cta;
+  const int nh = min(rows_per_cta, Ho - h0);
+  const long long n = blockIdx.x / bands;
+  const int span = (nh - 1) * step + D;
+  const int nrow = span * C;
+  const int max_rows = ((rows_per_cta - 1) * step + D) * C;
+  int *row_shift = (int *)(g3_rows + (size_t)max_rows * Wrow);   // -1: row outside the image
+  const long long total = (long long)B * C * H * W;
+  // phase 1: each input row [ih][0, W) of the band as aligned 16 B chunks
+  // (cp.async, zero fill past the end of the tensor); shift = row start % 4
+  const float inv_cpr = 1.f / (float)cpr;
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(g3_rows);
+  for (int v = threadIdx.x; v < nrow * cpr; v += blockDim.x) {
+    int r, jc;
+    fdivmod(v, cpr, inv_cpr, r, jc);
+    const int a = r / C, c = r - a * C;
+    const int ih = h0 * step - pad + a;
+    if (ih < 0 || ih >= H) continue;
+    const long long e0 = ((n * C + c) * H + ih) * (long long)W;
+    const long long a0 = e0 & ~3LL;
+    const long long e = a0 + 4LL * jc;
+    const int bytes = e + 4 <= total ? 16 : (e < total ? (int)(total - e) * 4 : 0);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(
+                     sbase + (uint32_t)((r * Wrow + 4 * jc) * 4)),
+                 "l"(x + (bytes ? e : 0)), "r"(bytes)
+                 : "memory");
+  }
+  for (int r = threadIdx.x; r < nrow; r += blockDim.x) {
+    const int a = r / C, c = r - a * C;
+    const int ih = h0 * step - pad + a;
+    row_shift[r] = (ih < 0 || ih >= H) ? -1 : (int)((((n * C + c) * H + ih) * (long long)W) & 3);
+  }
+  asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
+  __syncthreads();
+  // phase 2: thread = (pixel, 16 B output chunk); its chunk index is fixed
+  // (blockDim % chunks == 0), so the chunk's channel -> (row, column offset)
+  // map is computed once into registers
+  const int chunks = Kp / VN;
+  const int ch = threadIdx.x % chunks;
+  int rr[VN], bb[VN];
+#pragma unroll
+  for (int e = 0; e < VN; ++e) {
+    const int k = ch * VN + e;
+    if (k < K) {
+      const int ab = k / C, c = k - ab * C;
+      const int a = ab / D;
+      rr[e] = a * C + c;
+      bb[e] = ab - a * D - pad;
+    } else {
+      rr[e] = -1;
+      bb[e] = 0;
+    }
+  }
+  const int Wop = Wo + 2 * halo;
+  const int ppi = blockDim.x / chunks;               // pixels per pass
+  for (int hh = 0; hh < nh; ++hh) {
+    const int h = h0 + hh;
+    char *yrow = (char *)y + ((size_t)(n * (Ho + 2 * halo) + h + halo) * Wop + halo) *
+                                 (size_t)Kp * (ST == ST_BF16 ? 2 : 4);
+    // per channel of this thread's chunk: smem index of input column 0 of its
+    // row in this output row, minus the pad (can be negative: the sentinel for
+    // a row outside the image is NOROW)
+    constexpr int NOROW = -(1 << 30);
+    int base[VN];
+#pragma unroll
+    for (int e = 0; e < VN; ++e) {
+      base[e] = NOROW;
+      if (rr[e] >= 0) {
+        const int r = rr[e] + hh * step * C;
+        const int sh = row_shift[r];
+        if (sh >= 0) base[e] = r * Wrow + sh + bb[e];
+      }
+    }
+    for (int w = threadIdx.x / chunks; w < Wo; w += ppi) {
+      const int iw0 = w * step - pad;                // column of tap offset 0
+      const bool inner = iw0 >= 0 && iw0 + D <= W;
+      Vec16<ST> o;
+#pragma unroll
+      for (int e = 0; e < VN; ++e) {
+        float val = 0.f;
+        if (base[e] != NOROW) {
+          const int iw = w * step + bb[e];
+          if (inner || (iw >= 0 && iw < W)) val = g3_rows[base[e] + w * step];
+        }
+        o.v[e] = val;
+      }
+      o.store(yrow + ((size_t)w * chunks + ch) * 16, tf32_round);
+    }
+  }
+}
+
+static bool gather3_ok(int st, int W, int Kp, int D, int step) {
+  const int vn = st == ST_BF16 ? 8 : 4;
+  const int Wrow = (W + 3) / 4 * 4 + 4;
+  return Kp % vn == 0 && 256 % (Kp / vn) == 0 && D * D * 3 <= Kp &&
+         (size_t)D * 3 * (Wrow * sizeof(float) + sizeof(int)) <= 96 * 1024 && step >= 1;
+}
+
+static cudaError_t launch_gather3(const float *x, void *y, int st, int B, int H, int W, int Ho,
+                                  int Wo, int Kp, int D, int step, int pad, int halo,
+                                  int tf32_round, cudaStream_t s) {
+  static const int rows_env = [] {
+    const char *e = getenv("PCNN_STAGE_ROWS");
+    return e ? atoi(e) : 0;
+  }();
+  const int vn = st == ST_BF16 ? 8 : 4;
+  if (Kp % vn || 256 % (Kp / vn) || D * D * 3 > Kp) return cudaErrorInvalidValue;
+  const int Wrow = (W + 3) / 4 * 4 + 4;
+  auto smem_for = [&](int R) {
+    return (size_t)((R - 1) * step + D) * 3 * (Wrow * sizeof(float) + sizeof(int));
+  };
+  int R = rows_env > 0 ? rows_env : 1;
+  if (rows_env <= 0)
+    while (R < 8 && R < Ho && smem_for(R + 1) <= 40 * 1024) ++R;
+  const size_t smem = smem_for(R);
+  if (smem > 96 * 1024) return cudaErrorInvalidValue;
+  const unsigned grid = (unsigned)((long long)B * ((Ho + R - 1) / R));
+  if (st == ST_BF16) {
+    if (smem > 48 * 1024)
+      cudaFuncSetAttribute(stage_gather3_kernel<ST_BF16>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    stage_gather3_kernel<ST_BF16><<<grid, 256, smem, s>>>(x, y, B, H, W, Ho, Wo, Kp, D, step,
+                                                           pad, halo, R, 0);
+  } else {
+    if (smem > 48 * 1024)
+      cudaFuncSetAttribute(stage_gather3_kernel<ST_F32>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    stage_gather3_kernel<ST_F32><<<grid, 256, smem, s>>>(x, y, B, H, W, Ho, Wo, Kp, D, step,
+                                                          pad, halo, R, tf32_round);
+  }
+  return cudaGetLastError();
+}
+
 cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, int H, int W,
                                 int S, int stride, int pad, int Ho, int Wo, int Kp,
                                 int halo, int tf32_round, cudaStream_t s) {
   if (C != 3 || (S != 3 && S != 5)) return cudaErrorInvalidValue;
+  if (!getenv("PCNN_OLD_STAGE") && gather3_ok(st, W, Kp, S, stride))
+    return launch_gather3(x, y, st, B, H, W, Ho, Wo, Kp, S, stride, pad, halo, tf32_round, s);
   const size_t smem = (size_t)S * C * ((Wo - 1) * stride + S) * sizeof(float);
   if (smem > 48 * 1024) return cudaErrorInvalidValue;
   const unsigned grid = (unsigned)((long long)B * Ho);
@@ -308,6 +464,8 @@ cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, i
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
                                int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {
+  if (C == 3 && !getenv("PCNN_OLD_STAGE") && gather3_ok(st, W, Cs, blk, blk))
+    return launch_gather3(x, y, st, B, H, W, Hs, Ws, Cs, blk, blk, pad, 0, tf32_round, s);
   if (C == 3 && (blk == 4 || blk == 1) && W <= 4096) {
     const int Wp = ((Ws * blk + 3) & ~3) + 4;
     const size_t smem = (size_t)blk * C * Wp * sizeof(float);
@@ -529,6 +687,7 @@ struct LrnPoolArgs {
   int ocg, ocp;            // output group layout: ocg real channels padded to
                            // ocp per group (0 = compact, Cout == C)
   int hi, ho;              // zero halo of the input / output layout (pixels per side)
+  int R, nbands;           // band kernel: output rows per tile, bands per image
   Budget b;
 };
 
@@ -691,6 +850,175 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
   });
 }
 
+// LRN (+ optional pool) over bands of R output rows: the band's input rows
+// are staged once (cp.async, padded pixel pitch so per-pixel accesses are
+// conflict-free), normalised IN PLACE by one thread per pixel streaming its
+// channels in order (the 5-channel window of chunk j needs only the original
+// tail of chunk j-1, kept in registers, and the head of chunk j+1, not yet
+// overwritten), then pooled from smem.  Every input pixel is normalised once
+// per band (rows shared by two bands: (R*s + k - s) / (R*s) recompute) instead
+// of once per pooling window.  Same per-element arithmetic as lrn_pool_kernel
+// and the conv epilogue (sum order, lrn_scale_pow), so results are identical.
+template <int ST, int LS>
+__global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
+  extern __shared__ __align__(16) uint8_t lb_smem[];
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  constexpr int VN = Vec16<ST>::N;
+  constexpr int HALF = LS / 2;
+  static_assert(HALF <= VN, "LRN window wider than one neighbouring chunk");
+  const int C = a.C, chunks = C / VN;
+  const int pitch = C * ESZ + 16;
+  const long long tiles = (long long)a.B * a.nbands;
+  const int Hp = a.H + 2 * a.hi, Wp = a.W + 2 * a.hi;
+  const int Hop = a.Ho + 2 * a.ho, Wop = a.Wo + 2 * a.ho;
+  const float inv_chunks = 1.f / (float)chunks;
+
+  for_each_tile(a.b, tiles, [&](long long t) {
+    const int band = (int)(t % a.nbands);
+    const long long n = t / a.nbands;
+    const int p0 = band * a.R, p1 = min(p0 + a.R, a.Ho);
+    const int h0 = p0 * a.s, h1 = min((p1 - 1) * a.s + a.k, a.H);
+    const int nr = h1 - h0;
+    if (a.ho > 0) {
+      // zero the output halo cells this band owns: top / bottom halo rows
+      // with the first / last band, left / right columns of its rows
+      const int oc16 = a.Cout * ESZ / 16;
+      const uint4 z = make_uint4(0, 0, 0, 0);
+      uint4 *yb = (uint4 *)a.y;
+      if (p0 == 0)
+        for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
+          yb[(size_t)n * Hop * Wop * oc16 + v] = z;
+      if (p1 == a.Ho)
+        for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
+          yb[((size_t)n * Hop + a.Ho + a.ho) * Wop * oc16 + v] = z;
+      for (int v = threadIdx.x; v < (p1 - p0) * 2 * a.ho * oc16; v += blockDim.x) {
+        const int rr = v / (2 * a.ho * oc16), e = v - rr * 2 * a.ho * oc16;
+        const int side = e / (a.ho * oc16), o = e - side * a.ho * oc16;
+        const size_t rowb = ((size_t)n * Hop + p0 + rr + a.ho) * Wop * oc16;
+        yb[rowb + (side ? (size_t)(a.Wo + a.ho) * oc16 : 0) + o] = z;
+      }
+    }
+    __syncthreads();   // the previous band's pooling is done with smem
+    const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(lb_smem);
+    const int npix = nr * a.W;
+    for (int v = threadIdx.x; v < npix * chunks; v += blockDim.x) {
+      int pix, ch;
+      fdivmod(v, chunks, inv_chunks, pix, ch);
+      const int r = pix / a.W, col = pix - r * a.W;
+      const size_t src = (((size_t)n * Hp + h0 + r + a.hi) * Wp + col + a.hi) * C + (size_t)ch * VN;
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(
+                       sbase + (uint32_t)(pix * pitch + ch * 16)),
+                   "l"((const char *)a.x + src * ESZ)
+                   : "memory");
+    }
+    asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
+    __syncthreads();
+    if (LS > 0) {
+      for (int pix = threadIdx.x; pix < npix; pix += blockDim.x) {
+        uint8_t *px = lb_smem + pix * pitch;
+        float tail[HALF > 0 ? HALF : 1];
+#pragma unroll
+        for (int j = 0; j < HALF; ++j) tail[j] = 0.f;
+        Vec16<ST> cur, nxt;
+        cur.load(px);
+        for (int ch = 0; ch < chunks; ++ch) {
+          if (ch + 1 < chunks) nxt.load(px + (ch + 1) * 16);
+          else
+#pragma unroll
+            for (int j = 0; j < VN; ++j) nxt.v[j] = 0.f;
+          float sq[VN + 2 * HALF];
+#pragma unroll
+          for (int j = 0; j < VN + 2 * HALF; ++j) {
+            const int o = j - HALF;
+            const float xv = o < 0 ? tail[HALF + o] : (o < VN ? cur.v[o] : nxt.v[o - VN]);
+            sq[j] = xv * xv;
+          }
+          Vec16<ST> out;
+#pragma unroll
+          for (int j = 0; j < VN; ++j) {
+            float acc = 0.f;
+#pragma unroll
+            for (int w = 0; w < LS; ++w) acc += sq[j + w];
+            const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
+            out.v[j] = cur.v[j] * lrn_scale_pow(scale, a.lrn_beta);
+          }
+          out.store(px + ch * 16, a.tf32_round);
+#pragma unroll
+          for (int j = 0; j < HALF; ++j) tail[j] = cur.v[VN - HALF + j];
+          cur = nxt;
+        }
+      }
+      __syncthreads();
+    }
+    // pool (k = s = 1: copy) the normalised rows
+    const float inv = 1.f / (float)(a.k * a.k);
+    const int ochunks = a.Cout / VN;
+    const float inv_oc = 1.f / (float)ochunks;
+    const int grp_real = a.ocg / VN, grp_pad = a.ocp / VN;
+    const int nq = a.Wo * ochunks;
+    for (int v = threadIdx.x; v < (p1 - p0) * nq; v += blockDim.x) {
+      const int rr = v / nq;
+      int q, oc;
+      fdivmod(v - rr * nq, ochunks, inv_oc, q, oc);
+      const int pp = p0 + rr;
+      int ch = oc;
+      bool pad = false;
+      if (grp_pad > 0) {
+        const int gi = oc / grp_pad, j = oc - gi * grp_pad;
+        pad = j >= grp_real;
+        ch = gi * grp_real + j;
+      }
+      char *dst = (char *)a.y + ((((size_t)n * Hop + pp + a.ho) * Wop + q + a.ho) * a.Cout + oc * VN) * ESZ;
+      const int rs = pp * a.s - h0, re = min(rs + a.k, nr);
+      const int cs = q * a.s, ce = min(cs + a.k, a.W);
+      if (ST == ST_BF16 && a.is_max) {
+        __nv_bfloat162 m[4];
+        const __nv_bfloat162 ninf = __float2bfloat162_rn(-INFINITY);
+        const __nv_bfloat162 zero = __float2bfloat162_rn(0.f);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) m[j] = pad ? zero : ninf;
+        if (!pad)
+          for (int r = rs; r < re; ++r)
+            for (int col = cs; col < ce; ++col) {
+              const uint4 raw = *(const uint4 *)(lb_smem + (r * a.W + col) * pitch + ch * 16);
+              const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
+#pragma unroll
+              for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], h[j]);
+            }
+        *(uint4 *)dst = *(const uint4 *)m;
+        continue;
+      }
+      Vec16<ST> acc, cur;
+#pragma unroll
+      for (int j = 0; j < VN; ++j) acc.v[j] = pad ? 0.f : (a.is_max ? -INFINITY : 0.f);
+      if (!pad) {
+        for (int r = rs; r < re; ++r)
+          for (int col = cs; col < ce; ++col) {
+            cur.load(lb_smem + (r * a.W + col) * pitch + ch * 16);
+#pragma unroll
+            for (int j = 0; j < VN; ++j)
+              acc.v[j] = a.is_max ? fmaxf(acc.v[j], cur.v[j]) : acc.v[j] + cur.v[j];
+          }
+        if (!a.is_max)
+#pragma unroll
+          for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
+      }
+      acc.store(dst, a.is_max ? 0 : a.tf32_round);
+    }
+  });
+}
+
+constexpr int LB_SMEM_BUDGET = 100 * 1024;
+
+// output rows per band so that the band's staged rows fit LB_SMEM_BUDGET
+static int lrn_band_rows(int st, int W, int C, int k, int s, int Ho) {
+  const int esz = st == ST_BF16 ? 2 : 4;
+  const size_t row = (size_t)W * (C * esz + 16);
+  int R = 1;
+  while (R < Ho && (size_t)((R) * s + k) * row <= LB_SMEM_BUDGET) ++R;
+  return R;
+}
+
 constexpr int LP_SMEM_BUDGET = 48 * 1024;
 
 // Output columns per tile so that the staged rows fit the smem budget.
@@ -735,6 +1063,10 @@ static cudaError_t lrn_pool_dispatch(const LrnPoolArgs &a, int grid, size_t smem
 }
 
 long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int Ho, int Wo) {
+  if (lrn) {
+    const int R = lrn_band_rows(st, W, C, k, s, Ho);
+    return (long long)B * ((Ho + R - 1) / R);
+  }
   const int Q = lrn_pool_cols(st, W, C, lrn, k, s, Wo);
   return (long long)B * Ho * ((Wo + Q - 1) / Q);
 }
@@ -776,6 +1108,27 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.ho = out_halo;
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
+  if (lrn_size > 0 && (lrn_size == 5 || lrn_size == 3)) {
+    // band kernel (every LRN, fused with a following pool or not)
+    a.R = lrn_band_rows(st, W, C, k, s, Ho);
+    a.nbands = (Ho + a.R - 1) / a.R;
+    const size_t smem = (size_t)(min((a.R - 1) * s + k, H)) * W * (C * esz + 16);
+    if (smem > 200 * 1024) return cudaErrorInvalidValue;
+#define PCNN_LB(STT, LSS)                                                                       \
+  do {                                                                                          \
+    if (smem > 48 * 1024)                                                                       \
+      cudaFuncSetAttribute(lrn_band_kernel<STT, LSS>,                                           \
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);             \
+    lrn_band_kernel<STT, LSS><<<grid, 256, smem, stream>>>(a);                                  \
+  } while (0)
+    if (st == ST_BF16) {
+      if (lrn_size == 5) PCNN_LB(ST_BF16, 5); else PCNN_LB(ST_BF16, 3);
+    } else {
+      if (lrn_size == 5) PCNN_LB(ST_F32, 5); else PCNN_LB(ST_F32, 3);
+    }
+#undef PCNN_LB
+    return cudaGetLastError();
+  }
   const size_t smem = (size_t)k * ((a.Q - 1) * s + k) * C * esz * (lrn_size > 0 ? 2 : 1);
   if (smem > 200 * 1024) return cudaErrorInvalidValue;
   if (st == ST_BF16) return lrn_pool_dispatch<ST_BF16>(a, grid, smem, stream);

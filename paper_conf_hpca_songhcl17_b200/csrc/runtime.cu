@@ -392,7 +392,7 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
                                int groups, int S, int stride, int pad, int relu,
                                int in_c, int in_h, int in_w, int in_cs, bool is_fc,
                                const float *w, const float *bias, int out_mode,
-                               int pm_halo = 0) {
+                               int pm_halo = 0, bool pm_valid = false) {
   gs.release();
   gs.st = storage_of(precision);
   gs.engine = precision == PCNN_FP32_SIMT ? 0 : 1;
@@ -435,7 +435,18 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
     g.Nfg = Nf / groups;
     g.K = S * S * Cg_st;
     g.Kpad = round_up(g.K, k_align(precision));
-    if (pm_halo > 0) {
+    if (pm_halo > 0 && pm_valid) {
+      // a 'valid' stride-1 conv (pad 0, S = 2h + 1) read as a 'same' conv on
+      // its own input grid: the input is the halo-h grid of the output, the
+      // windows are shifted by the virtual pad h (layer 0 after space-to-depth)
+      if (gs.engine != 1 || stride != 1 || pad != 0 || S != 2 * pm_halo + 1)
+        return fail(PCNN_ERR_UNSUPPORTED, "valid padded-layout mode needs pad 0, S = 2h + 1");
+      g.pm = 1;
+      g.vh = pm_halo;
+      g.hv = in_h;
+      g.wv = in_w;
+      g.pad = pm_halo;
+    } else if (pm_halo > 0) {
       if (gs.engine != 1 || stride != 1 || S != 2 * pad + 1 || pad > pm_halo)
         return fail(PCNN_ERR_UNSUPPORTED, "padded-layout mode needs a stride-1 'same' conv");
       g.pm = 1;
@@ -847,7 +858,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
 static bool fuse_conv_lrn(const pcnn_net *net, int i) {
   if (!net->fuse_lrn_pool || i + 1 >= (int)net->layers.size()) return false;
   const Layer &c = net->layers[i], &l = net->layers[i + 1];
-  return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 &&
+  return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 && c.pm_halo == 0 &&
          c.exact.engine == 1 && c.variant == PCNN_VARIANT_EXACT && c.d.groups == 1 &&
          c.d.out_channels <= 128 && c.out_cs == c.d.out_channels;
 }
@@ -1265,6 +1276,19 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
       }
       for (bool changed = true; changed;) {
         changed = false;
+        if (net->stage_blk > 1 && n > 1 && kind(0) == PCNN_CONV) {
+          // space-to-depth first conv: Sp x Sp, stride 1, pad 0 on the staged
+          // grid -- a 'valid' pm conv when Sp is odd and its consumer reads a halo
+          const int Sp = (net->layers[0].d.kernel + net->stage_blk - 1) / net->stage_blk;
+          const int hh = (Sp % 2 == 1 && Sp > 1 && Sp <= 7 &&
+                          tc_slab_bytes(net->st, net->in_cs) == 128 &&
+                          (is_pool(1) || kind(1) == PCNN_LRN))
+                             ? (Sp - 1) / 2 : 0;
+          if (pmh[0] != hh) {
+            pmh[0] = hh;
+            changed = true;
+          }
+        }
         if (net->stage_im2col && n > 1) {
           const int h = kind(1) == PCNN_CONV && tc_slab_bytes(net->st, net->in_cs) ? pmh[1] : 0;
           if (pmh[0] != h) {
@@ -1288,7 +1312,7 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
     }
     for (int i = 0; i < n; ++i) {
       Layer &ly = net->layers[i];
-      ly.in_halo = i > 0 ? net->layers[i - 1].out_halo : pmh[0];
+      ly.in_halo = i > 0 ? net->layers[i - 1].out_halo : (net->stage_blk > 1 ? 0 : pmh[0]);
       ly.pm_halo = pmh[i];
       if (pmh[i]) ly.out_halo = pmh[i];
       else if (is_pool(i) && i + 1 < n && kind(i + 1) == PCNN_CONV) ly.out_halo = pmh[i + 1];
@@ -1315,7 +1339,8 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
         const int Sp = (ly.d.kernel + net->stage_blk - 1) / net->stage_blk;
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, 1, Sp, 1, 0, ly.d.relu,
                         net->stage_c, net->stage_h, net->stage_w, net->in_cs, false,
-                        s2d_w.data(), biases ? biases[i] : nullptr, mode);
+                        s2d_w.data(), biases ? biases[i] : nullptr, mode, ly.pm_halo,
+                        ly.pm_halo > 0);
       } else {
         s = build_stage(ly.exact, ly, prec, ly.d.out_channels, is_fc ? 1 : ly.d.groups,
                         is_fc ? 1 : ly.d.kernel, is_fc ? 1 : ly.d.stride,

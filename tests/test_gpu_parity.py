@@ -46,6 +46,34 @@ CONV_CASES = [
 ]
 
 
+# first-layer staging (a1): 3-channel inputs staged as im2col rows (S <= 5)
+# or space-to-depth (strided S = 11), in bands of output rows -- sizes that
+# span several bands with ragged last bands, checked element by element so a
+# single wrong tap in one band row cannot hide under the max-relative metric
+STAGE_CASES = [
+    # (out, k, stride, pad, H, W, B)
+    (32, 3, 1, 1, 40, 40, 3),
+    (16, 5, 1, 2, 45, 37, 2),
+    (96, 11, 4, 0, 67, 71, 2),
+    (64, 3, 1, 1, 23, 224, 1),
+]
+
+
+@pytest.mark.parametrize("prec", PRECS)
+@pytest.mark.parametrize("case", STAGE_CASES, ids=lambda c: "x".join(map(str, c)))
+def test_first_layer_staging_elementwise(orc, prec, case):
+    out_c, k, st, pad, H, W, B = case
+    net = dict(in_shape=(3, H, W), layers=[conv_layer(out_c, k, 3, st, pad, 1, relu=False)])
+    w, b = params(net, seed=41)
+    x = small_inputs((3, H, W), B, lo=-1, hi=1)
+    ref = orc.run_net(net, w, b, x).reshape(B, out_c, -1)
+    out = gpu_run(net, w, b, x, prec)["out"].reshape(B, out_c, -1)
+    scale = np.abs(ref).max()
+    # per output pixel: the worst channel's error, relative to the layer scale
+    per_pix = np.abs(out - ref).max(axis=1) / scale
+    assert per_pix.max() <= TOL[prec] / 4, np.argwhere(per_pix > TOL[prec] / 4)[:8]
+
+
 @pytest.mark.parametrize("prec", PRECS)
 @pytest.mark.parametrize("case", CONV_CASES, ids=lambda c: "x".join(map(str, c)))
 def test_conv_layer_parity(orc, prec, case):
