@@ -38,8 +38,8 @@ template <int ST>
 struct Vec16 {
   static constexpr int N = ST == ST_BF16 ? 8 : 4;
   float v[N];
-  __device__ __forceinline__ void load(const void *p) {
-    const uint4 raw = *(const uint4 *)p;
+  __device__ __forceinline__ void load(const void *p) { from_raw(*(const uint4 *)p); }
+  __device__ __forceinline__ void from_raw(const uint4 raw) {
     if constexpr (ST == ST_BF16) {
       const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
 #pragma unroll
@@ -1008,12 +1008,199 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
   });
 }
 
+// LRN (+ optional pool) over bands of R output rows, LRN in registers.
+// P lanes of one warp share a pixel, each owning CPT consecutive 16 B channel
+// chunks that it loads straight from global memory (a warp reads one
+// contiguous run of pixels); the 2 channels of the window that lie in the
+// neighbouring lanes' chunks come by warp shuffle, so there is no staging
+// pass and no serial walk along the channels.  The normalised band is written
+// once to shared memory (chunk c of pixel x at slot c ^ ((x*P + c/8) & 7) when
+// CPT == 8, so neither the writes nor the pooling reads conflict) and pooled
+// from there.  Same per-element arithmetic as the other LRN paths (sum order,
+// lrn_scale_pow), so the results are identical.
+template <int ST, int CPT>
+__global__ void __launch_bounds__(256) lrn_reg_kernel(const LrnPoolArgs a) {
+  extern __shared__ __align__(16) uint8_t lr_smem[];
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  constexpr int VN = Vec16<ST>::N;
+  constexpr int HALF = 2;                      // LRN size 5
+  constexpr bool SWZ = CPT == 8;
+  const int C = a.C, chunks = C / VN, P = chunks / CPT;
+  const long long tiles = (long long)a.B * a.nbands;
+  const int Hp = a.H + 2 * a.hi, Wp = a.W + 2 * a.hi;
+  const int Hop = a.Ho + 2 * a.ho, Wop = a.Wo + 2 * a.ho;
+  const int lane = threadIdx.x & 31;
+  auto slot = [&](int pix, int c) -> int {
+    return SWZ ? (c ^ ((pix * P + (c >> 3)) & 7)) : c;
+  };
+
+  for_each_tile(a.b, tiles, [&](long long t) {
+    const int band = (int)(t % a.nbands);
+    const long long n = t / a.nbands;
+    const int p0 = band * a.R, p1 = min(p0 + a.R, a.Ho);
+    const int h0 = p0 * a.s, h1 = min((p1 - 1) * a.s + a.k, a.H);
+    const int nr = h1 - h0;
+    if (a.ho > 0) {
+      const int oc16 = a.Cout * ESZ / 16;
+      const uint4 z = make_uint4(0, 0, 0, 0);
+      uint4 *yb = (uint4 *)a.y;
+      if (p0 == 0)
+        for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
+          yb[(size_t)n * Hop * Wop * oc16 + v] = z;
+      if (p1 == a.Ho)
+        for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
+          yb[((size_t)n * Hop + a.Ho + a.ho) * Wop * oc16 + v] = z;
+      for (int v = threadIdx.x; v < (p1 - p0) * 2 * a.ho * oc16; v += blockDim.x) {
+        const int rr = v / (2 * a.ho * oc16), e = v - rr * 2 * a.ho * oc16;
+        const int side = e / (a.ho * oc16), o = e - side * a.ho * oc16;
+        const size_t rowb = ((size_t)n * Hop + p0 + rr + a.ho) * Wop * oc16;
+        yb[rowb + (side ? (size_t)(a.Wo + a.ho) * oc16 : 0) + o] = z;
+      }
+    }
+    __syncthreads();   // the previous band's pooling is done with smem
+    const int npix = nr * a.W;
+    const int nv = (npix * P + 31) & ~31;     // warp-uniform trip count
+    for (int v = threadIdx.x; v < nv; v += blockDim.x) {
+      const int pix = v / P, part = v - pix * P;
+      const bool ok = pix < npix;
+      const int r = ok ? pix / a.W : 0, col = ok ? pix - r * a.W : 0;
+      const char *src = (const char *)a.x +
+          ((((size_t)n * Hp + h0 + r + a.hi) * Wp + col + a.hi) * C + (size_t)part * CPT * VN) * ESZ;
+      Vec16<ST> ch[CPT];
+#pragma unroll
+      for (int j = 0; j < CPT; ++j) {
+        if (ok) {
+          const uint4 raw = __ldg((const uint4 *)(src + j * 16));
+          ch[j].from_raw(raw);
+        } else {
+#pragma unroll
+          for (int i = 0; i < VN; ++i) ch[j].v[i] = 0.f;
+        }
+      }
+      // window neighbours held by the adjacent lanes of the same pixel
+      float tail[HALF], head[HALF];
+#pragma unroll
+      for (int i = 0; i < HALF; ++i) {
+        tail[i] = __shfl_up_sync(0xffffffffu, ch[CPT - 1].v[VN - HALF + i], 1);
+        head[i] = __shfl_down_sync(0xffffffffu, ch[0].v[i], 1);
+        if (part == 0) tail[i] = 0.f;
+        if (part == P - 1 || lane == 31) head[i] = 0.f;
+      }
+      if (ok) {
+        uint8_t *dst = lr_smem + (size_t)pix * chunks * 16;
+#pragma unroll
+        for (int j = 0; j < CPT; ++j) {
+          float sq[VN + 2 * HALF];
+#pragma unroll
+          for (int q = 0; q < VN + 2 * HALF; ++q) {
+            const int o = q - HALF;
+            float xv;
+            if (o < 0) xv = j > 0 ? ch[j - 1].v[VN + o] : tail[HALF + o];
+            else if (o < VN) xv = ch[j].v[o];
+            else xv = j + 1 < CPT ? ch[j + 1].v[o - VN] : head[o - VN];
+            sq[q] = xv * xv;
+          }
+          Vec16<ST> out;
+#pragma unroll
+          for (int q = 0; q < VN; ++q) {
+            float acc = 0.f;
+#pragma unroll
+            for (int w = 0; w < 2 * HALF + 1; ++w) acc += sq[q + w];
+            const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
+            out.v[q] = ch[j].v[q] * lrn_scale_pow(scale, a.lrn_beta);
+          }
+          out.store(dst + slot(pix, part * CPT + j) * 16, a.tf32_round);
+        }
+      }
+    }
+    __syncthreads();
+    // pool (k = s = 1: copy) the normalised rows
+    const float inv = 1.f / (float)(a.k * a.k);
+    const int ochunks = a.Cout / VN;
+    const float inv_oc = 1.f / (float)ochunks;
+    const int grp_real = a.ocg / VN, grp_pad = a.ocp / VN;
+    const int nq = a.Wo * ochunks;
+    for (int v = threadIdx.x; v < (p1 - p0) * nq; v += blockDim.x) {
+      const int rr = v / nq;
+      int q, oc;
+      fdivmod(v - rr * nq, ochunks, inv_oc, q, oc);
+      const int pp = p0 + rr;
+      int c = oc;
+      bool pad = false;
+      if (grp_pad > 0) {
+        const int gi = oc / grp_pad, j = oc - gi * grp_pad;
+        pad = j >= grp_real;
+        c = gi * grp_real + j;
+      }
+      char *dst = (char *)a.y + ((((size_t)n * Hop + pp + a.ho) * Wop + q + a.ho) * a.Cout + oc * VN) * ESZ;
+      const int rs = pp * a.s - h0, re = min(rs + a.k, nr);
+      const int cs = q * a.s, ce = min(cs + a.k, a.W);
+      if (ST == ST_BF16 && a.is_max) {
+        __nv_bfloat162 m[4];
+        const __nv_bfloat162 ninf = __float2bfloat162_rn(-INFINITY);
+        const __nv_bfloat162 zero = __float2bfloat162_rn(0.f);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) m[j] = pad ? zero : ninf;
+        if (!pad)
+          for (int r = rs; r < re; ++r)
+            for (int col = cs; col < ce; ++col) {
+              const int pix = r * a.W + col;
+              const uint4 raw =
+                  *(const uint4 *)(lr_smem + ((size_t)pix * chunks + slot(pix, c)) * 16);
+              const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
+#pragma unroll
+              for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], h[j]);
+            }
+        *(uint4 *)dst = *(const uint4 *)m;
+        continue;
+      }
+      Vec16<ST> acc, cur;
+#pragma unroll
+      for (int j = 0; j < VN; ++j) acc.v[j] = pad ? 0.f : (a.is_max ? -INFINITY : 0.f);
+      if (!pad) {
+        for (int r = rs; r < re; ++r)
+          for (int col = cs; col < ce; ++col) {
+            const int pix = r * a.W + col;
+            cur.load(lr_smem + ((size_t)pix * chunks + slot(pix, c)) * 16);
+#pragma unroll
+            for (int j = 0; j < VN; ++j)
+              acc.v[j] = a.is_max ? fmaxf(acc.v[j], cur.v[j]) : acc.v[j] + cur.v[j];
+          }
+        if (!a.is_max)
+#pragma unroll
+          for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
+      }
+      acc.store(dst, a.is_max ? 0 : a.tf32_round);
+    }
+  });
+}
+
+// chunks per lane of lrn_reg_kernel for C stored channels (0 = not supported):
+// 8 (swizzled) when the chunk count is a multiple of 8, else 6 or 3 with a
+// power-of-two lane count per pixel.
+static int lrn_reg_cpt(int st, int C) {
+  const int vn = st == ST_BF16 ? 8 : 4;
+  if (C % vn) return 0;
+  const int chunks = C / vn;
+  auto pow2_le32 = [](int p) { return p >= 1 && p <= 32 && (p & (p - 1)) == 0; };
+  if (chunks % 8 == 0 && pow2_le32(chunks / 8)) return 8;
+  if (chunks % 6 == 0 && pow2_le32(chunks / 6)) return 6;
+  if (chunks % 3 == 0 && pow2_le32(chunks / 3)) return 3;
+  return 0;
+}
+
 constexpr int LB_SMEM_BUDGET = 100 * 1024;
 
 // output rows per band so that the band's staged rows fit LB_SMEM_BUDGET
-static int lrn_band_rows(int st, int W, int C, int k, int s, int Ho) {
+static bool use_lrn_reg(int st, int C, int lrn) {
+  const char *e = getenv("PCNN_LRN_BAND");     // A/B tests: the staged band kernel
+  const bool off = e && e[0] == '1';
+  return lrn == 5 && !off && lrn_reg_cpt(st, C) > 0;
+}
+
+static int lrn_band_rows(int st, int W, int C, int k, int s, int Ho, int lrn) {
   const int esz = st == ST_BF16 ? 2 : 4;
-  const size_t row = (size_t)W * (C * esz + 16);
+  const size_t row = (size_t)W * (C * esz + (use_lrn_reg(st, C, lrn) ? 0 : 16));
   int R = 1;
   while (R < Ho && (size_t)((R) * s + k) * row <= LB_SMEM_BUDGET) ++R;
   return R;
@@ -1064,7 +1251,7 @@ static cudaError_t lrn_pool_dispatch(const LrnPoolArgs &a, int grid, size_t smem
 
 long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int Ho, int Wo) {
   if (lrn) {
-    const int R = lrn_band_rows(st, W, C, k, s, Ho);
+    const int R = lrn_band_rows(st, W, C, k, s, Ho, lrn);
     return (long long)B * ((Ho + R - 1) / R);
   }
   const int Q = lrn_pool_cols(st, W, C, lrn, k, s, Wo);
@@ -1108,9 +1295,30 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.ho = out_halo;
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
+  if (use_lrn_reg(st, C, lrn_size)) {
+    a.R = lrn_band_rows(st, W, C, k, s, Ho, lrn_size);
+    a.nbands = (Ho + a.R - 1) / a.R;
+    const size_t smem = (size_t)(min((a.R - 1) * s + k, H)) * W * C * esz;
+    if (smem > 200 * 1024) return cudaErrorInvalidValue;
+    const int cpt = lrn_reg_cpt(st, C);
+#define PCNN_LR(STT, CP)                                                                        \
+  do {                                                                                          \
+    if (smem > 48 * 1024)                                                                       \
+      cudaFuncSetAttribute(lrn_reg_kernel<STT, CP>,                                             \
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);             \
+    lrn_reg_kernel<STT, CP><<<grid, 256, smem, stream>>>(a);                                    \
+  } while (0)
+    if (st == ST_BF16) {
+      if (cpt == 8) PCNN_LR(ST_BF16, 8); else if (cpt == 6) PCNN_LR(ST_BF16, 6); else PCNN_LR(ST_BF16, 3);
+    } else {
+      if (cpt == 8) PCNN_LR(ST_F32, 8); else if (cpt == 6) PCNN_LR(ST_F32, 6); else PCNN_LR(ST_F32, 3);
+    }
+#undef PCNN_LR
+    return cudaGetLastError();
+  }
   if (lrn_size > 0 && (lrn_size == 5 || lrn_size == 3)) {
     // band kernel (every LRN, fused with a following pool or not)
-    a.R = lrn_band_rows(st, W, C, k, s, Ho);
+    a.R = lrn_band_rows(st, W, C, k, s, Ho, lrn_size);
     a.nbands = (Ho + a.R - 1) / a.R;
     const size_t smem = (size_t)(min((a.R - 1) * s + k, H)) * W * (C * esz + 16);
     if (smem > 200 * 1024) return cudaErrorInvalidValue;

@@ -893,7 +893,7 @@ static pcnn_status run_lrn_pool(pcnn_net *net, int li, int pi, int B, const void
     Ho = p.out_h;
     Wo = p.out_w;
   }
-  const long long tiles = lrn_pool_tiles(net->st, B, W, C, lrn > 0, k, st, Ho, Wo);
+  const long long tiles = lrn_pool_tiles(net->st, B, W, C, lrn, k, st, Ho, Wo);
   const bool gated = is_gated(net, ly);
   const int grid = gated ? net->num_sms * net->occ_lp : (int)std::min<long long>(tiles, 1 << 30);
   Budget b = make_budget(net, ly, 0, true);

@@ -253,3 +253,24 @@ def test_conv_lrn_epilogue_fusion(orc, prec, monkeypatch):
     assert rel_err(plain, ref) <= TOL[prec] / 4
     # same arithmetic and roundings up to FMA contraction: last-place differences
     assert rel_err(fused, plain) <= (2e-3 if prec == "tf32" else 8e-3)
+
+
+@pytest.mark.parametrize("shape", [(96, 55, 55), (256, 27, 27), (64, 13, 11)])
+def test_lrn_register_kernel_matches_band_kernel(orc, shape, monkeypatch):
+    """norm -> pool with the LRN window in registers (lane shuffles for the
+    neighbouring chunks, swizzled smem for C = 256) against the staged band
+    kernel and the oracle: AlexNet norm1 / norm2 shapes and a 6-chunk case."""
+    net = dict(in_shape=shape, layers=[
+        dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0),
+        dict(kind="maxpool", k=3, stride=2)])
+    x = small_inputs(shape, 2, lo=-128, hi=128)
+    ref = orc.run_net(net, [None, None], [None, None], x).reshape(2, -1)
+    for prec in PRECS:
+        reg = gpu_run(net, [None, None], [None, None], x, prec)["out"]
+        monkeypatch.setenv("PCNN_LRN_BAND", "1")
+        band = gpu_run(net, [None, None], [None, None], x, prec)["out"]
+        monkeypatch.delenv("PCNN_LRN_BAND")
+        assert rel_err(reg, ref) <= TOL[prec] / 4
+        # same per-element arithmetic; at most last-place differences
+        assert rel_err(reg, band) <= (8e-3 if prec == "bf16" else 1e-6)
+        assert np.mean(reg == band) > 0.99
