@@ -16,6 +16,9 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(ROOT, "build", "pcnn")
 LIB = os.path.join(PKG, "libpcnn.so")
+# role-profiling variant (tcgen05 barrier-wait counters compiled in), used by
+# tools/tc_roles.py through PCNN_LIB; never the product library
+PROF_LIB = os.path.join(ROOT, "build", "prof", "libpcnn_prof.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -32,18 +35,22 @@ def _newer(src_list, target):
     return any(os.path.getmtime(s) > t for s in src_list)
 
 
-def build(force=False, verbose=False):
-    os.makedirs(BUILD, exist_ok=True)
+def build(force=False, verbose=False, prof=False):
+    bdir = BUILD + ("_prof" if prof else "")
+    lib = PROF_LIB if prof else LIB
+    flags = FLAGS + (["-DPCNN_TC_PROF=1"] if prof else [])
+    os.makedirs(bdir, exist_ok=True)
+    os.makedirs(os.path.dirname(lib), exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [
         os.path.join(ROOT, "include", "pcnn.h")]
     objs, jobs = [], []
     for src in SOURCES:
         s = os.path.join(CSRC, src)
-        o = os.path.join(BUILD, src + ".o")
+        o = os.path.join(bdir, src + ".o")
         objs.append(o)
         if force or _newer([s] + hdrs, o):
             extra = ["-Xptxas", "-v"] if verbose and src.endswith(".cu") else []
-            jobs.append([NVCC] + ARCH + FLAGS + extra + ["-c", s, "-o", o])
+            jobs.append([NVCC] + ARCH + flags + extra + ["-c", s, "-o", o])
 
     def run(cmd):
         r = subprocess.run(cmd, capture_output=True, text=True)
@@ -55,12 +62,13 @@ def build(force=False, verbose=False):
         for out in ex.map(run, jobs):
             if verbose and out:
                 sys.stderr.write(out)
-    if force or jobs or _newer(objs, LIB):
-        tmp = LIB + ".tmp%d" % os.getpid()
+    if force or jobs or _newer(objs, lib):
+        tmp = lib + ".tmp%d" % os.getpid()
         run([NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-lpthread"])
-        os.replace(tmp, LIB)
-    return LIB
+        os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv))
+    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv,
+                prof="--prof" in sys.argv))

@@ -1060,23 +1060,30 @@ __global__ void __launch_bounds__(256) lrn_reg_kernel(const LrnPoolArgs a) {
     __syncthreads();   // the previous band's pooling is done with smem
     const int npix = nr * a.W;
     const int nv = (npix * P + 31) & ~31;     // warp-uniform trip count
+    // the next item's chunks are loaded before the current one is normalised,
+    // so every thread keeps two items' global loads in flight
+    auto load_item = [&](int v, uint4 (&raw)[CPT]) {
+      const int pix = v / P, part = v - pix * P;
+      if (pix < npix) {
+        const int r = pix / a.W, col = pix - r * a.W;
+        const char *src = (const char *)a.x +
+            ((((size_t)n * Hp + h0 + r + a.hi) * Wp + col + a.hi) * C + (size_t)part * CPT * VN) * ESZ;
+#pragma unroll
+        for (int j = 0; j < CPT; ++j) raw[j] = __ldg((const uint4 *)(src + j * 16));
+      } else {
+#pragma unroll
+        for (int j = 0; j < CPT; ++j) raw[j] = make_uint4(0, 0, 0, 0);
+      }
+    };
+    uint4 nraw[CPT];
+    if ((int)threadIdx.x < nv) load_item(threadIdx.x, nraw);
     for (int v = threadIdx.x; v < nv; v += blockDim.x) {
       const int pix = v / P, part = v - pix * P;
       const bool ok = pix < npix;
-      const int r = ok ? pix / a.W : 0, col = ok ? pix - r * a.W : 0;
-      const char *src = (const char *)a.x +
-          ((((size_t)n * Hp + h0 + r + a.hi) * Wp + col + a.hi) * C + (size_t)part * CPT * VN) * ESZ;
       Vec16<ST> ch[CPT];
 #pragma unroll
-      for (int j = 0; j < CPT; ++j) {
-        if (ok) {
-          const uint4 raw = __ldg((const uint4 *)(src + j * 16));
-          ch[j].from_raw(raw);
-        } else {
-#pragma unroll
-          for (int i = 0; i < VN; ++i) ch[j].v[i] = 0.f;
-        }
-      }
+      for (int j = 0; j < CPT; ++j) ch[j].from_raw(nraw[j]);
+      if (v + (int)blockDim.x < nv) load_item(v + blockDim.x, nraw);
       // window neighbours held by the adjacent lanes of the same pixel
       float tail[HALF], head[HALF];
 #pragma unroll
@@ -1183,6 +1190,9 @@ static int lrn_reg_cpt(int st, int C) {
   if (C % vn) return 0;
   const int chunks = C / vn;
   auto pow2_le32 = [](int p) { return p >= 1 && p <= 32 && (p & (p - 1)) == 0; };
+  const char *e = getenv("PCNN_LRN_CPT");        // tuning experiments
+  const int want = e ? atoi(e) : 0;
+  if (want == 3 && chunks % 3 == 0 && pow2_le32(chunks / 3)) return 3;
   if (chunks % 8 == 0 && pow2_le32(chunks / 8)) return 8;
   if (chunks % 6 == 0 && pow2_le32(chunks / 6)) return 6;
   if (chunks % 3 == 0 && pow2_le32(chunks / 3)) return 3;
@@ -1201,8 +1211,10 @@ static bool use_lrn_reg(int st, int C, int lrn) {
 static int lrn_band_rows(int st, int W, int C, int k, int s, int Ho, int lrn) {
   const int esz = st == ST_BF16 ? 2 : 4;
   const size_t row = (size_t)W * (C * esz + (use_lrn_reg(st, C, lrn) ? 0 : 16));
+  const char *e = getenv("PCNN_LB_KB");          // tuning experiments
+  const size_t budget = e ? (size_t)atoi(e) * 1024 : (size_t)LB_SMEM_BUDGET;
   int R = 1;
-  while (R < Ho && (size_t)((R) * s + k) * row <= LB_SMEM_BUDGET) ++R;
+  while (R < Ho && (size_t)((R) * s + k) * row <= budget) ++R;
   return R;
 }
 

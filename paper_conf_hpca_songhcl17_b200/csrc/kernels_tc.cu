@@ -79,12 +79,18 @@ size_t tc_smem_bytes() { return TC_SMEM_BYTES; }
 int tc_max_ktab() { return TC_MAX_KTAB; }
 int tc_block_k_elems(int st) { return st == ST_BF16 ? 64 : 32; }
 // Padded mode: one A stage is the (128 + 2 pad)-row window of one filter row
-// r and channel slab; one B stage is the weight slab of one tap (r, s).
-static int pm_a_stage_bytes(int slab_bytes, int S) {
-  return ((TC_BM + (S - 1)) * slab_bytes + 1023) / 1024 * 1024;
+// r and channel slab (msub = 2: two such windows, 128 rows apart, for two
+// M sub-tiles that share every weight slab); one B stage is the weight slab
+// of one tap (r, s).
+// rows from one sub-tile's window to the next: a whole number of 8-row
+// swizzle atoms, so every window starts swizzle-aligned
+__host__ __device__ constexpr int pm_sub_rows(int S) { return (TC_BM + S - 1 + 7) / 8 * 8; }
+static int pm_a_stage_bytes(int slab_bytes, int S, int msub) {
+  return ((msub - 1) * pm_sub_rows(S) * slab_bytes + (TC_BM + S - 1) * slab_bytes + 1023) /
+         1024 * 1024;
 }
-void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int *a_stages, int *b_stages) {
-  const int as_bytes = pm_a_stage_bytes(slab_bytes, S);
+void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages, int *b_stages) {
+  const int as_bytes = pm_a_stage_bytes(slab_bytes, S, msub);
   const int bs_bytes = bn / cg * slab_bytes;
   int na = TC_MAX_ASTAGES;
   while (na > 2 && na * as_bytes + 2 * S * bs_bytes > TC_STAGE_BUDGET) --na;
@@ -370,6 +376,7 @@ struct TcArgs {
   int prof;             // 1: accumulate per-role barrier-wait cycles (debug)
   int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
   int a_stages, b_stages, pm_a_stage;   // padded mode rings (g.pm)
+  int msub;             // padded mode: M sub-tiles of 128 rows per CTA sharing each B slab
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
   int tma_y;            // 1: full 32-column output chunks leave by TMA tensor store
   float lrn_a_over_n, lrn_beta, lrn_k;
@@ -483,11 +490,19 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
 //  6 epilogue busy cycles      7 CTAs
 __device__ unsigned long long g_tc_prof[8];
 
+// Role profiling is compiled in only with -DPCNN_TC_PROF=1 (tools/tc_roles.py
+// builds such a library): its clocks and 64-bit sums cost the issue loops
+// uniform registers.
+#ifndef PCNN_TC_PROF
+#define PCNN_TC_PROF 0
+#endif
+#define TC_PROF(a) (PCNN_TC_PROF && (a).prof)
+
 struct WaitClock {
   bool on;
   unsigned long long acc = 0;
   __device__ __forceinline__ void wait(uint32_t bar, uint32_t parity) {
-    if (on) {
+    if (PCNN_TC_PROF && on) {
       const long long t0 = clock64();
       mbar_wait(bar, parity);
       acc += (unsigned long long)(clock64() - t0);
@@ -530,7 +545,7 @@ __device__ __forceinline__ void mma_issuer_im2col(const TcArgs &a, uint32_t sbas
   const uint32_t a_stage16 = TC_A_STAGE / 16, b_stage16 = b_stage / 16;
   const int stages = a.stages, units = a.units, mtiles = a.mtiles, ntiles = a.ntiles;
   const int groups = a.g.groups, kblocks = a.kblocks, kbs = a.kb_per_split;
-  const bool prof = a.prof != 0, skip_mma = (a.skip & 4) != 0;
+  const bool prof = TC_PROF(a) != 0, skip_mma = (a.skip & 4) != 0;
   const bool leader = elect_one();
   WaitClock wfull{prof}, wtemp{prof};
   uint32_t stage = 0, phase = 0, lt = 0;
@@ -570,7 +585,7 @@ __device__ __forceinline__ void mma_issuer_im2col(const TcArgs &a, uint32_t sbas
 
 // Padded mode: per (slab, filter row) A window, S taps; tap s reads the
 // window shifted by s rows (SLAB / 16 descriptor units per row).
-template <int ST, int CG, int SLAB>
+template <int ST, int CG, int SLAB, int MSUB>
 __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, uint32_t sA,
                                               uint32_t sBp, uint32_t pm_b_bytes,
                                               uint32_t tmem_base, int pair, int npairs, int nj,
@@ -583,7 +598,9 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
   const uint64_t b_desc0 = umma_desc(sBp, SLAB);
   const uint32_t a_st16 = (uint32_t)a.pm_a_stage / 16, b_st16 = pm_b_bytes / 16;
   const int a_stages = a.a_stages, b_stages = a.b_stages, units = a.units, S = a.g.S;
-  const bool prof = a.prof != 0, skip_mma = (a.skip & 4) != 0;
+  // sub-tile 1's window starts pm_sub_rows(S) rows into the A stage
+  const uint32_t sub16 = (uint32_t)pm_sub_rows(S) * ROW16;
+  const bool prof = TC_PROF(a) != 0, skip_mma = (a.skip & 4) != 0;
   const bool leader = elect_one();
   WaitClock wfull{prof}, wtemp{prof};
   uint32_t as = 0, aph = 0, bs = 0, bph = 0, lt = 0;
@@ -602,9 +619,14 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
         const uint64_t bd = b_desc0 + bs * b_st16;
         if (leader) {
           if (!skip_mma) {
-            tc_mma<ST, CG>(dcol, aw, bd, idesc, (j > 0 || s2 > 0) ? 1u : 0u);
 #pragma unroll
-            for (int k = 1; k < KMMA; ++k) tc_mma<ST, CG>(dcol, aw + 2 * k, bd + 2 * k, idesc, 1u);
+            for (int sb = 0; sb < MSUB; ++sb) {
+              const uint64_t awb = aw + sb * sub16;
+              const uint32_t dc = dcol + sb * (TC_BN_MAX / 2);
+              tc_mma<ST, CG>(dc, awb, bd, idesc, (j > 0 || s2 > 0) ? 1u : 0u);
+#pragma unroll
+              for (int k = 1; k < KMMA; ++k) tc_mma<ST, CG>(dc, awb + 2 * k, bd + 2 * k, idesc, 1u);
+            }
           }
           tc_commit<CG>(sbase + SM_EMPTY + 8 * bs);
         }
@@ -629,7 +651,7 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
 }
 
 template <int ST, int CG, bool LRN>
-__global__ void __launch_bounds__(tc_threads<LRN>(), 1)
+__global__ void __launch_bounds__(tc_threads<LRN>(), 1) __maxnreg__(LRN ? 255 : 200)
 conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
                const __grid_constant__ CUtensorMap tmap_x,
                const __grid_constant__ CUtensorMap tmap_y, const TcArgs a) {
@@ -700,7 +722,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *(volatile uint32_t *)(smem + SM_TMEMPTR);
-  const long long t_start = a.prof ? clock64() : 0;
+  const long long t_start = TC_PROF(a) ? clock64() : 0;
   unsigned long long wtf_acc_out = 0, busy_out = 0;   // epilogue profile (warp 2)
 
   const int HoWo = g.Ho * g.Wo;
@@ -732,24 +754,27 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
       const uint32_t pm_a_bytes = (uint32_t)(TC_BM + 2 * g.pad) * slab_bytes;
       uint32_t as = 0, aph = 0, bs = 0, bph = 0;
-      WaitClock wc{a.prof != 0};
+      WaitClock wc{TC_PROF(a) != 0};
       unsigned long long nkb = 0;
       for (int u = pair; u < a.units; u += npairs) {
         int mt, nt, grp, sp;
         decode(u, mt, nt, grp, sp);
         nkb += pm_nj;
         const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
-        const int i0 = mt * (TC_BM * CG) + (int)rank * TC_BM;
+        const int i0 = (mt * CG + (int)rank) * TC_BM * a.msub;
         int cb = 0, r = 0;
         for (int j = 0; j < pm_nj; ++j) {
           wc.wait(sbase + SM_AEMPTY + 8 * as, aph ^ 1);
           const uint32_t fa = sbase + SM_AFULL + 8 * as;
-          if (rank == 0) mbar_arrive_expect_tx(fa, (a.skip & 1) ? 0 : CG * pm_a_bytes);
+          if (rank == 0) mbar_arrive_expect_tx(fa, (a.skip & 1) ? 0 : CG * a.msub * pm_a_bytes);
           if (!(a.skip & 1)) {
             const uint32_t dA = sA + as * (uint32_t)a.pm_a_stage;
             const int cc = grp * g.Cg + cb * pm_se, row = i0 + (r - g.pad) * g.wv - g.pad;
-            if constexpr (CG == 1) tma_load_2d(dA, &tmap_x, fa, cc, row);
-            else tma_load_2d_2sm(dA, &tmap_x, fa, cc, row);
+            for (int sb = 0; sb < a.msub; ++sb) {
+              const uint32_t d = dA + (uint32_t)(sb * pm_sub_rows(g.S) * slab_bytes);
+              if constexpr (CG == 1) tma_load_2d(d, &tmap_x, fa, cc, row + sb * TC_BM);
+              else tma_load_2d_2sm(d, &tmap_x, fa, cc, row + sb * TC_BM);
+            }
           }
           advance(as, aph, a.a_stages);
           for (int s2 = 0; s2 < g.S; ++s2) {
@@ -766,7 +791,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           if (++r == g.S) { r = 0; ++cb; }
         }
       }
-      if (a.prof) {
+      if (TC_PROF(a)) {
         atomicAdd(&g_tc_prof[0], wc.acc);
         atomicAdd(&g_tc_prof[5], nkb);
       }
@@ -775,13 +800,19 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     if (rank == 0) {
       // ---------------------------------------------- MMA issuer, padded mode
       unsigned long long af = 0, at = 0;
-      if (slab_bytes == 128)
-        mma_issuer_pm<ST, CG, 128>(a, sbase, sA, sBp, pm_b_bytes, tmem_base, pair, npairs, pm_nj, &af, &at);
-      else if (slab_bytes == 64)
-        mma_issuer_pm<ST, CG, 64>(a, sbase, sA, sBp, pm_b_bytes, tmem_base, pair, npairs, pm_nj, &af, &at);
-      else
-        mma_issuer_pm<ST, CG, 32>(a, sbase, sA, sBp, pm_b_bytes, tmem_base, pair, npairs, pm_nj, &af, &at);
-      if (a.prof && lane == 0) {
+#define PCNN_PM_ISSUE(SL, MS) \
+  mma_issuer_pm<ST, CG, SL, MS>(a, sbase, sA, sBp, pm_b_bytes, tmem_base, pair, npairs, pm_nj, &af, &at)
+      if (a.msub == 2) {
+        if (slab_bytes == 128) PCNN_PM_ISSUE(128, 2);
+        else if (slab_bytes == 64) PCNN_PM_ISSUE(64, 2);
+        else PCNN_PM_ISSUE(32, 2);
+      } else {
+        if (slab_bytes == 128) PCNN_PM_ISSUE(128, 1);
+        else if (slab_bytes == 64) PCNN_PM_ISSUE(64, 1);
+        else PCNN_PM_ISSUE(32, 1);
+      }
+#undef PCNN_PM_ISSUE
+      if (TC_PROF(a) && lane == 0) {
         atomicAdd(&g_tc_prof[1], af);
         atomicAdd(&g_tc_prof[2], at);
       }
@@ -792,7 +823,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
       uint32_t stage = 0, phase = 0;
-      WaitClock wc{a.prof != 0};
+      WaitClock wc{TC_PROF(a) != 0};
       unsigned long long nkb = 0;
       for (int u = pair; u < a.units; u += npairs) {
         int mt, nt, grp, sp, k0, k1;
@@ -853,7 +884,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           advance(stage, phase, stages);
         }
       }
-      if (a.prof) {
+      if (TC_PROF(a)) {
         atomicAdd(&g_tc_prof[0], wc.acc);
         atomicAdd(&g_tc_prof[5], nkb);
       }
@@ -868,7 +899,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         mma_issuer_im2col<ST, CG, 64>(a, sbase, sA, sB, b_stage, tmem_base, pair, npairs, &af, &at);
       else
         mma_issuer_im2col<ST, CG, 32>(a, sbase, sA, sB, b_stage, tmem_base, pair, npairs, &af, &at);
-      if (a.prof && lane == 0) {
+      if (TC_PROF(a) && lane == 0) {
         atomicAdd(&g_tc_prof[1], af);
         atomicAdd(&g_tc_prof[2], at);
       }
@@ -883,7 +914,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     const uint32_t tempty_leader =
         CG == 2 ? mapa(sbase + SM_TEMPTY, 0) : sbase + SM_TEMPTY;
     uint32_t lt = 0;
-    WaitClock wtf{a.prof != 0 && lane == 0 && warp == 2};
+    WaitClock wtf{TC_PROF(a) != 0 && lane == 0 && warp == 2};
     unsigned long long busy = 0;
     long long tb = 0;
     for (int u = pair; u < a.units; u += npairs, ++lt) {
@@ -894,6 +925,9 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       wtf.wait(sbase + SM_TFULL + 8 * buf, use & 1);
       if (wtf.on) tb = clock64();
       tc_fence_after();
+      for (int sb = 0; sb < a.msub; ++sb) {
+      // TMEM columns of this sub-tile's accumulator
+      const uint32_t tcol = buf * TC_BN_MAX + sb * (TC_BN_MAX / 2);
       int m;
       bool mok;
       if (rect) {
@@ -906,7 +940,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         mok = row < rect_rows && q < g.Wo && p < g.Ho && n * HoWo < g.M;
         m = (n * g.Ho + p) * g.Wo + q;
       } else {
-        m = mt * (TC_BM * CG) + (int)rank * TC_BM + row;
+        m = ((mt * CG + (int)rank) * a.msub + sb) * TC_BM + row;
         mok = m < g.M;
       }
       bool valid = true;      // padded mode: halo rows are stored as zeros
@@ -918,14 +952,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       }
       const size_t orow = (size_t)m * g.out_cs;
       if constexpr (LRN) {
-        epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX, mok,
+        epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + tcol, mok,
                          orow, stage, lane);
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) {
-          if (CG == 2 && rank != 0) mbar_arrive_cluster(tempty_leader + 8 * buf);
-          else mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
-        }
         continue;
       }
       if (a.tma_y) {
@@ -945,7 +973,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           float f[32];
           {
             uint32_t v[32];
-            tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0, v);
+            tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + tcol + c0, v);
             tmem_ld_wait();
 #pragma unroll
             for (int i = 0; i < 32; ++i) f[i] = __uint_as_float(v[i]);
@@ -1031,12 +1059,6 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
             epi_store_rows(stage, pc, np, rowp, lane);
           }
         }
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) {
-          if (CG == 2 && rank != 0) mbar_arrive_cluster(tempty_leader + 8 * buf);
-          else mbar_arrive(sbase + SM_TEMPTY + 8 * buf);
-        }
         continue;
       }
       // bias is zero-padded on the device, so whole float4s can be read.
@@ -1059,7 +1081,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         for (int h = 0; h < 2; ++h) {
           if (h == 0 || (out16 && c0 + 32 < cend)) {
             uint32_t v[32];
-            tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + buf * TC_BN_MAX + c0 + 32 * h, v);
+            tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + tcol + c0 + 32 * h, v);
             tmem_ld_wait();
 #pragma unroll
             for (int i = 0; i < 32; ++i) f[32 * h + i] = __uint_as_float(v[i]);
@@ -1111,6 +1133,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         char *rowp = mok ? obase + ((size_t)m * ocs + col) * eb : nullptr;
         epi_store_rows(stage, pc, np, rowp, lane);
       }
+      }   // sub-tiles
       tc_fence_before();
       __syncwarp();
       if (lane == 0) {
@@ -1125,14 +1148,14 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     busy_out = busy;
   }
 
-  if (a.prof && warp == 2 && lane == 0) {
+  if (TC_PROF(a) && warp == 2 && lane == 0) {
     atomicAdd(&g_tc_prof[3], wtf_acc_out);
     atomicAdd(&g_tc_prof[6], busy_out);
   }
   tc_fence_before();
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
-  if (a.prof && tid == 0) {
+  if (TC_PROF(a) && tid == 0) {
     atomicAdd(&g_tc_prof[4], (unsigned long long)(clock64() - t_start));
     atomicAdd(&g_tc_prof[7], 1ULL);
   }
@@ -1286,7 +1309,10 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.rects_h = p.rect_w ? (g.Ho + p.rect_h - 1) / p.rect_h : 0;
   args.a_stages = p.a_stages;
   args.b_stages = p.b_stages;
-  args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, g.S) : 0;
+  args.msub = p.msub > 1 ? p.msub : 1;
+  args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, g.S, args.msub) : 0;
+  if (args.msub > 2 || (args.msub == 2 && (!g.pm || p.bn > TC_BN_MAX / 2)))
+    return cudaErrorInvalidValue;
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
   if (g.pm && (p.splits != 1 || lrn || p.rect_w || g.stride != 1 || g.S != 2 * g.pad + 1 ||

@@ -95,6 +95,7 @@ struct TcPlan {
   int grid;        // CTAs = cg * min(units, SM budget / cg)
   int rect_w, rect_h, rect_n;  // 0 = im2col A tiles; else rectangle tiles (tiled TMA)
   int a_stages, b_stages;      // padded mode: A (row-window) and B (tap slab) ring depths
+  int msub;                    // padded mode: 128-row M sub-tiles per CTA sharing each B slab
 };
 // Launches the GEMM and, when p.splits > 1, the deterministic split-K
 // reduction (ws must hold splits * M * out_cs floats; a split-K output must
@@ -117,7 +118,8 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
 int tc_slab_bytes(int st, int cg_channels);
 int tc_stages_for(int bn, int cg);
 // padded mode: ring depths for an N tile, CTA grouping, slab width and kernel size
-void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int *a_stages, int *b_stages);
+void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages,
+                  int *b_stages);
 // debug: per-role barrier-wait cycle totals accumulated while PCNN_TC_PROFILE=1
 cudaError_t tc_profile(int reset, unsigned long long out[8]);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)

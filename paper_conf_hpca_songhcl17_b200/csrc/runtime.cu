@@ -731,35 +731,44 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz) {
   const int nj = g.Cg * esz / slab * g.S;
   const char *force_cg = getenv("PCNN_FORCE_CG");
   const char *force_bn = getenv("PCNN_FORCE_BN");
-  for (int cg = 1; cg <= 2; ++cg) {
-    if (force_cg && atoi(force_cg) != cg) continue;
-    const int mtiles = (int)(((long long)g.M + 128LL * cg - 1) / (128LL * cg));
-    const int slots = device_sms / cg;
-    for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {
-      if (force_bn && atoi(force_bn) != bn) continue;
-      const int ntiles = (g.Nfg + bn - 1) / bn;
-      const long long tiles = (long long)mtiles * ntiles * g.groups;
-      const double load = ((128.0 + g.S - 1) * slab + (double)g.S * slab * bn / cg) /
-                          kOperandBytesPerCycle;
-      const double mma = g.S * (slab / 128.0) * 2.05 * bn / kMmaEfficiency;
-      const double j_cycles = std::max(load, mma) + 40.0;
-      const long long waves = (tiles + slots - 1) / slots;
-      const double t = (double)waves * nj * j_cycles / f + 2e-6;
-      if (t < best_t * 0.999 ||
-          (t <= best_t * 1.001 && (long long)bn * cg > (long long)best.bn * best.cg)) {
-        best_t = t;
-        best.cg = cg;
-        best.bn = bn;
-        best.mtiles = mtiles;
-        best.ntiles = ntiles;
-        best.tiles = (int)tiles;
-        best.splits = 1;
-        best.kb_per_split = nj;
-        best.units = (int)tiles;
+  const char *force_ms = getenv("PCNN_PM_MSUB");           // 1 | 2 (experiments)
+  for (int ms = 1; ms <= 2; ++ms) {
+    if (force_ms && atoi(force_ms) != ms) continue;
+    for (int cg = 1; cg <= 2; ++cg) {
+      if (force_cg && atoi(force_cg) != cg) continue;
+      const long long rows = 128LL * cg * ms;
+      const int mtiles = (int)(((long long)g.M + rows - 1) / rows);
+      const int slots = device_sms / cg;
+      for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {
+        if (force_bn && atoi(force_bn) != bn) continue;
+        if (ms == 2 && bn > 128) continue;          // two accumulators per TMEM buffer
+        const int ntiles = (g.Nfg + bn - 1) / bn;
+        const long long tiles = (long long)mtiles * ntiles * g.groups;
+        // per (slab, filter row): ms windows of 128 + S - 1 rows and S weight
+        // slabs (shared by the ms sub-tiles) through L2, ms * S * slab/32 UMMAs
+        const double load = (ms * (128.0 + g.S - 1) * slab + (double)g.S * slab * bn / cg) /
+                            kOperandBytesPerCycle;
+        const double mma = ms * g.S * (slab / 128.0) * 2.05 * bn / kMmaEfficiency;
+        const double j_cycles = std::max(load, mma) + 40.0;
+        const long long waves = (tiles + slots - 1) / slots;
+        const double t = (double)waves * nj * j_cycles / f + 2e-6 * ms;
+        if (t < best_t * 0.999 ||
+            (t <= best_t * 1.001 && (long long)bn * cg > (long long)best.bn * best.cg)) {
+          best_t = t;
+          best.cg = cg;
+          best.bn = bn;
+          best.msub = ms;
+          best.mtiles = mtiles;
+          best.ntiles = ntiles;
+          best.tiles = (int)tiles;
+          best.splits = 1;
+          best.kb_per_split = nj;
+          best.units = (int)tiles;
+        }
       }
     }
   }
-  tc_pm_stages(best.bn, best.cg, slab, g.S, &best.a_stages, &best.b_stages);
+  tc_pm_stages(best.bn, best.cg, slab, g.S, best.msub, &best.a_stages, &best.b_stages);
   return best;
 }
 
@@ -801,7 +810,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
         stage_tmap(gs, p.bn / p.cg, g.pm ? tc_slab_bytes(gs.st, g.Cg) : 128);
     if (!tm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeTiled failed");
     if (info) {
-      info->tile_m = 128 * p.cg;
+      info->tile_m = 128 * p.cg * std::max(1, p.msub);
       info->tile_n = p.bn;
       info->tiles = p.tiles;
       info->grid = p.grid;

@@ -10,7 +10,8 @@ import ctypes
 import os
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libpcnn.so")
+# PCNN_LIB: A/B experiments against another build of the same library
+LIB_PATH = os.environ.get("PCNN_LIB") or os.path.join(PKG, "libpcnn.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

@@ -107,3 +107,25 @@ def test_padded_mode_batch_one_and_max_batch(orc):
     r = gpu_run(net, w, b, x, "bf16", max_batch=7)
     assert r["net"].query_layer(1, 1)["a_mode"] == 2
     assert rel_err(r["out"], ref) <= TOL["bf16"] / 2
+
+
+@pytest.mark.parametrize("cg", ["1", "2"])
+@pytest.mark.parametrize("groups", [1, 2])
+def test_padded_mode_two_subtiles_bitwise(orc, cg, groups, monkeypatch):
+    """msub = 2 (two 128-row M sub-tiles per CTA sharing every weight slab,
+    two TMEM accumulators) computes each sub-tile with the same UMMA sequence
+    as msub = 1: bitwise equal outputs, ragged last tile included."""
+    net = vgg_like(hw=36, c1=64 * groups, c2=128, groups=groups)
+    w, b = params(net, seed=13)
+    x = small_inputs((3, 36, 36), 3, lo=-128, hi=128)
+    ref = orc.run_net(net, w, b, x).reshape(3, -1)
+    monkeypatch.setenv("PCNN_FORCE_CG", cg)
+    out = {}
+    for ms in ("1", "2"):
+        monkeypatch.setenv("PCNN_PM_MSUB", ms)
+        r = gpu_run(net, w, b, x, "bf16")
+        f = r["net"].query_layer(1, 3)
+        assert f["a_mode"] == 2 and f["tile_m"] == 128 * int(cg) * int(ms)
+        out[ms] = r["out"]
+    np.testing.assert_array_equal(out["1"], out["2"])
+    assert rel_err(out["2"], ref) <= TOL["bf16"] / 2

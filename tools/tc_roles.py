@@ -5,6 +5,8 @@ per CTA each role spent blocked."""
 import ctypes, os, sys
 os.environ["PCNN_TC_PROFILE"] = "1"
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_hpca_songhcl17_b200 import build as _b   # counters need the -DPCNN_TC_PROF=1 build
+os.environ["PCNN_LIB"] = _b.build(prof=True)
 import torch
 import synth
 from paper_conf_hpca_songhcl17_b200 import pcnn
