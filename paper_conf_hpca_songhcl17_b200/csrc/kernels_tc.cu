@@ -356,8 +356,29 @@ __device__ __forceinline__ float tf32_rna_tc(float v) {
   return __uint_as_float(r);
 }
 
+// Division by a launch-invariant divisor d (Granlund-Montgomery, exact for
+// every 32-bit n): q = (t + ((n - t) >> 1)) >> (l - 1), t = umulhi(m, n),
+// l = ceil(log2 d), m = floor(2^32 (2^l - d) / d) + 1.  The epilogue's
+// per-tile index arithmetic (tile decode, halo test) runs on every lane, where
+// a hardware-less integer division costs ~20 instructions.
+struct FastDiv {
+  uint32_t d, m, l;
+  __host__ void init(uint32_t dd) {
+    d = dd < 1 ? 1 : dd;
+    l = 0;
+    while ((1ull << l) < d) ++l;
+    m = (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+  }
+  __device__ __forceinline__ uint32_t div(uint32_t n) const {
+    if (d == 1) return n;
+    const uint32_t t = __umulhi(m, n);
+    return (t + ((n - t) >> 1)) >> (l - 1);
+  }
+};
+
 struct TcArgs {
   ConvGeom g;
+  FastDiv fd_mt, fd_nt, fd_grp, fd_hw, fd_w;   // mtiles, ntiles, groups, hv*wv, wv
   void *y;
   float *ws;            // split-K partials [splits][M][out_cs] fp32 (splits > 1)
   const float *bias;
@@ -729,12 +750,12 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   // work unit u -> (m tile, n tile, group, split); m fastest so CTAs running
   // concurrently share one weight slice in L2.
   auto decode = [&](int u, int &mt, int &nt, int &grp, int &sp) {
-    mt = u % a.mtiles;
-    int r = u / a.mtiles;
-    nt = r % a.ntiles;
-    r /= a.ntiles;
-    grp = r % g.groups;
-    sp = r / g.groups;
+    int r = (int)a.fd_mt.div((uint32_t)u);
+    mt = u - r * a.mtiles;
+    const int r2 = (int)a.fd_nt.div((uint32_t)r);
+    nt = r - r2 * a.ntiles;
+    sp = (int)a.fd_grp.div((uint32_t)r2);
+    grp = r2 - sp * g.groups;
   };
   auto kb_range = [&](int sp, int &k0, int &k1) {
     k0 = sp * a.kb_per_split;
@@ -945,9 +966,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       }
       bool valid = true;      // padded mode: halo rows are stored as zeros
       if (g.pm) {
-        const int hvwv = g.hv * g.wv;
-        const int ni = m / hvwv, rem = m - ni * hvwv;
-        const int pv = rem / g.wv, qv = rem - pv * g.wv;
+        const int ni = (int)a.fd_hw.div((uint32_t)m), rem = m - ni * g.hv * g.wv;
+        const int pv = (int)a.fd_w.div((uint32_t)rem), qv = rem - pv * g.wv;
         valid = pv >= g.vh && pv < g.vh + g.Ho && qv >= g.vh && qv < g.vh + g.Wo;
       }
       const size_t orow = (size_t)m * g.out_cs;
@@ -970,6 +990,11 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           const int n = nt * a.bn + c0;
           if (n >= g.Nfg) break;                         // warp-uniform
           const int col = grp * g.Nfg + n;
+          // bias loads issued before the TMEM load so their latencies overlap
+          const float4 *bp = (const float4 *)(a.bias + col);
+          float4 bb[8];
+#pragma unroll
+          for (int q = 0; q < 8; ++q) bb[q] = __ldg(bp + q);
           float f[32];
           {
             uint32_t v[32];
@@ -978,14 +1003,12 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
 #pragma unroll
             for (int i = 0; i < 32; ++i) f[i] = __uint_as_float(v[i]);
           }
-          const float4 *bp = (const float4 *)(a.bias + col);
 #pragma unroll
           for (int q = 0; q < 8; ++q) {
-            const float4 bb = __ldg(bp + q);
-            f[4 * q] += bb.x;
-            f[4 * q + 1] += bb.y;
-            f[4 * q + 2] += bb.z;
-            f[4 * q + 3] += bb.w;
+            f[4 * q] += bb[q].x;
+            f[4 * q + 1] += bb[q].y;
+            f[4 * q + 2] += bb[q].z;
+            f[4 * q + 3] += bb[q].w;
           }
           if (g.relu)
 #pragma unroll
@@ -1288,6 +1311,11 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
     args.lrn_k = lrn[3];
   }
   args.g = g;
+  args.fd_mt.init(p.mtiles);
+  args.fd_nt.init(p.ntiles);
+  args.fd_grp.init(g.groups);
+  args.fd_hw.init(g.pm ? g.hv * g.wv : 1);
+  args.fd_w.init(g.pm ? g.wv : 1);
   args.y = y;
   args.tma_y = (tmap_y != nullptr && !lrn && p.splits == 1 && p.rect_w == 0) ? 1 : 0;
   args.ws = ws;
