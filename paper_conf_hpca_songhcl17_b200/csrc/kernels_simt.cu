@@ -41,12 +41,12 @@ struct Vec16 {
   __device__ __forceinline__ void load(const void *p) { from_raw(*(const uint4 *)p); }
   __device__ __forceinline__ void from_raw(const uint4 raw) {
     if constexpr (ST == ST_BF16) {
-      const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
+      // bf16 -> fp32 is a 16-bit shift of the bit pattern (exact)
+      const uint32_t w[4] = {raw.x, raw.y, raw.z, raw.w};
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
-        const float2 f = __bfloat1622float2(h[i]);
-        v[2 * i] = f.x;
-        v[2 * i + 1] = f.y;
+        v[2 * i] = __uint_as_float(w[i] << 16);
+        v[2 * i + 1] = __uint_as_float(w[i] & 0xFFFF0000u);
       }
     } else {
       const float *f = (const float *)&raw;
@@ -1127,10 +1127,12 @@ __global__ void __launch_bounds__(256) lrn_reg_kernel(const LrnPoolArgs a) {
     const float inv_oc = 1.f / (float)ochunks;
     const int grp_real = a.ocg / VN, grp_pad = a.ocp / VN;
     const int nq = a.Wo * ochunks;
+    const float inv_nq = 1.f / (float)nq;
     for (int v = threadIdx.x; v < (p1 - p0) * nq; v += blockDim.x) {
-      const int rr = v / nq;
-      int q, oc;
-      fdivmod(v - rr * nq, ochunks, inv_oc, q, oc);
+      int rr, q, oc;
+      if (nq <= 1024) fdivmod(v, nq, inv_nq, rr, q);   // fdivmod's exact range
+      else { rr = v / nq; q = v - rr * nq; }
+      fdivmod(q, ochunks, inv_oc, q, oc);
       const int pp = p0 + rr;
       int c = oc;
       bool pad = false;
@@ -1148,16 +1150,24 @@ __global__ void __launch_bounds__(256) lrn_reg_kernel(const LrnPoolArgs a) {
         const __nv_bfloat162 zero = __float2bfloat162_rn(0.f);
 #pragma unroll
         for (int j = 0; j < 4; ++j) m[j] = pad ? zero : ninf;
-        if (!pad)
-          for (int r = rs; r < re; ++r)
-            for (int col = cs; col < ce; ++col) {
-              const int pix = r * a.W + col;
-              const uint4 raw =
-                  *(const uint4 *)(lr_smem + ((size_t)pix * chunks + slot(pix, c)) * 16);
-              const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
+        auto take = [&](int pix) {
+          const uint4 raw = *(const uint4 *)(lr_smem + ((size_t)pix * chunks + slot(pix, c)) * 16);
+          const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
 #pragma unroll
-              for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], h[j]);
-            }
+          for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], h[j]);
+        };
+        if (!pad) {
+          if (re - rs == 3 && ce - cs == 3) {      // AlexNet's 3 x 3 windows, unclipped
+            const int pix0 = rs * a.W + cs;
+#pragma unroll
+            for (int dr = 0; dr < 3; ++dr)
+#pragma unroll
+              for (int dc = 0; dc < 3; ++dc) take(pix0 + dr * a.W + dc);
+          } else {
+            for (int r = rs; r < re; ++r)
+              for (int col = cs; col < ce; ++col) take(r * a.W + col);
+          }
+        }
         *(uint4 *)dst = *(const uint4 *)m;
         continue;
       }

@@ -688,10 +688,15 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
         // split-K candidates: none, or any split that keeps >= 4 K-blocks per unit
         const int max_split =
             (tiles >= slots || full_n) ? 1 : std::min(16, std::max(1, kblocks / 4));
+        static const int force_split = [] {              // tuning experiments
+          const char *e = getenv("PCNN_FORCE_SPLIT");
+          return e ? atoi(e) : 0;
+        }();
         for (int want = 1; want <= max_split; ++want) {
           const int kbs = (kblocks + want - 1) / want;
           const int splits = (kblocks + kbs - 1) / kbs;
           if (splits != want) continue;
+          if (force_split > 0 && splits != force_split) continue;
           const long long units = tiles * splits;
           const long long waves = (units + slots - 1) / slots;
           double t = (double)waves * kbs * kb_cycles / f + 2e-6;   // + per-tile drain
