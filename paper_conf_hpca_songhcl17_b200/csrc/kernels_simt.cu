@@ -782,14 +782,8 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
           sq[j] = xv * xv;
         }
         Vec16<ST> out;
-#pragma unroll
-        for (int j = 0; j < VN; ++j) {
-          float acc = 0.f;
-#pragma unroll
-          for (int w = 0; w < LS; ++w) acc += sq[j + w];
-          const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
-          out.v[j] = cur.v[j] * lrn_scale_pow(scale, a.lrn_beta);
-        }
+        lrn_normalise<ST == ST_BF16, LS, VN>(sq, cur.v, a.lrn_k, a.lrn_alpha_over_n, a.lrn_beta,
+                                             out.v);
         out.store(U + ((size_t)r * wc_max + col) * C * ESZ + (size_t)ch * 16, a.tf32_round);
       }
       __syncthreads();
@@ -858,7 +852,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
 // overwritten), then pooled from smem.  Every input pixel is normalised once
 // per band (rows shared by two bands: (R*s + k - s) / (R*s) recompute) instead
 // of once per pooling window.  Same per-element arithmetic as lrn_pool_kernel
-// and the conv epilogue (sum order, lrn_scale_pow), so results are identical.
+// and the conv epilogue (lrn_normalise), so results are identical.
 template <int ST, int LS>
 __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
   extern __shared__ __align__(16) uint8_t lb_smem[];
@@ -934,14 +928,8 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
             sq[j] = xv * xv;
           }
           Vec16<ST> out;
-#pragma unroll
-          for (int j = 0; j < VN; ++j) {
-            float acc = 0.f;
-#pragma unroll
-            for (int w = 0; w < LS; ++w) acc += sq[j + w];
-            const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
-            out.v[j] = cur.v[j] * lrn_scale_pow(scale, a.lrn_beta);
-          }
+          lrn_normalise<ST == ST_BF16, LS, VN>(sq, cur.v, a.lrn_k, a.lrn_alpha_over_n,
+                                               a.lrn_beta, out.v);
           out.store(px + ch * 16, a.tf32_round);
 #pragma unroll
           for (int j = 0; j < HALF; ++j) tail[j] = cur.v[VN - HALF + j];
@@ -1017,7 +1005,7 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
 // once to shared memory (chunk c of pixel x at slot c ^ ((x*P + c/8) & 7) when
 // CPT == 8, so neither the writes nor the pooling reads conflict) and pooled
 // from there.  Same per-element arithmetic as the other LRN paths (sum order,
-// lrn_scale_pow), so the results are identical.
+// lrn_normalise), so the results are identical.
 template <int ST, int CPT>
 __global__ void __launch_bounds__(256) lrn_reg_kernel(const LrnPoolArgs a) {
   extern __shared__ __align__(16) uint8_t lr_smem[];
@@ -1108,14 +1096,8 @@ __global__ void __launch_bounds__(256) lrn_reg_kernel(const LrnPoolArgs a) {
             sq[q] = xv * xv;
           }
           Vec16<ST> out;
-#pragma unroll
-          for (int q = 0; q < VN; ++q) {
-            float acc = 0.f;
-#pragma unroll
-            for (int w = 0; w < 2 * HALF + 1; ++w) acc += sq[q + w];
-            const float scale = a.lrn_k + a.lrn_alpha_over_n * acc;
-            out.v[q] = ch[j].v[q] * lrn_scale_pow(scale, a.lrn_beta);
-          }
+          lrn_normalise<ST == ST_BF16, 2 * HALF + 1, VN>(sq, ch[j].v, a.lrn_k, a.lrn_alpha_over_n,
+                                                         a.lrn_beta, out.v);
           out.store(dst + slot(pix, part * CPT + j) * 16, a.tf32_round);
         }
       }

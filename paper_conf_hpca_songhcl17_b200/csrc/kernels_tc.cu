@@ -476,15 +476,12 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
       constexpr int PER = 16 / EB;                       // channels per piece
       const int c0 = (pass * 128 + q * 16) / EB;
       float o[PER];
+      float sq8[PER + 4], x8[PER];
 #pragma unroll
-      for (int j = 0; j < PER; ++j) {
-        const int c = c0 + j;
-        float acc = 0.f;
+      for (int t = 0; t < PER + 4; ++t) sq8[t] = sq[(c0 + t) < MAXC + 4 ? c0 + t : MAXC + 3];
 #pragma unroll
-        for (int w = 0; w < 5; ++w) acc += sq[(c + w) < MAXC + 4 ? c + w : MAXC + 3];
-        const float scale = a.lrn_k + a.lrn_a_over_n * acc;
-        o[j] = (c < MAXC ? f[c < MAXC ? c : 0] : 0.f) * lrn_scale_pow(scale, a.lrn_beta);
-      }
+      for (int j = 0; j < PER; ++j) x8[j] = c0 + j < MAXC ? f[c0 + j < MAXC ? c0 + j : 0] : 0.f;
+      lrn_normalise<ST == ST_BF16, 5, PER>(sq8, x8, a.lrn_k, a.lrn_a_over_n, a.lrn_beta, o);
       if constexpr (ST == ST_BF16) {
         uint32_t *pw = (uint32_t *)&pc[q];
 #pragma unroll
