@@ -308,12 +308,33 @@ stage_gather3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, 
   const int cpr = Wrow / 4;                          // 16 B chunks loaded per row
   const int K = D * D * C;
   const int bands = (Ho + rows_per_cta - 1) / rows_per_cta;
-  const int h0 = (blockIdx.x % bands) * rows_per_cta;
+  const int max_rows = ((rows_per_cta - 1) * step + D) * C;
+  // this thread's output chunk is fixed (blockDim % chunks == 0), so its
+  // channel -> (row, column offset) map is computed once, outside the
+  // persistent band loop
+  const int chunks = Kp / VN;
+  const int ch = threadIdx.x % chunks;
+  int rr[VN], bb[VN];
+#pragma unroll
+  for (int e = 0; e < VN; ++e) {
+    const int k = ch * VN + e;
+    if (k < K) {
+      const int ab = k / C, c = k - ab * C;
+      const int a = ab / D;
+      rr[e] = a * C + c;
+      bb[e] = ab - a * D - pad;
+    } else {
+      rr[e] = -1;
+      bb[e] = 0;
+    }
+  }
+  for (long long t = blockIdx.x; t < (long long)B * bands; t += gridDim.x) {
+  const int h0 = (int)(t % bands) * rows_per_cta;
   const int nh = min(rows_per_cta, Ho - h0);
-  const long long n = blockIdx.x / bands;
+  const long long n = t / bands;
   const int span = (nh - 1) * step + D;
   const int nrow = span * C;
-  const int max_rows = ((rows_per_cta - 1) * step + D) * C;
+  __syncthreads();   // the previous band's rows are no longer read
   int *row_shift = (int *)(g3_rows + (size_t)max_rows * Wrow);   // -1: row outside the image
   const long long total = (long long)B * C * H * W;
   // phase 1: each input row [ih][0, W) of the band as aligned 16 B chunks
@@ -342,25 +363,7 @@ stage_gather3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, 
   }
   asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
   __syncthreads();
-  // phase 2: thread = (pixel, 16 B output chunk); its chunk index is fixed
-  // (blockDim % chunks == 0), so the chunk's channel -> (row, column offset)
-  // map is computed once into registers
-  const int chunks = Kp / VN;
-  const int ch = threadIdx.x % chunks;
-  int rr[VN], bb[VN];
-#pragma unroll
-  for (int e = 0; e < VN; ++e) {
-    const int k = ch * VN + e;
-    if (k < K) {
-      const int ab = k / C, c = k - ab * C;
-      const int a = ab / D;
-      rr[e] = a * C + c;
-      bb[e] = ab - a * D - pad;
-    } else {
-      rr[e] = -1;
-      bb[e] = 0;
-    }
-  }
+  // phase 2: thread = (pixel, 16 B output chunk)
   const int Wop = Wo + 2 * halo;
   const int ppi = blockDim.x / chunks;               // pixels per pass
   for (int hh = 0; hh < nh; ++hh) {
@@ -397,6 +400,7 @@ stage_gather3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, 
       o.store(yrow + ((size_t)w * chunks + ch) * 16, tf32_round);
     }
   }
+  }   // bands
 }
 
 static bool gather3_ok(int st, int W, int Kp, int D, int step) {
@@ -424,7 +428,17 @@ static cudaError_t launch_gather3(const float *x, void *y, int st, int B, int H,
     while (R < 8 && R < Ho && smem_for(R + 1) <= 40 * 1024) ++R;
   const size_t smem = smem_for(R);
   if (smem > 96 * 1024) return cudaErrorInvalidValue;
-  const unsigned grid = (unsigned)((long long)B * ((Ho + R - 1) / R));
+  const long long tiles = (long long)B * ((Ho + R - 1) / R);
+  // persistent CTAs: a full wave of resident CTAs walks the bands
+  int occ = 1;
+  if (st == ST_BF16)
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stage_gather3_kernel<ST_BF16>, 256, smem);
+  else
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stage_gather3_kernel<ST_F32>, 256, smem);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const unsigned grid = (unsigned)std::min<long long>(tiles, (long long)sms * std::max(occ, 1));
   if (st == ST_BF16) {
     if (smem > 48 * 1024)
       cudaFuncSetAttribute(stage_gather3_kernel<ST_BF16>,
@@ -461,10 +475,175 @@ cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, i
   return cudaGetLastError();
 }
 
+// Space-to-depth staging for 3-channel inputs, block 4, no padding (AlexNet
+// conv1 11x11/4 -> 3x3/1 on 48 channels).  A persistent CTA walks bands of R
+// staged rows; one thread copies each needed input row (all W floats of one
+// channel) into shared memory with a single bulk TMA copy of its 16 B-aligned
+// superset, the next band's copies in flight while the current band is
+// converted (two buffers, one mbarrier each).  Then one thread per staged
+// pixel reads its 4 x 3 row segments as 16 B vectors (re-aligned by the row's
+// start offset), permutes them into the (dr, ds, c) channel order and writes
+// the whole pixel (Cs channels, zero padded) with 16 B stores.
+template <int ST>
+__global__ void __launch_bounds__(256)
+stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Hs, int Ws,
+                  int Cs, int R, int tf32_round) {
+  constexpr int C = 3, BLK = 4;
+  constexpr int VN = Vec16<ST>::N;
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  extern __shared__ __align__(128) uint8_t s2_smem[];
+  const int pitch = ((W + 3) / 4 + 1) * 4;            // floats per smem row (16 B multiple)
+  const int rows = R * BLK * C;
+  float *bufs = (float *)s2_smem;                     // [2][rows][pitch]
+  uint64_t *bar = (uint64_t *)(s2_smem + (size_t)2 * rows * pitch * 4);
+  int *shift = (int *)(bar + 2);                      // [2][rows]: start offset, -1 = zero row
+  const int bands = (Hs + R - 1) / R;
+  const long long tiles = (long long)B * bands;
+  const uintptr_t xend = (uintptr_t)(x + (size_t)B * C * H * W);
+  const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bar);
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0));
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  // warp 0: start the copies of band t into buffer b, one row per lane; the
+  // bytes are announced after the copies (the mbarrier's tx-count may go
+  // negative within a phase, and the phase cannot complete before lane 0's
+  // arrive)
+  auto issue = [&](long long t, int b) {
+    const int lane = threadIdx.x & 31;
+    const long long n = t / bands;
+    const int h0 = (int)(t % bands) * R, nh = min(R, Hs - h0);
+    float *buf = bufs + (size_t)b * rows * pitch;
+    int *sh = shift + b * rows;
+    const uint32_t bb = bar0 + 8 * b;
+    uint32_t bytes = 0;
+    for (int lr = lane; lr < nh * BLK * C; lr += 32) {
+      const int a = lr / C, c = lr - a * C, ih = h0 * BLK + a;
+      if (ih >= H) {
+        sh[lr] = -1;
+        continue;
+      }
+      const uintptr_t src = (uintptr_t)(x + ((size_t)(n * C + c) * H + ih) * W);
+      const uintptr_t a0 = src & ~(uintptr_t)15;
+      const uint32_t nb = (uint32_t)(((src + (uintptr_t)W * 4 - a0) + 15) & ~(uintptr_t)15);
+      float *dst = buf + (size_t)lr * pitch;
+      if (a0 + nb > xend) {              // superset past the tensor: plain loads
+        for (int j = 0; j < W; ++j) dst[j] = __ldg((const float *)src + j);
+        sh[lr] = 0;
+        continue;
+      }
+      sh[lr] = (int)((src - a0) >> 2);
+      bytes += nb;
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+          ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(a0), "r"(nb), "r"(bb)
+          : "memory");
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
+    __syncwarp();                        // every lane's smem writes precede the arrive
+    if (lane == 0)
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bb), "r"(bytes)
+                   : "memory");
+  };
+  long long t = blockIdx.x;
+  if (threadIdx.x < 32 && t < tiles) issue(t, 0);
+  uint32_t phase[2] = {0, 0};
+  for (int b = 0; t < tiles; t += gridDim.x, b ^= 1) {
+    if (threadIdx.x < 32 && t + gridDim.x < tiles) issue(t + gridDim.x, b ^ 1);
+    {
+      const uint32_t bb = bar0 + 8 * b, par = phase[b];
+      asm volatile(
+          "{\n.reg .pred P1;\nW_%=:\nmbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+          "@!P1 bra W_%=;\n}\n" ::"r"(bb), "r"(par)
+          : "memory");
+      phase[b] ^= 1;
+    }
+    const long long n = t / bands;
+    const int h0 = (int)(t % bands) * R, nh = min(R, Hs - h0);
+    const float *buf = bufs + (size_t)b * rows * pitch;
+    const int *sh = shift + b * rows;
+    for (int p = threadIdx.x; p < nh * Ws; p += blockDim.x) {
+      const int hr = p / Ws, ws = p - hr * Ws;
+      float v[BLK * BLK * C];                       // channel (dr * BLK + ds) * C + c
+#pragma unroll
+      for (int dr = 0; dr < BLK; ++dr)
+#pragma unroll
+        for (int c = 0; c < C; ++c) {
+          const int lr = (hr * BLK + dr) * C + c;
+          const int o = sh[lr];
+          float q[4] = {0.f, 0.f, 0.f, 0.f};
+          if (o >= 0) {
+            const float *rp = buf + (size_t)lr * pitch + ws * BLK;
+            const float4 lo = *(const float4 *)rp;
+            const float4 hi = *(const float4 *)(rp + 4);
+            const float w8[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
+#pragma unroll
+            for (int ds = 0; ds < 4; ++ds) {
+              float val = w8[ds];
+              val = o == 1 ? w8[ds + 1] : val;
+              val = o == 2 ? w8[ds + 2] : val;
+              val = o == 3 ? w8[ds + 3] : val;
+              q[ds] = ws * BLK + ds < W ? val : 0.f;
+            }
+          }
+#pragma unroll
+          for (int ds = 0; ds < BLK; ++ds) v[(dr * BLK + ds) * C + c] = q[ds];
+        }
+      char *py = (char *)y + (((size_t)n * Hs + h0 + hr) * Ws + ws) * (size_t)Cs * ESZ;
+      constexpr int NREAL = BLK * BLK * C;
+      constexpr int NCH = (NREAL + VN - 1) / VN;      // chunks holding real channels
+#pragma unroll
+      for (int ch = 0; ch < NCH; ++ch) {
+        Vec16<ST> o;
+#pragma unroll
+        for (int j = 0; j < VN; ++j) o.v[j] = ch * VN + j < NREAL ? v[ch * VN + j] : 0.f;
+        o.store(py + ch * 16, tf32_round);
+      }
+      for (int ch = NCH; ch < Cs / VN; ++ch) *(uint4 *)(py + ch * 16) = make_uint4(0, 0, 0, 0);
+    }
+    __syncthreads();   // buffer b is refilled by the next-but-one band
+  }
+}
+
+static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int H, int W,
+                                     int Hs, int Ws, int Cs, int tf32_round, cudaStream_t s) {
+  static const int R = [] {                          // staged rows per band
+    const char *e = getenv("PCNN_S2D_ROWS");
+    return e && atoi(e) > 0 ? atoi(e) : 2;
+  }();
+  const int pitch = ((W + 3) / 4 + 1) * 4;
+  const size_t smem = (size_t)2 * R * 12 * pitch * 4 + 16 + 2 * R * 12 * 4;
+  if (smem > 200 * 1024) return cudaErrorInvalidValue;
+  const long long tiles = (long long)B * ((Hs + R - 1) / R);
+  int dev = 0, sms = 148, occ = 1;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+#define PCNN_S2D(STT)                                                                          \
+  do {                                                                                         \
+    if (smem > 48 * 1024)                                                                      \
+      cudaFuncSetAttribute(stage_s2d4_kernel<STT>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                           (int)smem);                                                         \
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stage_s2d4_kernel<STT>, 256, smem);    \
+    const unsigned grid = (unsigned)std::min<long long>(tiles, (long long)sms * std::max(occ, 1)); \
+    stage_s2d4_kernel<STT><<<grid, 256, smem, s>>>(x, y, B, H, W, Hs, Ws, Cs, R, tf32_round);  \
+  } while (0)
+  if (st == ST_BF16) PCNN_S2D(ST_BF16);
+  else PCNN_S2D(ST_F32);
+#undef PCNN_S2D
+  return cudaGetLastError();
+}
+
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
                                int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {
-  if (C == 3 && !getenv("PCNN_OLD_STAGE") && gather3_ok(st, W, Cs, blk, blk))
+  const char *old_stage = getenv("PCNN_OLD_STAGE");   // A/B: the staged-gather kernels
+  if (C == 3 && blk == 4 && pad == 0 && !old_stage && Cs >= 48 &&
+      Cs % (st == ST_BF16 ? 8 : 4) == 0 && Hs * 4 <= H + 3 && Ws * 4 <= W + 3)
+    return launch_stage_s2d4(x, y, st, B, H, W, Hs, Ws, Cs, tf32_round, s);
+  if (C == 3 && !old_stage && gather3_ok(st, W, Cs, blk, blk))
     return launch_gather3(x, y, st, B, H, W, Hs, Ws, Cs, blk, blk, pad, 0, tf32_round, s);
   if (C == 3 && (blk == 4 || blk == 1) && W <= 4096) {
     const int Wp = ((Ws * blk + 3) & ~3) + 4;
