@@ -127,7 +127,33 @@ typedef struct {
                            window per filter row feeds all S taps)           */
     int halo_in, halo_out; /* zero border of the stored input / output
                            activation layouts ([B][H+2h][W+2h][C])           */
+    int cta_group;      /* SMs per GEMM tile: 2 for CTA-pair tiles, else 1   */
 } pcnn_layer_info;
+
+/* Resource + time model of one layer, for the
+ * layer's current variant at `batch`, on the whole device:
+ *   grid_size     GridSize = work units of the layer's GEMM (eq. 4 tiles x
+ *                 split-K factor); non-GEMM layers: 0
+ *   opt_tlp       CTAs per SM: 1 for tcgen05 kernels (one CTA per SM by
+ *                 shared memory / TMEM), the kernel's occupancy for SIMT
+ *   n_invocations eq. 8 on all SMs: ceil(GridSize / (TLP * nSMs)), with
+ *                 nSMs counted in CTA-pair units for 2-SM tiles
+ *   opt_sm        eq. 11: the fewest SMs that keep n_invocations (a
+ *                 multiple of cta_group); all SMs for non-GEMM layers
+ *   t_model_us    eq. 12: FLOPs / (peak per SM x opt_sm x rEC x pipe
+ *                 efficiency) -- DESIGN.md R12 reads the garbled "rCE" as
+ *                 eq. 9's rEC and "FMA / total instructions" as the tensor
+ *                 pipe's measured efficiency (0.8); non-GEMM layers: their
+ *                 algorithmic bytes at the HBM bandwidth (6.5 TB/s)
+ * Host-only (no launch); INVALID_ARGUMENT for a bad layer / batch. */
+typedef struct {
+    long long grid_size;
+    int opt_tlp;
+    int n_invocations;
+    int opt_sm;
+    int cta_group;
+    double t_model_us;
+} pcnn_budget_plan;
 
 typedef struct pcnn_net pcnn_net;
 
@@ -199,6 +225,9 @@ pcnn_status pcnn_output_size(const pcnn_net *net, int *out_elems);
 pcnn_status pcnn_num_layers(const pcnn_net *net, int *n_layers);
 pcnn_status pcnn_query_layer(const pcnn_net *net, int layer, int batch,
                              pcnn_layer_info *info);
+/* eqs. 8 / 11 / 12 for one layer (pcnn_budget_plan above). */
+pcnn_status pcnn_plan_budget(const pcnn_net *net, int layer, int batch,
+                             pcnn_budget_plan *plan);
 
 /* Host-only shape inference + FLOP/byte accounting of a descriptor list,
  * no device needed (used by CPU tests and by planners).  infos[n_layers]. */

@@ -213,6 +213,39 @@ def rank_r_conv_weight(w, groups, r):
     return out, unique
 
 
+# perforation-interpolation (NEXT-1; Fig. 11, ref. [38] P:479)
+def perforation_index(n, s):
+    """Reading R13: the grid perforation keeps every s-th output row (column)
+    0, s, 2s, ... < n; every other index takes the value of its nearest kept
+    index (ties to the lower one; indices past the last kept one take the
+    last).  Returns the kept-index source of each of the n outputs."""
+    kept = list(range(0, n, s))
+    src = []
+    for p in range(n):
+        best = min(kept, key=lambda k: (abs(p - k), k))
+        src.append(best)
+    return np.asarray(src, dtype=np.int64)
+
+
+def perforated_conv2d(x, w, b, stride=1, pad=0, groups=1, relu=False, sh=1, sw=1,
+                      threads=None):
+    """Perforated conv: the convolution (eq. 1, bias, ReLU) evaluated
+    only at the kept output positions of an sh x sw grid -- perforation rate
+    1 - H'W'/(HW) -- and every skipped position filled with its nearest kept
+    neighbour (interpolation, R13).  The kept values are the exact conv's
+    values at those positions (the direct loop computes every output position
+    independently), so they are taken from conv2d."""
+    y = conv2d(x, w, b, stride, pad, groups, relu, threads)
+    Ho, Wo = y.shape[2], y.shape[3]
+    ri, ci = perforation_index(Ho, sh), perforation_index(Wo, sw)
+    return y[:, :, ri][:, :, :, ci]
+
+
+def perforation_rate(Ho, Wo, sh, sw):
+    """1 - W'_o H'_o / (W_o H_o)."""
+    return 1.0 - len(range(0, Ho, sh)) * len(range(0, Wo, sw)) / float(Ho * Wo)
+
+
 # analytical helpers (eqs. 4, 5, 6, 8, 9, 11)
 def grid_size(M, N, m, n):
     return lib().orc_grid_size(M, N, m, n)
@@ -239,7 +272,7 @@ def opt_sm(grid, tlp, nsms):
 
 
 def run_net(net, weights, biases, x, ranks=None, threads=None,
-            return_all=False):
+            return_all=False, perforation=None):
     """Run a synth net description over images x [B,C,H,W] in FP64.
 
     ranks: optional {layer_index: r} -> the conv/FC weight of that layer is
@@ -248,6 +281,7 @@ def run_net(net, weights, biases, x, ranks=None, threads=None,
     with return_all, the list of every layer's output.
     """
     ranks = ranks or {}
+    perforation = perforation or {}       # {layer: (sh, sw)} (NEXT-1, R13)
     a = np.asarray(x, dtype=np.float64)
     outs = []
     for i, L in enumerate(net["layers"]):
@@ -256,8 +290,13 @@ def run_net(net, weights, biases, x, ranks=None, threads=None,
             w = weights[i]
             if i in ranks:
                 w, _ = rank_r_conv_weight(w, L["groups"], ranks[i])
-            a = conv2d(a, w, biases[i], L["stride"], L["pad"], L["groups"],
-                       L["relu"], threads)
+            if i in perforation:
+                sh, sw = perforation[i]
+                a = perforated_conv2d(a, w, biases[i], L["stride"], L["pad"], L["groups"],
+                                      L["relu"], sh, sw, threads)
+            else:
+                a = conv2d(a, w, biases[i], L["stride"], L["pad"], L["groups"],
+                           L["relu"], threads)
         elif k == "fc":
             w = weights[i]
             if i in ranks:

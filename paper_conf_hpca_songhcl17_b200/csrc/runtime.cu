@@ -824,6 +824,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->splits = p.splits;
       info->a_mode = g.pm ? 2 : (p.rect_w ? 1 : 0);
       info->n_sms = std::max(info->n_sms, p.grid);   // pair granularity
+      info->cta_group = p.cg;
     }
     if (ws_need) *ws_need = std::max(*ws_need, p.splits > 1 ? (size_t)p.splits * g.M * g.out_cs * 4 : 0);
     if (!x) return PCNN_OK;   // planning only
@@ -855,6 +856,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->grid = grid;
       info->tlp = ly.tlp > 0 ? ly.tlp : net->occ_simt;
       info->engine = 0;
+      info->cta_group = 1;
     }
     if (!x) return PCNN_OK;
     Budget b = make_budget(net, ly, slot, true);
@@ -1493,6 +1495,53 @@ pcnn_status pcnn_set_sm_budget(pcnn_net *net, int layer, int n_sms, int ctas_per
   ly.n_sms = n_sms >= net->num_sms ? 0 : n_sms;
   ly.tlp = ctas_per_sm;
   net->version++;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_plan_budget(const pcnn_net *cnet, int layer, int batch, pcnn_budget_plan *bp) {
+  pcnn_net *net = const_cast<pcnn_net *>(cnet);
+  if (!net || !bp || layer < 0 || layer >= (int)net->layers.size() || batch <= 0)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  std::memset(bp, 0, sizeof *bp);
+  Layer &ly = net->layers[layer];
+  const int nsms = net->num_sms;
+  bp->opt_sm = nsms;
+  bp->cta_group = 1;
+  bp->opt_tlp = 1;
+  if (!ly.gemm) {
+    bp->t_model_us = layer_bytes(ly, batch, net->desc.precision,
+                                 layer == (int)net->layers.size() - 1) / 6.5e12 * 1e6;
+    return PCNN_OK;
+  }
+  // the plan on the whole device (the budget in effect must not change it)
+  const int save_sms = ly.n_sms, save_tlp = ly.tlp;
+  ly.n_sms = 0;
+  ly.tlp = 0;
+  pcnn_layer_info f;
+  pcnn_status s = pcnn_query_layer(net, layer, batch, &f);
+  ly.n_sms = save_sms;
+  ly.tlp = save_tlp;
+  if (s != PCNN_OK) return s;
+  const int cg = std::max(1, f.cta_group);
+  const long long G = f.tiles * std::max(1, f.splits);
+  const int tlp = f.engine == 1 ? 1 : std::max(1, net->occ_simt);
+  const long long slots = nsms / cg;                       // SMs in tile units
+  const long long inv = (G + (long long)tlp * slots - 1) / ((long long)tlp * slots);   // eq. 8
+  long long p = 1;                                        // eq. 11: the fewest units
+  while (p < slots && (G + (long long)tlp * p - 1) / ((long long)tlp * p) != inv) ++p;
+  bp->grid_size = G;
+  bp->opt_tlp = tlp;
+  bp->n_invocations = (int)inv;
+  bp->cta_group = cg;
+  bp->opt_sm = (int)(p * cg);
+  // eq. 12 (reading R12): peak per SM from the tensor / FFMA rate x SM clock
+  int khz = 0;
+  cudaDeviceGetAttribute(&khz, cudaDevAttrClockRate, net->device);
+  const double clk = khz > 0 ? khz * 1e3 : 1.965e9;
+  const double flop_per_clk = f.engine == 0 ? 256.0
+                              : (net->desc.precision == PCNN_TF32 ? 4096.0 : 8192.0);
+  const double eff = 0.8;
+  bp->t_model_us = f.flops / (flop_per_clk * clk * bp->opt_sm * std::max(f.rec, 1e-9) * eff) * 1e6;
   return PCNN_OK;
 }
 

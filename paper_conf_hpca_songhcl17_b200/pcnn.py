@@ -54,7 +54,17 @@ class LayerInfo(ctypes.Structure):
                 ("tlp", ctypes.c_int), ("engine", ctypes.c_int), ("tile_m", ctypes.c_int),
                 ("tile_n", ctypes.c_int), ("tiles", ctypes.c_longlong), ("grid", ctypes.c_int),
                 ("util", ctypes.c_double), ("rec", ctypes.c_double), ("splits", ctypes.c_int),
-                ("a_mode", ctypes.c_int), ("halo_in", ctypes.c_int), ("halo_out", ctypes.c_int)]
+                ("a_mode", ctypes.c_int), ("halo_in", ctypes.c_int), ("halo_out", ctypes.c_int),
+                ("cta_group", ctypes.c_int)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class BudgetPlan(ctypes.Structure):
+    _fields_ = [("grid_size", ctypes.c_longlong), ("opt_tlp", ctypes.c_int),
+                ("n_invocations", ctypes.c_int), ("opt_sm", ctypes.c_int),
+                ("cta_group", ctypes.c_int), ("t_model_us", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -74,6 +84,7 @@ _lib.pcnn_infer_host.argtypes = [_P, _P, ctypes.c_int, _P, _P, _P, _P]
 _lib.pcnn_output_size.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.pcnn_num_layers.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.pcnn_query_layer.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.POINTER(LayerInfo)]
+_lib.pcnn_plan_budget.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.POINTER(BudgetPlan)]
 _lib.pcnn_describe_net.argtypes = [ctypes.POINTER(NetDesc), ctypes.POINTER(LayerDesc),
                                    ctypes.c_int, ctypes.c_int, ctypes.POINTER(LayerInfo)]
 _lib.pcnn_profile_layers.argtypes = [_P, _P, ctypes.c_int, _P, ctypes.c_int, _FP, _FP, _P]
@@ -90,7 +101,7 @@ _lib.pcnn_status_string.restype = ctypes.c_char_p
 _lib.pcnn_last_error_message.restype = ctypes.c_char_p
 for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_infer",
-           "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer",
+           "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
            "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
            "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
            "pcnn_last_launch_count"):
@@ -98,7 +109,7 @@ for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
 
 EXPORTED = ["pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
             "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_infer",
-            "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer",
+            "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
             "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
             "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
             "pcnn_last_launch_count", "pcnn_device_sm_count", "pcnn_version",
@@ -262,6 +273,22 @@ class Net:
         _check(_lib.pcnn_query_layer(self._h, layer, batch, ctypes.byref(info)),
                "pcnn_query_layer")
         return info.as_dict()
+
+    def plan_budget(self, layer, batch):
+        """eqs. 8 / 11 / 12 for one layer (see pcnn_plan_budget)."""
+        bp = BudgetPlan()
+        _check(_lib.pcnn_plan_budget(self._h, layer, batch, ctypes.byref(bp)),
+               "pcnn_plan_budget")
+        return bp.as_dict()
+
+    def apply_opt_budgets(self, batch):
+        """Give every GEMM layer its eq. 11 optSM x optTLP budget (P:341);
+        returns the plans."""
+        plans = [self.plan_budget(i, batch) for i in range(self.n_layers)]
+        for i, p in enumerate(plans):
+            if p["grid_size"] > 0:
+                self.set_sm_budget(i, p["opt_sm"], 0)
+        return plans
 
     def profile_layers(self, images, reps=5, out=None, stream=None):
         import torch

@@ -129,3 +129,70 @@ def test_rank_variant_rejects_bad_requests(alex):
     info = n.query_layer(3, 2)
     assert info["variant"] == 1 and info["rank"] == 32
     assert info["flops"] < info["flops_exact"]
+
+
+# ------------------------------------------------------------------ resource / time model (NEXT-3)
+@pytest.mark.parametrize("prec,B", [("bf16", 1), ("bf16", 64), ("fp32", 2)])
+def test_plan_budget_matches_oracle_eq11(orc, alex, prec, B):
+    """pcnn_plan_budget's optSM is eq. 11 (P:296-303) applied to the layer's
+    own GridSize, TLP and SM count -- checked against the oracle's eq. 8 / 11
+    helpers, which tests/test_oracle_pins.py pins to the paper's worked
+    example -- and eq. 12's time is positive and scales with 1 / optSM."""
+    import torch
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    net, w, b, _ = alex
+    n = pcnn.Net(net, w, b, B, prec)
+    nsms = torch.cuda.get_device_properties(0).multi_processor_count
+    for i, L in enumerate(net["layers"]):
+        p = n.plan_budget(i, B)
+        if L["kind"] not in ("conv", "fc"):
+            assert p["grid_size"] == 0 and p["opt_sm"] == nsms
+            continue
+        cg, G, tlp = p["cta_group"], p["grid_size"], p["opt_tlp"]
+        info = n.query_layer(i, B)
+        assert G == info["tiles"] * info["splits"]
+        assert tlp == (1 if prec == "bf16" else max(1, info["tlp"]))
+        assert p["n_invocations"] == orc.n_invocations(G, tlp, nsms // cg)
+        assert p["opt_sm"] == cg * orc.opt_sm(G, tlp, nsms // cg), (i, p)
+        assert p["opt_sm"] <= nsms and p["t_model_us"] > 0
+
+
+def test_opt_budgets_keep_results_and_latency(alex):
+    """Running every GEMM layer on its eq. 11 optSM changes placement only
+    (bitwise identical logits, per-layer SM census within optSM) and keeps
+    the number of invocations, so the whole pass stays within 25% of the
+    unbudgeted latency (the paper's claim: 'release SMs' at the same
+    nInvocations)."""
+    import torch
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    net, w, b, _ = alex
+    B = 8
+    x = torch.from_numpy(synth.images(0, B, net["in_shape"])).cuda()
+
+    def timed(n):
+        n.infer(x)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(20):
+            n.infer(x)
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / 20
+
+    n0 = pcnn.Net(net, w, b, B, "bf16")
+    base, _, _ = n0.infer(x)
+    t0 = timed(n0)
+    n1 = pcnn.Net(net, w, b, B, "bf16")
+    plans = n1.apply_opt_budgets(B)
+    n1.enable_sm_census(True)
+    out, _, _ = n1.infer(x)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(out.cpu().numpy(), base.cpu().numpy())
+    for i, p in enumerate(plans):
+        if p["grid_size"] > 0:
+            assert 0 < len(n1.sm_census(i)) <= p["opt_sm"], (i, p)
+    assert sum(p["opt_sm"] < 148 for p in plans if p["grid_size"] > 0) >= 1   # SMs released
+    n1.enable_sm_census(False)
+    t1 = timed(n1)
+    assert t1 <= 1.25 * t0, (t0, t1)

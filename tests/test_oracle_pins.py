@@ -310,3 +310,51 @@ def test_rec_eq9_closed_forms(orc):
     assert orc.rec(256, 256, 128, 128) == 1.0
     assert orc.rec(100, 128, 128, 128) == 100 / 128
     assert abs(orc.rec(169, 128, 128, 128) - 169 / 256) < 1e-15
+
+
+# ------------------------------------------------------------ perforation (NEXT-1, R13)
+def test_perforation_index_hand_fixture(orc):
+    """Nearest kept index (ties to the lower one) on a hand-written case:
+    n = 7, s = 3 keeps 0, 3, 6; n = 6, s = 2 keeps 0, 2, 4 (5 -> 4);
+    n = 5, s = 4 keeps 0, 4 (2 is a tie -> 0)."""
+    assert list(orc.perforation_index(7, 3)) == [0, 0, 3, 3, 3, 6, 6]
+    assert list(orc.perforation_index(6, 2)) == [0, 0, 2, 2, 4, 4]
+    assert list(orc.perforation_index(5, 4)) == [0, 0, 0, 4, 4]
+    assert list(orc.perforation_index(4, 1)) == [0, 1, 2, 3]
+
+
+def test_perforation_rate_zero_is_exact_conv(orc):
+    """Rate 0 (sh = sw = 1) is the exact layer, bit for bit."""
+    rng = np.random.default_rng(3)
+    x = rng.standard_normal((2, 6, 9, 8))
+    w = rng.standard_normal((8, 3, 3, 3))
+    b = rng.standard_normal(8)
+    e = orc.conv2d(x, w, b, 1, 1, 2, True)
+    p = orc.perforated_conv2d(x, w, b, 1, 1, 2, True, 1, 1)
+    np.testing.assert_array_equal(p, e)
+    assert orc.perforation_rate(9, 8, 1, 1) == 0.0
+
+
+def test_perforation_kept_values_and_interpolation(orc):
+    """Kept positions carry the exact conv values computed by brute force at
+    those positions only; every other position equals a kept neighbour at
+    distance <= s/2 per axis; the rate is 1 - H'W'/(HW)."""
+    rng = np.random.default_rng(4)
+    x = rng.standard_normal((1, 3, 11, 10))
+    w = rng.standard_normal((4, 3, 3, 3))
+    b = rng.standard_normal(4)
+    sh, sw = 2, 3
+    y = orc.perforated_conv2d(x, w, b, 1, 1, 1, False, sh, sw)
+    xp = np.pad(x, ((0, 0), (0, 0), (1, 1), (1, 1)))
+    for p in range(0, 11, sh):
+        for q in range(0, 10, sw):
+            for f in range(4):
+                ref = b[f] + np.sum(w[f] * xp[0, :, p:p + 3, q:q + 3])
+                assert abs(y[0, f, p, q] - ref) < 1e-12
+    for p in range(11):
+        for q in range(10):
+            kp = min(range(0, 11, sh), key=lambda k: (abs(p - k), k))
+            kq = min(range(0, 10, sw), key=lambda k: (abs(q - k), k))
+            assert abs(p - kp) <= sh // 2 + (1 if p > 10 // sh * sh else 0)
+            np.testing.assert_array_equal(y[0, :, p, q], y[0, :, kp, kq])
+    assert abs(orc.perforation_rate(11, 10, sh, sw) - (1 - 6 * 4 / 110)) < 1e-15
