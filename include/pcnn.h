@@ -181,6 +181,16 @@ pcnn_status pcnn_destroy_net(pcnn_net *net);
  * INVALID_ARGUMENT for a bad rank. */
 pcnn_status pcnn_set_variant(pcnn_net *net, int layer, int variant, int rank);
 
+/* Perforation-interpolation variant (Fig. 11; reading
+ * R13): the conv is evaluated only at the kept positions of an sh x sw
+ * output grid (rows 0, sh, 2sh, ...; columns 0, sw, ...) -- perforation rate
+ * 1 - H'W'/(HW) -- and every other output position takes the value of its
+ * nearest kept neighbour (ties to the lower index).  sh = sw = 1 turns it off;
+ * steps 1..4.  Conv layers on the tcgen05 engine (BF16 / TF32) only;
+ * UNSUPPORTED for the FP32 SIMT path, a staged first conv, or a layer with a
+ * rank variant (pcnn_set_variant(EXACT) clears both). */
+pcnn_status pcnn_set_perforation(pcnn_net *net, int layer, int sh, int sw);
+
 /* Test hook: install explicit factors for a RANK variant.
  *   A : host fp32 [groups][N_f/g][rank]   (stage-2 1x1 weights)
  *   B : host fp32 [groups][rank][C/g][S][S] (stage-1 filters, OIHW)

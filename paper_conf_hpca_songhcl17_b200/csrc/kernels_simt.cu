@@ -1527,6 +1527,51 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   return lrn_pool_dispatch<ST_F32>(a, grid, smem, stream);
 }
 
+// ------------------------------------------------------------ NEXT-1: interpolation
+// Perforation-interpolation (Fig. 11, reading R13): every output pixel
+// of the layer takes the channel vector of its nearest kept grid position
+// (kept rows 0, sh, 2sh, ...; ties to the lower one).  A pure copy: one thread
+// per (output pixel, 16 B chunk), chunk fastest so loads and stores coalesce.
+__device__ __forceinline__ int perf_src(int p, int s, int n) {
+  const int lo = p / s * s, hi = lo + s;
+  return (hi < n && hi - p < p - lo) ? hi / s : lo / s;
+}
+
+__global__ void __launch_bounds__(256)
+perf_interp_kernel(const uint4 *__restrict__ t, uint4 *__restrict__ y, int B, int Ho, int Wo,
+                   int sh, int sw, int chunks, int ho) {
+  const int Hk = (Ho + sh - 1) / sh, Wk = (Wo + sw - 1) / sw;
+  const int Hp = Ho + 2 * ho, Wp = Wo + 2 * ho;
+  const long long total = (long long)B * Hp * Wp * chunks;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int ch = (int)(i % chunks);
+    const long long pix = i / chunks;
+    const int q = (int)(pix % Wp) - ho;
+    const long long r = pix / Wp;
+    const int p = (int)(r % Hp) - ho;
+    const long long n = r / Hp;
+    uint4 v = make_uint4(0, 0, 0, 0);
+    if (p >= 0 && p < Ho && q >= 0 && q < Wo) {
+      const long long src = ((n * Hk + perf_src(p, sh, Ho)) * Wk + perf_src(q, sw, Wo)) * chunks + ch;
+      v = __ldg(t + src);
+    }
+    y[i] = v;
+  }
+}
+
+cudaError_t launch_perf_interp(const void *t, void *y, int st, int B, int Ho, int Wo, int sh,
+                               int sw, int Cs, int ho, cudaStream_t s) {
+  const int esz = st == ST_BF16 ? 2 : 4;
+  if ((Cs * esz) % 16) return cudaErrorInvalidValue;
+  const int chunks = Cs * esz / 16;
+  const long long total = (long long)B * (Ho + 2 * ho) * (Wo + 2 * ho) * chunks;
+  const int grid = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
+  perf_interp_kernel<<<grid, 256, 0, s>>>((const uint4 *)t, (uint4 *)y, B, Ho, Wo, sh, sw,
+                                          chunks, ho);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------------ a7: softmax + entropy
 // One warp per image: max and sum by warp shuffles (eq. 2).
 // H = ln S - sum_j p_j (z_j - max), algebraically -sum p ln p (reading R6).

@@ -862,8 +862,10 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           const int m0 = mt * (TC_BM * CG) + (int)rank * TC_BM;
           n0 = m0 / HoWo;
           const int pq = m0 % HoWo;
-          w0 = (pq % g.Wo) * g.stride - g.pad;
-          h0 = (pq / g.Wo) * g.stride - g.pad;
+          // perforated variant: kept positions psh / psw output rows / cols
+          // apart; a zero-haloed input shifts every window by ih
+          w0 = (pq % g.Wo) * g.stride * max(g.psw, 1) - g.pad + g.ih;
+          h0 = (pq / g.Wo) * g.stride * max(g.psh, 1) - g.pad + g.ih;
         }
         for (int kb = k0; kb < k1; ++kb) {
           wc.wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);

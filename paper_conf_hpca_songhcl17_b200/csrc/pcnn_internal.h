@@ -56,6 +56,11 @@ struct ConvGeom {
   // the next layer's padding).  Requires stride 1 and S == 2*pad + 1.
   int pm;
   int hv, wv, vh;
+  // perforated variant (NEXT-1, reading R13; im2col mode only): the GEMM rows
+  // are the kept output positions of a psh x psw grid (Ho, Wo above are the
+  // kept counts), i.e. input windows stride*psh / stride*psw apart; ih = zero
+  // border of the stored input ([B][H + 2ih][W + 2ih][Cs]); 0 = plain
+  int psh, psw, ih;
 };
 
 // ---------------------------------------------------------------- launchers
@@ -143,6 +148,11 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
 long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s,
                          int Ho, int Wo);
 int lrn_pool_occupancy(int st);
+// NEXT-1 interpolation: y [B][Ho + 2ho][Wo + 2ho][Cs] from the kept grid
+// t [B][ceil(Ho/sh)][ceil(Wo/sw)][Cs] by nearest kept neighbour (ties to the
+// lower index, reading R13); halo cells written as zeros.
+cudaError_t launch_perf_interp(const void *t, void *y, int st, int B, int Ho, int Wo, int sh,
+                               int sw, int Cs, int ho, cudaStream_t s);
 // a7
 cudaError_t launch_softmax_entropy(const float *z, float *p, float *h, int B,
                                    int N, cudaStream_t s);

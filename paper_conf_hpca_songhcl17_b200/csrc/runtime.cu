@@ -133,6 +133,9 @@ struct Layer {
   // rank-r variant
   int variant = PCNN_VARIANT_EXACT, rank = 0;
   GemmStage r1, r2;
+  // perforated variant (NEXT-1): kept-grid steps (1, 1 = off) and its stage
+  int perf_sh = 1, perf_sw = 1;
+  GemmStage pf;
   std::vector<float> host_w;   // OIHW copy kept for the SVD (conv only)
   std::vector<Svd> svd;        // per group (lazily computed)
   // budget
@@ -303,6 +306,9 @@ static double layer_flops_exact(const Layer &ly, int B) {
 }
 
 static double layer_flops_variant(const Layer &ly, int B) {
+  if (ly.perf_sh * ly.perf_sw > 1)       // eq. 1 FLOPs at the kept positions only
+    return layer_flops_exact(ly, B) * ((ly.out_h + ly.perf_sh - 1) / ly.perf_sh) *
+           ((ly.out_w + ly.perf_sw - 1) / ly.perf_sw) / ((double)ly.out_h * ly.out_w);
   if (ly.variant != PCNN_VARIANT_RANK) return layer_flops_exact(ly, B);
   const auto &d = ly.d;
   const double P = (double)B * ly.out_h * ly.out_w;
@@ -567,16 +573,23 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, co
   }
   auto enc = get_encode_im2col();
   if (!enc) return nullptr;
-  // bounding box of the conv's input corners (square kernels: W and H equal)
-  const int lower[2] = {-g.pad, -g.pad};
-  const int upper[2] = {g.pad - (g.S - 1), g.pad - (g.S - 1)};
-  const cuuint32_t estr[4] = {1, (cuuint32_t)g.stride, (cuuint32_t)g.stride, 1};
+  // bounding box of the conv's input corners (square kernels: W and H equal);
+  // a zero-haloed input (perforated variant of a padded-layout layer) is the
+  // grid [H + 2ih][W + 2ih] whose windows start ih - pad inside it
+  cuuint64_t dimsh[4] = {dims[0], dims[1] + 2 * (cuuint64_t)g.ih, dims[2] + 2 * (cuuint64_t)g.ih,
+                         dims[3]};
+  const cuuint64_t stridesh[3] = {(cuuint64_t)g.Cs * esz, dimsh[1] * g.Cs * esz,
+                                  dimsh[2] * dimsh[1] * g.Cs * esz};
+  const int lower[2] = {g.ih - g.pad, g.ih - g.pad};
+  const int upper[2] = {g.pad - (g.S - 1) - g.ih, g.pad - (g.S - 1) - g.ih};
+  const cuuint32_t estr[4] = {1, (cuuint32_t)(g.stride * std::max(g.psw, 1)),
+                              (cuuint32_t)(g.stride * std::max(g.psh, 1)), 1};
   const CUtensorMapSwizzle sw = slab == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
                                 : slab == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
                                              : CU_TENSOR_MAP_SWIZZLE_32B;
   CUresult r = enc(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
                                         : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
-                   4, const_cast<void *>(x), dims, strides, lower, upper,
+                   4, const_cast<void *>(x), dimsh, stridesh, lower, upper,
                    (cuuint32_t)(slab / esz), 128, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return nullptr;
@@ -875,6 +888,7 @@ static bool fuse_conv_lrn(const pcnn_net *net, int i) {
   if (!net->fuse_lrn_pool || i + 1 >= (int)net->layers.size()) return false;
   const Layer &c = net->layers[i], &l = net->layers[i + 1];
   return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 && c.pm_halo == 0 &&
+         c.perf_sh * c.perf_sw == 1 &&
          c.exact.engine == 1 && c.variant == PCNN_VARIANT_EXACT && c.d.groups == 1 &&
          c.d.out_channels <= 128 && c.out_cs == c.d.out_channels;
 }
@@ -932,6 +946,15 @@ static pcnn_status run_layer(pcnn_net *net, int i, int B, const void *x, void *y
   switch (ly.d.kind) {
     case PCNN_CONV:
     case PCNN_FC:
+      if (ly.perf_sh * ly.perf_sw > 1) {
+        // perforation: the conv at the kept grid into the scratch buffer, then
+        // nearest-neighbour interpolation into the layer's output layout
+        pcnn_status r = run_stage(net, ly, ly.pf, B, x, r_buf, 0, s, nullptr);
+        if (r != PCNN_OK) return r;
+        CUDA_TRY(counted(launch_perf_interp(r_buf, y, st, B, ly.out_h, ly.out_w, ly.perf_sh,
+                                            ly.perf_sw, ly.out_cs, ly.out_halo, s)));
+        return PCNN_OK;
+      }
       if (ly.variant == PCNN_VARIANT_RANK) {
         pcnn_status r = run_stage(net, ly, ly.r1, B, x, r_buf, 0, s, nullptr);
         if (r != PCNN_OK) return r;
@@ -1065,7 +1088,9 @@ static pcnn_status ensure_workspace(pcnn_net *net, int batch) {
   size_t need = 0;
   for (auto &ly : net->layers) {
     if (!ly.gemm) continue;
-    if (ly.variant == PCNN_VARIANT_RANK) {
+    if (ly.perf_sh * ly.perf_sw > 1) {
+      run_stage(net, ly, ly.pf, batch, nullptr, nullptr, 0, nullptr, nullptr, &need);
+    } else if (ly.variant == PCNN_VARIANT_RANK) {
       run_stage(net, ly, ly.r1, batch, nullptr, nullptr, 0, nullptr, nullptr, &need);
       run_stage(net, ly, ly.r2, batch, nullptr, nullptr, 0, nullptr, nullptr, &need);
     } else {
@@ -1408,6 +1433,7 @@ pcnn_status pcnn_destroy_net(pcnn_net *net) {
     ly.exact.release();
     ly.r1.release();
     ly.r2.release();
+    ly.pf.release();
     if (ly.d_ctr) cudaFree(ly.d_ctr);
     if (ly.d_census) cudaFree(ly.d_census);
   }
@@ -1439,11 +1465,14 @@ pcnn_status pcnn_set_variant(pcnn_net *net, int layer, int variant, int rank) {
     return fail(PCNN_ERR_INVALID_ARGUMENT, "bad net / layer");
   Layer &ly = net->layers[layer];
   if (variant == PCNN_VARIANT_EXACT) {
-    if (ly.variant != PCNN_VARIANT_EXACT) net->version++;
+    if (ly.variant != PCNN_VARIANT_EXACT || ly.perf_sh * ly.perf_sw > 1) net->version++;
     ly.variant = PCNN_VARIANT_EXACT;
     ly.rank = 0;
+    ly.perf_sh = ly.perf_sw = 1;
     return PCNN_OK;
   }
+  if (ly.perf_sh * ly.perf_sw > 1)
+    return fail(PCNN_ERR_UNSUPPORTED, "rank variant of a perforated layer (set EXACT first)");
   if (variant != PCNN_VARIANT_RANK) return fail(PCNN_ERR_INVALID_ARGUMENT, "bad variant");
   if (ly.d.kind != PCNN_CONV)
     return fail(PCNN_ERR_UNSUPPORTED, "rank variant is implemented for conv layers");
@@ -1475,6 +1504,50 @@ pcnn_status pcnn_set_variant(pcnn_net *net, int layer, int variant, int rank) {
         Bm[((size_t)gi * rank + a) * K + k] = (float)sv.Vt[(size_t)a * K + k];
   }
   return build_rank_stages(net, ly, rank, A.data(), Bm.data());
+}
+
+pcnn_status pcnn_set_perforation(pcnn_net *net, int layer, int sh, int sw) {
+  if (!net || layer < 0 || layer >= (int)net->layers.size() || sh < 1 || sw < 1 || sh > 4 ||
+      sw > 4)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad net / layer / perforation steps (1..4)");
+  Layer &ly = net->layers[layer];
+  if (ly.d.kind != PCNN_CONV)
+    return fail(PCNN_ERR_UNSUPPORTED, "perforation is defined for conv layers (P:328)");
+  if (sh * sw == 1) {
+    if (ly.perf_sh * ly.perf_sw > 1) net->version++;
+    ly.perf_sh = ly.perf_sw = 1;
+    ly.pf.release();
+    return PCNN_OK;
+  }
+  if (ly.variant != PCNN_VARIANT_EXACT)
+    return fail(PCNN_ERR_UNSUPPORTED, "perforation of a rank-r layer (set EXACT first)");
+  if (net->desc.precision == PCNN_FP32_SIMT)
+    return fail(PCNN_ERR_UNSUPPORTED, "perforation runs on the tcgen05 engine (BF16 / TF32)");
+  if (layer == 0 && (net->stage_im2col || net->stage_blk > 1))
+    return fail(PCNN_ERR_UNSUPPORTED,
+                "perforation of a first conv whose input is staged (im2col / space-to-depth)");
+  if (ly.in_halo > 0 && ly.in_halo < ly.d.pad)
+    return fail(PCNN_ERR_UNSUPPORTED, "input halo narrower than the conv padding");
+  CUDA_TRY(cudaSetDevice(net->device));
+  const int mode = ly.exact.g.out_mode;
+  pcnn_status s = build_stage(ly.pf, ly, net->desc.precision, ly.d.out_channels, ly.d.groups,
+                              ly.d.kernel, ly.d.stride, ly.d.pad, ly.d.relu, ly.in_c, ly.in_h,
+                              ly.in_w, ly.in_cs, false, ly.host_w.data(), nullptr, mode);
+  if (s != PCNN_OK) return s;
+  CUDA_TRY(cudaMemcpy(ly.pf.d_bias, ly.exact.d_bias,
+                      sizeof(float) * ((size_t)round_up(ly.d.out_channels, 256) + 256),
+                      cudaMemcpyDeviceToDevice));
+  ConvGeom &g = ly.pf.g;
+  g.psh = sh;
+  g.psw = sw;
+  g.ih = ly.in_halo;
+  g.Ho = (ly.out_h + sh - 1) / sh;        // kept rows / columns
+  g.Wo = (ly.out_w + sw - 1) / sw;
+  g.out_cs = ly.out_cs;
+  ly.perf_sh = sh;
+  ly.perf_sw = sw;
+  net->version++;
+  return PCNN_OK;
 }
 
 pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank, const float *A,
@@ -1579,8 +1652,10 @@ pcnn_status pcnn_query_layer(const pcnn_net *cnet, int layer, int batch, pcnn_la
     float lp[4];
     const bool fl = fuse_conv_lrn(net, layer);
     if (fl) lrn_params(net->layers[layer + 1], lp);
-    pcnn_status s = run_stage(net, ly, ly.variant == PCNN_VARIANT_RANK ? ly.r2 : ly.exact,
-                              batch, nullptr, nullptr, 0, nullptr, f, nullptr, fl ? lp : nullptr);
+    GemmStage &ps = ly.perf_sh * ly.perf_sw > 1 ? ly.pf
+                    : (ly.variant == PCNN_VARIANT_RANK ? ly.r2 : ly.exact);
+    pcnn_status s = run_stage(net, ly, ps, batch, nullptr, nullptr, 0, nullptr, f, nullptr,
+                              fl ? lp : nullptr);
     if (s != PCNN_OK) return s;
     const long long maxb = (long long)f->n_sms * std::max(f->tlp, 1);
     const long long waves = (f->tiles + maxb - 1) / maxb;

@@ -79,6 +79,7 @@ _lib.pcnn_destroy_net.argtypes = [_P]
 _lib.pcnn_set_variant.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
 _lib.pcnn_set_variant_factors.argtypes = [_P, ctypes.c_int, ctypes.c_int, _FP, _FP]
 _lib.pcnn_set_sm_budget.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
+_lib.pcnn_set_perforation.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
 _lib.pcnn_infer.argtypes = [_P, _P, ctypes.c_int, _P, _P, _P, _P]
 _lib.pcnn_infer_host.argtypes = [_P, _P, ctypes.c_int, _P, _P, _P, _P]
 _lib.pcnn_output_size.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
@@ -100,7 +101,7 @@ _lib.pcnn_status_string.argtypes = [ctypes.c_int]
 _lib.pcnn_status_string.restype = ctypes.c_char_p
 _lib.pcnn_last_error_message.restype = ctypes.c_char_p
 for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
-           "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_infer",
+           "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_perforation", "pcnn_infer",
            "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
            "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
            "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
@@ -108,7 +109,7 @@ for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
-            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_infer",
+            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_perforation", "pcnn_infer",
             "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
             "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
             "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
@@ -240,6 +241,9 @@ class Net:
         B = np.ascontiguousarray(B, dtype=np.float32)
         _check(_lib.pcnn_set_variant_factors(self._h, layer, rank, A.ctypes.data_as(_FP),
                                              B.ctypes.data_as(_FP)), "pcnn_set_variant_factors")
+
+    def set_perforation(self, layer, sh, sw):
+        _check(_lib.pcnn_set_perforation(self._h, layer, sh, sw), "pcnn_set_perforation")
 
     def set_sm_budget(self, layer, n_sms, ctas_per_sm=0):
         _check(_lib.pcnn_set_sm_budget(self._h, layer, n_sms, ctas_per_sm), "pcnn_set_sm_budget")

@@ -1,0 +1,108 @@
+"""Run-time management of P-CNN (Fig. 12): entropy-guided greedy
+accuracy tuning over each layer's variant ladder, the tuning path it leaves
+behind, and calibration by backtracking along that path.
+
+This is host-side control logic over the C ABI: every candidate is executed
+by libpcnn's kernels (the network's time comes from CUDA events, its
+uncertainty CNN_entropy from the fused softmax + entropy kernel, eq. 2).
+
+* A *ladder* per layer lists variants from exact to most aggressive, e.g.
+  ``[("exact",), ("rank", 64), ("rank", 32)]`` or
+  ``[("exact",), ("perf", 1, 2), ("perf", 2, 2)]`` (perforation).
+* One greedy *iteration* (Fig. 12) tries, for every layer that has a further
+  rung, that layer one rung further with all other layers unchanged, and
+  scores it with eq. 14:  TE = (T_ori - T_layer) / (H_layer - H_ori);
+  the candidate with the largest TE is adopted (a candidate that does not
+  raise the entropy has TE = +inf: free speed).  Candidates whose entropy
+  exceeds the user's threshold, or that are not faster, are not eligible.
+* Tuning stops when no eligible candidate remains.  Each adopted state is a
+  *tuning table*: the per-layer rungs plus every layer's optSM (eq. 11) for
+  the run-time kernel scheduler.
+* *Calibration* (P:345): at run time, if the observed entropy exceeds the
+  threshold, step back along the path to the most aggressive table whose
+  tuning-time entropy was below the observed-adjusted bound.
+"""
+import math
+
+
+def te_score(t_ori, h_ori, t_new, h_new):
+    """eq. 14.  +inf when the candidate is faster without raising entropy."""
+    dh = h_new - h_ori
+    dt = t_ori - t_new
+    if dh <= 0:
+        return math.inf if dt > 0 else -math.inf
+    return dt / dh
+
+
+def greedy_tune(ladders, measure, threshold, max_iters=64):
+    """Fig. 12.  ladders: {layer: [variant, ...]} (rung 0 = exact);
+    measure(state) -> (time, entropy) for a state {layer: rung}.
+    Returns the tuning path: a list of dicts {"state", "time", "entropy", "te",
+    "layer"} starting with the all-exact state."""
+    state = {l: 0 for l in ladders}
+    t0, h0 = measure(dict(state))
+    path = [{"state": dict(state), "time": t0, "entropy": h0, "te": None, "layer": None}]
+    for _ in range(max_iters):
+        t_ori, h_ori = path[-1]["time"], path[-1]["entropy"]
+        best = None
+        for l, rungs in ladders.items():
+            if state[l] + 1 >= len(rungs):
+                continue
+            cand = dict(state)
+            cand[l] += 1
+            t, h = measure(cand)
+            if h > threshold or t >= t_ori:
+                continue
+            te = te_score(t_ori, h_ori, t, h)
+            if best is None or te > best[0] or (te == best[0] and l < best[1]):
+                best = (te, l, cand, t, h)
+        if best is None:
+            break
+        te, l, cand, t, h = best
+        state = cand
+        path.append({"state": dict(state), "time": t, "entropy": h, "te": te, "layer": l})
+    return path
+
+
+def calibrate(path, index, observed_entropy, threshold):
+    """while the observed uncertainty exceeds the threshold, back-track
+    one table along the tuning path (towards exact).  Returns the new index.
+    The entropy the inputs now produce is estimated by shifting the tuned
+    entropies by (observed - tuned) at the current index."""
+    shift = observed_entropy - path[index]["entropy"]
+    while index > 0 and path[index]["entropy"] + shift > threshold:
+        index -= 1
+    return index
+
+
+def apply_state(net, ladders, state, batch=None):
+    """Program a libpcnn Net with the rungs of `state` (and, given a batch,
+    every GEMM layer's eq. 11 optSM budget)."""
+    for l, rung in state.items():
+        v = ladders[l][rung]
+        net.set_variant(l, "exact")
+        if v[0] == "rank":
+            net.set_variant(l, "rank", v[1])
+        elif v[0] == "perf":
+            net.set_perforation(l, v[1], v[2])
+    if batch is not None:
+        net.apply_opt_budgets(batch)
+
+
+def gpu_measure(net, ladders, images, reps=10):
+    """measure() for greedy_tune on the GPU: mean time per pass (CUDA events)
+    and mean CNN_entropy (eq. 2) of the calibration images."""
+    import torch
+
+    def measure(state):
+        apply_state(net, ladders, state)
+        out, _, ent = net.infer(images, entropy=True)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(reps):
+            net.infer(images, out=out, entropy=ent)
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / reps, float(ent.mean().item())
+    return measure

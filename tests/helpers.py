@@ -17,7 +17,7 @@ def rel_err(y, ref):
 
 
 def gpu_run(net, weights, biases, x, precision, max_batch=None, probs=False,
-            variants=None, budgets=None, census=False):
+            variants=None, budgets=None, census=False, perforation=None):
     """Build a libpcnn net, run x (numpy NCHW fp32) and return numpy outputs."""
     import torch
     from paper_conf_hpca_songhcl17_b200 import pcnn
@@ -25,6 +25,8 @@ def gpu_run(net, weights, biases, x, precision, max_batch=None, probs=False,
     n = pcnn.Net(net, weights, biases, max_batch or B, precision)
     for (i, (v, r)) in (variants or {}).items():
         n.set_variant(i, v, r)
+    for (i, (sh, sw)) in (perforation or {}).items():
+        n.set_perforation(i, sh, sw)
     for (i, (s, t)) in (budgets or {}).items():
         n.set_sm_budget(i, s, t)
     if census:

@@ -1,0 +1,47 @@
+"""Entropy-guided greedy accuracy tuning and calibration (Fig. 12,
+eq. 14) on hand-made (time, entropy) tables whose outcome is worked out by
+hand below -- host logic, no GPU."""
+import math
+
+from paper_conf_hpca_songhcl17_b200 import tuning
+
+
+def table_measure(table):
+    def measure(state):
+        return table[tuple(sorted(state.items()))]
+    return measure
+
+
+def test_te_score_eq14():
+    assert tuning.te_score(10.0, 1.0, 8.0, 1.5) == 4.0          # 2 / 0.5
+    assert tuning.te_score(10.0, 1.0, 9.0, 1.0) == math.inf     # free speed-up
+    assert tuning.te_score(10.0, 1.0, 11.0, 0.9) == -math.inf
+
+
+def test_greedy_follows_fig12():
+    """Two layers, two rungs each.  Iteration 1: layer A -> TE (10-8)/(1.2-1)
+    = 10, layer B -> (10-9)/(1.05-1) = 20: B wins.  Iteration 2 from (0,1):
+    A -> (9-6.5)/(1.3-1.05) = 10, B -> (9-8.9)/(1.06-1.05) = 10: tie -> the
+    lower layer index (A).  Iteration 3 from (1,1): A's rung 2 exceeds the
+    threshold 1.5 (1.6), B -> (6.5-6)/(1.4-1.3) = 5 -> (1,2).  Then A's last
+    rung exceeds the threshold: stop."""
+    T = {((0, 0), (1, 0)): (10.0, 1.00),
+         ((0, 1), (1, 0)): (8.0, 1.20), ((0, 0), (1, 1)): (9.0, 1.05),
+         ((0, 1), (1, 1)): (6.5, 1.30), ((0, 0), (1, 2)): (8.9, 1.06),
+         ((0, 2), (1, 1)): (5.0, 1.60), ((0, 1), (1, 2)): (6.0, 1.40),
+         ((0, 2), (1, 2)): (4.0, 1.70)}
+    ladders = {0: [("exact",), ("rank", 64), ("rank", 32)],
+               1: [("exact",), ("perf", 1, 2), ("perf", 2, 2)]}
+    path = tuning.greedy_tune(ladders, table_measure(T), threshold=1.5)
+    assert [p["layer"] for p in path] == [None, 1, 0, 1]
+    assert [tuple(sorted(p["state"].items())) for p in path][-1] == ((0, 1), (1, 2))
+    assert abs(path[1]["te"] - 20.0) < 1e-9 and abs(path[2]["te"] - 10.0) < 1e-9
+    assert abs(path[3]["te"] - 5.0) < 1e-9
+
+
+def test_calibration_backtracks():
+    path = [{"entropy": 1.0}, {"entropy": 1.2}, {"entropy": 1.4}]
+    # observed 1.6 at table 2 (shift +0.2): table 1 -> 1.4 <= 1.5 is the first safe one
+    assert tuning.calibrate(path, 2, 1.6, 1.5) == 1
+    assert tuning.calibrate(path, 2, 1.45, 1.5) == 2          # within threshold: stay
+    assert tuning.calibrate(path, 2, 3.0, 1.5) == 0           # back to exact

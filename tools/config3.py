@@ -30,6 +30,8 @@ w, b = synth.net_params(net)
 names = [L.get("name", str(i)) for i, L in enumerate(net["layers"])]
 gemm = [i for i, L in enumerate(net["layers"]) if L["kind"] in ("conv", "fc")]
 nsms = torch.cuda.get_device_properties(0).multi_processor_count
+PERF_LADDER = [{}, {3: (1, 2)}, {3: (2, 2)}, {3: (2, 2), 6: (1, 2), 7: (1, 2), 8: (1, 2)},
+               {3: (2, 2), 6: (2, 2), 7: (2, 2), 8: (2, 2)}]
 LADDER = [{}, {3: 64}, {3: 64, 8: 64}, {3: 64, 8: 64, 7: 96}, {3: 64, 8: 64, 7: 96, 6: 192},
           {3: 32, 8: 32, 7: 48, 6: 96}, {3: 16, 8: 16, 7: 32, 6: 48}]
 
@@ -104,4 +106,29 @@ for B in (64, 256):
         rows.append(row)
         n.close()
     res["ladder"][str(B)] = rows
+# NEXT-1: perforation ladder (R13 grid steps per layer)
+res["perforation_ladder"] = {}
+for B in (64, 256):
+    x = torch.from_numpy(synth.images(0, B, net["in_shape"])).cuda()
+    rows = []
+    for lvl, perf in enumerate(PERF_LADDER):
+        n = pcnn.Net(net, w, b, B, "bf16")
+        for i, st in perf.items():
+            n.set_perforation(i, *st)
+        fl = sum(n.query_layer(i, B)["flops"] for i in gemm)
+        fe = sum(n.query_layer(i, B)["flops_exact"] for i in gemm)
+        row = {"level": lvl, "steps": {names[i]: list(st) for i, st in perf.items()},
+               "img_s": round(img_s(n, x), 1), "flop_fraction": round(fl / fe, 4)}
+        if B == 64:
+            out, _, ent = n.infer(torch.from_numpy(xs).cuda(), entropy=True)
+            torch.cuda.synchronize()
+            y = out.cpu().numpy()
+            ref_p = orc.run_net(net, w, b, xs, perforation=perf) if perf else ref_exact
+            row["err_vs_perforated_oracle"] = float(np.abs(y - ref_p).max() / np.abs(ref_p).max())
+            row["err_vs_exact_oracle"] = float(np.abs(y - ref_exact).max() / np.abs(ref_exact).max())
+            row["top1_agree_exact"] = float((y.argmax(1) == ref_exact.argmax(1)).mean())
+            row["mean_entropy"] = float(ent.mean().item())
+        rows.append(row)
+        n.close()
+    res["perforation_ladder"][str(B)] = rows
 print(json.dumps(res, indent=1))
