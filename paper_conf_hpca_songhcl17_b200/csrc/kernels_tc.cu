@@ -42,6 +42,7 @@ constexpr int TC_BM = 128;              // UMMA M (cta_group::1)
 constexpr int TC_BN_MAX = 256;          // max UMMA N
 constexpr int TC_ROW_BYTES = 128;       // one K-block row = one 128B swizzle row
 constexpr int TC_MAX_STAGES = 12;
+constexpr int TC_MAX_BSTAGES = 24;      // padded mode with narrow (SW64/SW32) slabs
 constexpr int TC_A_STAGE = TC_BM * TC_ROW_BYTES;          // 16 KB
 constexpr int TC_STAGE_BUDGET = 176 * 1024;               // operand stages per CTA
 constexpr int TC_MAX_KTAB = 1024;       // slab-table entries kept in smem
@@ -64,14 +65,15 @@ constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 constexpr int SM_EPI = TC_STAGE_BUDGET;
 constexpr int SM_BAR = SM_EPI + 8 * EPI_WARP_BYTES;
 constexpr int SM_FULL = SM_BAR;
-constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_STAGES;
-constexpr int SM_TFULL = SM_EMPTY + 8 * TC_MAX_STAGES;
+constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_BSTAGES;
+constexpr int SM_TFULL = SM_EMPTY + 8 * TC_MAX_BSTAGES;
 constexpr int SM_TEMPTY = SM_TFULL + 16;
 constexpr int SM_TMEMPTR = SM_TEMPTY + 16;
-constexpr int TC_MAX_ASTAGES = 4;       // padded mode: A row-window ring
+constexpr int TC_MAX_ASTAGES = 8;       // padded mode: A row-window ring
 constexpr int SM_AFULL = SM_TMEMPTR + 16;
 constexpr int SM_AEMPTY = SM_AFULL + 8 * TC_MAX_ASTAGES;
-constexpr int SM_KTAB = SM_BAR + 512;
+constexpr int SM_KTAB = SM_BAR + 1024;
+static_assert(SM_AEMPTY + 8 * TC_MAX_ASTAGES <= SM_KTAB, "barrier area");
 constexpr int SM_TOTAL = SM_KTAB + 4 * TC_MAX_KTAB;
 constexpr size_t TC_SMEM_BYTES = SM_TOTAL + 1024;         // + alignment slack
 
@@ -92,10 +94,13 @@ static int pm_a_stage_bytes(int slab_bytes, int S, int msub) {
 void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages, int *b_stages) {
   const int as_bytes = pm_a_stage_bytes(slab_bytes, S, msub);
   const int bs_bytes = bn / cg * slab_bytes;
-  int na = TC_MAX_ASTAGES;
+  // 128 B slabs keep the tuned ring depths (4 windows, 12 tap slabs); narrow
+  // slabs carry 2-4x less work per stage and get deeper rings
+  int na = slab_bytes == 128 ? 4 : TC_MAX_ASTAGES;
   while (na > 2 && na * as_bytes + 2 * S * bs_bytes > TC_STAGE_BUDGET) --na;
   int nb = (TC_STAGE_BUDGET - na * as_bytes) / bs_bytes;
-  if (nb > TC_MAX_STAGES) nb = TC_MAX_STAGES;
+  const int nb_max = slab_bytes == 128 ? TC_MAX_STAGES : TC_MAX_BSTAGES;
+  if (nb > nb_max) nb = nb_max;
   *a_stages = na;
   *b_stages = nb;
 }
@@ -706,7 +711,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     }
   }
   if (tid == 0) {
-    for (int s = 0; s < (g.pm ? a.b_stages : stages); ++s) {
+    for (int s = 0; s < (g.pm ? a.b_stages : stages); ++s) {   // b_stages <= TC_MAX_BSTAGES
       mbar_init(sbase + SM_FULL + 8 * s, 1);
       mbar_init(sbase + SM_EMPTY + 8 * s, 1);
     }
@@ -1344,7 +1349,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
   if (g.pm && (p.splits != 1 || lrn || p.rect_w || g.stride != 1 || g.S != 2 * g.pad + 1 ||
                g.Cg % (args.slab_bytes / (st == ST_BF16 ? 2 : 4)) || p.a_stages < 2 ||
-               p.b_stages < 2 || p.a_stages > TC_MAX_ASTAGES || p.b_stages > TC_MAX_STAGES))
+               p.b_stages < 2 || p.a_stages > TC_MAX_ASTAGES || p.b_stages > TC_MAX_BSTAGES))
     return cudaErrorInvalidValue;
   cudaError_t e;
   const bool L = args.lrn != 0;

@@ -1227,7 +1227,11 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   // padded to a multiple of 128 bytes instead (zeros; packed weights are zero
   // there too), so the conv loads full SW128 slabs.
   const int slab128 = 128 / esz;
-  if (prec != PCNN_FP32_SIMT) {
+  // PCNN_NARROW_PM=1 (experiment): keep such groups unpadded and run the conv
+  // in padded-layout mode on narrow (SW32 / SW64) slabs -- no K padding waste
+  const char *narrow_env = getenv("PCNN_NARROW_PM");
+  const bool narrow_pm = narrow_env && narrow_env[0] == '1';
+  if (prec != PCNN_FP32_SIMT && !narrow_pm) {
     for (int i = 1; i < n_layers; ++i) {
       Layer &ly = net->layers[i];
       Layer &pv = net->layers[i - 1];
@@ -1311,7 +1315,8 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
         if (ly.d.kind != PCNN_CONV) continue;
         const int S = ly.d.kernel, P = ly.d.pad, g = ly.d.groups;
         if (ly.d.stride != 1 || S != 2 * P + 1 || P < 1 || P > 3 || ly.in_cs % g) continue;
-        if (tc_slab_bytes(net->st, ly.in_cs / g) != 128) continue;
+        const int sb = tc_slab_bytes(net->st, ly.in_cs / g);
+        if (sb == 0 || (sb != 128 && !narrow_pm)) continue;
         if ((double)(ly.in_h + 2 * P) * (ly.in_w + 2 * P) > pm_max_halo * ly.in_h * ly.in_w) continue;
         pmh[i] = P;
       }

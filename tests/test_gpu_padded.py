@@ -129,3 +129,20 @@ def test_padded_mode_two_subtiles_bitwise(orc, cg, groups, monkeypatch):
         out[ms] = r["out"]
     np.testing.assert_array_equal(out["1"], out["2"])
     assert rel_err(out["2"], ref) <= TOL["bf16"] / 2
+
+
+@pytest.mark.parametrize("prec", ["bf16", "tf32"])
+def test_padded_mode_narrow_slabs(orc, prec, monkeypatch):
+    """PCNN_NARROW_PM=1: a grouped conv with 48 channels per group (AlexNet
+    conv2's input) stays unpadded and runs in padded-layout mode on SW32
+    (BF16) / SW64 (TF32) slabs, each tap's window shifted by one narrow row."""
+    monkeypatch.setenv("PCNN_NARROW_PM", "1")
+    net = dict(in_shape=(96, 27, 27), layers=[
+        dict(kind="maxpool", k=1, stride=1),
+        conv_layer(256, 5, 96, 1, 2, 2), dict(kind="maxpool", k=3, stride=2)])
+    w, b = params(net, seed=12)
+    x = small_inputs((96, 27, 27), 2, lo=-2, hi=2)
+    ref = orc.run_net(net, w, b, x).reshape(2, -1)
+    r = gpu_run(net, w, b, x, prec)
+    assert r["net"].query_layer(1, 2)["a_mode"] == 2
+    assert rel_err(r["out"], ref) <= TOL[prec] / 2
