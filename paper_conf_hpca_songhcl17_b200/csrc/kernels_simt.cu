@@ -1575,6 +1575,9 @@ cudaError_t launch_perf_interp(const void *t, void *y, int st, int B, int Ho, in
 // ------------------------------------------------------------ a7: softmax + entropy
 // One warp per image: max and sum by warp shuffles (eq. 2).
 // H = ln S - sum_j p_j (z_j - max), algebraically -sum p ln p (reading R6).
+// NR > 0: the row (N <= 32 * NR) is held in registers, read once; NR = 0:
+// generic strided loops.  Same per-element arithmetic either way.
+template <int NR>
 __global__ void softmax_entropy_kernel(const float *__restrict__ z, float *p,
                                        float *h, int B, int N) {
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) / 32;
@@ -1582,30 +1585,63 @@ __global__ void softmax_entropy_kernel(const float *__restrict__ z, float *p,
   if (warp >= B) return;
   const float *zr = z + (size_t)warp * N;
   float m = -INFINITY;
-  for (int j = lane; j < N; j += 32) m = fmaxf(m, zr[j]);
+  float v[NR > 0 ? NR : 1];
+  if constexpr (NR > 0) {
+#pragma unroll
+    for (int i = 0; i < NR; ++i) {
+      const int j = lane + 32 * i;
+      v[i] = j < N ? __ldg(zr + j) : -INFINITY;
+      m = fmaxf(m, v[i]);
+    }
+  } else {
+    for (int j = lane; j < N; j += 32) m = fmaxf(m, zr[j]);
+  }
   for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
   float s = 0.f, sz = 0.f;
-  for (int j = lane; j < N; j += 32) {
-    const float d = zr[j] - m;
-    const float e = expf(d);
-    s += e;
-    sz += e * d;
+  if constexpr (NR > 0) {
+#pragma unroll
+    for (int i = 0; i < NR; ++i) {
+      if (lane + 32 * i < N) {
+        const float d = v[i] - m;
+        const float e = expf(d);
+        s += e;
+        sz += e * d;
+        v[i] = e;
+      }
+    }
+  } else {
+    for (int j = lane; j < N; j += 32) {
+      const float d = zr[j] - m;
+      const float e = expf(d);
+      s += e;
+      sz += e * d;
+    }
   }
   for (int o = 16; o; o >>= 1) {
     s += __shfl_xor_sync(0xffffffffu, s, o);
     sz += __shfl_xor_sync(0xffffffffu, sz, o);
   }
   const float inv = 1.f / s;
-  if (p)
-    for (int j = lane; j < N; j += 32) p[(size_t)warp * N + j] = expf(zr[j] - m) * inv;
+  if (p) {
+    if constexpr (NR > 0) {
+#pragma unroll
+      for (int i = 0; i < NR; ++i)
+        if (lane + 32 * i < N) p[(size_t)warp * N + lane + 32 * i] = v[i] * inv;
+    } else {
+      for (int j = lane; j < N; j += 32) p[(size_t)warp * N + j] = expf(zr[j] - m) * inv;
+    }
+  }
   if (h && lane == 0) h[warp] = logf(s) - sz * inv;
 }
-
 cudaError_t launch_softmax_entropy(const float *z, float *p, float *h, int B,
                                    int N, cudaStream_t s) {
-  const int warps_per_block = 8;
+  // two warps (images) per CTA: a 256-image batch spreads over 128 SMs
+  const int warps_per_block = 2;
   const int grid = (B + warps_per_block - 1) / warps_per_block;
-  softmax_entropy_kernel<<<grid, warps_per_block * 32, 0, s>>>(z, p, h, B, N);
+  if (N <= 32 * 32)
+    softmax_entropy_kernel<32><<<grid, warps_per_block * 32, 0, s>>>(z, p, h, B, N);
+  else
+    softmax_entropy_kernel<0><<<grid, warps_per_block * 32, 0, s>>>(z, p, h, B, N);
   return cudaGetLastError();
 }
 
