@@ -223,7 +223,12 @@ pcnn_status pcnn_infer(pcnn_net *net, const float *d_images, int batch,
 /* End-to-end form of pcnn_infer with HOST buffers: copies h_images to a
  * library-owned device buffer, runs the hot path, copies the outputs back and
  * synchronises `stream` before returning.  Host buffers should be pinned for
- * full PCIe bandwidth.  h_probs / h_entropy may be NULL. */
+ * full PCIe bandwidth.  h_probs / h_entropy may be NULL.  When the images take
+ * much longer to copy than to infer (batch >= 64 and the copy per image > 2x
+ * the modelled compute per image, e.g. AlexNet), the batch runs as 4 chunks
+ * whose host->device copies (on a library stream) overlap the previous
+ * chunk's inference; per-image results then come from chunk-sized launches
+ * (same values up to the split-K grouping of the FC layers). */
 pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch,
                             float *h_out, float *h_probs, float *h_entropy,
                             void *stream);

@@ -161,6 +161,10 @@ struct pcnn_net {
   void *d_act[3] = {nullptr, nullptr, nullptr};
   float *d_host_in = nullptr, *d_host_out = nullptr, *d_host_p = nullptr,
         *d_host_h = nullptr;
+  // pcnn_infer_host pipelining: host->device copies of later chunks on their
+  // own stream while earlier chunks compute
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_copy[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
   int out_elems = 0;
   int occ_simt = 1, occ_lp = 1;
   // input staging geometry (space-to-depth by `blk` for a strided first conv)
@@ -1445,6 +1449,9 @@ pcnn_status pcnn_destroy_net(pcnn_net *net) {
   for (auto &p : net->d_act)
     if (p) cudaFree(p);
   if (net->d_ws) cudaFree(net->d_ws);
+  if (net->copy_stream) cudaStreamDestroy(net->copy_stream);
+  for (auto &e : net->ev_copy)
+    if (e) cudaEventDestroy(e);
   if (net->d_host_in) cudaFree(net->d_host_in);
   if (net->d_host_out) cudaFree(net->d_host_out);
   if (net->d_host_p) cudaFree(net->d_host_p);
@@ -1736,20 +1743,47 @@ pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch, flo
     CUDA_TRY(cudaMalloc(&net->d_host_h, sizeof(float) * maxb));
   }
   cudaStream_t s = (cudaStream_t)stream;
-  CUDA_TRY(cudaMemcpyAsync(net->d_host_in, h_images, sizeof(float) * in_elems * batch,
-                           cudaMemcpyHostToDevice, s));
-  pcnn_status r = pcnn_infer(net, net->d_host_in, batch, net->d_host_out,
-                             h_probs ? net->d_host_p : nullptr,
-                             h_entropy ? net->d_host_h : nullptr, stream);
-  if (r != PCNN_OK) return r;
-  CUDA_TRY(cudaMemcpyAsync(h_out, net->d_host_out, sizeof(float) * net->out_elems * batch,
-                           cudaMemcpyDeviceToHost, s));
-  if (h_probs)
-    CUDA_TRY(cudaMemcpyAsync(h_probs, net->d_host_p, sizeof(float) * net->out_elems * batch,
+  // When the images take much longer to cross PCIe (~50 GB/s) than to infer
+  // (FLOPs at ~700 TFLOP/s), split the batch into 4 chunks: chunk i+1's
+  // host->device copy (own stream) overlaps chunk i's inference.  Images are
+  // independent, so the chunks compute the same per-image results.
+  double flops = 0;
+  for (auto &ly : net->layers) flops += layer_flops_exact(ly, 1);
+  const double h2d_img = sizeof(float) * in_elems / 50e9, comp_img = flops / 7e14;
+  const int k = (batch >= 64 && h2d_img > 2.0 * comp_img) ? 4 : 1;
+  const int chunk = (batch + k - 1) / k;
+  if (k > 1 && !net->copy_stream) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&net->copy_stream, cudaStreamNonBlocking));
+    for (auto &e : net->ev_copy) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
+  if (k > 1) {     // copies start after the caller's prior work on `stream`
+    CUDA_TRY(cudaEventRecord(net->ev_copy[4], s));
+    CUDA_TRY(cudaStreamWaitEvent(net->copy_stream, net->ev_copy[4], 0));
+  }
+  for (int c = 0, b0 = 0; b0 < batch; ++c, b0 += chunk) {
+    const int nb = std::min(chunk, batch - b0);
+    CUDA_TRY(cudaMemcpyAsync(net->d_host_in + (size_t)b0 * in_elems, h_images + (size_t)b0 * in_elems,
+                             sizeof(float) * in_elems * nb, cudaMemcpyHostToDevice,
+                             k > 1 ? net->copy_stream : s));
+    if (k > 1) CUDA_TRY(cudaEventRecord(net->ev_copy[c], net->copy_stream));
+  }
+  for (int c = 0, b0 = 0; b0 < batch; ++c, b0 += chunk) {
+    const int nb = std::min(chunk, batch - b0);
+    if (k > 1) CUDA_TRY(cudaStreamWaitEvent(s, net->ev_copy[c], 0));
+    const size_t oo = (size_t)b0 * net->out_elems;
+    pcnn_status r = pcnn_infer(net, net->d_host_in + (size_t)b0 * in_elems, nb,
+                               net->d_host_out + oo, h_probs ? net->d_host_p + oo : nullptr,
+                               h_entropy ? net->d_host_h + b0 : nullptr, stream);
+    if (r != PCNN_OK) return r;
+    CUDA_TRY(cudaMemcpyAsync(h_out + oo, net->d_host_out + oo, sizeof(float) * net->out_elems * nb,
                              cudaMemcpyDeviceToHost, s));
-  if (h_entropy)
-    CUDA_TRY(cudaMemcpyAsync(h_entropy, net->d_host_h, sizeof(float) * batch,
-                             cudaMemcpyDeviceToHost, s));
+    if (h_probs)
+      CUDA_TRY(cudaMemcpyAsync(h_probs + oo, net->d_host_p + oo,
+                               sizeof(float) * net->out_elems * nb, cudaMemcpyDeviceToHost, s));
+    if (h_entropy)
+      CUDA_TRY(cudaMemcpyAsync(h_entropy + b0, net->d_host_h + b0, sizeof(float) * nb,
+                               cudaMemcpyDeviceToHost, s));
+  }
   CUDA_TRY(cudaStreamSynchronize(s));
   return PCNN_OK;
 }

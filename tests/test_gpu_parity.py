@@ -274,3 +274,28 @@ def test_lrn_register_kernel_matches_band_kernel(orc, shape, monkeypatch):
         # same per-element arithmetic; at most last-place differences
         assert rel_err(reg, band) <= (8e-3 if prec == "bf16" else 1e-6)
         assert np.mean(reg == band) > 0.99
+
+
+def test_infer_host_pipelined_chunks(orc):
+    """AlexNet at B = 64 through pcnn_infer_host takes the pipelined path (4
+    chunks, copies overlapping inference): same logits as the device call up
+    to FC split-K grouping, identical top-1, and the oracle's tolerance."""
+    import torch
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    net = synth.alexnet()
+    w, b = params(net)
+    B = 64
+    x = synth.images(0, B, net["in_shape"])
+    n = pcnn.Net(net, w, b, B, "bf16")
+    dev, _, _ = n.infer(torch.from_numpy(x).cuda())
+    torch.cuda.synchronize()
+    xh = torch.from_numpy(x).pin_memory()
+    oh = torch.empty((B, 1000)).pin_memory()
+    hh = torch.empty((B,)).pin_memory()
+    n.infer_host(xh, oh, None, hh)
+    d = dev.cpu().numpy()
+    assert rel_err(oh.numpy(), d) <= 2e-3
+    assert (oh.numpy().argmax(1) == d.argmax(1)).all()
+    ref = orc.run_net(net, w, b, x[:2])
+    assert rel_err(oh.numpy()[:2], ref) <= TOL["bf16"]
+    assert np.isfinite(hh.numpy()).all() and (hh.numpy() >= 0).all()
