@@ -440,7 +440,8 @@ __device__ __forceinline__ void epi_store_rows(uint8_t *stage, const uint4 (&pc)
 // form), so the result is bitwise identical to conv -> store -> LRN.
 template <int ST>
 __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bool mok,
-                                             size_t orow, uint8_t *stage, int lane) {
+                                             bool valid, size_t orow, uint8_t *stage,
+                                             int lane) {
   const ConvGeom &g = a.g;
   constexpr int MAXC = 128;
   float f[MAXC];
@@ -462,7 +463,7 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
     // the value the stand-alone conv would have stored
     if constexpr (ST == ST_BF16) x = __bfloat162float(__float2bfloat16_rn(x));
     else if (g.out_mode == OUT_F32_TF32) x = tf32_rna_tc(x);
-    f[i] = i < C ? x : 0.f;
+    f[i] = (i < C && valid) ? x : 0.f;   // padded-layout halo rows are stored as zeros
   }
   float sq[MAXC + 4];
   sq[0] = sq[1] = sq[MAXC + 2] = sq[MAXC + 3] = 0.f;
@@ -977,7 +978,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       const size_t orow = (size_t)m * g.out_cs;
       if constexpr (LRN) {
         epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + tcol, mok,
-                         orow, stage, lane);
+                         valid, orow, stage, lane);
         continue;
       }
       if (a.tma_y) {
@@ -1347,7 +1348,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
     return cudaErrorInvalidValue;
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
-  if (g.pm && (p.splits != 1 || lrn || p.rect_w || g.stride != 1 || g.S != 2 * g.pad + 1 ||
+  if (g.pm && (p.splits != 1 || p.rect_w || g.stride != 1 || g.S != 2 * g.pad + 1 ||
                g.Cg % (args.slab_bytes / (st == ST_BF16 ? 2 : 4)) || p.a_stages < 2 ||
                p.b_stages < 2 || p.a_stages > TC_MAX_ASTAGES || p.b_stages > TC_MAX_BSTAGES))
     return cudaErrorInvalidValue;

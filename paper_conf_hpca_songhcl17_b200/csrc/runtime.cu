@@ -744,7 +744,7 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
 // Padded-layout plan: per (slab, filter row) window the SM loads
 // (128 + S - 1) A rows once plus S weight slabs and issues S x slab/32 UMMAs;
 // no split-K (a split would need the halo zeroing in the reduction).
-static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz) {
+static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n = false) {
   TcPlan best{};
   double best_t = 1e300;
   const int nmax = std::min(256, round_up(g.Nfg, 32));
@@ -762,7 +762,8 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz) {
       const int mtiles = (int)(((long long)g.M + rows - 1) / rows);
       const int slots = device_sms / cg;
       for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {
-        if (force_bn && atoi(force_bn) != bn) continue;
+        if (full_n && bn != round_up(g.Nfg, 32)) continue;     // one N tile (fused LRN)
+        if (force_bn && !full_n && atoi(force_bn) != bn) continue;
         if (ms == 2 && bn > 128) continue;          // two accumulators per TMEM buffer
         const int ntiles = (g.Nfg + bn - 1) / bn;
         const long long tiles = (long long)mtiles * ntiles * g.groups;
@@ -820,8 +821,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
   ConvGeom g = gs.g;
   g.M = g.pm ? B * g.hv * g.wv : B * g.Ho * g.Wo;
   if (gs.engine == 1) {
-    if (g.pm && lrn) return fail(PCNN_ERR_UNSUPPORTED, "LRN fusion in padded-layout mode");
-    TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st))
+    TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st), lrn != nullptr)
                     : plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st),
                               lrn != nullptr);
     // the budget caps concurrent units; a CTA pair needs at least 2 SMs
@@ -891,8 +891,13 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
 static bool fuse_conv_lrn(const pcnn_net *net, int i) {
   if (!net->fuse_lrn_pool || i + 1 >= (int)net->layers.size()) return false;
   const Layer &c = net->layers[i], &l = net->layers[i + 1];
-  return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 && c.pm_halo == 0 &&
-         c.perf_sh * c.perf_sw == 1 &&
+  // padded-layout convs fuse LRN only on request (PCNN_PM_LRN=1): the LRN
+  // epilogue (4 warps, one pixel's channel vector per thread) made AlexNet
+  // conv1 279 us against 79 us conv + 92 us register-LRN/pool kernel
+  const char *pe = getenv("PCNN_PM_LRN");
+  const bool pm_lrn = pe && pe[0] == '1';
+  return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 &&
+         (c.pm_halo == 0 || pm_lrn) && c.perf_sh * c.perf_sw == 1 &&
          c.exact.engine == 1 && c.variant == PCNN_VARIANT_EXACT && c.d.groups == 1 &&
          c.d.out_channels <= 128 && c.out_cs == c.d.out_channels;
 }
@@ -1366,6 +1371,8 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
       ly.pm_halo = pmh[i];
       if (pmh[i]) ly.out_halo = pmh[i];
       else if (is_pool(i) && i + 1 < n && kind(i + 1) == PCNN_CONV) ly.out_halo = pmh[i + 1];
+      else if (kind(i) == PCNN_LRN && i > 0 && pmh[i - 1] && i + 1 < n && is_pool(i + 1))
+        ly.out_halo = pmh[i - 1];   // keeps the conv's layout: conv + LRN may run fused
       else ly.out_halo = 0;
     }
   }

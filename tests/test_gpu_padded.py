@@ -146,3 +146,25 @@ def test_padded_mode_narrow_slabs(orc, prec, monkeypatch):
     r = gpu_run(net, w, b, x, prec)
     assert r["net"].query_layer(1, 2)["a_mode"] == 2
     assert rel_err(r["out"], ref) <= TOL[prec] / 2
+
+
+@pytest.mark.parametrize("prec", ["bf16", "tf32"])
+def test_padded_mode_conv_lrn_fusion(orc, prec, monkeypatch):
+    """AlexNet conv1 -> norm1 -> pool1 shape (space-to-depth conv in padded-
+    layout mode): LRN fused into the conv epilogue writes the halo layout the
+    pool reads; agrees with the unfused kernels and the oracle."""
+    net = dict(in_shape=(3, 67, 67), layers=[
+        conv_layer(96, 11, 3, 4, 0, 1, relu=True),
+        dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0),
+        dict(kind="maxpool", k=3, stride=2)])
+    w, b = params(net, seed=21)
+    x = small_inputs((3, 67, 67), 2, lo=-128, hi=128)
+    ref = orc.run_net(net, w, b, x).reshape(2, -1)
+    monkeypatch.setenv("PCNN_PM_LRN", "1")
+    fused = gpu_run(net, w, b, x, prec)
+    assert fused["net"].query_layer(0, 2)["a_mode"] == 2
+    monkeypatch.setenv("PCNN_NO_FUSE", "1")
+    plain = gpu_run(net, w, b, x, prec)["out"]
+    assert rel_err(fused["out"], ref) <= TOL[prec] / 4
+    assert rel_err(plain, ref) <= TOL[prec] / 4
+    assert rel_err(fused["out"], plain) <= (2e-3 if prec == "tf32" else 8e-3)
