@@ -455,10 +455,164 @@ static cudaError_t launch_gather3(const float *x, void *y, int st, int B, int H,
   return cudaGetLastError();
 }
 
+// Warp-cooperative bulk staging of input rows for the first-layer staging
+// kernels: rows [row0, row0 + nrows) of the C channels of image n (row lr =
+// a * C + c at buf + lr * pitch), one bulk TMA copy per row of its 16 B-aligned
+// superset, one row per lane.  sh[lr] = the row's start offset in floats, -1
+// for rows outside the image (read as zeros).  The bytes are announced after
+// the copies (the mbarrier tx-count may go negative within a phase; the phase
+// cannot complete before lane 0's arrive).  Rows whose superset would run
+// past the tensor are loaded with plain loads.
+__device__ __forceinline__ void bulk_rows(const float *__restrict__ x, uintptr_t xend,
+                                          long long n, int C, int H, int W, int row0,
+                                          int nrows, float *buf, int *sh, int pitch,
+                                          uint32_t bar) {
+  const int lane = threadIdx.x & 31;
+  uint32_t bytes = 0;
+  for (int lr = lane; lr < nrows * C; lr += 32) {
+    const int a = lr / C, c = lr - a * C, ih = row0 + a;
+    if (ih < 0 || ih >= H) {
+      sh[lr] = -1;
+      continue;
+    }
+    const uintptr_t src = (uintptr_t)(x + ((size_t)(n * C + c) * H + ih) * W);
+    const uintptr_t a0 = src & ~(uintptr_t)15;
+    const uint32_t nb = (uint32_t)(((src + (uintptr_t)W * 4 - a0) + 15) & ~(uintptr_t)15);
+    float *dst = buf + (size_t)lr * pitch;
+    if (a0 + nb > xend) {
+      for (int j = 0; j < W; ++j) dst[j] = __ldg((const float *)src + j);
+      sh[lr] = 0;
+      continue;
+    }
+    sh[lr] = (int)((src - a0) >> 2);
+    bytes += nb;
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+        ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(a0), "r"(nb), "r"(bar)
+        : "memory");
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
+  __syncwarp();
+  if (lane == 0)
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait_parity(uint32_t bar, uint32_t par) {
+  asm volatile(
+      "{\n.reg .pred P1;\nW_%=:\nmbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra W_%=;\n}\n" ::"r"(bar), "r"(par)
+      : "memory");
+}
+
+// First-layer im2col staging for 3-channel inputs, S x S taps, stride 1,
+// pad S/2 (VGG conv1_1): persistent CTAs over bands of R output rows; the
+// band's R + S - 1 input rows per channel arrive by bulk TMA copies (two
+// buffers); one thread per output pixel gathers its S*S*3 values (rows
+// re-aligned by their start offset, zeros outside the image) in (r, s, c)
+// order, zero-pads to Kp channels and writes the pixel with 16 B stores into
+// the interior of the halo-h output grid.
+template <int ST, int S>
+__global__ void __launch_bounds__(256)
+stage_im2c3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Kp, int halo,
+                   int R, int tf32_round) {
+  constexpr int C = 3, PAD = S / 2, NREAL = S * S * C;
+  constexpr int VN = Vec16<ST>::N;
+  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
+  extern __shared__ __align__(128) uint8_t ic_smem[];
+  const int pitch = ((W + 3) / 4 + 1) * 4;
+  const int rows = (R + S - 1) * C;
+  float *bufs = (float *)ic_smem;
+  uint64_t *bar = (uint64_t *)(ic_smem + (size_t)2 * rows * pitch * 4);
+  int *shift = (int *)(bar + 2);
+  const int bands = (H + R - 1) / R;
+  const long long tiles = (long long)B * bands;
+  const uintptr_t xend = (uintptr_t)(x + (size_t)B * C * H * W);
+  const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bar);
+  const int Hp = H + 2 * halo, Wp = W + 2 * halo;
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0));
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](long long t, int b) {
+    const long long n = t / bands;
+    const int p0 = (int)(t % bands) * R, nh = min(R, H - p0);
+    bulk_rows(x, xend, n, C, H, W, p0 - PAD, nh + S - 1, bufs + (size_t)b * rows * pitch,
+              shift + b * rows, pitch, bar0 + 8 * b);
+  };
+  long long t = blockIdx.x;
+  if (threadIdx.x < 32 && t < tiles) issue(t, 0);
+  uint32_t phase[2] = {0, 0};
+  for (int b = 0; t < tiles; t += gridDim.x, b ^= 1) {
+    if (threadIdx.x < 32 && t + gridDim.x < tiles) issue(t + gridDim.x, b ^ 1);
+    mbar_wait_parity(bar0 + 8 * b, phase[b]);
+    phase[b] ^= 1;
+    const long long n = t / bands;
+    const int p0 = (int)(t % bands) * R, nh = min(R, H - p0);
+    const float *buf = bufs + (size_t)b * rows * pitch;
+    const int *sh = shift + b * rows;
+    for (int pix = threadIdx.x; pix < nh * W; pix += blockDim.x) {
+      const int hr = pix / W, q = pix - hr * W;
+      float v[NREAL];                               // channel (r * S + s) * C + c
+#pragma unroll
+      for (int r = 0; r < S; ++r)
+#pragma unroll
+        for (int c = 0; c < C; ++c) {
+          const int lr = (hr + r) * C + c, o = sh[lr];
+          const float *rp = buf + (size_t)lr * pitch + o;
+#pragma unroll
+          for (int s2 = 0; s2 < S; ++s2) {
+            const int col = q + s2 - PAD;
+            v[(r * S + s2) * C + c] = (o >= 0 && col >= 0 && col < W) ? rp[col] : 0.f;
+          }
+        }
+      char *py = (char *)y + ((((size_t)n * Hp + p0 + hr + halo) * Wp + q + halo) * (size_t)Kp) * ESZ;
+      constexpr int NCH = (NREAL + VN - 1) / VN;
+#pragma unroll
+      for (int ch = 0; ch < NCH; ++ch) {
+        Vec16<ST> o;
+#pragma unroll
+        for (int j = 0; j < VN; ++j) o.v[j] = ch * VN + j < NREAL ? v[ch * VN + j] : 0.f;
+        o.store(py + ch * 16, tf32_round);
+      }
+      for (int ch = NCH; ch < Kp / VN; ++ch) *(uint4 *)(py + ch * 16) = make_uint4(0, 0, 0, 0);
+    }
+    __syncthreads();
+  }
+}
+
 cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, int H, int W,
                                 int S, int stride, int pad, int Ho, int Wo, int Kp,
                                 int halo, int tf32_round, cudaStream_t s) {
   if (C != 3 || (S != 3 && S != 5)) return cudaErrorInvalidValue;
+  if (!getenv("PCNN_OLD_STAGE") && S == 3 && stride == 1 && pad == 1 && Ho == H && Wo == W &&
+      Kp >= 27 && Kp % (st == ST_BF16 ? 8 : 4) == 0) {
+    const int R = 2;
+    const int pitch = ((W + 3) / 4 + 1) * 4;
+    const size_t smem = (size_t)2 * (R + 2) * 3 * pitch * 4 + 16 + 2 * (R + 2) * 3 * 4;
+    if (smem <= 200 * 1024) {
+      const long long tiles = (long long)B * ((H + R - 1) / R);
+      int dev = 0, sms = 148, occ = 1;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+#define PCNN_IC3(STT)                                                                          \
+  do {                                                                                         \
+    if (smem > 48 * 1024)                                                                      \
+      cudaFuncSetAttribute(stage_im2c3_kernel<STT, 3>,                                         \
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stage_im2c3_kernel<STT, 3>, 256, smem); \
+    const unsigned grid = (unsigned)std::min<long long>(tiles, (long long)sms * std::max(occ, 1)); \
+    stage_im2c3_kernel<STT, 3><<<grid, 256, smem, s>>>(x, y, B, H, W, Kp, halo, R, tf32_round); \
+  } while (0)
+      if (st == ST_BF16) PCNN_IC3(ST_BF16);
+      else PCNN_IC3(ST_F32);
+#undef PCNN_IC3
+      return cudaGetLastError();
+    }
+  }
   if (!getenv("PCNN_OLD_STAGE") && gather3_ok(st, W, Kp, S, stride))
     return launch_gather3(x, y, st, B, H, W, Ho, Wo, Kp, S, stride, pad, halo, tf32_round, s);
   const size_t smem = (size_t)S * C * ((Wo - 1) * stride + S) * sizeof(float);
@@ -507,46 +661,11 @@ stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  // warp 0: start the copies of band t into buffer b, one row per lane; the
-  // bytes are announced after the copies (the mbarrier's tx-count may go
-  // negative within a phase, and the phase cannot complete before lane 0's
-  // arrive)
   auto issue = [&](long long t, int b) {
-    const int lane = threadIdx.x & 31;
     const long long n = t / bands;
     const int h0 = (int)(t % bands) * R, nh = min(R, Hs - h0);
-    float *buf = bufs + (size_t)b * rows * pitch;
-    int *sh = shift + b * rows;
-    const uint32_t bb = bar0 + 8 * b;
-    uint32_t bytes = 0;
-    for (int lr = lane; lr < nh * BLK * C; lr += 32) {
-      const int a = lr / C, c = lr - a * C, ih = h0 * BLK + a;
-      if (ih >= H) {
-        sh[lr] = -1;
-        continue;
-      }
-      const uintptr_t src = (uintptr_t)(x + ((size_t)(n * C + c) * H + ih) * W);
-      const uintptr_t a0 = src & ~(uintptr_t)15;
-      const uint32_t nb = (uint32_t)(((src + (uintptr_t)W * 4 - a0) + 15) & ~(uintptr_t)15);
-      float *dst = buf + (size_t)lr * pitch;
-      if (a0 + nb > xend) {              // superset past the tensor: plain loads
-        for (int j = 0; j < W; ++j) dst[j] = __ldg((const float *)src + j);
-        sh[lr] = 0;
-        continue;
-      }
-      sh[lr] = (int)((src - a0) >> 2);
-      bytes += nb;
-      asm volatile(
-          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-          ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(a0), "r"(nb), "r"(bb)
-          : "memory");
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
-    __syncwarp();                        // every lane's smem writes precede the arrive
-    if (lane == 0)
-      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bb), "r"(bytes)
-                   : "memory");
+    bulk_rows(x, xend, n, C, H, W, h0 * BLK, nh * BLK, bufs + (size_t)b * rows * pitch,
+              shift + b * rows, pitch, bar0 + 8 * b);
   };
   long long t = blockIdx.x;
   if (threadIdx.x < 32 && t < tiles) issue(t, 0);
@@ -1441,6 +1560,77 @@ long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int
   return (long long)B * Ho * ((Wo + Q - 1) / Q);
 }
 
+// Plain pooling (no LRN, no group padding) straight from global memory: one
+// thread per (output pixel, 16 B channel chunk), chunk fastest, so each warp
+// reads whole runs of input pixels; K = 2 / 3 windows are unrolled (VGG 2x2
+// s2, AlexNet 3x3 s2), overlapping windows re-hit L1.  Writes the output
+// halo zeros.  Same max / mean arithmetic as lrn_pool_kernel.
+template <int ST, int K>
+__global__ void __launch_bounds__(256)
+pool_direct_kernel(const uint4 *__restrict__ x, uint4 *__restrict__ y, int B, int H, int W,
+                   int chunks, int kk, int s, int is_max, int Ho, int Wo, int hi, int ho,
+                   int tf32_round, Budget bud) {
+  constexpr int VN = Vec16<ST>::N;
+  const int k = K > 0 ? K : kk;
+  const int Hp = H + 2 * hi, Wp = W + 2 * hi, Hop = Ho + 2 * ho, Wop = Wo + 2 * ho;
+  const long long total = (long long)B * Hop * Wop * chunks;
+  const float inv = 1.f / (float)(k * k);
+  if (threadIdx.x == 0) census_mark(bud);
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int ch = (int)(i % chunks);
+    const long long pix = i / chunks;
+    const int q = (int)(pix % Wop) - ho;
+    const long long t = pix / Wop;
+    const int p = (int)(t % Hop) - ho;
+    const long long n = t / Hop;
+    if (p < 0 || p >= Ho || q < 0 || q >= Wo) {
+      y[i] = make_uint4(0, 0, 0, 0);
+      continue;
+    }
+    const int r0 = p * s, c0 = q * s;
+    const int re = min(r0 + k, H), ce = min(c0 + k, W);
+    const uint4 *base = x + (((size_t)n * Hp + r0 + hi) * Wp + c0 + hi) * chunks + ch;
+    if (ST == ST_BF16 && is_max) {
+      __nv_bfloat162 m[4];
+      const __nv_bfloat162 ninf = __float2bfloat162_rn(-INFINITY);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) m[j] = ninf;
+      auto take = [&](const uint4 *ptr) {
+        const uint4 raw = __ldg(ptr);
+        const __nv_bfloat162 *h2 = (const __nv_bfloat162 *)&raw;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], h2[j]);
+      };
+      if (K > 0 && re - r0 == K && ce - c0 == K) {
+#pragma unroll
+        for (int dr = 0; dr < (K > 0 ? K : 1); ++dr)
+#pragma unroll
+          for (int dc = 0; dc < (K > 0 ? K : 1); ++dc) take(base + ((size_t)dr * Wp + dc) * chunks);
+      } else {
+        for (int r = r0; r < re; ++r)
+          for (int c = c0; c < ce; ++c) take(base + ((size_t)(r - r0) * Wp + (c - c0)) * chunks);
+      }
+      y[i] = *(const uint4 *)m;
+      continue;
+    }
+    Vec16<ST> acc, cur;
+#pragma unroll
+    for (int j = 0; j < VN; ++j) acc.v[j] = is_max ? -INFINITY : 0.f;
+    for (int r = r0; r < re; ++r)
+      for (int c = c0; c < ce; ++c) {
+        cur.from_raw(__ldg(base + ((size_t)(r - r0) * Wp + (c - c0)) * chunks));
+#pragma unroll
+        for (int j = 0; j < VN; ++j)
+          acc.v[j] = is_max ? fmaxf(acc.v[j], cur.v[j]) : acc.v[j] + cur.v[j];
+      }
+    if (!is_max)
+#pragma unroll
+      for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
+    acc.store(y + i, is_max ? 0 : tf32_round);
+  }
+}
+
 cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int B, int H, int W,
                             int C, int lrn_size, float alpha, float beta, float kk, int k,
                             int s, int is_max, int Ho, int Wo, int out_groups, int out_cg_pad,
@@ -1452,6 +1642,22 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   const int ocp = out_groups > 0 ? out_cg_pad : 0;
   if (out_groups > 0 && (C % out_groups || ocg % vn || ocp % vn || ocp < ocg))
     return cudaErrorInvalidValue;
+  if (lrn_size == 0 && out_groups == 0 && !b.gated && !getenv("PCNN_OLD_POOL")) {
+    const int chunks = C / vn;
+    const long long total = (long long)B * (Ho + 2 * out_halo) * (Wo + 2 * out_halo) * chunks;
+    const int g = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
+#define PCNN_PD(STT, KK)                                                                       \
+  pool_direct_kernel<STT, KK><<<g, 256, 0, stream>>>((const uint4 *)x, (uint4 *)y, B, H, W,    \
+                                                     chunks, k, s, is_max, Ho, Wo, in_halo,    \
+                                                     out_halo, tf32_round, b)
+    if (st == ST_BF16) {
+      if (k == 2) PCNN_PD(ST_BF16, 2); else if (k == 3) PCNN_PD(ST_BF16, 3); else PCNN_PD(ST_BF16, 0);
+    } else {
+      if (k == 2) PCNN_PD(ST_F32, 2); else if (k == 3) PCNN_PD(ST_F32, 3); else PCNN_PD(ST_F32, 0);
+    }
+#undef PCNN_PD
+    return cudaGetLastError();
+  }
   LrnPoolArgs a;
   a.x = x;
   a.y = y;
