@@ -182,6 +182,26 @@ __device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap *map
   }
 }
 
+// tiled 3-D TMA load (row-perforated padded mode: {channels, wv, grid rows}
+// box, grid rows traversed with the perforation stride)
+template <int CG>
+__device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap *map, uint32_t bar,
+                                            int c0, int c1, int c2) {
+  if constexpr (CG == 1) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
+        "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
+        : "memory");
+  } else {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
+        "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c0), "r"(c1), "r"(c2)
+        : "memory");
+  }
+}
+
 // 2-SM form: lands in this CTA's smem, bytes counted on the leader's barrier.
 __device__ __forceinline__ void tma_im2col_2sm(uint32_t dst, const CUtensorMap *map,
                                                uint32_t bar, int c, int w, int h, int n,
@@ -776,7 +796,9 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     if (lane == 0) {
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_w) : "memory");
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
-      const uint32_t pm_a_bytes = (uint32_t)(TC_BM + 2 * g.pad) * slab_bytes;
+      // pm = 2: nseg segments of wv + 2 pad columns (grid columns -pad ..)
+      const uint32_t pm_a_bytes = g.pm == 2 ? (uint32_t)(g.nseg * (g.wv + 2 * g.pad)) * slab_bytes
+                                            : (uint32_t)(TC_BM + 2 * g.pad) * slab_bytes;
       uint32_t as = 0, aph = 0, bs = 0, bph = 0;
       WaitClock wc{TC_PROF(a) != 0};
       unsigned long long nkb = 0;
@@ -791,7 +813,15 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           wc.wait(sbase + SM_AEMPTY + 8 * as, aph ^ 1);
           const uint32_t fa = sbase + SM_AFULL + 8 * as;
           if (rank == 0) mbar_arrive_expect_tx(fa, (a.skip & 1) ? 0 : CG * a.msub * pm_a_bytes);
-          if (!(a.skip & 1)) {
+          if (!(a.skip & 1) && g.pm == 2) {
+            // kept rows tb*nseg .. of image n, filter row r: a {slab, wv + 2 pad,
+            // nseg} box starting pad columns left of the row, rows psh apart
+            const uint32_t dA = sA + as * (uint32_t)a.pm_a_stage;
+            const int T = mt * CG + (int)rank, n = T / g.tpi, tb = T - n * g.tpi;
+            const int cc = grp * g.Cg + cb * pm_se;
+            const int grow = n * g.hv + g.vh + g.psh * tb * g.nseg + r - g.pad;
+            tma_load_3d<CG>(dA, &tmap_x, fa, cc, -g.pad, grow);
+          } else if (!(a.skip & 1)) {
             const uint32_t dA = sA + as * (uint32_t)a.pm_a_stage;
             const int cc = grp * g.Cg + cb * pm_se, row = i0 + (r - g.pad) * g.wv - g.pad;
             for (int sb = 0; sb < a.msub; ++sb) {
@@ -970,7 +1000,17 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         mok = m < g.M;
       }
       bool valid = true;      // padded mode: halo rows are stored as zeros
-      if (g.pm) {
+      if (g.pm == 2) {
+        // row-perforated: MMA row = (kept row k of the tile, segment position
+        // v; segments are wv + 2 pad long); only interior columns of existing
+        // kept rows are stored (compact)
+        const int T = mt * CG + (int)rank, n = T / g.tpi, tb = T - n * g.tpi;
+        const int k = (int)a.fd_w.div((uint32_t)row), v = row - k * (g.wv + 2 * g.pad);
+        const int pk = tb * g.nseg + k;
+        mok = k < g.nseg && pk < g.hk && v >= g.vh && v < g.vh + g.Wo && T * TC_BM < g.M;
+        m = (n * g.hk + pk) * g.Wo + (v - g.vh);
+        valid = mok;
+      } else if (g.pm) {
         const int ni = (int)a.fd_hw.div((uint32_t)m), rem = m - ni * g.hv * g.wv;
         const int pv = (int)a.fd_w.div((uint32_t)rem), qv = rem - pv * g.wv;
         valid = pv >= g.vh && pv < g.vh + g.Ho && qv >= g.vh && qv < g.vh + g.Wo;
@@ -1320,9 +1360,9 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.fd_nt.init(p.ntiles);
   args.fd_grp.init(g.groups);
   args.fd_hw.init(g.pm ? g.hv * g.wv : 1);
-  args.fd_w.init(g.pm ? g.wv : 1);
+  args.fd_w.init(g.pm == 2 ? g.wv + 2 * g.pad : g.pm ? g.wv : 1);
   args.y = y;
-  args.tma_y = (tmap_y != nullptr && !lrn && p.splits == 1 && p.rect_w == 0) ? 1 : 0;
+  args.tma_y = (tmap_y != nullptr && !lrn && p.splits == 1 && p.rect_w == 0 && g.pm != 2) ? 1 : 0;
   args.ws = ws;
   args.bias = bias;
   args.ktab = ktab;
@@ -1344,7 +1384,8 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.b_stages = p.b_stages;
   args.msub = p.msub > 1 ? p.msub : 1;
   args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, g.S, args.msub) : 0;
-  if (args.msub > 2 || (args.msub == 2 && (!g.pm || p.bn > TC_BN_MAX / 2)))
+  if (args.msub > 2 || (args.msub == 2 && (!g.pm || g.pm == 2 || p.bn > TC_BN_MAX / 2)) ||
+      (g.pm == 2 && (g.nseg < 1 || g.nseg * (g.wv + 2 * g.pad) > TC_BM || g.tpi < 1)))
     return cudaErrorInvalidValue;
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;

@@ -61,6 +61,12 @@ struct ConvGeom {
   // kept counts), i.e. input windows stride*psh / stride*psw apart; ih = zero
   // border of the stored input ([B][H + 2ih][W + 2ih][Cs]); 0 = plain
   int psh, psw, ih;
+  // row-perforated padded mode (pm = 2): the kept output rows p' (p = psh p')
+  // of each image form segments of wv virtual rows; a CTA tile is nseg
+  // consecutive kept rows of one image (nseg * wv <= 128 MMA rows), tpi tiles
+  // per image, hk kept rows per image; M = B * tpi * 128.  The output is the
+  // compact kept grid [B][hk][Wo][out_cs].
+  int nseg, tpi, hk;
 };
 
 // ---------------------------------------------------------------- launchers

@@ -530,6 +530,27 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, co
   const int esz = esz_of(gs.st);
   const int slab = tc_slab_bytes(gs.st, g.Cg);
   CUtensorMap m;
+  if (g.pm == 2) {
+    // row-perforated padded layout: {channels, wv, grid rows} with the grid
+    // rows traversed psh apart; a box is nseg kept rows of one filter row
+    auto enct = get_encode_tiled();
+    if (!enct) return nullptr;
+    const cuuint64_t d3[3] = {(cuuint64_t)g.Cs, (cuuint64_t)g.wv, (cuuint64_t)batch * g.hv};
+    const cuuint64_t s3[2] = {(cuuint64_t)g.Cs * esz, (cuuint64_t)g.wv * g.Cs * esz};
+    const cuuint32_t box[3] = {(cuuint32_t)(slab / esz), (cuuint32_t)(g.wv + 2 * g.pad),
+                               (cuuint32_t)(g.nseg * g.psh)};
+    const cuuint32_t estr[3] = {1, 1, (cuuint32_t)g.psh};
+    const CUtensorMapSwizzle sw = slab == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                  : slab == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                               : CU_TENSOR_MAP_SWIZZLE_32B;
+    CUresult r = enct(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                           : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                      3, const_cast<void *>(x), d3, s3, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                      sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return nullptr;
+    if (gs.xmaps.size() > 64) gs.xmaps.clear();
+    return &(gs.xmaps[key] = m);
+  }
   if (g.pm) {
     // padded layout: the input is a plain [B*hv*wv][Cs] matrix; a box is the
     // (128 + S - 1)-row window of one filter row (rows outside the tensor --
@@ -756,6 +777,7 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
   const char *force_ms = getenv("PCNN_PM_MSUB");           // 1 | 2 (experiments)
   for (int ms = 1; ms <= 2; ++ms) {
     if (force_ms && atoi(force_ms) != ms) continue;
+    if (g.pm == 2 && ms > 1) continue;          // row-perforated tiles: one sub-tile
     for (int cg = 1; cg <= 2; ++cg) {
       if (force_cg && atoi(force_cg) != cg) continue;
       const long long rows = 128LL * cg * ms;
@@ -819,7 +841,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
                              void *y, int slot, cudaStream_t s, pcnn_layer_info *info,
                              size_t *ws_need = nullptr, const float *lrn = nullptr) {
   ConvGeom g = gs.g;
-  g.M = g.pm ? B * g.hv * g.wv : B * g.Ho * g.Wo;
+  g.M = g.pm == 2 ? B * g.tpi * 128 : g.pm ? B * g.hv * g.wv : B * g.Ho * g.Wo;
   if (gs.engine == 1) {
     TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st), lrn != nullptr)
                     : plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st),
@@ -855,8 +877,8 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       const char *e = getenv("PCNN_NO_TMA_STORE");
       return e && e[0] == '1';
     }();
-    const CUtensorMap *ym =
-        (p.splits == 1 && !lrn && !p.rect_w && !no_tma_store) ? stage_ymap(gs, y, g.M) : nullptr;
+    const CUtensorMap *ym = (p.splits == 1 && !lrn && !p.rect_w && !no_tma_store && g.pm != 2)
+                                ? stage_ymap(gs, y, g.M) : nullptr;
     CUDA_TRY(counted(launch_conv_tc(g, gs.st, xm, tm, gs.d_bias, y, gs.d_ktab, p, net->d_ws,
                                     b, s, lrn, ym)));
   } else {
@@ -1549,9 +1571,15 @@ pcnn_status pcnn_set_perforation(pcnn_net *net, int layer, int sh, int sw) {
     return fail(PCNN_ERR_UNSUPPORTED, "input halo narrower than the conv padding");
   CUDA_TRY(cudaSetDevice(net->device));
   const int mode = ly.exact.g.out_mode;
+  // rows only, on a padded-layout layer whose grid rows fit one MMA tile:
+  // the kept rows run in padded-layout mode (pm = 2, row-strided windows)
+  const char *e2 = getenv("PCNN_PERF_IM2COL");           // A/B: force the im2col kept grid
+  const bool pm2 = sw == 1 && ly.exact.g.pm == 1 && ly.pm_halo > 0 &&
+                   ly.exact.g.wv + 2 * ly.exact.g.pad <= 128 && !(e2 && e2[0] == '1');
   pcnn_status s = build_stage(ly.pf, ly, net->desc.precision, ly.d.out_channels, ly.d.groups,
                               ly.d.kernel, ly.d.stride, ly.d.pad, ly.d.relu, ly.in_c, ly.in_h,
-                              ly.in_w, ly.in_cs, false, ly.host_w.data(), nullptr, mode);
+                              ly.in_w, ly.in_cs, false, ly.host_w.data(), nullptr, mode,
+                              pm2 ? ly.pm_halo : 0);
   if (s != PCNN_OK) return s;
   CUDA_TRY(cudaMemcpy(ly.pf.d_bias, ly.exact.d_bias,
                       sizeof(float) * ((size_t)round_up(ly.d.out_channels, 256) + 256),
@@ -1559,10 +1587,17 @@ pcnn_status pcnn_set_perforation(pcnn_net *net, int layer, int sh, int sw) {
   ConvGeom &g = ly.pf.g;
   g.psh = sh;
   g.psw = sw;
-  g.ih = ly.in_halo;
-  g.Ho = (ly.out_h + sh - 1) / sh;        // kept rows / columns
-  g.Wo = (ly.out_w + sw - 1) / sw;
   g.out_cs = ly.out_cs;
+  if (pm2) {
+    g.pm = 2;
+    g.hk = (ly.out_h + sh - 1) / sh;
+    g.nseg = 128 / (g.wv + 2 * g.pad);   // segments: grid columns -pad .. wv + pad
+    g.tpi = (g.hk + g.nseg - 1) / g.nseg;
+  } else {
+    g.ih = ly.in_halo;
+    g.Ho = (ly.out_h + sh - 1) / sh;      // kept rows / columns
+    g.Wo = (ly.out_w + sw - 1) / sw;
+  }
   ly.perf_sh = sh;
   ly.perf_sw = sw;
   net->version++;

@@ -103,3 +103,34 @@ def test_perforation_rejections():
     n.set_variant(3, "exact")
     n.set_perforation(3, 2, 2)
     n.close()
+
+
+@pytest.mark.parametrize("prec", ["bf16", "tf32"])
+@pytest.mark.parametrize("sh", [2, 3])
+def test_row_perforation_padded_layout(orc, prec, sh, monkeypatch):
+    """Row perforation (s_w = 1) of padded-layout layers runs the kept rows in
+    padded-layout mode (row-strided 3-D TMA windows, segments of W + 2h + 2p
+    rows): oracle parity, agreement with the im2col kept grid, and the
+    AlexNet conv2 shape (5x5, groups 2) included."""
+    net = vgg_like()
+    w, b = params(net, seed=31)
+    x = small_inputs((3, 36, 36), 3, lo=-128, hi=128)
+    perf = {1: (sh, 1), 4: (sh, 1)}
+    ref = orc.run_net(net, w, b, x, perforation=perf).reshape(3, -1)
+    r = gpu_run(net, w, b, x, prec, perforation=perf)
+    assert r["net"].query_layer(1, 3)["a_mode"] == 2
+    assert rel_err(r["out"], ref) <= TOL[prec] / 2
+    monkeypatch.setenv("PCNN_PERF_IM2COL", "1")
+    r2 = gpu_run(net, w, b, x, prec, perforation=perf)
+    assert r2["net"].query_layer(1, 3)["a_mode"] == 0
+    assert rel_err(r["out"], r2["out"]) <= TOL[prec] / 4
+    monkeypatch.delenv("PCNN_PERF_IM2COL")
+    anet = dict(in_shape=(96, 27, 27), layers=[
+        dict(kind="maxpool", k=1, stride=1), conv_layer(256, 5, 96, 1, 2, 2),
+        dict(kind="maxpool", k=3, stride=2)])
+    aw, ab = params(anet, seed=9)
+    ax = small_inputs((96, 27, 27), 2, lo=-2, hi=2)
+    aref = orc.run_net(anet, aw, ab, ax, perforation={1: (sh, 1)}).reshape(2, -1)
+    ar = gpu_run(anet, aw, ab, ax, prec, perforation={1: (sh, 1)})
+    assert ar["net"].query_layer(1, 2)["a_mode"] == 2
+    assert rel_err(ar["out"], aref) <= TOL[prec] / 2

@@ -30,8 +30,10 @@ w, b = synth.net_params(net)
 names = [L.get("name", str(i)) for i, L in enumerate(net["layers"])]
 gemm = [i for i, L in enumerate(net["layers"]) if L["kind"] in ("conv", "fc")]
 nsms = torch.cuda.get_device_properties(0).multi_processor_count
-PERF_LADDER = [{}, {3: (1, 2)}, {3: (2, 2)}, {3: (2, 2), 6: (1, 2), 7: (1, 2), 8: (1, 2)},
-               {3: (2, 2), 6: (2, 2), 7: (2, 2), 8: (2, 2)}]
+PERF_LADDER = [{}, {3: (2, 1)}, {3: (2, 1), 8: (2, 1)}, {3: (2, 1), 8: (2, 1), 7: (2, 1)},
+               {3: (2, 1), 8: (2, 1), 7: (2, 1), 6: (2, 1)},
+               {3: (3, 1), 8: (3, 1), 7: (3, 1), 6: (3, 1)},
+               {3: (2, 2), 8: (2, 2), 7: (2, 2), 6: (2, 2)}]
 LADDER = [{}, {3: 64}, {3: 64, 8: 64}, {3: 64, 8: 64, 7: 96}, {3: 64, 8: 64, 7: 96, 6: 192},
           {3: 32, 8: 32, 7: 48, 6: 96}, {3: 16, 8: 16, 7: 32, 6: 48}]
 

@@ -15,6 +15,9 @@ names = [L.get("name", str(i)) for i, L in enumerate(net["layers"])]
 for label, setup in [("exact", {}), ("rank conv2=64", {"rank": {3: 64}}),
                      ("rank conv2=32 conv3=96", {"rank": {3: 32, 6: 96}}),
                      ("perf conv2 2x2", {"perf": {3: (2, 2)}}),
+                     ("perf conv2 2x1", {"perf": {3: (2, 1)}}),
+                     ("perf conv2-5 2x1", {"perf": {3: (2, 1), 6: (2, 1), 7: (2, 1), 8: (2, 1)}}),
+                     ("perf conv2-5 3x1", {"perf": {3: (3, 1), 6: (3, 1), 7: (3, 1), 8: (3, 1)}}),
                      ("perf conv3 2x2", {"perf": {6: (2, 2)}})]:
     n = pcnn.Net(net, w, b, B, "bf16")
     for i, r in setup.get("rank", {}).items():
