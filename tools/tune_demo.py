@@ -1,0 +1,47 @@
+"""Run-time management demo: entropy-guided greedy tuning of
+AlexNet (BF16, one batch of seeded images) over per-layer rank-r and
+perforation ladders, then calibration along the tuning path.  Prints JSON:
+the path (state, ms per pass, mean CNN_entropy, TE), each table's eq. 11
+optSM per layer, and calibration decisions for a few observed entropies.
+
+    python tools/tune_demo.py [B] [entropy_margin_nats] > profiles/r01_tuning_path.json
+"""
+import json
+import os
+import sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+import synth  # noqa: E402
+from paper_conf_hpca_songhcl17_b200 import pcnn, tuning  # noqa: E402
+
+B = int(sys.argv[1]) if len(sys.argv) > 1 else 64
+margin = float(sys.argv[2]) if len(sys.argv) > 2 else 0.5
+net = synth.alexnet()
+w, b = synth.net_params(net)
+names = [L.get("name", str(i)) for i, L in enumerate(net["layers"])]
+x = torch.from_numpy(synth.images(0, B, net["in_shape"])).cuda()
+n = pcnn.Net(net, w, b, B, "bf16")
+ladders = {3: [("exact",), ("perf", 2, 1), ("rank", 64), ("rank", 32)],
+           6: [("exact",), ("rank", 192), ("rank", 96), ("perf", 2, 1)],
+           7: [("exact",), ("rank", 96), ("rank", 48)],
+           8: [("exact",), ("rank", 64), ("perf", 2, 1)]}
+measure = tuning.gpu_measure(n, ladders, x, reps=10)
+t0, h0 = measure({l: 0 for l in ladders})
+threshold = h0 + margin
+path = tuning.greedy_tune(ladders, measure, threshold)
+out = {"net": "alexnet", "batch": B, "precision": "bf16", "threshold_nats": threshold,
+       "ladders": {names[l]: [list(v) for v in r] for l, r in ladders.items()}, "path": []}
+for step in path:
+    tuning.apply_state(n, ladders, step["state"])
+    plans = [n.plan_budget(i, B) for i in range(n.n_layers)]
+    out["path"].append({
+        "layer": names[step["layer"]] if step["layer"] is not None else None,
+        "state": {names[l]: list(ladders[l][r]) for l, r in step["state"].items()},
+        "ms": round(step["time"], 5), "entropy": round(step["entropy"], 5),
+        "te": None if step["te"] is None else (str(step["te"]) if step["te"] == float("inf")
+                                               else round(step["te"], 5)),
+        "opt_sm": {names[i]: p["opt_sm"] for i, p in enumerate(plans) if p["grid_size"] > 0}})
+last = len(path) - 1
+out["calibration"] = {str(h): tuning.calibrate(path, last, h, threshold)
+                      for h in (path[last]["entropy"], threshold, threshold + 0.5, 1e9)}
+print(json.dumps(out, indent=1))
