@@ -106,3 +106,23 @@ def gpu_measure(net, ladders, images, reps=10):
         torch.cuda.synchronize()
         return e0.elapsed_time(e1) / reps, float(ent.mean().item())
     return measure
+
+
+# ---------------------------------------------------------------- batch selection (NEXT-4)
+def background_batch(util_of_layer, layers, max_batch):
+    """P:259 (background task): the optimal batch is the smallest one at which
+    every GEMM layer -- in practice the last, least-utilised one (Table V) --
+    reaches Util = 1 (eq. 6); beyond it throughput cannot grow.  util_of_layer
+    (layer, batch) -> eq. 6 Util.  Returns max_batch when no batch reaches 1."""
+    for bsz in range(1, max_batch + 1):
+        if all(util_of_layer(l, bsz) >= 1.0 - 1e-9 for l in layers):
+            return bsz
+    return max_batch
+
+
+def rescale_batch(t_user, t_model, batch):
+    """eq. 13: new batch size = T_user / T x batch (floored, >= 1),
+    applied when the modelled time T exceeds the user's requirement."""
+    if t_model <= t_user:
+        return batch
+    return max(1, int(math.floor(t_user / t_model * batch)))

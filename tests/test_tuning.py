@@ -45,3 +45,17 @@ def test_calibration_backtracks():
     assert tuning.calibrate(path, 2, 1.6, 1.5) == 1
     assert tuning.calibrate(path, 2, 1.45, 1.5) == 2          # within threshold: stay
     assert tuning.calibrate(path, 2, 3.0, 1.5) == 0           # back to exact
+
+
+def test_background_batch_rule():
+    """the smallest batch at which every layer's Util (eq. 6) is 1.
+    Hand table: layer 0 saturates at 3, layer 1 (the 'last layer') at 5."""
+    util = {0: lambda b: min(1.0, b / 3.0), 1: lambda b: min(1.0, b / 5.0)}
+    assert tuning.background_batch(lambda l, b: util[l](b), [0, 1], 64) == 5
+    assert tuning.background_batch(lambda l, b: 0.5, [0], 8) == 8
+
+
+def test_eq13_rescale():
+    assert tuning.rescale_batch(10.0, 40.0, 64) == 16      # T_user / T = 1/4
+    assert tuning.rescale_batch(10.0, 5.0, 64) == 64       # already fast enough
+    assert tuning.rescale_batch(1.0, 1000.0, 64) == 1

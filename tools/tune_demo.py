@@ -44,4 +44,15 @@ for step in path:
 last = len(path) - 1
 out["calibration"] = {str(h): tuning.calibrate(path, last, h, threshold)
                       for h in (path[last]["entropy"], threshold, threshold + 0.5, 1e9)}
+# NEXT-4: background-task batch (every conv layer at Util = 1, eq. 6) on this
+# net's own tile plans, and eq. 13's rescaled batch for a 0.2 ms requirement
+nb = pcnn.Net(net, w, b, 256, "bf16")
+convs = [i for i, L in enumerate(net["layers"]) if L["kind"] == "conv"]
+out["background_batch"] = tuning.background_batch(
+    lambda l, bsz: nb.query_layer(l, bsz)["util"], convs, 256)
+out["util_at_background_batch"] = {names[l]: round(nb.query_layer(l, out["background_batch"])["util"], 4)
+                                   for l in convs}
+t_model = sum(nb.plan_budget(i, B)["t_model_us"] for i in range(nb.n_layers)) / 1000
+out["eq13"] = {"t_user_ms": 0.2, "t_model_ms": round(t_model, 5), "batch": B,
+               "new_batch": tuning.rescale_batch(0.2, t_model, B)}
 print(json.dumps(out, indent=1))
