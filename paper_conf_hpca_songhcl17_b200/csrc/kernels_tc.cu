@@ -815,12 +815,17 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           if (rank == 0) mbar_arrive_expect_tx(fa, (a.skip & 1) ? 0 : CG * a.msub * pm_a_bytes);
           if (!(a.skip & 1) && g.pm == 2) {
             // kept rows tb*nseg .. of image n, filter row r: a {slab, wv + 2 pad,
-            // nseg} box starting pad columns left of the row, rows psh apart
+            // nseg} box starting pad columns left of the row, rows psh apart;
+            // one box per M sub-tile
             const uint32_t dA = sA + as * (uint32_t)a.pm_a_stage;
-            const int T = mt * CG + (int)rank, n = T / g.tpi, tb = T - n * g.tpi;
             const int cc = grp * g.Cg + cb * pm_se;
-            const int grow = n * g.hv + g.vh + g.psh * tb * g.nseg + r - g.pad;
-            tma_load_3d<CG>(dA, &tmap_x, fa, cc, -g.pad, grow);
+            for (int sb = 0; sb < a.msub; ++sb) {
+              const int T = (mt * CG + (int)rank) * a.msub + sb, n = T / g.tpi,
+                        tb = T - n * g.tpi;
+              const int grow = n * g.hv + g.vh + g.psh * tb * g.nseg + r - g.pad;
+              tma_load_3d<CG>(dA + (uint32_t)(sb * pm_sub_rows(g.S) * slab_bytes), &tmap_x, fa,
+                              cc, -g.pad, grow);
+            }
           } else if (!(a.skip & 1)) {
             const uint32_t dA = sA + as * (uint32_t)a.pm_a_stage;
             const int cc = grp * g.Cg + cb * pm_se, row = i0 + (r - g.pad) * g.wv - g.pad;
@@ -1001,15 +1006,16 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       }
       bool valid = true;      // padded mode: halo rows are stored as zeros
       if (g.pm == 2) {
-        // row-perforated: MMA row = (kept row k of the tile, segment position
-        // v; segments are wv + 2 pad long); only interior columns of existing
-        // kept rows are stored (compact)
-        const int T = mt * CG + (int)rank, n = T / g.tpi, tb = T - n * g.tpi;
+        // row-perforated: MMA row = (kept row k of the tile, grid column v;
+        // segments are wv + 2 pad long).  m = the kept row's own position on
+        // the layer's output grid; the store below copies it to every output
+        // row whose nearest kept row it is (R13), halo columns as zeros.
+        const int T = (mt * CG + (int)rank) * a.msub + sb, n = T / g.tpi, tb = T - n * g.tpi;
         const int k = (int)a.fd_w.div((uint32_t)row), v = row - k * (g.wv + 2 * g.pad);
         const int pk = tb * g.nseg + k;
-        mok = k < g.nseg && pk < g.hk && v >= g.vh && v < g.vh + g.Wo && T * TC_BM < g.M;
-        m = (n * g.hk + pk) * g.Wo + (v - g.vh);
-        valid = mok;
+        mok = k < g.nseg && pk < g.hk && v < g.wv && T * TC_BM < g.M;
+        m = (n * g.hv + g.vh + pk * g.psh) * g.wv + v;
+        valid = mok && v >= g.vh && v < g.vh + g.Wo;
       } else if (g.pm) {
         const int ni = (int)a.fd_hw.div((uint32_t)m), rem = m - ni * g.hv * g.wv;
         const int pv = (int)a.fd_w.div((uint32_t)rem), qv = rem - pv * g.wv;
@@ -1199,7 +1205,22 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         // pieces of this pass inside both the group (Nfg) and this N tile (bn)
         const int np = min(8, (min(min(g.Nfg - n, cend - c0), pass_cols) * eb) / 16);
         char *rowp = mok ? obase + ((size_t)m * ocs + col) * eb : nullptr;
-        epi_store_rows(stage, pc, np, rowp, lane);
+        if (g.pm == 2) {
+          // kept output row p = pk * psh -> every row q with nearest kept row p
+          const int p = m / g.wv % g.hv - g.vh;
+          for (int d = -((g.psh - 1) / 2); d < g.psh; ++d) {     // warp-uniform bounds
+            const int q = p + d;
+            bool ok = rowp != nullptr && q >= 0 && q < g.Ho;
+            if (ok) {
+              const int lo = q / g.psh * g.psh, hi = lo + g.psh;
+              ok = ((hi < g.Ho && hi - q < q - lo) ? hi : lo) == p;
+            }
+            epi_store_rows(stage, pc, np,
+                           ok ? rowp + (ptrdiff_t)d * g.wv * ocs * eb : nullptr, lane);
+          }
+        } else {
+          epi_store_rows(stage, pc, np, rowp, lane);
+        }
       }
       }   // sub-tiles
       tc_fence_before();
@@ -1384,7 +1405,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.b_stages = p.b_stages;
   args.msub = p.msub > 1 ? p.msub : 1;
   args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, g.S, args.msub) : 0;
-  if (args.msub > 2 || (args.msub == 2 && (!g.pm || g.pm == 2 || p.bn > TC_BN_MAX / 2)) ||
+  if (args.msub > 2 || (args.msub == 2 && (!g.pm || p.bn > TC_BN_MAX / 2)) ||
       (g.pm == 2 && (g.nseg < 1 || g.nseg * (g.wv + 2 * g.pad) > TC_BM || g.tpi < 1)))
     return cudaErrorInvalidValue;
   args.b = b;

@@ -777,7 +777,6 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
   const char *force_ms = getenv("PCNN_PM_MSUB");           // 1 | 2 (experiments)
   for (int ms = 1; ms <= 2; ++ms) {
     if (force_ms && atoi(force_ms) != ms) continue;
-    if (g.pm == 2 && ms > 1) continue;          // row-perforated tiles: one sub-tile
     for (int cg = 1; cg <= 2; ++cg) {
       if (force_cg && atoi(force_cg) != cg) continue;
       const long long rows = 128LL * cg * ms;
@@ -977,6 +976,20 @@ static pcnn_status run_layer(pcnn_net *net, int i, int B, const void *x, void *y
   switch (ly.d.kind) {
     case PCNN_CONV:
     case PCNN_FC:
+      if (ly.perf_sh * ly.perf_sw > 1 && ly.pf.g.pm == 2) {
+        // row perforation in padded-layout mode: the epilogue writes each
+        // kept row to every output row it stands for (R13); the halo rows
+        // above / below the image are zeroed here
+        pcnn_status r = run_stage(net, ly, ly.pf, B, x, y, 0, s, nullptr);
+        if (r != PCNN_OK) return r;
+        const ConvGeom &g = ly.pf.g;
+        const size_t rowb = (size_t)g.wv * ly.out_cs * esz_of(ly.pf.st);
+        const size_t img = (size_t)g.hv * rowb;
+        CUDA_TRY(cudaMemset2DAsync(y, img, 0, (size_t)g.vh * rowb, B, s));
+        CUDA_TRY(cudaMemset2DAsync((char *)y + (size_t)(g.vh + g.Ho) * rowb, img, 0,
+                                   (size_t)(g.hv - g.vh - g.Ho) * rowb, B, s));
+        return PCNN_OK;
+      }
       if (ly.perf_sh * ly.perf_sw > 1) {
         // perforation: the conv at the kept grid into the scratch buffer, then
         // nearest-neighbour interpolation into the layer's output layout

@@ -134,3 +134,18 @@ def test_row_perforation_padded_layout(orc, prec, sh, monkeypatch):
     ar = gpu_run(anet, aw, ab, ax, prec, perforation={1: (sh, 1)})
     assert ar["net"].query_layer(1, 2)["a_mode"] == 2
     assert rel_err(ar["out"], aref) <= TOL[prec] / 2
+
+
+@pytest.mark.parametrize("sh", [2, 4])
+def test_row_perforation_feeding_padded_conv(orc, sh):
+    """A row-perforated padded-layout layer whose consumer is another
+    padded-layout conv: the direct multi-row epilogue stores and the halo-row
+    zeroing must leave exactly the zero border the consumer reads."""
+    net = vgg_like()
+    w, b = params(net, seed=33)
+    x = small_inputs((3, 36, 36), 2, lo=-128, hi=128)
+    perf = {3: (sh, 1)}                 # conv 3 feeds padded-layout conv 4
+    ref = orc.run_net(net, w, b, x, perforation=perf).reshape(2, -1)
+    r = gpu_run(net, w, b, x, "bf16", perforation=perf)
+    assert r["net"].query_layer(3, 2)["a_mode"] == 2
+    assert rel_err(r["out"], ref) <= TOL["bf16"] / 2
