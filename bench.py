@@ -53,6 +53,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--net", default="alexnet", choices=["alexnet", "vgg16"])
     ap.add_argument("--batch", type=int, default=None)
+    ap.add_argument("--global-batch", type=int, default=None,
+                    help="strong scaling (configs[4]): split this many images over the ranks")
     ap.add_argument("--precision", default="bf16", choices=["bf16", "tf32", "fp32"])
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -221,6 +223,10 @@ def main():
 
     net = synth.get_net(a.net)
     B = a.batch
+    if a.global_batch:                     # configs[4]: e.g. VGG-16 1024 images over N GPUs
+        if a.global_batch % world:
+            raise SystemExit("--global-batch must be a multiple of the GPU count")
+        B = a.global_batch // world
     # weights: generated on rank 0, broadcast once over NCCL (C1)
     t_b = time.perf_counter()
     if world > 1:
@@ -364,7 +370,7 @@ def main():
         "warmup": a.warmup,
         "ms_per_step": round(total_step_ms, 4),
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "strong" if a.global_batch else "weak",
         "vs_baseline": None,
         "dtype": a.precision,
         "data": "synthetic (seeded He-normal weights, U[-128,128) images, BF16-representable)",
