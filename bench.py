@@ -324,6 +324,29 @@ def main():
         sampler.mark(False)
     clocks = sampler.stop() if sampler else None
 
+    # ---------------- board energy per image (NVML counter over >= 1 s of steps,
+    # after the clock sampling of the timed / e2e regions;
+    # the eq. 15 SoC denominator, DESIGN.md NEXT-4)
+    from paper_conf_hpca_songhcl17_b200 import tuning as ptuning
+    meter = ptuning.EnergyMeter(local)
+    energy = None
+    if meter.read_j() is not None:
+        # the same step count on every rank (steps carry collectives): ~1 s
+        # at the all-reduced step time
+        n_e = max(10, int(1000.0 / max(ms_max / a.steps, 1e-3)))
+        barrier()
+        torch.cuda.synchronize()
+        e0j, t0 = meter.read_j(), time.perf_counter()
+        for _ in range(n_e):
+            step()
+        torch.cuda.synchronize()
+        el = time.perf_counter() - t0
+        dj = meter.read_j() - e0j
+        energy = {"j_per_image": round(dj / (n_e * B), 6), "avg_power_w": round(dj / el, 1),
+                  "window_s": round(el, 3), "source": "nvmlDeviceGetTotalEnergyConsumption "
+                  "(board, this rank's GPU)"}
+
+
     # ---------------- per-layer plan, roofline of the dominant kernel (conv)
     infos = [n.query_layer(i, B) for i in range(n.n_layers)]
     conv_idx = [i for i, f in enumerate(infos) if f["kind"] == pcnn.CONV]
@@ -399,6 +422,7 @@ def main():
         "value_graph_replay": round(value_graph, 1),
         "per_layer": per_layer,
         "weights_broadcast_ms": round(bcast_ms, 3),
+        "energy": energy,
         "clocks": clocks,
         "paper_context": PAPER_CONTEXT[a.net],
     }

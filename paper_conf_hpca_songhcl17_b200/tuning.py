@@ -126,3 +126,47 @@ def rescale_batch(t_user, t_model, batch):
     if t_model <= t_user:
         return batch
     return max(1, int(math.floor(t_user / t_model * batch)))
+
+
+# ---------------------------------------------------------------- SoC (NEXT-4, eq. 15)
+def soc_time(t, t_i, t_t):
+    """P:69 / P:364: 1 in the imperceptible region (0, T_i], 0 in the
+    unusable region (T_t, inf), linear in between (reading R15: linear from
+    1 at T_i to 0 at T_t)."""
+    if t <= t_i:
+        return 1.0
+    if t >= t_t:
+        return 0.0
+    return (t_t - t) / (t_t - t_i)
+
+
+def soc_accuracy(entropy, threshold):
+    """1 when CNN_entropy <= CNN_threshold, else threshold / entropy."""
+    return 1.0 if entropy <= threshold else threshold / entropy
+
+
+def soc(t, entropy, energy_j, t_i, t_t, threshold):
+    """eq. 15: SoC = SoC_time x SoC_accuracy / energy consumption."""
+    return soc_time(t, t_i, t_t) * soc_accuracy(entropy, threshold) / energy_j
+
+
+class EnergyMeter:
+    """Board energy from NVML's total-energy counter (mJ since driver load;
+    SM power gating is not software-controllable on B200, so this is the
+    board-level figure eq. 15 divides by).  Unavailable -> None."""
+
+    def __init__(self, device=0):
+        self.h = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device)
+            pynvml.nvmlDeviceGetTotalEnergyConsumption(self.h)
+        except Exception:
+            self.h = None
+
+    def read_j(self):
+        if self.h is None:
+            return None
+        return self._nv.nvmlDeviceGetTotalEnergyConsumption(self.h) / 1000.0

@@ -59,3 +59,13 @@ def test_eq13_rescale():
     assert tuning.rescale_batch(10.0, 40.0, 64) == 16      # T_user / T = 1/4
     assert tuning.rescale_batch(10.0, 5.0, 64) == 64       # already fast enough
     assert tuning.rescale_batch(1.0, 1000.0, 64) == 1
+
+
+def test_soc_eq15():
+    """eq. 15 and its two factors on hand-worked values."""
+    assert tuning.soc_time(0.05, 0.1, 1.0) == 1.0
+    assert abs(tuning.soc_time(0.55, 0.1, 1.0) - 0.5) < 1e-12
+    assert tuning.soc_time(2.0, 0.1, 1.0) == 0.0
+    assert tuning.soc_accuracy(0.4, 0.5) == 1.0
+    assert tuning.soc_accuracy(1.0, 0.5) == 0.5
+    assert abs(tuning.soc(0.55, 1.0, 2.0, 0.1, 1.0, 0.5) - 0.125) < 1e-12

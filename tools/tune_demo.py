@@ -41,6 +41,33 @@ for step in path:
         "te": None if step["te"] is None else (str(step["te"]) if step["te"] == float("inf")
                                                else round(step["te"], 5)),
         "opt_sm": {names[i]: p["opt_sm"] for i, p in enumerate(plans) if p["grid_size"] > 0}})
+# eq. 15 SoC of the first and last tables: board energy per pass over ~1 s
+meter = tuning.EnergyMeter(0)
+
+
+def energy_per_pass(state):
+    tuning.apply_state(n, ladders, state)
+    o, _, e = n.infer(x, entropy=True)
+    torch.cuda.synchronize()
+    import time
+    j0, t0, k = meter.read_j(), time.perf_counter(), 0
+    while time.perf_counter() - t0 < 1.0:
+        for _ in range(10):
+            n.infer(x, out=o, entropy=e)
+        k += 10
+        torch.cuda.synchronize()
+    return (meter.read_j() - j0) / k
+
+
+if meter.read_j() is not None:
+    t_i, t_t = 0.5, 2.0          # ms: imperceptible / unusable bounds of this demo (R15)
+    out["soc"] = []
+    for idx in (0, len(path) - 1):
+        ej = energy_per_pass(path[idx]["state"])
+        out["soc"].append({"table": idx, "j_per_pass": round(ej, 5),
+                           "soc": tuning.soc(path[idx]["time"], path[idx]["entropy"], ej,
+                                             t_i, t_t, threshold),
+                           "t_i_ms": t_i, "t_t_ms": t_t})
 last = len(path) - 1
 out["calibration"] = {str(h): tuning.calibrate(path, last, h, threshold)
                       for h in (path[last]["entropy"], threshold, threshold + 0.5, 1e9)}
