@@ -299,3 +299,23 @@ def test_infer_host_pipelined_chunks(orc):
     ref = orc.run_net(net, w, b, x[:2])
     assert rel_err(oh.numpy()[:2], ref) <= TOL["bf16"]
     assert np.isfinite(hh.numpy()).all() and (hh.numpy() >= 0).all()
+
+
+# ------------------------------------------------------------ bench configurations, full size
+@pytest.mark.parametrize("name,B,samples", [("alexnet", 256, (0, 131, 255)), ("vgg16", 64, (0, 63))])
+def test_bench_workload_sampled_parity(orc, name, B, samples):
+    """The workloads bench.py times (AlexNet B = 256, VGG-16 B = 64, BF16, the
+    same launch plan and CUDA graph): sampled images against the oracle one by
+    one, and properties that hold for every image of the batch (finite logits,
+    softmax rows summing to 1, entropy in [0, ln 1000])."""
+    net = synth.get_net(name)
+    w, b = params(net)
+    x = synth.images(0, B, net["in_shape"])
+    r = gpu_run(net, w, b, x, "bf16", probs=True)
+    out, probs, ent = r["out"], r["probs"], r["entropy"]
+    assert np.isfinite(out).all()
+    assert np.abs(probs.sum(1) - 1.0).max() < 1e-4
+    assert (ent >= -1e-5).all() and (ent <= np.log(1000) + 1e-4).all()
+    for i in samples:
+        ref = orc.run_net(net, w, b, x[i:i + 1])
+        assert rel_err(out[i:i + 1], ref) <= TOL["bf16"], (name, i)
