@@ -191,10 +191,16 @@ pcnn_status pcnn_set_variant(pcnn_net *net, int layer, int variant, int rank);
  * rank variant (pcnn_set_variant(EXACT) clears both). */
 pcnn_status pcnn_set_perforation(pcnn_net *net, int layer, int sh, int sw);
 
-/* Test hook: install explicit factors for a RANK variant.
- *   A : host fp32 [groups][N_f/g][rank]   (stage-2 1x1 weights)
- *   B : host fp32 [groups][rank][C/g][S][S] (stage-1 filters, OIHW)
- * so that the layer computes conv(x, A_g B_g) + bias. */
+/* Install explicit factors for a RANK variant (conv: test hook; FC: the way
+ * to get an FC rank-r variant -- the library computes SVDs only for conv
+ * layers, whose per-group matrices are small).
+ *   conv: A host fp32 [groups][N_f/g][rank]   (stage-2 1x1 weights)
+ *         B host fp32 [groups][rank][C/g][S][S] (stage-1 filters, OIHW)
+ *         -> conv(x, A_g B_g) + bias
+ *   FC:   A host fp32 [N][rank], B host fp32 [rank][C*H*W] (columns in the
+ *         input's C,H,W order like the FC weight) -> (A B) x + bias
+ * INVALID_ARGUMENT for a rank outside [1, min(N, K)]; UNSUPPORTED for other
+ * layer kinds or a perforated layer. */
 pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank,
                                      const float *A, const float *B);
 

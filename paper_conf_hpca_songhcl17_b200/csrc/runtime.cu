@@ -310,6 +310,8 @@ static double layer_flops_exact(const Layer &ly, int B) {
 }
 
 static double layer_flops_variant(const Layer &ly, int B) {
+  if (ly.variant == PCNN_VARIANT_RANK && ly.d.kind == PCNN_FC)   // 2 B r (K + N)
+    return 2.0 * B * ly.rank * ((double)ly.in_c * ly.in_h * ly.in_w + ly.d.out_channels);
   if (ly.perf_sh * ly.perf_sw > 1)       // eq. 1 FLOPs at the kept positions only
     return layer_flops_exact(ly, B) * ((ly.out_h + ly.perf_sh - 1) / ly.perf_sh) *
            ((ly.out_w + ly.perf_sw - 1) / ly.perf_sw) / ((double)ly.out_h * ly.out_w);
@@ -1617,14 +1619,50 @@ pcnn_status pcnn_set_perforation(pcnn_net *net, int layer, int sh, int sw) {
   return PCNN_OK;
 }
 
+// FC rank-r (the conv form with S = 1): stage 1 = FC K -> r
+// with B's rows (CHW-ordered columns, permuted like the exact fc), stage 2 =
+// FC r -> N with A + bias (+ ReLU).
+static pcnn_status build_rank_stages_fc(pcnn_net *net, Layer &ly, int r, const float *A,
+                                        const float *Bf) {
+  const auto &d = ly.d;
+  const int prec = net->desc.precision, st = net->st, N = d.out_channels;
+  const size_t K = (size_t)ly.in_c * ly.in_h * ly.in_w;
+  const int rs = round_up(r, 64);                 // one full K-block of stage 2
+  std::vector<float> w1((size_t)rs * K, 0.f), w2((size_t)N * rs, 0.f);
+  std::memcpy(w1.data(), Bf, sizeof(float) * (size_t)r * K);
+  for (int f = 0; f < N; ++f)
+    for (int a = 0; a < r; ++a) w2[(size_t)f * rs + a] = A[(size_t)f * r + a];
+  const int mode1 = st == ST_BF16 ? OUT_BF16 : (prec == PCNN_TF32 ? OUT_F32_TF32 : OUT_F32);
+  pcnn_status s1 = build_stage(ly.r1, ly, prec, rs, 1, 1, 1, 0, 0, ly.in_c, ly.in_h, ly.in_w,
+                               ly.in_cs, true, w1.data(), nullptr, mode1);
+  if (s1 != PCNN_OK) return s1;
+  const GemmStage &ex = ly.exact;
+  pcnn_status s2 = build_stage(ly.r2, ly, prec, N, 1, 1, 1, 0, d.relu, rs, 1, 1, rs, true,
+                               w2.data(), nullptr, ex.g.out_mode);
+  if (s2 != PCNN_OK) return s2;
+  CUDA_TRY(cudaMemcpy(ly.r2.d_bias, ex.d_bias, sizeof(float) * N, cudaMemcpyDeviceToDevice));
+  ly.rank = r;
+  ly.variant = PCNN_VARIANT_RANK;
+  net->version++;
+  return PCNN_OK;
+}
+
 pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank, const float *A,
                                      const float *B) {
   if (!net || layer < 0 || layer >= (int)net->layers.size() || !A || !B)
     return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
   Layer &ly = net->layers[layer];
-  if (ly.d.kind != PCNN_CONV) return fail(PCNN_ERR_UNSUPPORTED, "conv layers only");
+  if (ly.d.kind != PCNN_CONV && ly.d.kind != PCNN_FC)
+    return fail(PCNN_ERR_UNSUPPORTED, "conv / fc layers only");
   if (rank < 1 || rank > 4096) return fail(PCNN_ERR_INVALID_ARGUMENT, "bad rank");
+  if (ly.perf_sh * ly.perf_sw > 1)
+    return fail(PCNN_ERR_UNSUPPORTED, "rank variant of a perforated layer (set EXACT first)");
   CUDA_TRY(cudaSetDevice(net->device));
+  if (ly.d.kind == PCNN_FC) {
+    if (rank > std::min<long long>(ly.d.out_channels, (long long)ly.in_c * ly.in_h * ly.in_w))
+      return fail(PCNN_ERR_INVALID_ARGUMENT, "rank out of [1, min(N, K)]");
+    return build_rank_stages_fc(net, ly, rank, A, B);
+  }
   return build_rank_stages(net, ly, rank, A, B);
 }
 

@@ -196,3 +196,32 @@ def test_opt_budgets_keep_results_and_latency(alex):
     n1.enable_sm_census(False)
     t1 = timed(n1)
     assert t1 <= 1.25 * t0, (t0, t1)
+
+
+@pytest.mark.parametrize("prec", ["tf32", "bf16"])
+def test_fc_rank_variant_factors(orc, prec):
+    """FC rank-r: factors A = U_r S_r, B = V_r^T installed
+    through pcnn_set_variant_factors (B's columns in the input's C,H,W order,
+    so the CHW -> HWC permutation of the first FC applies) match the oracle's
+    rank-r operator (its own SVD algorithm) end to end."""
+    net = dict(in_shape=(16, 8, 8), layers=[
+        conv_layer(32, 3, 16, 1, 1), dict(kind="maxpool", k=2, stride=2),
+        dict(kind="fc", out=96, in_f=32 * 4 * 4, relu=True),
+        dict(kind="fc", out=16, in_f=96, relu=False)])
+    w, b = params(net, seed=41)
+    x = small_inputs((16, 8, 8), 3, lo=-2, hi=2)
+    ranks = {2: 32, 3: 8}
+    ref = orc.run_net(net, w, b, x, ranks=ranks).reshape(3, -1)
+    import torch
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    n = pcnn.Net(net, w, b, 3, prec)
+    for i, r in ranks.items():
+        U, S, Vt = np.linalg.svd(np.asarray(w[i], dtype=np.float64), full_matrices=False)
+        n.set_variant_factors(i, r, U[:, :r] * S[:r], Vt[:r])
+        f = n.query_layer(i, 3)
+        assert f["rank"] == r and f["flops"] < f["flops_exact"]
+    out, _, _ = n.infer(torch.from_numpy(x).cuda())
+    torch.cuda.synchronize()
+    assert rel_err(out.cpu().numpy(), ref) <= TOL[prec] / 2
+    with pytest.raises(pcnn.PcnnError):
+        n.set_variant_factors(3, 17, np.zeros((16, 17)), np.zeros((17, 96)))   # rank > min(N, K)
