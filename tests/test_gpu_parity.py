@@ -319,3 +319,15 @@ def test_bench_workload_sampled_parity(orc, name, B, samples):
     for i in samples:
         ref = orc.run_net(net, w, b, x[i:i + 1])
         assert rel_err(out[i:i + 1], ref) <= TOL["bf16"], (name, i)
+
+
+def test_vgg16_tf32_bench_batch_sampled(orc):
+    """VGG-16 TF32 (configs[3]'s second precision) at the bench batch: one
+    sampled image against the oracle within the TF32 tolerance."""
+    net = synth.vgg16()
+    w, b = params(net)
+    x = synth.images(0, 64, net["in_shape"])
+    out = gpu_run(net, w, b, x, "tf32")["out"]
+    assert np.isfinite(out).all()
+    ref = orc.run_net(net, w, b, x[17:18])
+    assert rel_err(out[17:18], ref) <= TOL["tf32"]
