@@ -103,3 +103,37 @@ def net_params(net, seed=WEIGHT_SEED):
         ws.append(he_weights(wshape, fan_in, i, seed))
         bs.append(biases(bshape[0], i, seed))
     return ws, bs
+
+
+PROTO_TENSOR_ID = 1 << 20        # planted-class prototypes
+NOISE_TENSOR_ID = (1 << 20) + 1
+
+
+def prototypes(count, shape, seed=IMAGE_SEED, block=16):
+    """Planted-class prototypes [count, C, H, W]: a
+    block x block piecewise-constant low-frequency field at U[-128, 128) per
+    channel plus U[-32, 32) texture.  Pure generation, no method arithmetic."""
+    C, H, W = shape
+    bh, bw = (H + block - 1) // block, (W + block - 1) // block
+    out = np.empty((count, C, H, W), dtype=np.float32)
+    for k in range(count):
+        coarse = uniform(seed, PROTO_TENSOR_ID, k * C * bh * bw, C * bh * bw,
+                         -128.0, 128.0).reshape(C, bh, bw)
+        field = np.repeat(np.repeat(coarse, block, axis=1), block, axis=2)[:, :H, :W]
+        tex = uniform(seed, PROTO_TENSOR_ID + 2, k * C * H * W, C * H * W,
+                      -32.0, 32.0).reshape(C, H, W)
+        out[k] = field + tex
+    return round_to_bf16(out)
+
+
+def planted_images(n_start, count, shape, n_classes, seed=IMAGE_SEED):
+    """Images of the planted-class set: image n is prototype (n mod n_classes)
+    plus N(0, sigma^2) noise, sigma = U[0.02, 0.08) x 128 per image; returns
+    (images [count, C, H, W], labels [count])."""
+    per = int(np.prod(shape))
+    labels = (np.arange(n_start, n_start + count) % n_classes).astype(np.int64)
+    protos = prototypes(n_classes, shape, seed)
+    sig = uniform(seed, NOISE_TENSOR_ID + 1, n_start, count, 0.02 * 128, 0.08 * 128)
+    noise = normal(seed, NOISE_TENSOR_ID, n_start * per, count * per).reshape((count,) + tuple(shape))
+    x = protos[labels] + noise * sig[:, None, None, None].astype(np.float32)
+    return round_to_bf16(x), labels

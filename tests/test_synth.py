@@ -40,3 +40,16 @@ def test_net_params_shapes():
     assert shapes[3] == (256, 48, 5, 5)
     assert shapes[10] == (4096, 9216)
     assert bs[12].shape == (1000,)
+
+
+def test_planted_set_generator():
+    """Planted-class images: deterministic by global index, label = index mod
+    classes, image = its prototype plus small noise."""
+    shp = (3, 40, 36)
+    x1, l1 = synth.planted_images(5, 3, shp, 4)
+    x2, l2 = synth.planted_images(5, 3, shp, 4)
+    assert (x1 == x2).all() and list(l1) == [1, 2, 3]
+    p = synth.prototypes(4, shp)
+    d = np.abs(x1 - p[l1]).max(axis=(1, 2, 3))
+    assert (d < 0.12 * 128 * 6).all() and (d > 0).all()
+    assert np.abs(p[0] - p[1]).mean() > 20          # distinct prototypes
