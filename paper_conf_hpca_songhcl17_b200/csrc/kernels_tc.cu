@@ -423,6 +423,8 @@ struct TcArgs {
   int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
   int a_stages, b_stages, pm_a_stage;   // padded mode rings (g.pm)
   int msub;             // padded mode: M sub-tiles of 128 rows per CTA sharing each B slab
+  int kmma_last;        // padded mode: UMMAs (32 B of K each) of the last channel slab that
+                        // touch real channels; the rest multiply zero padding and are skipped
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
   int tma_y;            // 1: full 32-column output chunks leave by TMA tensor store
   float lrn_a_over_n, lrn_beta, lrn_k;
@@ -642,6 +644,7 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
   const uint64_t b_desc0 = umma_desc(sBp, SLAB);
   const uint32_t a_st16 = (uint32_t)a.pm_a_stage / 16, b_st16 = pm_b_bytes / 16;
   const int a_stages = a.a_stages, b_stages = a.b_stages, units = a.units, S = a.g.S;
+  const int j_last = nj - S, kmma_last = a.kmma_last;   // windows of the last channel slab
   // sub-tile 1's window starts pm_sub_rows(S) rows into the A stage
   const uint32_t sub16 = (uint32_t)pm_sub_rows(S) * ROW16;
   const bool prof = TC_PROF(a) != 0, skip_mma = (a.skip & 4) != 0;
@@ -656,6 +659,7 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
     for (int j = 0; j < nj; ++j) {
       wfull.wait(sbase + SM_AFULL + 8 * as, aph);
       const uint64_t ad = a_desc0 + as * a_st16;
+      const int kk = j >= j_last ? kmma_last : KMMA;
       for (int s2 = 0; s2 < S; ++s2) {
         wfull.wait(sbase + SM_FULL + 8 * bs, bph);
         tc_fence_after();
@@ -669,7 +673,8 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
               const uint32_t dc = dcol + sb * (TC_BN_MAX / 2);
               tc_mma<ST, CG>(dc, awb, bd, idesc, (j > 0 || s2 > 0) ? 1u : 0u);
 #pragma unroll
-              for (int k = 1; k < KMMA; ++k) tc_mma<ST, CG>(dc, awb + 2 * k, bd + 2 * k, idesc, 1u);
+              for (int k = 1; k < KMMA; ++k)
+                if (k < kk) tc_mma<ST, CG>(dc, awb + 2 * k, bd + 2 * k, idesc, 1u);
             }
           }
           tc_commit<CG>(sbase + SM_EMPTY + 8 * bs);
@@ -1404,6 +1409,17 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.a_stages = p.a_stages;
   args.b_stages = p.b_stages;
   args.msub = p.msub > 1 ? p.msub : 1;
+  {
+    // padded mode: UMMAs of the last channel slab that reach real channels
+    const int se = args.slab_bytes / (st == ST_BF16 ? 2 : 4);
+    const int creal = g.Creal > 0 && g.Creal <= g.Cg ? g.Creal : g.Cg;
+    const int ncb = se > 0 ? g.Cg / se : 1;
+    const int valid_b = (creal - (ncb - 1) * se) * (st == ST_BF16 ? 2 : 4);
+    const char *ek = getenv("PCNN_NO_KSKIP");           // A/B: multiply the padding too
+    args.kmma_last = args.slab_bytes / 32;
+    if (!(ek && ek[0] == '1') && valid_b > 0)
+      args.kmma_last = std::min(args.slab_bytes / 32, (valid_b + 31) / 32);
+  }
   args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, g.S, args.msub) : 0;
   if (args.msub > 2 || (args.msub == 2 && (!g.pm || p.bn > TC_BN_MAX / 2)) ||
       (g.pm == 2 && (g.nseg < 1 || g.nseg * (g.wv + 2 * g.pad) > TC_BM || g.tpi < 1)))

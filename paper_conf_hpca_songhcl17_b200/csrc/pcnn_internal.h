@@ -67,6 +67,9 @@ struct ConvGeom {
   // per image, hk kept rows per image; M = B * tpi * 128.  The output is the
   // compact kept grid [B][hk][Wo][out_cs].
   int nseg, tpi, hk;
+  // real (unpadded) channels per group, 0 = Cg: padded-layout UMMAs over the
+  // zero channel padding of the last slab are skipped (their products are 0)
+  int Creal;
 };
 
 // ---------------------------------------------------------------- launchers

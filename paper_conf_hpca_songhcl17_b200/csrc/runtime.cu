@@ -447,6 +447,7 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
     g.Nfg = Nf / groups;
     g.K = S * S * Cg_st;
     g.Kpad = round_up(g.K, k_align(precision));
+    g.Creal = Cg_log;
     if (pm_halo > 0 && pm_valid) {
       // a 'valid' stride-1 conv (pad 0, S = 2h + 1) read as a 'same' conv on
       // its own input grid: the input is the halo-h grid of the output, the

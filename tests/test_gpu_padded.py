@@ -168,3 +168,20 @@ def test_padded_mode_conv_lrn_fusion(orc, prec, monkeypatch):
     assert rel_err(fused["out"], ref) <= TOL[prec] / 4
     assert rel_err(plain, ref) <= TOL[prec] / 4
     assert rel_err(fused["out"], plain) <= (2e-3 if prec == "tf32" else 8e-3)
+
+
+@pytest.mark.parametrize("prec", ["bf16", "tf32"])
+def test_padded_mode_skips_channel_padding_bitwise(prec, monkeypatch):
+    """AlexNet conv2-shaped grouped conv (48 real channels per group stored
+    as 64): skipping the UMMAs that only multiply the zero padding gives
+    bitwise the same result as multiplying it."""
+    net = dict(in_shape=(96, 27, 27), layers=[
+        dict(kind="maxpool", k=1, stride=1),
+        conv_layer(256, 5, 96, 1, 2, 2), dict(kind="maxpool", k=3, stride=2)])
+    w, b = params(net, seed=12)
+    x = small_inputs((96, 27, 27), 2, lo=-2, hi=2)
+    fast = gpu_run(net, w, b, x, prec)
+    assert fast["net"].query_layer(1, 2)["a_mode"] == 2
+    monkeypatch.setenv("PCNN_NO_KSKIP", "1")
+    full = gpu_run(net, w, b, x, prec)["out"]
+    np.testing.assert_array_equal(fast["out"], full)
