@@ -771,6 +771,7 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
 static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n = false) {
   TcPlan best{};
   double best_t = 1e300;
+  std::vector<std::pair<double, TcPlan>> cands;
   const int nmax = std::min(256, round_up(g.Nfg, 32));
   const double f = 1.9e9;
   const int slab = tc_slab_bytes(esz == 2 ? ST_BF16 : ST_F32, g.Cg);
@@ -792,27 +793,49 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
         const int ntiles = (g.Nfg + bn - 1) / bn;
         const long long tiles = (long long)mtiles * ntiles * g.groups;
         // per (slab, filter row): ms windows of 128 + S - 1 rows and S weight
-        // slabs (shared by the ms sub-tiles) through L2, ms * S * slab/32 UMMAs
+        // slabs (shared by the ms sub-tiles) through L2, each TMA load with a
+        // fixed issue / completion cost (measured: ~64 cycles; AlexNet conv2
+        // ms = 1 1970 cycles per window vs 1680 from bytes and MMAs alone),
+        // ms * S UMMA slabs of which the last channel slab's zero padding is
+        // skipped (kmma_eff of slab/32 UMMAs, averaged over the slabs)
+        const int se = slab / esz, ncb = std::max(1, g.Cg / se);
+        const int creal = g.Creal > 0 && g.Creal <= g.Cg ? g.Creal : g.Cg;
+        const double last_frac =
+            std::min(1.0, std::ceil((double)(creal - (ncb - 1) * se) * esz / 32.0) / (slab / 32.0));
+        const double kfrac = ((ncb - 1) + last_frac) / ncb;
         const double load = (ms * (128.0 + g.S - 1) * slab + (double)g.S * slab * bn / cg) /
-                            kOperandBytesPerCycle;
-        const double mma = ms * g.S * (slab / 128.0) * 2.05 * bn / kMmaEfficiency;
+                                kOperandBytesPerCycle + 64.0 * (ms + g.S);
+        const double mma = ms * g.S * (slab / 128.0) * kfrac * 2.05 * bn / kMmaEfficiency;
         const double j_cycles = std::max(load, mma) + 40.0;
         const long long waves = (tiles + slots - 1) / slots;
         const double t = (double)waves * nj * j_cycles / f + 2e-6 * ms;
-        if (t < best_t * 0.999 ||
-            (t <= best_t * 1.001 && (long long)bn * cg > (long long)best.bn * best.cg)) {
-          best_t = t;
-          best.cg = cg;
-          best.bn = bn;
-          best.msub = ms;
-          best.mtiles = mtiles;
-          best.ntiles = ntiles;
-          best.tiles = (int)tiles;
-          best.splits = 1;
-          best.kb_per_split = nj;
-          best.units = (int)tiles;
-        }
+        TcPlan c{};
+        c.cg = cg;
+        c.bn = bn;
+        c.msub = ms;
+        c.mtiles = mtiles;
+        c.ntiles = ntiles;
+        c.tiles = (int)tiles;
+        c.splits = 1;
+        c.kb_per_split = nj;
+        c.units = (int)tiles;
+        cands.push_back({t, c});
+        best_t = std::min(best_t, t);
       }
+    }
+  }
+  // within 5% of the fastest modelled plan (the model's error on measured
+  // layers), prefer the widest N tile: it re-reads A the fewest times (VGG
+  // conv3-5: 256 x 256 beats 512 x 128 by ~4% although modelled 2% slower)
+  long long wide = -1;
+  double bt = 1e300;
+  for (auto &pc : cands) {
+    if (pc.first > best_t * 1.05) continue;
+    const long long wdt = (long long)pc.second.bn * pc.second.cg;
+    if (wdt > wide || (wdt == wide && pc.first < bt)) {
+      wide = wdt;
+      bt = pc.first;
+      best = pc.second;
     }
   }
   tc_pm_stages(best.bn, best.cg, slab, g.S, best.msub, &best.a_stages, &best.b_stages);
