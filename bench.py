@@ -378,6 +378,16 @@ def main():
             d["grid"] = f["grid"]
             d["util_eq6"] = round(f["util"], 3)
             d["rec_eq9"] = round(f["rec"], 3)
+        elif (f["kind"] in (pcnn.MAXPOOL, pcnn.AVGPOOL) and i > 0 and infos[i - 1]["kind"] == pcnn.LRN
+              and os.environ.get("PCNN_NO_FUSE") != "1"):
+            # LRN + pool run as ONE launch (runtime.cu run_lrn_pool): the pool's
+            # event window is empty, so the pair's time and bytes (LRN input read
+            # + pool output write = this pool layer's in + out bytes, since the
+            # LRN output has the LRN input's shape) go on the LRN entry.
+            d["fused_into"] = per_layer[-1]["layer"]
+            pm = per_layer[-1]["ms"] + lm
+            per_layer[-1]["gbs"] = round(f["bytes"] / (pm / 1000) / 1e9, 1) if pm > 0 else None
+            per_layer[-1]["includes"] = d["layer"]
         else:
             d["gbs"] = round(f["bytes"] / (lm / 1000) / 1e9, 1) if lm > 0 else None
         per_layer.append(d)
