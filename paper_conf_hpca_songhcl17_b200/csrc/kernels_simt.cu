@@ -731,7 +731,7 @@ static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int
                                      int Hs, int Ws, int Cs, int tf32_round, cudaStream_t s) {
   static const int R = [] {                          // staged rows per band
     const char *e = getenv("PCNN_S2D_ROWS");
-    return e && atoi(e) > 0 ? atoi(e) : 2;
+    return e && atoi(e) > 0 ? atoi(e) : 3;
   }();
   const int pitch = ((W + 3) / 4 + 1) * 4;
   const size_t smem = (size_t)2 * R * 12 * pitch * 4 + 16 + 2 * R * 12 * 4;
@@ -1304,8 +1304,8 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
 // CPT == 8, so neither the writes nor the pooling reads conflict) and pooled
 // from there.  Same per-element arithmetic as the other LRN paths (sum order,
 // lrn_normalise), so the results are identical.
-template <int ST, int CPT>
-__global__ void __launch_bounds__(256) lrn_reg_kernel(const LrnPoolArgs a) {
+template <int ST, int CPT, int MINB = 0>
+__global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a) {
   extern __shared__ __align__(16) uint8_t lr_smem[];
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
   constexpr int VN = Vec16<ST>::N;
@@ -1690,12 +1690,23 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
     const size_t smem = (size_t)(min((a.R - 1) * s + k, H)) * W * C * esz;
     if (smem > 200 * 1024) return cudaErrorInvalidValue;
     const int cpt = lrn_reg_cpt(st, C);
+    static const bool occ3 = [] {                 // experiment: 3 CTAs / SM (<= 85 regs)
+      const char *e = getenv("PCNN_LRN_OCC3");
+      return e && e[0] == '1';
+    }();
 #define PCNN_LR(STT, CP)                                                                        \
   do {                                                                                          \
-    if (smem > 48 * 1024)                                                                       \
-      cudaFuncSetAttribute(lrn_reg_kernel<STT, CP>,                                             \
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);             \
-    lrn_reg_kernel<STT, CP><<<grid, 256, smem, stream>>>(a);                                    \
+    if (occ3) {                                                                                 \
+      if (smem > 48 * 1024)                                                                     \
+        cudaFuncSetAttribute(lrn_reg_kernel<STT, CP, 3>,                                        \
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);           \
+      lrn_reg_kernel<STT, CP, 3><<<grid, 256, smem, stream>>>(a);                               \
+    } else {                                                                                    \
+      if (smem > 48 * 1024)                                                                     \
+        cudaFuncSetAttribute(lrn_reg_kernel<STT, CP>,                                           \
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);           \
+      lrn_reg_kernel<STT, CP><<<grid, 256, smem, stream>>>(a);                                  \
+    }                                                                                           \
   } while (0)
     if (st == ST_BF16) {
       if (cpt == 8) PCNN_LR(ST_BF16, 8); else if (cpt == 6) PCNN_LR(ST_BF16, 6); else PCNN_LR(ST_BF16, 3);
