@@ -1272,9 +1272,23 @@ __global__ void splitk_reduce_kernel(const float *__restrict__ ws, void *y,
        i += (long long)gridDim.x * blockDim.x) {
     const long long e = i * 4;
     const int col = (int)(e % N);
+    // partials summed in split order (fixed, so every SM budget gives the
+    // same bits); the loads of three splits are issued before their adds so
+    // a thread has three L2 round trips in flight instead of one
+    const size_t sMN = (size_t)M * N;
     float4 acc = *(const float4 *)(ws + e);
-    for (int s = 1; s < splits; ++s) {
-      const float4 v = *(const float4 *)(ws + (size_t)s * M * N + e);
+    int s = 1;
+    for (; s + 2 < splits; s += 3) {
+      const float4 v0 = *(const float4 *)(ws + (size_t)s * sMN + e);
+      const float4 v1 = *(const float4 *)(ws + (size_t)(s + 1) * sMN + e);
+      const float4 v2 = *(const float4 *)(ws + (size_t)(s + 2) * sMN + e);
+      acc.x = ((acc.x + v0.x) + v1.x) + v2.x;
+      acc.y = ((acc.y + v0.y) + v1.y) + v2.y;
+      acc.z = ((acc.z + v0.z) + v1.z) + v2.z;
+      acc.w = ((acc.w + v0.w) + v1.w) + v2.w;
+    }
+    for (; s < splits; ++s) {
+      const float4 v = *(const float4 *)(ws + (size_t)s * sMN + e);
       acc.x += v.x;
       acc.y += v.y;
       acc.z += v.z;
