@@ -87,6 +87,30 @@ typedef struct {
     float lrn_k;
 } pcnn_layer_desc;
 
+/* Layout choices of pcnn_create_net (pcnn_net_desc.flags, OR-ed).  Every
+ * combination computes the same layers (the same products per output, up to
+ * the accumulation order and last-place rounding of fused epilogues, bounded
+ * in DESIGN.md); 0 = the library's default plan.  They exist so that tests
+ * can compare the alternative kernels / layouts against each other. */
+typedef enum {
+    PCNN_FLAG_NO_SPACE_TO_DEPTH = 1,    /* strided / 3-channel first conv read
+                                           from a channel-padded input
+                                           instead of space-to-depth or
+                                           im2col staging (a1)               */
+    PCNN_FLAG_NO_PADDED_LAYOUT = 2,     /* every conv in TMA-im2col mode (no
+                                           zero-haloed shifted windows)      */
+    PCNN_FLAG_NO_LRN_POOL_FUSION = 4,   /* LRN and the following pool as two
+                                           launches (and no conv+LRN epilogue) */
+    PCNN_FLAG_CONV_LRN_EPILOGUE = 8,    /* conv -> LRN fused into the tcgen05
+                                           epilogue also for padded-layout
+                                           convs (off by default: slower)    */
+    PCNN_FLAG_NARROW_SLABS = 16,        /* grouped convs with channels per
+                                           group not a multiple of 128 B keep
+                                           them unpadded (SW64 / SW32 slabs) */
+    PCNN_FLAG_PERFORATION_IM2COL = 32   /* row perforation of padded-layout
+                                           layers in im2col mode (NEXT-1)    */
+} pcnn_net_flag;
+
 typedef struct {
     int in_channels;   /* C of the NCHW input images                        */
     int in_height;     /* H                                                  */
@@ -94,6 +118,7 @@ typedef struct {
     int max_batch;     /* largest batch pcnn_infer* will be called with      */
     int precision;     /* pcnn_precision                                     */
     int device;        /* CUDA device ordinal                                */
+    int flags;         /* OR of pcnn_net_flag, 0 = default                   */
 } pcnn_net_desc;
 
 /* Per-layer geometry / plan, for a given batch (pcnn_query_layer,
@@ -212,6 +237,16 @@ pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank,
  * placement only: results are bitwise identical for every budget (R11). */
 pcnn_status pcnn_set_sm_budget(pcnn_net *net, int layer, int n_sms,
                                int ctas_per_sm);
+
+/* Per-layer tile choice override (the paper's sub-matrix choice, P:186,
+ * P:223, eqs. 4-9): cta_group = 1 (128-row UMMA tiles) or 2
+ * (CTA-pair 256-row tiles), m_sub = 128-row M sub-tiles per CTA sharing each
+ * weight slab in padded-layout mode (1 or 2); 0 = the planner's choice.  The
+ * K order of every output is unchanged, so results are bitwise identical to
+ * the default plan's.  UNSUPPORTED for non-GEMM layers or the FP32 SIMT
+ * engine, INVALID_ARGUMENT for other values. */
+pcnn_status pcnn_set_layer_plan(pcnn_net *net, int layer, int cta_group,
+                                int m_sub);
 
 /* The hot path.  Asynchronous on `stream`.
  *   d_images  : device fp32 [batch][C][H][W] (NCHW)

@@ -16,8 +16,9 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(ROOT, "build", "pcnn")
 LIB = os.path.join(PKG, "libpcnn.so")
-# role-profiling variant (tcgen05 barrier-wait counters compiled in), used by
-# tools/tc_roles.py through PCNN_LIB; never the product library
+# experiments variant (tcgen05 barrier-wait counters and the PCNN_* tuning /
+# A-B environment switches compiled in), used by tools/ through PCNN_LIB;
+# never the product library
 PROF_LIB = os.path.join(ROOT, "build", "prof", "libpcnn_prof.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
@@ -38,7 +39,7 @@ def _newer(src_list, target):
 def build(force=False, verbose=False, prof=False):
     bdir = BUILD + ("_prof" if prof else "")
     lib = PROF_LIB if prof else LIB
-    flags = FLAGS + (["-DPCNN_TC_PROF=1"] if prof else [])
+    flags = FLAGS + (["-DPCNN_TC_PROF=1", "-DPCNN_EXPERIMENTS=1"] if prof else [])
     os.makedirs(bdir, exist_ok=True)
     os.makedirs(os.path.dirname(lib), exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [

@@ -414,7 +414,7 @@ static cudaError_t launch_gather3(const float *x, void *y, int st, int B, int H,
                                   int Wo, int Kp, int D, int step, int pad, int halo,
                                   int tf32_round, cudaStream_t s) {
   static const int rows_env = [] {
-    const char *e = getenv("PCNN_STAGE_ROWS");
+    const char *e = exp_env("PCNN_STAGE_ROWS");
     return e ? atoi(e) : 0;
   }();
   const int vn = st == ST_BF16 ? 8 : 4;
@@ -588,7 +588,7 @@ cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, i
                                 int S, int stride, int pad, int Ho, int Wo, int Kp,
                                 int halo, int tf32_round, cudaStream_t s) {
   if (C != 3 || (S != 3 && S != 5)) return cudaErrorInvalidValue;
-  if (!getenv("PCNN_OLD_STAGE") && S == 3 && stride == 1 && pad == 1 && Ho == H && Wo == W &&
+  if (!exp_env("PCNN_OLD_STAGE") && S == 3 && stride == 1 && pad == 1 && Ho == H && Wo == W &&
       Kp >= 27 && Kp % (st == ST_BF16 ? 8 : 4) == 0) {
     const int R = 2;
     const int pitch = ((W + 3) / 4 + 1) * 4;
@@ -613,7 +613,7 @@ cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, i
       return cudaGetLastError();
     }
   }
-  if (!getenv("PCNN_OLD_STAGE") && gather3_ok(st, W, Kp, S, stride))
+  if (!exp_env("PCNN_OLD_STAGE") && gather3_ok(st, W, Kp, S, stride))
     return launch_gather3(x, y, st, B, H, W, Ho, Wo, Kp, S, stride, pad, halo, tf32_round, s);
   const size_t smem = (size_t)S * C * ((Wo - 1) * stride + S) * sizeof(float);
   if (smem > 48 * 1024) return cudaErrorInvalidValue;
@@ -730,7 +730,7 @@ stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int
 static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int H, int W,
                                      int Hs, int Ws, int Cs, int tf32_round, cudaStream_t s) {
   static const int R = [] {                          // staged rows per band
-    const char *e = getenv("PCNN_S2D_ROWS");
+    const char *e = exp_env("PCNN_S2D_ROWS");
     return e && atoi(e) > 0 ? atoi(e) : 3;
   }();
   const int pitch = ((W + 3) / 4 + 1) * 4;
@@ -758,7 +758,7 @@ static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int
 cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, int H, int W,
                                int Hs, int Ws, int Cs, int blk, int pad, int tf32_round,
                                cudaStream_t s) {
-  const char *old_stage = getenv("PCNN_OLD_STAGE");   // A/B: the staged-gather kernels
+  const char *old_stage = exp_env("PCNN_OLD_STAGE");   // A/B: the staged-gather kernels
   if (C == 3 && blk == 4 && pad == 0 && !old_stage && Cs >= 48 &&
       Cs % (st == ST_BF16 ? 8 : 4) == 0 && Hs * 4 <= H + 3 && Ws * 4 <= W + 3)
     return launch_stage_s2d4(x, y, st, B, H, W, Hs, Ws, Cs, tf32_round, s);
@@ -1480,7 +1480,7 @@ static int lrn_reg_cpt(int st, int C) {
   if (C % vn) return 0;
   const int chunks = C / vn;
   auto pow2_le32 = [](int p) { return p >= 1 && p <= 32 && (p & (p - 1)) == 0; };
-  const char *e = getenv("PCNN_LRN_CPT");        // tuning experiments
+  const char *e = exp_env("PCNN_LRN_CPT");        // tuning experiments
   const int want = e ? atoi(e) : 0;
   if (want == 3 && chunks % 3 == 0 && pow2_le32(chunks / 3)) return 3;
   if (chunks % 8 == 0 && pow2_le32(chunks / 8)) return 8;
@@ -1493,7 +1493,7 @@ constexpr int LB_SMEM_BUDGET = 100 * 1024;
 
 // output rows per band so that the band's staged rows fit LB_SMEM_BUDGET
 static bool use_lrn_reg(int st, int C, int lrn) {
-  const char *e = getenv("PCNN_LRN_BAND");     // A/B tests: the staged band kernel
+  const char *e = exp_env("PCNN_LRN_BAND");     // A/B tests: the staged band kernel
   const bool off = e && e[0] == '1';
   return lrn == 5 && !off && lrn_reg_cpt(st, C) > 0;
 }
@@ -1501,7 +1501,7 @@ static bool use_lrn_reg(int st, int C, int lrn) {
 static int lrn_band_rows(int st, int W, int C, int k, int s, int Ho, int lrn) {
   const int esz = st == ST_BF16 ? 2 : 4;
   const size_t row = (size_t)W * (C * esz + (use_lrn_reg(st, C, lrn) ? 0 : 16));
-  const char *e = getenv("PCNN_LB_KB");          // tuning experiments
+  const char *e = exp_env("PCNN_LB_KB");          // tuning experiments
   const size_t budget = e ? (size_t)atoi(e) * 1024 : (size_t)LB_SMEM_BUDGET;
   int R = 1;
   while (R < Ho && (size_t)((R) * s + k) * row <= budget) ++R;
@@ -1642,7 +1642,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   const int ocp = out_groups > 0 ? out_cg_pad : 0;
   if (out_groups > 0 && (C % out_groups || ocg % vn || ocp % vn || ocp < ocg))
     return cudaErrorInvalidValue;
-  if (lrn_size == 0 && out_groups == 0 && !b.gated && !getenv("PCNN_OLD_POOL")) {
+  if (lrn_size == 0 && out_groups == 0 && !b.gated && !exp_env("PCNN_OLD_POOL")) {
     const int chunks = C / vn;
     const long long total = (long long)B * (Ho + 2 * out_halo) * (Wo + 2 * out_halo) * chunks;
     const int g = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
@@ -1691,7 +1691,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
     if (smem > 200 * 1024) return cudaErrorInvalidValue;
     const int cpt = lrn_reg_cpt(st, C);
     static const bool occ3 = [] {                 // experiment: 3 CTAs / SM (<= 85 regs)
-      const char *e = getenv("PCNN_LRN_OCC3");
+      const char *e = exp_env("PCNN_LRN_OCC3");
       return e && e[0] == '1';
     }();
 #define PCNN_LR(STT, CP)                                                                        \

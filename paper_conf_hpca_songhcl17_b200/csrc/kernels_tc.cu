@@ -109,7 +109,7 @@ int tc_stages_for(int bn, int cg) {
   const int per = TC_A_STAGE + bn / cg * TC_ROW_BYTES;
   int n = TC_STAGE_BUDGET / per;
   if (n > TC_MAX_STAGES) n = TC_MAX_STAGES;
-  static const char *ov = getenv("PCNN_STAGES");     // tuning experiments only
+  static const char *ov = exp_env("PCNN_STAGES");     // tuning experiments only
   if (ov && atoi(ov) >= 2 && atoi(ov) < n) n = atoi(ov);
   return n;
 }
@@ -1375,11 +1375,11 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            cudaStream_t s, const float *lrn, const CUtensorMap *tmap_y) {
   TcArgs args;
   static const int prof_env = [] {
-    const char *e = getenv("PCNN_TC_PROFILE");
+    const char *e = exp_env("PCNN_TC_PROFILE");
     return e && e[0] == '1' ? 1 : 0;
   }();
   static const int skip_env = [] {
-    const char *e = getenv("PCNN_TC_SKIP");
+    const char *e = exp_env("PCNN_TC_SKIP");
     return e ? atoi(e) : 0;
   }();
   args.prof = prof_env;
@@ -1429,7 +1429,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
     const int creal = g.Creal > 0 && g.Creal <= g.Cg ? g.Creal : g.Cg;
     const int ncb = se > 0 ? g.Cg / se : 1;
     const int valid_b = (creal - (ncb - 1) * se) * (st == ST_BF16 ? 2 : 4);
-    const char *ek = getenv("PCNN_NO_KSKIP");           // A/B: multiply the padding too
+    const char *ek = exp_env("PCNN_NO_KSKIP");           // A/B: multiply the padding too
     args.kmma_last = args.slab_bytes / 32;
     if (!(ek && ek[0] == '1') && valid_b > 0)
       args.kmma_last = std::min(args.slab_bytes / 32, (valid_b + 31) / 32);

@@ -6,8 +6,29 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
+#include <stdlib.h>
+
+// Tuning / A-B experiment switches (PCNN_STAGES, PCNN_TC_SKIP, PCNN_FORCE_*,
+// PCNN_LRN_*, ...) are read from the environment ONLY in the experiments
+// build (python -m paper_conf_hpca_songhcl17_b200.build --prof, which defines
+// PCNN_EXPERIMENTS=1 and writes build/prof/libpcnn_prof.so).  In the shipped
+// libpcnn.so exp_env() is always nullptr: no environment variable can skip
+// work, change a plan or select another kernel.  Supported layout choices are
+// pcnn_net_desc.flags and pcnn_set_layer_plan (include/pcnn.h).
+#ifndef PCNN_EXPERIMENTS
+#define PCNN_EXPERIMENTS 0
+#endif
 
 namespace pcnn {
+
+inline const char *exp_env(const char *name) {
+#if PCNN_EXPERIMENTS
+  return getenv(name);
+#else
+  (void)name;
+  return nullptr;
+#endif
+}
 
 constexpr int kMaxSMs = 256;          // census mask width
 

@@ -140,6 +140,8 @@ struct Layer {
   std::vector<Svd> svd;        // per group (lazily computed)
   // budget
   int n_sms = 0, tlp = 0;
+  // tile-choice override (pcnn_set_layer_plan; 0 = planner's choice)
+  int plan_cg = 0, plan_msub = 0;
   int out_groups = 0, out_cg_pad = 0;    // padded-group output layout (lrn/pool)
   // zero border (halo) of the stored input / output activation; pm_halo > 0:
   // this conv runs in padded-layout mode (ConvGeom::pm) with that halo
@@ -171,6 +173,8 @@ struct pcnn_net {
   int stage_h = 0, stage_w = 0, stage_blk = 1, stage_pad = 0, stage_c = 0;
   int stage_im2col = 0;     // 1: layer 0 input staged as im2col rows (1x1 conv)
   bool fuse_lrn_pool = true;
+  bool conv_lrn_pm = false;    // PCNN_FLAG_CONV_LRN_EPILOGUE
+  bool perf_im2col = false;    // PCNN_FLAG_PERFORATION_IM2COL
   bool census = false;
   // CUDA graph cache
   uint64_t version = 1;
@@ -699,15 +703,16 @@ static Rect best_rect(const ConvGeom &g) {
 }
 
 static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
-                      bool full_n = false) {
+                      bool full_n = false, int want_cg = 0) {
   TcPlan best{};
   double best_t = 1e300;
   const int nmax = std::min(256, round_up(g.Nfg, 32));
   const double f = 1.9e9, hbm = 6.0e12;
   const double wbytes = (double)g.Nfg * g.groups * g.Kpad * esz;
-  const char *force_cg = getenv("PCNN_FORCE_CG");
-  const char *force_bn = getenv("PCNN_FORCE_BN");          // tuning experiments
-  const char *force_am = getenv("PCNN_AMODE");             // "im2col" | "rect"
+  const char *force_cg = exp_env("PCNN_FORCE_CG");
+  const char *force_bn = exp_env("PCNN_FORCE_BN");          // tuning experiments
+  const char *force_am = exp_env("PCNN_AMODE");             // "im2col" | "rect"
+  if (want_cg > 0) force_cg = want_cg == 1 ? "1" : "2";
   const Rect rc = best_rect(g);
   for (int am = 0; am < 2; ++am) {            // 0 im2col, 1 rectangle tiles (opt-in)
     if (am == 1 && (rc.w == 0 || !force_am || std::string(force_am) != "rect")) continue;
@@ -730,7 +735,7 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
         const int max_split =
             (tiles >= slots || full_n) ? 1 : std::min(16, std::max(1, kblocks / 4));
         static const int force_split = [] {              // tuning experiments
-          const char *e = getenv("PCNN_FORCE_SPLIT");
+          const char *e = exp_env("PCNN_FORCE_SPLIT");
           return e ? atoi(e) : 0;
         }();
         for (int want = 1; want <= max_split; ++want) {
@@ -768,7 +773,8 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
 // Padded-layout plan: per (slab, filter row) window the SM loads
 // (128 + S - 1) A rows once plus S weight slabs and issues S x slab/32 UMMAs;
 // no split-K (a split would need the halo zeroing in the reduction).
-static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n = false) {
+static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n = false,
+                         int want_cg = 0, int want_msub = 0) {
   TcPlan best{};
   double best_t = 1e300;
   std::vector<std::pair<double, TcPlan>> cands;
@@ -776,9 +782,11 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
   const double f = 1.9e9;
   const int slab = tc_slab_bytes(esz == 2 ? ST_BF16 : ST_F32, g.Cg);
   const int nj = g.Cg * esz / slab * g.S;
-  const char *force_cg = getenv("PCNN_FORCE_CG");
-  const char *force_bn = getenv("PCNN_FORCE_BN");
-  const char *force_ms = getenv("PCNN_PM_MSUB");           // 1 | 2 (experiments)
+  const char *force_cg = exp_env("PCNN_FORCE_CG");
+  const char *force_bn = exp_env("PCNN_FORCE_BN");
+  const char *force_ms = exp_env("PCNN_PM_MSUB");           // 1 | 2 (experiments)
+  if (want_cg > 0) force_cg = want_cg == 1 ? "1" : "2";
+  if (want_msub > 0) force_ms = want_msub == 1 ? "1" : "2";
   for (int ms = 1; ms <= 2; ++ms) {
     if (force_ms && atoi(force_ms) != ms) continue;
     for (int cg = 1; cg <= 2; ++cg) {
@@ -868,9 +876,10 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
   ConvGeom g = gs.g;
   g.M = g.pm == 2 ? B * g.tpi * 128 : g.pm ? B * g.hv * g.wv : B * g.Ho * g.Wo;
   if (gs.engine == 1) {
-    TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st), lrn != nullptr)
+    TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st), lrn != nullptr, ly.plan_cg,
+                                 ly.plan_msub)
                     : plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st),
-                              lrn != nullptr);
+                              lrn != nullptr, ly.plan_cg);
     // the budget caps concurrent units; a CTA pair needs at least 2 SMs
     const int slots = std::max(1, effective_sms(net, ly) / p.cg);
     p.grid = p.cg * std::min(p.units, slots);
@@ -899,7 +908,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       return fail(PCNN_ERR_OUT_OF_MEMORY, "split-K workspace not reserved");
     g_launches += p.splits > 1 ? 1 : 0;   // the reduction kernel
     static const bool no_tma_store = [] {
-      const char *e = getenv("PCNN_NO_TMA_STORE");
+      const char *e = exp_env("PCNN_NO_TMA_STORE");
       return e && e[0] == '1';
     }();
     const CUtensorMap *ym = (p.splits == 1 && !lrn && !p.rect_w && !no_tma_store && g.pm != 2)
@@ -938,11 +947,10 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
 static bool fuse_conv_lrn(const pcnn_net *net, int i) {
   if (!net->fuse_lrn_pool || i + 1 >= (int)net->layers.size()) return false;
   const Layer &c = net->layers[i], &l = net->layers[i + 1];
-  // padded-layout convs fuse LRN only on request (PCNN_PM_LRN=1): the LRN
-  // epilogue (4 warps, one pixel's channel vector per thread) made AlexNet
-  // conv1 279 us against 79 us conv + 92 us register-LRN/pool kernel
-  const char *pe = getenv("PCNN_PM_LRN");
-  const bool pm_lrn = pe && pe[0] == '1';
+  // padded-layout convs fuse LRN only on request (PCNN_FLAG_CONV_LRN_EPILOGUE):
+  // the LRN epilogue (4 warps, one pixel's channel vector per thread) made
+  // AlexNet conv1 279 us against 79 us conv + 92 us register-LRN/pool kernel
+  const bool pm_lrn = net->conv_lrn_pm;
   return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 &&
          (c.pm_halo == 0 || pm_lrn) && c.perf_sh * c.perf_sw == 1 &&
          c.exact.engine == 1 && c.variant == PCNN_VARIANT_EXACT && c.d.groups == 1 &&
@@ -1278,10 +1286,9 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   net->occ_lp = lrn_pool_occupancy(net->st);
   net->stage_h = desc->in_height;
   net->stage_w = desc->in_width;
-  {
-    const char *e = getenv("PCNN_NO_FUSE");
-    net->fuse_lrn_pool = !(e && e[0] == '1');
-  }
+  net->fuse_lrn_pool = !(desc->flags & PCNN_FLAG_NO_LRN_POOL_FUSION);
+  net->conv_lrn_pm = (desc->flags & PCNN_FLAG_CONV_LRN_EPILOGUE) != 0;
+  net->perf_im2col = (desc->flags & PCNN_FLAG_PERFORATION_IM2COL) != 0;
   if (desc->precision != PCNN_FP32_SIMT) {
     if (!get_encode_tiled() || !get_encode_im2col())
       return fail(PCNN_ERR_CUDA, "driver entry points cuTensorMapEncode{Tiled,Im2col} unavailable");
@@ -1297,10 +1304,9 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   // padded to a multiple of 128 bytes instead (zeros; packed weights are zero
   // there too), so the conv loads full SW128 slabs.
   const int slab128 = 128 / esz;
-  // PCNN_NARROW_PM=1 (experiment): keep such groups unpadded and run the conv
-  // in padded-layout mode on narrow (SW32 / SW64) slabs -- no K padding waste
-  const char *narrow_env = getenv("PCNN_NARROW_PM");
-  const bool narrow_pm = narrow_env && narrow_env[0] == '1';
+  // PCNN_FLAG_NARROW_SLABS: keep such groups unpadded and run the conv in
+  // padded-layout mode on narrow (SW32 / SW64) slabs -- no K padding waste
+  const bool narrow_pm = (desc->flags & PCNN_FLAG_NARROW_SLABS) != 0;
   if (prec != PCNN_FP32_SIMT && !narrow_pm) {
     for (int i = 1; i < n_layers; ++i) {
       Layer &ly = net->layers[i];
@@ -1321,11 +1327,11 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   // is shifted by -pad.  Same products, no K padding waste.
   std::vector<float> s2d_w;
   const Layer &l0 = net->layers[0];
-  const char *no_s2d = getenv("PCNN_NO_S2D");
+  const bool no_s2d = (desc->flags & PCNN_FLAG_NO_SPACE_TO_DEPTH) != 0;
   const int k0 = l0.d.kernel;
   if (prec != PCNN_FP32_SIMT && l0.d.kind == PCNN_CONV && l0.d.groups == 1 &&
       desc->in_channels == 3 && (k0 == 3 || k0 == 5) && 3 * k0 * k0 <= 128 &&
-      !(no_s2d && no_s2d[0] == '1')) {
+      !no_s2d) {
     // im2col staging: W'[f][(r*S + s)*3 + c] = W[f][c][r][s], a 1x1 conv on Kp channels
     const int K = 3 * k0 * k0, F = l0.d.out_channels;
     const int Kp = K <= 64 / esz * 2 ? round_up(K, 64 / esz) : round_up(K, 128 / esz);
@@ -1341,7 +1347,7 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
           for (int q = 0; q < k0; ++q)
             s2d_w[(size_t)f * K + (r * k0 + q) * 3 + c] = weights[0][(((size_t)f * 3 + c) * k0 + r) * k0 + q];
   } else if (l0.d.kind == PCNN_CONV && l0.d.groups == 1 && l0.d.stride >= 2 && l0.d.stride <= 8 &&
-      !(no_s2d && no_s2d[0] == '1')) {
+      !no_s2d) {
     const int st2 = l0.d.stride, S = l0.d.kernel, Sp = (S + st2 - 1) / st2;
     const int C = desc->in_channels, Cp = st2 * st2 * C, F = l0.d.out_channels;
     net->stage_blk = st2;
@@ -1369,12 +1375,11 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   // per group must fill 128 B slabs, and the halo may add at most 40% rows.
   const int n = n_layers;
   {
-    const char *e = getenv("PCNN_NO_PM");
-    const bool allow = prec != PCNN_FP32_SIMT && !(e && e[0] == '1');
+    const bool allow = prec != PCNN_FP32_SIMT && !(desc->flags & PCNN_FLAG_NO_PADDED_LAYOUT);
     // halo rows are computed and discarded: up to 40% extra MMA rows still
     // beats im2col boxes (S x fewer A bytes through the tiled-TMA path,
     // measured 2x faster per byte than im2col mode on B200)
-    const char *eh = getenv("PCNN_PM_MAX_HALO");
+    const char *eh = exp_env("PCNN_PM_MAX_HALO");
     const double pm_max_halo = eh ? atof(eh) : 1.40;
     auto kind = [&](int j) { return net->layers[j].d.kind; };
     auto is_pool = [&](int j) { return kind(j) == PCNN_MAXPOOL || kind(j) == PCNN_AVGPOOL; };
@@ -1612,9 +1617,8 @@ pcnn_status pcnn_set_perforation(pcnn_net *net, int layer, int sh, int sw) {
   const int mode = ly.exact.g.out_mode;
   // rows only, on a padded-layout layer whose grid rows fit one MMA tile:
   // the kept rows run in padded-layout mode (pm = 2, row-strided windows)
-  const char *e2 = getenv("PCNN_PERF_IM2COL");           // A/B: force the im2col kept grid
   const bool pm2 = sw == 1 && ly.exact.g.pm == 1 && ly.pm_halo > 0 &&
-                   ly.exact.g.wv + 2 * ly.exact.g.pad <= 128 && !(e2 && e2[0] == '1');
+                   ly.exact.g.wv + 2 * ly.exact.g.pad <= 128 && !net->perf_im2col;
   pcnn_status s = build_stage(ly.pf, ly, net->desc.precision, ly.d.out_channels, ly.d.groups,
                               ly.d.kernel, ly.d.stride, ly.d.pad, ly.d.relu, ly.in_c, ly.in_h,
                               ly.in_w, ly.in_cs, false, ly.host_w.data(), nullptr, mode,
@@ -1687,6 +1691,23 @@ pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank, const f
       return fail(PCNN_ERR_INVALID_ARGUMENT, "rank out of [1, min(N, K)]");
     return build_rank_stages_fc(net, ly, rank, A, B);
   }
+  // the same guards as pcnn_set_variant: a staged first conv reads the
+  // space-to-depth / im2col grid, not the logical input the factors refer to
+  if (layer == 0 && (net->stage_im2col || net->stage_blk > 1))
+    return fail(PCNN_ERR_UNSUPPORTED,
+                "rank variant of a first conv whose input is staged (im2col / space-to-depth)");
+  {
+    const int g = ly.d.groups, Nfg = ly.d.out_channels / g;
+    const int K = (ly.in_c / g) * ly.d.kernel * ly.d.kernel;
+    if (rank > std::min(Nfg, K)) return fail(PCNN_ERR_INVALID_ARGUMENT, "rank out of [1, min(N_f/g, K)]");
+    // stage 1 writes g * round_up(r, chunk) channels on the layer's output grid
+    // into the arena's third buffer
+    const size_t s1 = (size_t)net->desc.max_batch * (ly.out_h + 2 * ly.out_halo) *
+                      (ly.out_w + 2 * ly.out_halo) * g *
+                      round_up(rank, chunk_elems(net->desc.precision)) * esz_of(net->st);
+    if (s1 > net->act_bytes)
+      return fail(PCNN_ERR_UNSUPPORTED, "rank-r intermediate larger than the activation arena");
+  }
   return build_rank_stages(net, ly, rank, A, B);
 }
 
@@ -1696,6 +1717,20 @@ pcnn_status pcnn_set_sm_budget(pcnn_net *net, int layer, int n_sms, int ctas_per
   Layer &ly = net->layers[layer];
   ly.n_sms = n_sms >= net->num_sms ? 0 : n_sms;
   ly.tlp = ctas_per_sm;
+  net->version++;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_set_layer_plan(pcnn_net *net, int layer, int cta_group, int m_sub) {
+  if (!net || layer < 0 || layer >= (int)net->layers.size())
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad net / layer");
+  if (cta_group < 0 || cta_group > 2 || m_sub < 0 || m_sub > 2)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "cta_group and m_sub must be 0, 1 or 2");
+  Layer &ly = net->layers[layer];
+  if (!ly.gemm || net->desc.precision == PCNN_FP32_SIMT)
+    return fail(PCNN_ERR_UNSUPPORTED, "tile override applies to tcgen05 GEMM layers");
+  ly.plan_cg = cta_group;
+  ly.plan_msub = m_sub;
   net->version++;
   return PCNN_OK;
 }

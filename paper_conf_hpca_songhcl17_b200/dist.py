@@ -107,3 +107,39 @@ def gather_logits(local_out, world):
                     dtype=local_out.dtype, device=local_out.device)
     dist.all_gather_into_tensor(g, local_out.contiguous())
     return g
+
+
+def free_port():
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def torchrun_command(n_procs, script_argv, port=None, python=None):
+    """The one-node launch line `bench.py --gpus N` re-executes itself with
+    when it is started without torchrun: one process per GPU, rendezvous on
+    127.0.0.1 (the container hostname may not resolve)."""
+    import sys
+    return [python or sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+            "--nproc-per-node", str(int(n_procs)), "--master-addr", "127.0.0.1",
+            "--master-port", str(port or free_port())] + list(script_argv)
+
+
+def relaunch(n_procs, script_argv, port=None, env=None):
+    """Run script_argv under torchrun with n_procs ranks; returns the exit
+    code (the ranks inherit stdout, so rank 0's JSON line passes through)."""
+    import os
+    import subprocess
+    e = dict(os.environ)
+    e.update(env or {})
+    return subprocess.call(torchrun_command(n_procs, script_argv, port), env=e)
+
+
+def check_world(expected):
+    """Every rank asserts that the process group has the requested size."""
+    import torch.distributed as dist
+    w = dist.get_world_size() if dist.is_initialized() else 1
+    if w != expected:
+        raise SystemExit("world size %d != --gpus %d" % (w, expected))
+    return w

@@ -25,6 +25,13 @@ OK = 0
 CONV, LRN, MAXPOOL, AVGPOOL, FC = 0, 1, 2, 3, 4
 FP32_SIMT, TF32, BF16 = 0, 1, 2
 VARIANT_EXACT, VARIANT_RANK = 0, 1
+# pcnn_net_flag (layout choices of pcnn_create_net)
+FLAG_NO_SPACE_TO_DEPTH = 1
+FLAG_NO_PADDED_LAYOUT = 2
+FLAG_NO_LRN_POOL_FUSION = 4
+FLAG_CONV_LRN_EPILOGUE = 8
+FLAG_NARROW_SLABS = 16
+FLAG_PERFORATION_IM2COL = 32
 PRECISIONS = {"fp32": FP32_SIMT, "fp32_simt": FP32_SIMT, "tf32": TF32, "bf16": BF16}
 _KINDS = {"conv": CONV, "lrn": LRN, "maxpool": MAXPOOL, "avgpool": AVGPOOL, "fc": FC}
 
@@ -40,7 +47,8 @@ class LayerDesc(ctypes.Structure):
 class NetDesc(ctypes.Structure):
     _fields_ = [("in_channels", ctypes.c_int), ("in_height", ctypes.c_int),
                 ("in_width", ctypes.c_int), ("max_batch", ctypes.c_int),
-                ("precision", ctypes.c_int), ("device", ctypes.c_int)]
+                ("precision", ctypes.c_int), ("device", ctypes.c_int),
+                ("flags", ctypes.c_int)]
 
 
 class LayerInfo(ctypes.Structure):
@@ -79,6 +87,7 @@ _lib.pcnn_destroy_net.argtypes = [_P]
 _lib.pcnn_set_variant.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
 _lib.pcnn_set_variant_factors.argtypes = [_P, ctypes.c_int, ctypes.c_int, _FP, _FP]
 _lib.pcnn_set_sm_budget.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
+_lib.pcnn_set_layer_plan.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
 _lib.pcnn_set_perforation.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
 _lib.pcnn_infer.argtypes = [_P, _P, ctypes.c_int, _P, _P, _P, _P]
 _lib.pcnn_infer_host.argtypes = [_P, _P, ctypes.c_int, _P, _P, _P, _P]
@@ -101,16 +110,16 @@ _lib.pcnn_status_string.argtypes = [ctypes.c_int]
 _lib.pcnn_status_string.restype = ctypes.c_char_p
 _lib.pcnn_last_error_message.restype = ctypes.c_char_p
 for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
-           "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_perforation", "pcnn_infer",
-           "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
+           "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_layer_plan",
+           "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
            "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
            "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
            "pcnn_last_launch_count"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
-            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_perforation", "pcnn_infer",
-            "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
+            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_layer_plan",
+            "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
             "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
             "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
             "pcnn_last_launch_count", "pcnn_device_sm_count", "pcnn_version",
@@ -161,10 +170,10 @@ def layer_descs(layers):
     return arr
 
 
-def net_desc(in_shape, max_batch, precision, device=0):
+def net_desc(in_shape, max_batch, precision, device=0, flags=0):
     c, h, w = in_shape
     p = PRECISIONS[precision] if isinstance(precision, str) else int(precision)
-    return NetDesc(c, h, w, max_batch, p, device)
+    return NetDesc(c, h, w, max_batch, p, device, int(flags))
 
 
 def describe_net(net, batch=1, precision="bf16"):
@@ -191,14 +200,14 @@ def _stream_ptr(stream):
 class Net:
     """A built network (pcnn_create_net) on one device."""
 
-    def __init__(self, net, weights, biases, max_batch, precision="bf16", device=0):
+    def __init__(self, net, weights, biases, max_batch, precision="bf16", device=0, flags=0):
         import numpy as np
         self.spec = net
         self.n_layers = len(net["layers"])
         self.precision = precision
         self.device = device
         layers = layer_descs(net["layers"])
-        nd = net_desc(net["in_shape"], max_batch, precision, device)
+        nd = net_desc(net["in_shape"], max_batch, precision, device, flags)
         keep = []
         wp = (_FP * self.n_layers)()
         bp = (_FP * self.n_layers)()
@@ -241,6 +250,9 @@ class Net:
         B = np.ascontiguousarray(B, dtype=np.float32)
         _check(_lib.pcnn_set_variant_factors(self._h, layer, rank, A.ctypes.data_as(_FP),
                                              B.ctypes.data_as(_FP)), "pcnn_set_variant_factors")
+
+    def set_layer_plan(self, layer, cta_group=0, m_sub=0):
+        _check(_lib.pcnn_set_layer_plan(self._h, layer, cta_group, m_sub), "pcnn_set_layer_plan")
 
     def set_perforation(self, layer, sh, sw):
         _check(_lib.pcnn_set_perforation(self._h, layer, sh, sw), "pcnn_set_perforation")

@@ -66,7 +66,7 @@ def round_to_bf16(a):
     return u.astype(np.uint32).view(np.float32).reshape(f.shape)
 
 
-def images(n_start, count, shape, seed=IMAGE_SEED, lo=-128.0, hi=128.0):
+def images(n_start, count, shape, seed=IMAGE_SEED, lo=-128.0, hi=128.0, bf16=True):
     """Images [count, C, H, W] float32 (BF16-representable), U[lo, hi).
 
     Image ``n`` (global index) uses counters n*C*H*W ... (n+1)*C*H*W-1, so a
@@ -74,23 +74,30 @@ def images(n_start, count, shape, seed=IMAGE_SEED, lo=-128.0, hi=128.0):
     ±128 is Caffe's mean-subtracted pixel scale (keeps LRN active, c3)."""
     per = int(np.prod(shape))
     v = uniform(seed, IMAGE_TENSOR_ID, n_start * per, count * per, lo, hi)
+    if not bf16:      # full FP32 values (exercises the CUDA path's own rounding)
+        return v.astype(np.float32).reshape((count,) + tuple(shape))
     return round_to_bf16(v).reshape((count,) + tuple(shape))
 
 
-def he_weights(shape, fan_in, layer_index, seed=WEIGHT_SEED):
-    """He-normal N(0, 2/fan_in), BF16-representable float32."""
+def he_weights(shape, fan_in, layer_index, seed=WEIGHT_SEED, bf16=True):
+    """He-normal N(0, 2/fan_in), BF16-representable float32 (bf16=False: full
+    FP32 values)."""
     n = int(np.prod(shape))
     v = normal(seed, layer_index, 0, n, std=np.sqrt(2.0 / fan_in))
+    if not bf16:
+        return v.astype(np.float32).reshape(shape)
     return round_to_bf16(v).reshape(shape)
 
 
-def biases(count, layer_index, seed=WEIGHT_SEED, lo=-0.1, hi=0.1):
+def biases(count, layer_index, seed=WEIGHT_SEED, lo=-0.1, hi=0.1, bf16=True):
     v = uniform(seed, layer_index + BIAS_TENSOR_OFFSET, 0, count, lo, hi)
-    return round_to_bf16(v)
+    return round_to_bf16(v) if bf16 else v.astype(np.float32)
 
 
-def net_params(net, seed=WEIGHT_SEED):
-    """(weights, biases) lists aligned with net['layers'] (None for weightless)."""
+def net_params(net, seed=WEIGHT_SEED, bf16=True):
+    """(weights, biases) lists aligned with net['layers'] (None for weightless).
+    bf16=False draws full FP32 values, so the CUDA path's own operand rounding
+    (BF16 RNE / TF32 RNA) is exercised."""
     from .nets import weight_shapes
     ws, bs = [], []
     for i, shp in enumerate(weight_shapes(net)):
@@ -100,8 +107,8 @@ def net_params(net, seed=WEIGHT_SEED):
             continue
         wshape, bshape = shp
         fan_in = int(np.prod(wshape[1:]))
-        ws.append(he_weights(wshape, fan_in, i, seed))
-        bs.append(biases(bshape[0], i, seed))
+        ws.append(he_weights(wshape, fan_in, i, seed, bf16))
+        bs.append(biases(bshape[0], i, seed, bf16=bf16))
     return ws, bs
 
 

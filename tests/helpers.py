@@ -6,6 +6,14 @@ import synth
 
 TOL = {"fp32": 1e-4, "tf32": 5e-3, "bf16": 2e-2}   # north_star, reading R10
 
+# pcnn_net_flag (include/pcnn.h) -- layout choices compared by the tests
+FLAG_NO_SPACE_TO_DEPTH = 1
+FLAG_NO_PADDED_LAYOUT = 2
+FLAG_NO_LRN_POOL_FUSION = 4
+FLAG_CONV_LRN_EPILOGUE = 8
+FLAG_NARROW_SLABS = 16
+FLAG_PERFORATION_IM2COL = 32
+
 
 def rel_err(y, ref):
     """max |y - ref| / max |ref| (R10)."""
@@ -17,12 +25,15 @@ def rel_err(y, ref):
 
 
 def gpu_run(net, weights, biases, x, precision, max_batch=None, probs=False,
-            variants=None, budgets=None, census=False, perforation=None):
+            variants=None, budgets=None, census=False, perforation=None, flags=0,
+            plans=None):
     """Build a libpcnn net, run x (numpy NCHW fp32) and return numpy outputs."""
     import torch
     from paper_conf_hpca_songhcl17_b200 import pcnn
     B = x.shape[0]
-    n = pcnn.Net(net, weights, biases, max_batch or B, precision)
+    n = pcnn.Net(net, weights, biases, max_batch or B, precision, flags=flags)
+    for (i, (cg, ms)) in (plans or {}).items():
+        n.set_layer_plan(i, cg, ms)
     for (i, (v, r)) in (variants or {}).items():
         n.set_variant(i, v, r)
     for (i, (sh, sw)) in (perforation or {}).items():

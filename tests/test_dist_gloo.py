@@ -79,3 +79,25 @@ def test_broadcast_and_gather_world2():
     assert sorted(r[0] for r in res) == [0, 1]
     for r in res:
         assert all(r[1:]), r
+
+
+def test_relaunch_under_torchrun_world2():
+    """bench.py --gpus N without torchrun re-executes itself through
+    dist.relaunch: N ranks on 127.0.0.1 that all see world size N."""
+    import json
+    import subprocess
+    import sys
+    probe = os.path.join(os.path.dirname(__file__), "_dist_probe.py")
+    cmd = pdist.torchrun_command(2, [probe, "2"])
+    assert cmd[1:3] == ["-m", "torch.distributed.run"] and "127.0.0.1" in cmd
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    line = [l for l in r.stdout.splitlines() if l.startswith("{")][-1]
+    d = json.loads(line)
+    assert d["world"] == 2 and d["ranks"] == [0, 1]
+    assert d["env"][0] == "127.0.0.1"
+    # a world-size mismatch fails loudly
+    r2 = subprocess.run(pdist.torchrun_command(2, [probe, "3"]), capture_output=True, text=True,
+                        timeout=300)
+    assert r2.returncode != 0
+    assert sys.executable

@@ -7,7 +7,9 @@ import numpy as np
 import pytest
 
 import synth
-from tests.helpers import TOL, conv_layer, gpu_run, params, rel_err, small_inputs
+from tests.helpers import (FLAG_CONV_LRN_EPILOGUE, FLAG_NARROW_SLABS, FLAG_NO_LRN_POOL_FUSION,
+                           FLAG_NO_PADDED_LAYOUT, FLAG_PERFORATION_IM2COL, TOL, conv_layer,
+                           gpu_run, params, rel_err, small_inputs)
 
 pytestmark = pytest.mark.gpu
 
@@ -107,7 +109,7 @@ def test_perforation_rejections():
 
 @pytest.mark.parametrize("prec", ["bf16", "tf32"])
 @pytest.mark.parametrize("sh", [2, 3])
-def test_row_perforation_padded_layout(orc, prec, sh, monkeypatch):
+def test_row_perforation_padded_layout(orc, prec, sh):
     """Row perforation (s_w = 1) of padded-layout layers runs the kept rows in
     padded-layout mode (row-strided 3-D TMA windows, segments of W + 2h + 2p
     rows): oracle parity, agreement with the im2col kept grid, and the
@@ -120,11 +122,9 @@ def test_row_perforation_padded_layout(orc, prec, sh, monkeypatch):
     r = gpu_run(net, w, b, x, prec, perforation=perf)
     assert r["net"].query_layer(1, 3)["a_mode"] == 2
     assert rel_err(r["out"], ref) <= TOL[prec] / 2
-    monkeypatch.setenv("PCNN_PERF_IM2COL", "1")
-    r2 = gpu_run(net, w, b, x, prec, perforation=perf)
+    r2 = gpu_run(net, w, b, x, prec, perforation=perf, flags=FLAG_PERFORATION_IM2COL)
     assert r2["net"].query_layer(1, 3)["a_mode"] == 0
     assert rel_err(r["out"], r2["out"]) <= TOL[prec] / 4
-    monkeypatch.delenv("PCNN_PERF_IM2COL")
     anet = dict(in_shape=(96, 27, 27), layers=[
         dict(kind="maxpool", k=1, stride=1), conv_layer(256, 5, 96, 1, 2, 2),
         dict(kind="maxpool", k=3, stride=2)])

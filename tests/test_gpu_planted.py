@@ -1,17 +1,31 @@
-"""Top-1 on the planted-class set (SURVEY.md §8(d) / DESIGN.md R10), where
-top-1 is meaningful: images are noisy copies of class prototypes and fc8's
-first rows are the normalised, centred FP64 fc7 features of those
-prototypes (built here by the oracle).  north_star: identical top-1 on
->= 99.9% of images -- with 64 images that is all of them."""
+"""Top-1 on the planted-class sets (BASELINE.md "Parity
+sets": AlexNet >= 1000 and VGG-16 >= 1000 planted-class images; DESIGN.md
+R10), where top-1 is meaningful: images are noisy copies of class prototypes
+and fc8's first rows are the normalised, centred FP64 fc7 features of those
+prototypes, computed by the oracle.
+
+north_star asks for the oracle's top-1 on >= 99.9% of images.  The oracle
+runs on a sample (FP64 VGG-16 costs ~1 s per image per core); for every other
+image the identity follows from parity: where the CUDA logits' top-1 / top-2
+margin exceeds 2 x tol x max|logit| (max over the whole set) and the logits
+are within tol x max|logit|
+of the oracle's (checked on the sample), the oracle's top-1 is the same
+class.  So each image counts only when (a) its CUDA top-1 is the planted
+label and (b) its margin clears that band.
+"""
+import os
+
 import numpy as np
 import pytest
 import torch
 
 import synth
-from tests.helpers import TOL, gpu_run, params, rel_err
+from tests.helpers import TOL, rel_err
 
 pytestmark = pytest.mark.gpu
 N_CLASSES = 100
+N_IMAGES = 1024
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -20,13 +34,28 @@ def _need_gpu():
         pytest.skip("no GPU")
 
 
-@pytest.fixture(scope="module")
-def planted(orc):
-    net = synth.alexnet()
-    w, b = params(net)
+def _prototype_features(orc, name, net, w, b):
+    """fc7 features of the prototypes: the committed oracle output
+    (tools/make_planted_golden.py) when present, else computed here."""
+    path = os.path.join(GOLD, "planted_%s_fc7.npz" % name)
+    if os.path.exists(path):
+        d = np.load(path)
+        if int(d["n_classes"]) == N_CLASSES and int(d["seed_w"]) == synth.WEIGHT_SEED:
+            return np.asarray(d["feats"], dtype=np.float64)
     protos = synth.prototypes(N_CLASSES, net["in_shape"])
     _, outs = orc.run_net(net, w, b, protos, return_all=True)
-    feats = np.asarray(outs[-2], dtype=np.float64)          # fc7 output [n, 4096]
+    return np.asarray(outs[-2], dtype=np.float64)
+
+
+_CACHE = {}
+
+
+def planted(orc, name):
+    if name in _CACHE:
+        return _CACHE[name]
+    net = synth.get_net(name)
+    w, b = synth.net_params(net)
+    feats = _prototype_features(orc, name, net, w, b)
     mean = feats.mean(0)
     F = feats - mean
     F /= np.linalg.norm(F, axis=1, keepdims=True)
@@ -36,17 +65,42 @@ def planted(orc):
     b = list(b)
     w[-1] = synth.round_to_bf16(W8)
     b[-1] = synth.round_to_bf16(-(W8 @ mean))
-    return net, w, b
+    _CACHE[name] = (net, w, b)
+    return _CACHE[name]
 
 
-@pytest.mark.parametrize("prec", ["bf16", "tf32"])
-def test_planted_top1(orc, planted, prec):
-    net, w, b = planted
-    x, labels = synth.planted_images(0, 64, net["in_shape"], N_CLASSES)
-    out = gpu_run(net, w, b, x, prec)["out"]
-    top1 = out.argmax(1)
-    assert (top1 == labels).mean() >= 0.999, (top1 != labels).sum()
-    ref = orc.run_net(net, w, b, x[:8])
-    assert (ref.argmax(1) == labels[:8]).all()
-    assert (top1[:8] == ref.argmax(1)).all()
-    assert rel_err(out[:8], ref) <= TOL[prec]
+def _run_all(net, w, b, prec, chunk):
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    n = pcnn.Net(net, w, b, max_batch=chunk, precision=prec)
+    outs, labels = [], []
+    for s in range(0, N_IMAGES, chunk):
+        x, lab = synth.planted_images(s, chunk, net["in_shape"], N_CLASSES)
+        o, _, _ = n.infer(torch.from_numpy(x).cuda())
+        outs.append(o.cpu().numpy())
+        labels.append(lab)
+    n.close()
+    return np.concatenate(outs), np.concatenate(labels)
+
+
+@pytest.mark.parametrize("name,prec,n_oracle", [
+    ("alexnet", "bf16", 32), ("alexnet", "tf32", 32),
+    ("vgg16", "bf16", 3), ("vgg16", "tf32", 3)])
+def test_planted_top1_1024(orc, name, prec, n_oracle):
+    net, w, b = planted(orc, name)
+    out, labels = _run_all(net, w, b, prec, 256 if name == "alexnet" else 128)
+    assert out.shape == (N_IMAGES, 1000)
+    tol = TOL[prec]
+    # parity on the oracle sample (spread over the set)
+    idx = np.linspace(0, N_IMAGES - 1, n_oracle).astype(int)
+    xs = np.concatenate([synth.planted_images(int(i), 1, net["in_shape"], N_CLASSES)[0]
+                         for i in idx])
+    ref = orc.run_net(net, w, b, xs)
+    assert rel_err(out[idx], ref) <= tol
+    assert (ref.argmax(1) == labels[idx]).all()
+    # every image: planted label and a margin outside the parity band
+    srt = np.sort(out, axis=1)
+    margin = srt[:, -1] - srt[:, -2]
+    safe = margin > 2 * tol * np.abs(out).max()
+    hit = out.argmax(1) == labels
+    frac = float((hit & safe).mean())
+    assert frac >= 0.999, (frac, int((~hit).sum()), int((~safe).sum()))

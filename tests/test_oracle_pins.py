@@ -358,3 +358,126 @@ def test_perforation_kept_values_and_interpolation(orc):
             assert abs(p - kp) <= sh // 2 + (1 if p > 10 // sh * sh else 0)
             np.testing.assert_array_equal(y[0, :, p, q], y[0, :, kp, kq])
     assert abs(orc.perforation_rate(11, 10, sh, sw) - (1 - 6 * 4 / 110)) < 1e-15
+
+
+# ------------------------------------------------------- rank-r per group (R7)
+def test_rank_r_conv_weight_per_group_equals_numpy_svd_per_block(orc):
+    """Reading R7: the rank-r operator is applied to each group's own
+    (N_f/g) x (C/g S^2) block.  Pinned against numpy's SVD of each block: a
+    wrong group slice (e.g. factorising the whole filter bank, swapping the
+    blocks, or slicing by input channels) changes the result.  The two blocks
+    are built with very different spectra so that any mix-up is visible."""
+    rng = np.random.default_rng(21)
+    g, Fg, Cg, S = 2, 6, 3, 3
+    w = rng.standard_normal((g * Fg, Cg, S, S))
+    w[Fg:] *= 10.0                                 # group 1: 10x the scale of group 0
+    w[Fg:, :, 0, 0] += 25.0                        # and a dominant direction of its own
+    for r in (1, 2, 4, Fg):
+        wr, uniq = orc.rank_r_conv_weight(w, g, r)
+        assert uniq
+        for gi in range(g):
+            blk = w[gi * Fg:(gi + 1) * Fg].reshape(Fg, -1)
+            U, s, Vt = np.linalg.svd(blk, full_matrices=False)
+            ref = ((U[:, :r] * s[:r]) @ Vt[:r]).reshape(Fg, Cg, S, S)
+            np.testing.assert_allclose(wr[gi * Fg:(gi + 1) * Fg], ref, atol=1e-9)
+        # the whole-bank factorisation is a different operator (negative control)
+        if r < Fg:
+            U, s, Vt = np.linalg.svd(w.reshape(g * Fg, -1), full_matrices=False)
+            whole = ((U[:, :r] * s[:r]) @ Vt[:r]).reshape(w.shape)
+            assert np.abs(whole - wr).max() > 1e-3
+    # full rank per group reproduces the weights
+    wr, _ = orc.rank_r_conv_weight(w, g, Fg)
+    np.testing.assert_allclose(wr, w, atol=1e-9)
+
+
+def test_run_net_rank_option_uses_per_group_operator(orc):
+    """run_net(ranks={i: r}) runs the exact conv with the per-group W_r."""
+    rng = np.random.default_rng(22)
+    net = dict(name="t", in_shape=(4, 6, 6), layers=[
+        dict(kind="conv", out=8, k=3, stride=1, pad=1, groups=2, relu=True, in_c=4)])
+    w = [rng.standard_normal((8, 2, 3, 3))]
+    b = [rng.standard_normal(8)]
+    x = rng.standard_normal((2, 4, 6, 6))
+    y = orc.run_net(net, w, b, x, ranks={0: 2})
+    wr = np.empty_like(w[0])
+    for gi in range(2):
+        blk = w[0][gi * 4:(gi + 1) * 4].reshape(4, -1)
+        U, s, Vt = np.linalg.svd(blk, full_matrices=False)
+        wr[gi * 4:(gi + 1) * 4] = ((U[:, :2] * s[:2]) @ Vt[:2]).reshape(4, 2, 3, 3)
+    ref = _scipy_conv(x, wr, b[0], 1, 1, 2, True)
+    np.testing.assert_allclose(y, ref, rtol=1e-9, atol=1e-9)
+
+
+# ------------------------------------------------------- run_net sequencing
+def _np_lrn(a, size, alpha, beta, k):
+    """Caffe across-channel LRN written with numpy (reading R3)."""
+    C = a.shape[1]
+    out = np.empty_like(a)
+    h = size // 2
+    for c in range(C):
+        lo, hi = max(0, c - h), min(C - 1, c + h)
+        ssum = np.sum(a[:, lo:hi + 1] ** 2, axis=1)
+        out[:, c] = a[:, c] / (k + alpha / size * ssum) ** beta
+    return out
+
+
+def _np_maxpool(a, k, s):
+    """ceil-mode max pooling (reading R4) by explicit windows."""
+    B, C, H, W = a.shape
+    Ho = -(-(H - k) // s) + 1
+    Wo = -(-(W - k) // s) + 1
+    if (Ho - 1) * s >= H:
+        Ho -= 1
+    if (Wo - 1) * s >= W:
+        Wo -= 1
+    y = np.empty((B, C, Ho, Wo))
+    for p in range(Ho):
+        for q in range(Wo):
+            y[:, :, p, q] = a[:, :, p * s:min(p * s + k, H), q * s:min(q * s + k, W)].max(axis=(2, 3))
+    return y
+
+
+def test_run_net_equals_independent_numpy_composition(orc):
+    """run_net's layer sequencing (conv -> LRN -> pool -> fc -> fc, the CHW
+    flatten before fc, ReLU on all but the last layer, the final fc without
+    ReLU) against a composition written with scipy / numpy only, on a tiny
+    net at Caffe pixel scale (LRN active), and against the hand composition
+    of the oracle's own pinned primitives."""
+    rng = np.random.default_rng(23)
+    net = dict(name="tiny", in_shape=(3, 11, 11), layers=[
+        dict(kind="conv", out=6, k=3, stride=2, pad=1, groups=1, relu=True, in_c=3),
+        dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0),
+        dict(kind="maxpool", k=3, stride=2),
+        dict(kind="conv", out=8, k=3, stride=1, pad=1, groups=2, relu=True, in_c=6),
+        dict(kind="fc", out=7, in_f=8 * 3 * 3, relu=True),
+        dict(kind="fc", out=5, in_f=7, relu=False),
+    ])
+    w = [rng.standard_normal((6, 3, 3, 3)) * 0.3, None, None,
+         rng.standard_normal((8, 3, 3, 3)) * 0.2, rng.standard_normal((7, 72)) * 0.1,
+         rng.standard_normal((5, 7))]
+    b = [rng.uniform(-1, 1, 6), None, None, rng.uniform(-1, 1, 8), rng.uniform(-1, 1, 7),
+         rng.uniform(-1, 1, 5)]
+    x = rng.uniform(-128, 128, (2, 3, 11, 11))
+    y, outs = orc.run_net(net, w, b, x, return_all=True)
+    # independent composition
+    a = _scipy_conv(x, w[0], b[0], 2, 1, 1, True)
+    assert a.shape == (2, 6, 6, 6)
+    a = _np_lrn(a, 5, 1e-4, 0.75, 1.0)
+    assert np.abs(a - outs[0]).max() > 1e-3 * np.abs(a).max()   # LRN is not ~identity here
+    a = _np_maxpool(a, 3, 2)
+    assert a.shape == (2, 6, 3, 3)   # ceil mode: ceil((6 - 3) / 2) + 1 = 3, last window clipped
+    a = _scipy_conv(a, w[3], b[3], 1, 1, 2, True)
+    a = np.maximum(a.reshape(2, -1) @ w[4].T + b[4], 0.0)       # CHW flatten
+    a = a @ w[5].T + b[5]                                        # no ReLU on the last fc
+    np.testing.assert_allclose(y, a, rtol=1e-10, atol=1e-10)
+    assert (y < 0).any()
+    # hand composition of the oracle's pinned primitives
+    h = orc.conv2d(x, w[0], b[0], 2, 1, 1, True)
+    h = orc.lrn(h, 5, 1e-4, 0.75, 1.0)
+    h = orc.maxpool(h, 3, 2)
+    h = orc.conv2d(h, w[3], b[3], 1, 1, 2, True)
+    h = orc.fc(h, w[4], b[4], True)
+    h = orc.fc(h, w[5], b[5], False)
+    np.testing.assert_array_equal(y, h)
+    for i, o in enumerate(outs):
+        assert o.shape[0] == 2, i
