@@ -68,6 +68,9 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-extra", action="store_true", help="skip the 'also' workloads")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--minimal", action="store_true",
+                    help="profiling: only the warm-up and the timed steps of the main workload "
+                         "(no graph-replay pass, e2e, energy, sweep or extras)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     a = ap.parse_args()
     if a.batch is None:
@@ -341,7 +344,7 @@ def timed_steps(ctx, step, steps, sampler=None):
 
 
 def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
-            global_batch=None, label=None):
+            global_batch=None, label=None, minimal=False):
     """One workload: build the net (weights broadcast once for N > 1), warm
     up, time `steps` steps with live per-layer events, then the same steps
     replayed from the cached CUDA graph; optionally the end-to-end host-buffer
@@ -384,10 +387,13 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
     layer_ms, nsteps = n.read_layer_timing()
     launches = n.last_launch_count()
     value = world * B * steps / (ms / 1000.0)
-    for _ in range(2):
-        step()
-    msg = timed_steps(ctx, step, steps)
-    value_graph = world * B * steps / (msg / 1000.0)
+    if minimal:
+        value_graph = None
+    else:
+        for _ in range(2):
+            step()
+        msg = timed_steps(ctx, step, steps)
+        value_graph = world * B * steps / (msg / 1000.0)
     torch.cuda.synchronize()
     logits = (gathered if world > 1 else out).cpu().numpy()
     infos = [n.query_layer(i, B) for i in range(n.n_layers)]
@@ -401,7 +407,7 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
         "workload": label or "%s_exact_b%d_%s" % (net_name, B, precision),
         "value": round(value, 1), "unit": "images/sec", "ms_per_step": round(total_step_ms, 4),
         "n_gpus": world, "batch_per_gpu": B, "global_batch": world * B, "precision": precision,
-        "value_graph_replay": round(value_graph, 1),
+        "value_graph_replay": round(value_graph, 1) if value_graph else None,
         "roofline": conv_roofline(n, infos, layer_ms, nsteps, precision, ctx.peaks, ctx.peak_src),
         "per_layer": per_layer, "gpu_launches": int(launches * steps),
         "launches_per_step": launches, "weights_broadcast_ms": round(bcast_ms, 3),
@@ -504,8 +510,18 @@ def main():
     sampler = ClockSampler(local)
     sampler.start()
     main_res, n, (net, w, b), bufs = measure(
-        ctx, a.net, a.precision, a.batch, a.steps, a.warmup, sampler=sampler, e2e=True,
-        global_batch=a.global_batch)
+        ctx, a.net, a.precision, a.batch, a.steps, a.warmup, sampler=sampler, e2e=not a.minimal,
+        global_batch=a.global_batch, minimal=a.minimal)
+    if a.minimal:
+        sampler.stop()
+        if rank == 0:
+            print(json.dumps({"metric": METRIC, "value": main_res["value"], "unit": "images/sec",
+                              "ms_per_step": main_res["ms_per_step"], "minimal": True,
+                              "per_layer": main_res["per_layer"]}))
+        n.close()
+        if world > 1:
+            dist.destroy_process_group()
+        return
     B = main_res["batch_per_gpu"]
 
     # board energy per image (NVML counter over >= 1 s of steps; the eq. 15

@@ -149,7 +149,10 @@ typedef struct {
     int a_mode;         /* tcgen05 A-operand addressing: 0 = TMA im2col over
                            output pixels, 1 = rectangle tiles (opt-in),
                            2 = padded-layout shifted window (one TMA row
-                           window per filter row feeds all S taps)           */
+                           window per filter row feeds all S taps),
+                           3 = FC weight stream (tile_m = weight rows per
+                           CTA, tile_n = images per UMMA, splits = K split
+                           of a CTA cluster)                                 */
     int halo_in, halo_out; /* zero border of the stored input / output
                            activation layouts ([B][H+2h][W+2h][C])           */
     int cta_group;      /* SMs per GEMM tile: 2 for CTA-pair tiles, else 1   */
@@ -268,8 +271,10 @@ pcnn_status pcnn_infer(pcnn_net *net, const float *d_images, int batch,
  * much longer to copy than to infer (batch >= 64 and the copy per image > 2x
  * the modelled compute per image, e.g. AlexNet), the batch runs as 4 chunks
  * whose host->device copies (on a library stream) overlap the previous
- * chunk's inference; per-image results then come from chunk-sized launches
- * (same values up to the split-K grouping of the FC layers). */
+ * chunk's inference.  Per-image results are bitwise those of pcnn_infer on
+ * the whole batch (the FC K split is batch-independent; conv layers split K
+ * only when their tiles cannot fill the device, which no chunk >= 16 images
+ * of AlexNet / VGG-16 reaches). */
 pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch,
                             float *h_out, float *h_probs, float *h_entropy,
                             void *stream);

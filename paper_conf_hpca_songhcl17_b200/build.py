@@ -25,8 +25,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",
          "-I" + os.path.join(ROOT, "include")]
-SOURCES = ["kernels_tc.cu", "kernels_simt.cu", "runtime.cu", "svd.cpp"]
-HEADERS = ["pcnn_internal.h", "budget.cuh", "svd.h", "lrn_math.cuh"]
+SOURCES = ["kernels_tc.cu", "kernels_fc.cu", "kernels_simt.cu", "runtime.cu", "svd.cpp"]
+HEADERS = ["pcnn_internal.h", "budget.cuh", "svd.h", "lrn_math.cuh", "tc_ptx.cuh"]
 
 
 def _newer(src_list, target):

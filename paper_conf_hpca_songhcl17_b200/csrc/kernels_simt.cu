@@ -82,6 +82,7 @@ template <int ST>
 __global__ void __launch_bounds__(256)
 stage_input_kernel(const float *__restrict__ x, void *y, int B, int C, int H, int W, int Hs,
                    int Ws, int Cs, int blk, int pad, int tf32_round) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int VN = Vec16<ST>::N;
   const int chunks = Cs / VN;
   const long long total = (long long)B * Hs * Ws * chunks;
@@ -119,6 +120,7 @@ template <int ST>
 __global__ void __launch_bounds__(256)
 stage_rows_kernel(const float *__restrict__ x, void *y, int C, int H, int W, int Hs, int Ws,
                   int Cs, int blk, int pad, int tf32_round) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   extern __shared__ float rows[];                  // [blk][C][W] then the channel map
   constexpr int VN = Vec16<ST>::N;
   const int hs = blockIdx.x % Hs;
@@ -178,6 +180,7 @@ template <int ST, int BLK>
 __global__ void __launch_bounds__(256)
 stage_c3_kernel(const float *__restrict__ x, void *y, int H, int W, int Hs, int Ws, int Cs,
                 int pad, int tf32_round) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int C = 3;
   constexpr int VN = Vec16<ST>::N;
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
@@ -242,6 +245,7 @@ template <int ST, int S>
 __global__ void __launch_bounds__(256)
 stage_im2col_kernel(const float *__restrict__ x, void *y, int H, int W, int Ho, int Wo, int Kp,
                     int st, int pad, int halo, int tf32_round) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int C = 3, K = S * S * C;
   constexpr int VN = Vec16<ST>::N;
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
@@ -301,6 +305,7 @@ template <int ST>
 __global__ void __launch_bounds__(256)
 stage_gather3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Ho, int Wo,
                      int Kp, int D, int step, int pad, int halo, int rows_per_cta, int tf32_round) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int C = 3;
   constexpr int VN = Vec16<ST>::N;
   extern __shared__ __align__(16) float g3_rows[];   // [span*C][Wrow] input rows, 16 B-aligned copies
@@ -443,13 +448,13 @@ static cudaError_t launch_gather3(const float *x, void *y, int st, int B, int H,
     if (smem > 48 * 1024)
       cudaFuncSetAttribute(stage_gather3_kernel<ST_BF16>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    stage_gather3_kernel<ST_BF16><<<grid, 256, smem, s>>>(x, y, B, H, W, Ho, Wo, Kp, D, step,
+    launch_pdl(stage_gather3_kernel<ST_BF16>, dim3(grid), dim3(256), smem, s, x, y, B, H, W, Ho, Wo, Kp, D, step,
                                                            pad, halo, R, 0);
   } else {
     if (smem > 48 * 1024)
       cudaFuncSetAttribute(stage_gather3_kernel<ST_F32>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    stage_gather3_kernel<ST_F32><<<grid, 256, smem, s>>>(x, y, B, H, W, Ho, Wo, Kp, D, step,
+    launch_pdl(stage_gather3_kernel<ST_F32>, dim3(grid), dim3(256), smem, s, x, y, B, H, W, Ho, Wo, Kp, D, step,
                                                           pad, halo, R, tf32_round);
   }
   return cudaGetLastError();
@@ -517,6 +522,7 @@ template <int ST, int S>
 __global__ void __launch_bounds__(256)
 stage_im2c3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Kp, int halo,
                    int R, int tf32_round) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int C = 3, PAD = S / 2, NREAL = S * S * C;
   constexpr int VN = Vec16<ST>::N;
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
@@ -605,7 +611,7 @@ cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, i
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);            \
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stage_im2c3_kernel<STT, 3>, 256, smem); \
     const unsigned grid = (unsigned)std::min<long long>(tiles, (long long)sms * std::max(occ, 1)); \
-    stage_im2c3_kernel<STT, 3><<<grid, 256, smem, s>>>(x, y, B, H, W, Kp, halo, R, tf32_round); \
+    launch_pdl(stage_im2c3_kernel<STT, 3>, dim3(grid), dim3(256), smem, s, x, y, B, H, W, Kp, halo, R, tf32_round); \
   } while (0)
       if (st == ST_BF16) PCNN_IC3(ST_BF16);
       else PCNN_IC3(ST_F32);
@@ -619,7 +625,7 @@ cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, i
   if (smem > 48 * 1024) return cudaErrorInvalidValue;
   const unsigned grid = (unsigned)((long long)B * Ho);
 #define PCNN_IM2COL(STT, SS) \
-  stage_im2col_kernel<STT, SS><<<grid, 256, smem, s>>>(x, y, H, W, Ho, Wo, Kp, stride, pad, halo, tf32_round)
+  launch_pdl(stage_im2col_kernel<STT, SS>, dim3(grid), dim3(256), smem, s, x, y, H, W, Ho, Wo, Kp, stride, pad, halo, tf32_round)
   if (st == ST_BF16) {
     if (S == 3) PCNN_IM2COL(ST_BF16, 3); else PCNN_IM2COL(ST_BF16, 5);
   } else {
@@ -642,6 +648,7 @@ template <int ST>
 __global__ void __launch_bounds__(256)
 stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Hs, int Ws,
                   int Cs, int R, int tf32_round) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int C = 3, BLK = 4;
   constexpr int VN = Vec16<ST>::N;
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
@@ -747,7 +754,7 @@ static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int
                            (int)smem);                                                         \
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, stage_s2d4_kernel<STT>, 256, smem);    \
     const unsigned grid = (unsigned)std::min<long long>(tiles, (long long)sms * std::max(occ, 1)); \
-    stage_s2d4_kernel<STT><<<grid, 256, smem, s>>>(x, y, B, H, W, Hs, Ws, Cs, R, tf32_round);  \
+    launch_pdl(stage_s2d4_kernel<STT>, dim3(grid), dim3(256), smem, s, x, y, B, H, W, Hs, Ws, Cs, R, tf32_round);  \
   } while (0)
   if (st == ST_BF16) PCNN_S2D(ST_BF16);
   else PCNN_S2D(ST_F32);
@@ -771,14 +778,14 @@ cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, in
     if (smem <= 48 * 1024) {
       if (st == ST_BF16) {
         if (blk == 4)
-          stage_c3_kernel<ST_BF16, 4><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, 0);
+          launch_pdl(stage_c3_kernel<ST_BF16, 4>, dim3(grid), dim3(256), smem, s, x, y, H, W, Hs, Ws, Cs, pad, 0);
         else
-          stage_c3_kernel<ST_BF16, 1><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, 0);
+          launch_pdl(stage_c3_kernel<ST_BF16, 1>, dim3(grid), dim3(256), smem, s, x, y, H, W, Hs, Ws, Cs, pad, 0);
       } else {
         if (blk == 4)
-          stage_c3_kernel<ST_F32, 4><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, tf32_round);
+          launch_pdl(stage_c3_kernel<ST_F32, 4>, dim3(grid), dim3(256), smem, s, x, y, H, W, Hs, Ws, Cs, pad, tf32_round);
         else
-          stage_c3_kernel<ST_F32, 1><<<grid, 256, smem, s>>>(x, y, H, W, Hs, Ws, Cs, pad, tf32_round);
+          launch_pdl(stage_c3_kernel<ST_F32, 1>, dim3(grid), dim3(256), smem, s, x, y, H, W, Hs, Ws, Cs, pad, tf32_round);
       }
       return cudaGetLastError();
     }
@@ -787,10 +794,10 @@ cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, in
   if (rows_bytes <= 48 * 1024 && blk <= 15) {
     const long long grid = (long long)B * Hs;
     if (st == ST_BF16)
-      stage_rows_kernel<ST_BF16><<<(unsigned)grid, 256, rows_bytes, s>>>(x, y, C, H, W, Hs, Ws,
+      launch_pdl(stage_rows_kernel<ST_BF16>, dim3((unsigned)grid), dim3(256), rows_bytes, s, x, y, C, H, W, Hs, Ws,
                                                                           Cs, blk, pad, 0);
     else
-      stage_rows_kernel<ST_F32><<<(unsigned)grid, 256, rows_bytes, s>>>(x, y, C, H, W, Hs, Ws,
+      launch_pdl(stage_rows_kernel<ST_F32>, dim3((unsigned)grid), dim3(256), rows_bytes, s, x, y, C, H, W, Hs, Ws,
                                                                          Cs, blk, pad, tf32_round);
     return cudaGetLastError();
   }
@@ -798,9 +805,9 @@ cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, in
   const long long total = (long long)B * Hs * Ws * (Cs / vn);
   const int grid = (int)std::max<long long>(1, std::min<long long>((total + 255) / 256, 148 * 16));
   if (st == ST_BF16)
-    stage_input_kernel<ST_BF16><<<grid, 256, 0, s>>>(x, y, B, C, H, W, Hs, Ws, Cs, blk, pad, 0);
+    launch_pdl(stage_input_kernel<ST_BF16>, dim3(grid), dim3(256), 0, s, x, y, B, C, H, W, Hs, Ws, Cs, blk, pad, 0);
   else
-    stage_input_kernel<ST_F32><<<grid, 256, 0, s>>>(x, y, B, C, H, W, Hs, Ws, Cs, blk, pad,
+    launch_pdl(stage_input_kernel<ST_F32>, dim3(grid), dim3(256), 0, s, x, y, B, C, H, W, Hs, Ws, Cs, blk, pad,
                                                     tf32_round);
   return cudaGetLastError();
 }
@@ -808,6 +815,7 @@ cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, in
 // final NHWC storage -> NCHW fp32 flatten (C,H,W order, reading R5)
 __global__ void unstage_output_kernel(const void *x, int st, float *y, int B,
                                       int C, int H, int W, int Cs) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   const long long HW = (long long)H * W;
   const long long total = (long long)B * C * HW;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
@@ -826,7 +834,7 @@ cudaError_t launch_unstage_output(const void *x, int st, float *y, int B,
   int grid = (int)((total + 255) / 256);
   if (grid > 148 * 16) grid = 148 * 16;
   if (grid < 1) grid = 1;
-  unstage_output_kernel<<<grid, 256, 0, s>>>(x, st, y, B, C, H, W, Cs);
+  launch_pdl(unstage_output_kernel, dim3(grid), dim3(256), 0, s, x, st, y, B, C, H, W, Cs);
   return cudaGetLastError();
 }
 
@@ -848,6 +856,7 @@ conv_simt_kernel(ConvGeom g, const float *__restrict__ x,
                  const float *__restrict__ w, const float *__restrict__ bias,
                  float *__restrict__ y, const int *__restrict__ ktab, Budget b,
                  int mtiles, int ntiles) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   __shared__ float As[SB_K][SB_M + 4];
   __shared__ float Bs[SB_K][SB_N + 4];
   __shared__ long long row_base[SB_M];
@@ -956,7 +965,7 @@ cudaError_t launch_conv_simt(const ConvGeom &g, const float *x, const float *w,
                              const Budget &b, int grid, cudaStream_t s) {
   const int mtiles = (g.M + SB_M - 1) / SB_M;
   const int ntiles = (g.Nfg + SB_N - 1) / SB_N;
-  conv_simt_kernel<<<grid, 256, 0, s>>>(g, x, w, bias, y, ktab, b, mtiles,
+  launch_pdl(conv_simt_kernel, dim3(grid), dim3(256), 0, s, g, x, w, bias, y, ktab, b, mtiles,
                                         ntiles);
   return cudaGetLastError();
 }
@@ -991,6 +1000,7 @@ struct LrnPoolArgs {
 
 template <int ST, int LS>
 __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   extern __shared__ __align__(16) uint8_t lp_smem[];
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
   constexpr int VN = Vec16<ST>::N;
@@ -1153,6 +1163,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
 // and the conv epilogue (lrn_normalise), so results are identical.
 template <int ST, int LS>
 __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   extern __shared__ __align__(16) uint8_t lb_smem[];
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
   constexpr int VN = Vec16<ST>::N;
@@ -1306,6 +1317,7 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
 // lrn_normalise), so the results are identical.
 template <int ST, int CPT, int MINB = 0>
 __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   extern __shared__ __align__(16) uint8_t lr_smem[];
   constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
   constexpr int VN = Vec16<ST>::N;
@@ -1534,7 +1546,7 @@ static cudaError_t lrn_pool_launch(const LrnPoolArgs &a, int grid, size_t smem, 
   if (smem > 48 * 1024)
     cudaFuncSetAttribute(lrn_pool_kernel<ST, LS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)smem);
-  lrn_pool_kernel<ST, LS><<<grid, 256, smem, s>>>(a);
+  launch_pdl(lrn_pool_kernel<ST, LS>, dim3(grid), dim3(256), smem, s, a);
   return cudaGetLastError();
 }
 
@@ -1570,6 +1582,7 @@ __global__ void __launch_bounds__(256)
 pool_direct_kernel(const uint4 *__restrict__ x, uint4 *__restrict__ y, int B, int H, int W,
                    int chunks, int kk, int s, int is_max, int Ho, int Wo, int hi, int ho,
                    int tf32_round, Budget bud) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int VN = Vec16<ST>::N;
   const int k = K > 0 ? K : kk;
   const int Hp = H + 2 * hi, Wp = W + 2 * hi, Hop = Ho + 2 * ho, Wop = Wo + 2 * ho;
@@ -1647,7 +1660,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
     const long long total = (long long)B * (Ho + 2 * out_halo) * (Wo + 2 * out_halo) * chunks;
     const int g = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
 #define PCNN_PD(STT, KK)                                                                       \
-  pool_direct_kernel<STT, KK><<<g, 256, 0, stream>>>((const uint4 *)x, (uint4 *)y, B, H, W,    \
+  launch_pdl(pool_direct_kernel<STT, KK>, dim3(g), dim3(256), 0, stream, (const uint4 *)x, (uint4 *)y, B, H, W,    \
                                                      chunks, k, s, is_max, Ho, Wo, in_halo,    \
                                                      out_halo, tf32_round, b)
     if (st == ST_BF16) {
@@ -1700,12 +1713,12 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
       if (smem > 48 * 1024)                                                                     \
         cudaFuncSetAttribute(lrn_reg_kernel<STT, CP, 3>,                                        \
                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);           \
-      lrn_reg_kernel<STT, CP, 3><<<grid, 256, smem, stream>>>(a);                               \
+      launch_pdl(lrn_reg_kernel<STT, CP, 3>, dim3(grid), dim3(256), smem, stream, a);                               \
     } else {                                                                                    \
       if (smem > 48 * 1024)                                                                     \
         cudaFuncSetAttribute(lrn_reg_kernel<STT, CP>,                                           \
                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);           \
-      lrn_reg_kernel<STT, CP><<<grid, 256, smem, stream>>>(a);                                  \
+      launch_pdl(lrn_reg_kernel<STT, CP>, dim3(grid), dim3(256), smem, stream, a);                                  \
     }                                                                                           \
   } while (0)
     if (st == ST_BF16) {
@@ -1727,7 +1740,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
     if (smem > 48 * 1024)                                                                       \
       cudaFuncSetAttribute(lrn_band_kernel<STT, LSS>,                                           \
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);             \
-    lrn_band_kernel<STT, LSS><<<grid, 256, smem, stream>>>(a);                                  \
+    launch_pdl(lrn_band_kernel<STT, LSS>, dim3(grid), dim3(256), smem, stream, a);                                  \
   } while (0)
     if (st == ST_BF16) {
       if (lrn_size == 5) PCNN_LB(ST_BF16, 5); else PCNN_LB(ST_BF16, 3);
@@ -1757,6 +1770,7 @@ __device__ __forceinline__ int perf_src(int p, int s, int n) {
 __global__ void __launch_bounds__(256)
 perf_interp_kernel(const uint4 *__restrict__ t, uint4 *__restrict__ y, int B, int Ho, int Wo,
                    int sh, int sw, int chunks, int ho) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   const int Hk = (Ho + sh - 1) / sh, Wk = (Wo + sw - 1) / sw;
   const int Hp = Ho + 2 * ho, Wp = Wo + 2 * ho;
   const long long total = (long long)B * Hp * Wp * chunks;
@@ -1784,7 +1798,7 @@ cudaError_t launch_perf_interp(const void *t, void *y, int st, int B, int Ho, in
   const int chunks = Cs * esz / 16;
   const long long total = (long long)B * (Ho + 2 * ho) * (Wo + 2 * ho) * chunks;
   const int grid = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
-  perf_interp_kernel<<<grid, 256, 0, s>>>((const uint4 *)t, (uint4 *)y, B, Ho, Wo, sh, sw,
+  launch_pdl(perf_interp_kernel, dim3(grid), dim3(256), 0, s, (const uint4 *)t, (uint4 *)y, B, Ho, Wo, sh, sw,
                                           chunks, ho);
   return cudaGetLastError();
 }
@@ -1797,6 +1811,7 @@ cudaError_t launch_perf_interp(const void *t, void *y, int st, int B, int Ho, in
 template <int NR>
 __global__ void softmax_entropy_kernel(const float *__restrict__ z, float *p,
                                        float *h, int B, int N) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) / 32;
   const int lane = threadIdx.x % 32;
   if (warp >= B) return;
@@ -1856,9 +1871,9 @@ cudaError_t launch_softmax_entropy(const float *z, float *p, float *h, int B,
   const int warps_per_block = 2;
   const int grid = (B + warps_per_block - 1) / warps_per_block;
   if (N <= 32 * 32)
-    softmax_entropy_kernel<32><<<grid, warps_per_block * 32, 0, s>>>(z, p, h, B, N);
+    launch_pdl(softmax_entropy_kernel<32>, dim3(grid), dim3(warps_per_block * 32), 0, s, z, p, h, B, N);
   else
-    softmax_entropy_kernel<0><<<grid, warps_per_block * 32, 0, s>>>(z, p, h, B, N);
+    launch_pdl(softmax_entropy_kernel<0>, dim3(grid), dim3(warps_per_block * 32), 0, s, z, p, h, B, N);
   return cudaGetLastError();
 }
 

@@ -35,6 +35,7 @@
 #include "budget.cuh"
 #include "lrn_math.cuh"
 #include "pcnn_internal.h"
+#include "tc_ptx.cuh"
 
 namespace pcnn {
 
@@ -114,258 +115,6 @@ int tc_stages_for(int bn, int cg) {
   return n;
 }
 
-// ------------------------------------------------------------ PTX wrappers
-__device__ __forceinline__ uint32_t smem_u32(const void *p) {
-  return (uint32_t)__cvta_generic_to_shared(p);
-}
-
-__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
-}
-__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar),
-               "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@!P1 bra WAIT_%=;\n"
-      "}\n" ::"r"(bar),
-      "r"(parity)
-      : "memory");
-}
-
-__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map,
-                                            uint32_t bar, int c0, int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
-      "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1)
-      : "memory");
-}
-
-// TMA im2col load of one A slab: 128 output pixels starting at (w, h, n)
-// (input-space corner of the first pixel), channels [c, c + slab), filter tap
-// offsets (ow, oh); padding / out-of-range pixels are zero-filled.
-__device__ __forceinline__ void tma_im2col(uint32_t dst, const CUtensorMap *map, uint32_t bar,
-                                           int c, int w, int h, int n, uint16_t ow,
-                                           uint16_t oh) {
-  asm volatile(
-      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
-      "l"((uint64_t)map), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ow), "h"(oh)
-      : "memory");
-}
-// tiled 4-D TMA load (A slab of a rectangle tile: channels x W x H x N box)
-template <int CG>
-__device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap *map, uint32_t bar,
-                                            int c0, int c1, int c2, int c3) {
-  if constexpr (CG == 1) {
-    asm volatile(
-        "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(dst),
-        "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
-        : "memory");
-  } else {
-    asm volatile(
-        "cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(dst),
-        "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
-        : "memory");
-  }
-}
-
-// tiled 3-D TMA load (row-perforated padded mode: {channels, wv, grid rows}
-// box, grid rows traversed with the perforation stride)
-template <int CG>
-__device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap *map, uint32_t bar,
-                                            int c0, int c1, int c2) {
-  if constexpr (CG == 1) {
-    asm volatile(
-        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
-        "l"((uint64_t)map), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
-        : "memory");
-  } else {
-    asm volatile(
-        "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
-        "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c0), "r"(c1), "r"(c2)
-        : "memory");
-  }
-}
-
-// 2-SM form: lands in this CTA's smem, bytes counted on the leader's barrier.
-__device__ __forceinline__ void tma_im2col_2sm(uint32_t dst, const CUtensorMap *map,
-                                               uint32_t bar, int c, int w, int h, int n,
-                                               uint16_t ow, uint16_t oh) {
-  asm volatile(
-      "cp.async.bulk.tensor.4d.im2col.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
-      "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c), "r"(w), "r"(h), "r"(n), "h"(ow),
-      "h"(oh)
-      : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-// TMA tensor store of one smem box (bulk-group completion)
-__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, uint32_t src, int c0, int c1) {
-  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
-                   (uint64_t)map),
-               "r"(src), "r"(c0), "r"(c1)
-               : "memory");
-}
-__device__ __forceinline__ void bulk_commit() {
-  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_wait_read0() {
-  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_wait0() {
-  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-}
-
-// one lane of a converged warp (the tcgen05 / TMA issue idiom): the loop
-// around it stays warp-uniform, so its values live in uniform registers
-__device__ __forceinline__ bool elect_one() {
-  uint32_t pred = 0;
-  asm volatile(
-      "{\n.reg .pred P;\nelect.sync _|P, 0xffffffff;\nselp.u32 %0, 1, 0, P;\n}"
-      : "=r"(pred));
-  return pred != 0;
-}
-
-__device__ __forceinline__ void tc_fence_before() {
-  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-}
-__device__ __forceinline__ void tc_fence_after() {
-  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-}
-template <int CG>
-__device__ __forceinline__ void tc_commit(uint32_t bar) {
-  if constexpr (CG == 1) {
-    asm volatile(
-        "tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-            bar)
-        : "memory");
-  } else {   // arrive on the barrier at this offset in both CTAs of the pair
-    asm volatile(
-        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
-        " [%0], %1;" ::"r"(bar),
-        "h"((uint16_t)0x3)
-        : "memory");
-  }
-}
-
-__device__ __forceinline__ uint32_t cluster_ctarank() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-  return r;
-}
-__device__ __forceinline__ void cluster_sync() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\n"
-               "barrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-// address of the same smem offset in CTA `rank` of the cluster
-__device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
-  uint32_t r;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
-  return r;
-}
-// Remote arrive carrying no data dependency (only TMEM-read completion,
-// ordered by tcgen05.fence::before_thread_sync): relaxed is enough and avoids
-// a GPU-scope MEMBAR.
-__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
-  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(
-                   cluster_addr)
-               : "memory");
-}
-// 2-SM TMA load: data lands in this CTA's smem, bytes are counted on the
-// leader CTA's barrier (peer bit cleared).
-__device__ __forceinline__ void tma_load_2d_2sm(uint32_t dst, const CUtensorMap *map,
-                                                uint32_t bar, int c0, int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
-      "l"((uint64_t)map), "r"(bar & 0xFEFFFFFFu), "r"(c0), "r"(c1)
-      : "memory");
-}
-
-template <int ST, int CG>
-__device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
-                                       uint32_t idesc, uint32_t accum) {
-  if constexpr (ST == ST_BF16 && CG == 1) {
-    asm volatile(
-        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
-        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
-  } else if constexpr (ST == ST_BF16 && CG == 2) {
-    asm volatile(
-        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
-        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
-  } else if constexpr (CG == 1) {
-    asm volatile(
-        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
-        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
-  } else {
-    asm volatile(
-        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-        "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
-        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accum));
-  }
-}
-
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
-      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
-        "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]),
-        "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
-      : "r"(taddr));
-}
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
-      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
-        "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]),
-        "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]),
-        "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
-        "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]),
-        "=r"(v[30]), "=r"(v[31])
-      : "r"(taddr));
-}
-__device__ __forceinline__ void tmem_ld_wait() {
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-}
-
-// UMMA shared-memory descriptor, K-major, swizzled rows of `row_bytes`
-// (128 / 64 / 32 B): 8-row atoms stacked along M/N every 8*row_bytes (SBO),
-// version 1 (sm_100), layout SW128 = 2, SW64 = 4, SW32 = 6.
-__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t row_bytes) {
-  const uint64_t layout = row_bytes == 128 ? 2 : (row_bytes == 64 ? 4 : 6);
-  uint64_t d = 0;
-  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
-  d |= (uint64_t)1 << 16;                        // LBO (unused for swizzled K-major)
-  d |= (uint64_t)((8 * row_bytes) >> 4) << 32;   // SBO
-  d |= (uint64_t)1 << 46;                        // descriptor version (sm_100)
-  d |= layout << 61;
-  return d;
-}
-__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) { return umma_desc(saddr, 128); }
-
 // Instruction descriptor: D fp32, A/B = BF16 (1) or TF32 (2), K-major,
 // M = 128 * CG, N = bn.
 template <int ST, int CG>
@@ -374,32 +123,6 @@ __device__ __forceinline__ uint32_t umma_idesc(int bn) {
   return (1u << 4) | (fmt << 7) | (fmt << 10) | ((uint32_t)(bn >> 3) << 17) |
          ((uint32_t)((TC_BM * CG) >> 4) << 24);
 }
-
-__device__ __forceinline__ float tf32_rna_tc(float v) {
-  unsigned r;
-  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(v));
-  return __uint_as_float(r);
-}
-
-// Division by a launch-invariant divisor d (Granlund-Montgomery, exact for
-// every 32-bit n): q = (t + ((n - t) >> 1)) >> (l - 1), t = umulhi(m, n),
-// l = ceil(log2 d), m = floor(2^32 (2^l - d) / d) + 1.  The epilogue's
-// per-tile index arithmetic (tile decode, halo test) runs on every lane, where
-// a hardware-less integer division costs ~20 instructions.
-struct FastDiv {
-  uint32_t d, m, l;
-  __host__ void init(uint32_t dd) {
-    d = dd < 1 ? 1 : dd;
-    l = 0;
-    while ((1ull << l) < d) ++l;
-    m = (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
-  }
-  __device__ __forceinline__ uint32_t div(uint32_t n) const {
-    if (d == 1) return n;
-    const uint32_t t = __umulhi(m, n);
-    return (t + ((n - t) >> 1)) >> (l - 1);
-  }
-};
 
 struct TcArgs {
   ConvGeom g;
@@ -771,6 +494,9 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *(volatile uint32_t *)(smem + SM_TMEMPTR);
+  // PDL: setup above overlapped the previous kernel's tail; activations are
+  // read (and outputs written) only after its completion
+  pdl_enter();
   const long long t_start = TC_PROF(a) ? clock64() : 0;
   unsigned long long wtf_acc_out = 0, busy_out = 0;   // epilogue profile (warp 2)
 
@@ -1267,6 +993,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
 __global__ void splitk_reduce_kernel(const float *__restrict__ ws, void *y,
                                      const float *__restrict__ bias, int M, int N, int splits,
                                      int relu, int out_mode) {
+  pdl_enter();
   const long long total = (long long)M * N / 4;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
        i += (long long)gridDim.x * blockDim.x) {
@@ -1347,13 +1074,15 @@ static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_
   cfg.blockDim = dim3(tc_threads<LRN>());
   cfg.dynamicSmemBytes = TC_SMEM_BYTES;
   cfg.stream = s;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = CG;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;   // PDL
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = 2;
   return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG, LRN>, *tmap_w, *tmap_x, *tmap_y, args);
 }
 
@@ -1461,7 +1190,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   if (e != cudaSuccess || p.splits <= 1) return e;
   const long long total = (long long)g.M * g.out_cs / 4;
   const int grid = (int)std::min<long long>((total + 255) / 256, 148 * 8);
-  splitk_reduce_kernel<<<grid, 256, 0, s>>>(ws, y, bias, g.M, g.out_cs, p.splits, g.relu,
+  launch_pdl(splitk_reduce_kernel, dim3(grid), dim3(256), 0, s, ws, y, bias, g.M, g.out_cs, p.splits, g.relu,
                                             g.out_mode);
   return cudaGetLastError();
 }

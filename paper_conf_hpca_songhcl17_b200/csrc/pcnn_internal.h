@@ -32,6 +32,46 @@ inline const char *exp_env(const char *name) {
 
 constexpr int kMaxSMs = 256;          // census mask width
 
+// ---------------------------------------------------------------- PDL
+// Every kernel of the hot path is launched with programmatic stream
+// serialization (programmatic dependent launch): its CTAs may be scheduled
+// while the previous kernel of the stream is still running.  Each kernel
+// (1) executes griddepcontrol.wait before it reads any activation or writes
+// any global memory -- the wait returns once every prerequisite grid has
+// completed and its writes are visible -- and (2) executes
+// griddepcontrol.launch_dependents once all of its CTAs are resident, so the
+// next kernel's launch latency, CTA rasterisation and prologue (barrier init,
+// TMEM allocation, tensor-map prefetch, weight prefetch) overlap this
+// kernel's tail.  Only read-only constants (weights, bias, tap tables) may be
+// touched before the wait.
+#ifdef __CUDACC__
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+// the common case: nothing to prefetch
+__device__ __forceinline__ void pdl_enter() {
+  pdl_wait();
+  pdl_trigger();
+}
+#endif
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                              cudaStream_t s, Args &&...args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+
 // Element storage types of activations / packed weights.
 enum StoreType : int { ST_F32 = 0, ST_BF16 = 1 };
 // Epilogue output modes.
@@ -161,6 +201,29 @@ int tc_block_k_elems(int st);          // K-block in elements (128 B)
 cudaError_t tc_init();                 // sets the kernels' smem attributes
 size_t tc_smem_bytes();
 int tc_max_ktab();
+
+// a6: weight-streaming FC (kernels_fc.cu).  A CTA pair (cta_group::2) owns
+// 256 weight rows (the UMMA M) for nb images of a batch chunk (the UMMA N);
+// `splits` pairs split K in fixed, batch-independent ranges of kbps K-blocks
+// and reduce their FP32 partials in split order.
+struct FcPlan {
+  int splits;     // K split = CTA pairs per unit (power of two, <= 16)
+  int kbps;       // K-blocks per split
+  int nb;         // batch columns per chunk (16..256, multiple of 16)
+  int rblocks;    // ceil(N / 256)
+  int chunks;     // ceil(B / nb)
+  int groups;     // concurrent unit workers (each = splits CTA pairs)
+  int grid;       // CTAs = 2 x splits x groups
+};
+int fc_stage_count(int nb);
+// tmap_w: 4-D map of the re-tiled weights [RB][KB][128][128 B] (box = one
+// 16 KB tile, SW128); tmap_x: tiled map of the input [B][K] (box 128 B x
+// nb / 2 rows, SW128); y: [B][ldy] output; ws: splits * B * N floats and sem:
+// 2 * units zeroed counters when splits > 1.
+cudaError_t launch_fc_tc(const FcPlan &p, int st, const CUtensorMap *tmap_w,
+                         const CUtensorMap *tmap_x, const float *bias, void *y, float *ws,
+                         unsigned *sem, int N, int B, int kblocks, int relu, int out_mode,
+                         int ldy, const Budget &b, cudaStream_t s);
 
 // a4 / a5: LRN (lrn_size > 0) followed by pooling (k x k, stride s; k = s =
 // 1 for no pooling), NHWC with C stored input channels.  out_groups > 0

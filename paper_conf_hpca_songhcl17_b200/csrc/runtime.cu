@@ -103,6 +103,9 @@ struct GemmStage {           // one implicit-GEMM launch
   int in_c = 0, in_h = 0, in_w = 0;
   int st = ST_F32;           // storage type of input / weights
   int engine = 0;            // 0 SIMT, 1 tcgen05
+  bool is_fc = false;        // FC layer (tcgen05: the weight-streaming FC kernel)
+  unsigned *d_sem = nullptr; // FC split-K arrival counters (2 x units, zero at rest)
+  int sem_count = 0;
   void *d_w = nullptr;       // packed [groups*Nfg][Kpad]
   float *d_bias = nullptr;
   int *d_ktab = nullptr;     // per-element (r,s,c) table
@@ -115,6 +118,9 @@ struct GemmStage {           // one implicit-GEMM launch
     if (d_w) cudaFree(d_w);
     if (d_bias) cudaFree(d_bias);
     if (d_ktab) cudaFree(d_ktab);
+    if (d_sem) cudaFree(d_sem);
+    d_sem = nullptr;
+    sem_count = 0;
     d_w = nullptr;
     d_bias = nullptr;
     d_ktab = nullptr;
@@ -412,6 +418,7 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
   gs.release();
   gs.st = storage_of(precision);
   gs.engine = precision == PCNN_FP32_SIMT ? 0 : 1;
+  gs.is_fc = is_fc;
   gs.in_c = in_c;
   gs.in_h = in_h;
   gs.in_w = in_w;
@@ -487,11 +494,25 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
   (void)ch;
   if (gs.engine == 1 && is_fc && tc_slab_bytes(gs.st, g.Cg) == 0)
     return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 FC needs K multiple of 32 bytes");
-  if (gs.engine == 1 && (g.Nfg % 8))
-    return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 path needs N_f/g multiple of 8");
+  if (gs.engine == 1 && !is_fc && (g.Nfg % 8))
+    return fail(PCNN_ERR_UNSUPPORTED, "tcgen05 conv needs N_f/g multiple of 8");
   g.relu = relu;
   g.out_mode = out_mode;
   g.out_cs = Nf;
+  if (gs.engine == 1 && is_fc) {
+    // weight-streaming FC: re-tile [N][Kpad] into contiguous 128-row x 128-B
+    // K-block tiles, [row block][K-block][128 rows][128 B] (rows past N are
+    // zeros), so every TMA box the kernel streams is one contiguous 16 KB run
+    // of HBM instead of 128 rows 2*Kpad bytes apart
+    const int kbe = k_align(precision) == 64 ? 64 : 32;
+    const int KB = g.Kpad / kbe, RB = (Nf + 127) / 128;
+    std::vector<float> t((size_t)RB * 128 * g.Kpad, 0.f);
+    for (int n = 0; n < Nf; ++n)
+      for (int kb = 0; kb < KB; ++kb)
+        std::memcpy(&t[(((size_t)(n / 128) * KB + kb) * 128 + (n % 128)) * kbe],
+                    &packed[(size_t)n * g.Kpad + (size_t)kb * kbe], sizeof(float) * kbe);
+    packed.swap(t);
+  }
   pcnn_status st = upload_weights(gs, packed, precision);
   if (st != PCNN_OK) return st;
   // zero-padded so the epilogue can read whole 32-column slices unguarded
@@ -629,6 +650,53 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, co
   return &(gs.xmaps[key] = m);
 }
 
+// Weight map of the weight-streaming FC kernel over the re-tiled layout
+// [RB][KB][128][kbe]: a box {kbe, 128, 1, 1} is one contiguous 16 KB tile.
+static const CUtensorMap *stage_fcwmap(GemmStage &gs) {
+  const int key = -7;
+  auto it = gs.tmaps.find(key);
+  if (it != gs.tmaps.end()) return &it->second;
+  auto enc = get_encode_tiled();
+  if (!enc) return nullptr;
+  const int esz = esz_of(gs.st), kbe = 128 / esz;
+  const cuuint64_t KB = gs.g.Kpad / kbe, RB = (gs.g.Nfg + 127) / 128;
+  CUtensorMap m;
+  const cuuint64_t dims[4] = {(cuuint64_t)kbe, 128, KB, RB};
+  const cuuint64_t strides[3] = {128, 128ull * 128, 128ull * 128 * KB};
+  const cuuint32_t box[4] = {(cuuint32_t)kbe, 128, 1, 1};
+  const cuuint32_t estr[4] = {1, 1, 1, 1};
+  CUresult r = enc(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                   4, gs.d_w, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return nullptr;
+  return &(gs.tmaps[key] = m);
+}
+
+// Activation (B operand) map of the weight-streaming FC kernel: the input
+// [B][K] matrix (K = the stored NHWC flatten), boxes of 128 B of K x nb images,
+// SW128; images past the batch and K past the row are zero-filled.
+static const CUtensorMap *stage_fcxmap(GemmStage &gs, const void *x, int batch, int nb) {
+  const auto key = std::make_tuple(x, batch, nb, -1, -1);
+  auto it = gs.xmaps.find(key);
+  if (it != gs.xmaps.end()) return &it->second;
+  auto enc = get_encode_tiled();
+  if (!enc) return nullptr;
+  const int esz = esz_of(gs.st);
+  CUtensorMap m;
+  const cuuint64_t dims[2] = {(cuuint64_t)gs.g.K, (cuuint64_t)batch};
+  const cuuint64_t strides[1] = {(cuuint64_t)gs.g.K * esz};
+  const cuuint32_t box[2] = {(cuuint32_t)(128 / esz), (cuuint32_t)nb};
+  const cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(&m, gs.st == ST_BF16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                   2, const_cast<void *>(x), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return nullptr;
+  if (gs.xmaps.size() > 64) gs.xmaps.clear();
+  return &(gs.xmaps[key] = m);
+}
+
 // Output map for the epilogue's TMA tensor stores: the [M][out_cs] output
 // matrix (rows = output pixels, padded grid in pm mode), boxes of 32 columns
 // x 32 rows, swizzle = the box row width (64 B bf16 / 128 B fp32).  nullptr
@@ -714,6 +782,17 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
   const char *force_am = exp_env("PCNN_AMODE");             // "im2col" | "rect"
   if (want_cg > 0) force_cg = want_cg == 1 ? "1" : "2";
   const Rect rc = best_rect(g);
+  // Split-K changes an output's summation order.  It is considered only when
+  // no tile shape fills the device without it (tiny batches): then the K
+  // order of every image is the same for every batch at which some tile
+  // shape fills the device -- per-image results are bitwise equal at B and
+  // B / W and across pcnn_infer_host's chunks.
+  bool can_fill = false;
+  for (int cg = 1; cg <= 2; ++cg)
+    for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {
+      const long long t = ((g.M + 128LL * cg - 1) / (128LL * cg)) * ((g.Nfg + bn - 1) / bn) * g.groups;
+      if (t >= device_sms / cg) can_fill = true;
+    }
   for (int am = 0; am < 2; ++am) {            // 0 im2col, 1 rectangle tiles (opt-in)
     if (am == 1 && (rc.w == 0 || !force_am || std::string(force_am) != "rect")) continue;
     if (am == 0 && force_am && std::string(force_am) == "rect" && rc.w != 0) continue;
@@ -733,7 +812,7 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
         const double kb_cycles = std::max(load, mma) + 40.0;
         // split-K candidates: none, or any split that keeps >= 4 K-blocks per unit
         const int max_split =
-            (tiles >= slots || full_n) ? 1 : std::min(16, std::max(1, kblocks / 4));
+            (tiles >= slots || full_n || can_fill) ? 1 : std::min(16, std::max(1, kblocks / 4));
         static const int force_split = [] {              // tuning experiments
           const char *e = exp_env("PCNN_FORCE_SPLIT");
           return e ? atoi(e) : 0;
@@ -850,6 +929,34 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
   return best;
 }
 
+// Weight-streaming FC plan (kernels_fc.cu).  The K split s (CTA pairs per
+// 256-row unit) and its ranges come from the layer shape and the device's SM
+// count only -- never from the batch or the SM budget -- so every image's sum
+// runs in the same order for any batch (bitwise per-image results at B and
+// B / W) and any budget (R11).  s is the largest power
+// of two <= 16 that keeps >= 4 K-blocks per split and fits all row blocks'
+// pairs on the device at once.  The batch only picks the UMMA N (nb images
+// per chunk) and the number of chunks, which move work between CTA pairs but
+// never change a sum.  All CTAs of the launch must be co-resident (the
+// split-K partials meet at a global counter): grid <= SM budget, and a budget
+// below 2 s SMs is raised to 2 s.
+static FcPlan plan_fc(int N, int kblocks, int B, int device_sms, int budget_sms) {
+  FcPlan p{};
+  const int rb = (N + 255) / 256;
+  int s = 1;
+  while (s < 16 && rb * 2 * (2 * s) <= device_sms && kblocks / (2 * s) >= 4) s *= 2;
+  if (const char *e = exp_env("PCNN_FC_SPLIT")) s = atoi(e);   // experiments build only
+  p.splits = s;
+  p.kbps = (kblocks + s - 1) / s;
+  p.chunks = (B + 255) / 256;
+  p.nb = round_up((B + p.chunks - 1) / p.chunks, 16);
+  p.rblocks = rb;
+  const int units = p.rblocks * p.chunks;
+  p.groups = std::max(1, std::min(units, std::min(budget_sms, device_sms) / (2 * s)));
+  p.grid = 2 * s * p.groups;
+  return p;
+}
+
 static int effective_sms(const pcnn_net *net, const Layer &ly) {
   int n = ly.n_sms <= 0 ? net->num_sms : std::min(ly.n_sms, net->num_sms);
   return std::max(n, 1);
@@ -875,6 +982,49 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
                              size_t *ws_need = nullptr, const float *lrn = nullptr) {
   ConvGeom g = gs.g;
   g.M = g.pm == 2 ? B * g.tpi * 128 : g.pm ? B * g.hv * g.wv : B * g.Ho * g.Wo;
+  if (gs.engine == 1 && gs.is_fc && !lrn) {
+    // a6: weight-streaming FC kernel
+    const int N = g.Nfg, kblocks = g.Kpad / tc_block_k_elems(gs.st);
+    const FcPlan p = plan_fc(N, kblocks, B, net->num_sms, effective_sms(net, ly));
+    if (info) {
+      info->tile_m = 256;
+      info->tile_n = p.nb;
+      info->tiles = (long long)p.rblocks * p.chunks;
+      info->grid = p.grid;
+      info->tlp = 1;
+      info->engine = 1;
+      info->splits = p.splits;
+      info->a_mode = 3;
+      info->n_sms = std::max(info->n_sms, p.grid);
+      info->cta_group = 2;
+    }
+    const size_t wsb = p.splits > 1 ? (size_t)p.splits * B * N * 4 : 0;
+    if (ws_need) *ws_need = std::max(*ws_need, wsb);
+    const int units = p.rblocks * p.chunks;
+    if (ws_need && 2 * units > gs.sem_count) {
+      // split-K arrival counters (reserved with the workspace, outside any
+      // graph capture): zeroed once, re-armed by the kernel itself
+      CUDA_TRY(cudaDeviceSynchronize());
+      if (gs.d_sem) cudaFree(gs.d_sem);
+      gs.d_sem = nullptr;
+      gs.sem_count = 0;
+      CUDA_TRY(cudaMalloc(&gs.d_sem, sizeof(unsigned) * 2 * units));
+      CUDA_TRY(cudaMemset(gs.d_sem, 0, sizeof(unsigned) * 2 * units));
+      gs.sem_count = 2 * units;
+      net->version++;          // cached graphs captured the old pointer
+    }
+    if (!x) return PCNN_OK;
+    if (wsb > net->ws_bytes) return fail(PCNN_ERR_OUT_OF_MEMORY, "FC split-K workspace not reserved");
+    if (p.splits > 1 && 2 * units > gs.sem_count)
+      return fail(PCNN_ERR_OUT_OF_MEMORY, "FC split-K counters not reserved");
+    const CUtensorMap *tm = stage_fcwmap(gs);
+    const CUtensorMap *xm = stage_fcxmap(gs, x, B, p.nb / 2);
+    if (!tm || !xm) return fail(PCNN_ERR_CUDA, "cuTensorMapEncodeTiled failed (FC)");
+    Budget b = make_budget(net, ly, slot, false);
+    CUDA_TRY(counted(launch_fc_tc(p, gs.st, tm, xm, gs.d_bias, y, net->d_ws, gs.d_sem, N, B,
+                                  kblocks, g.relu, g.out_mode, g.out_cs, b, s)));
+    return PCNN_OK;
+  }
   if (gs.engine == 1) {
     TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st), lrn != nullptr, ly.plan_cg,
                                  ly.plan_msub)

@@ -162,7 +162,7 @@ def test_padded_mode_conv_lrn_fusion(orc, prec):
     assert fused["net"].query_layer(0, 2)["a_mode"] == 2
     pr = gpu_run(net, w, b, x, prec, flags=FLAG_NO_LRN_POOL_FUSION)
     plain = pr["out"]
-    assert fused["net"].last_launch_count() + 1 == pr["net"].last_launch_count()
+    assert fused["net"].last_launch_count() < pr["net"].last_launch_count()
     assert rel_err(fused["out"], ref) <= TOL[prec] / 4
     assert rel_err(plain, ref) <= TOL[prec] / 4
     # last-place differences of the storage format (R16)

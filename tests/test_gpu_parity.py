@@ -257,8 +257,9 @@ def test_conv_lrn_epilogue_fusion(orc, prec):
     fr = gpu_run(net, w, b, x, prec, flags=FLAG_NO_PADDED_LAYOUT)
     pr = gpu_run(net, w, b, x, prec, flags=FLAG_NO_PADDED_LAYOUT | FLAG_NO_LRN_POOL_FUSION)
     fused, plain = fr["out"], pr["out"]
-    # the fusion really happened: conv+LRN and pool are 2 launches, not 3
-    assert fr["net"].last_launch_count() + 1 == pr["net"].last_launch_count()
+    # the fusion really happened: the conv+LRN epilogue saves the LRN launch
+    assert fr["net"].last_launch_count() < pr["net"].last_launch_count()
+    assert fr["net"].query_layer(0, 2)["tile_n"] >= 96          # one N tile holds all channels
     assert rel_err(fused, ref) <= TOL[prec] / 4
     assert rel_err(plain, ref) <= TOL[prec] / 4
     ulp = 2.0 ** -8 if prec == "bf16" else 2.0 ** -10
@@ -283,8 +284,9 @@ def test_lrn_pool_kernel_shapes(orc, shape):
 
 def test_infer_host_pipelined_chunks(orc):
     """AlexNet at B = 64 through pcnn_infer_host takes the pipelined path (4
-    chunks, copies overlapping inference): same logits as the device call up
-    to FC split-K grouping, identical top-1, and the oracle's tolerance."""
+    chunks, copies overlapping inference): bitwise the device call's logits
+    (the FC K split is batch-independent and no conv layer splits K at 16
+    images), and the oracle's tolerance."""
     import torch
     from paper_conf_hpca_songhcl17_b200 import pcnn
     net = synth.alexnet()
@@ -299,8 +301,7 @@ def test_infer_host_pipelined_chunks(orc):
     hh = torch.empty((B,)).pin_memory()
     n.infer_host(xh, oh, None, hh)
     d = dev.cpu().numpy()
-    assert rel_err(oh.numpy(), d) <= 2e-3
-    assert (oh.numpy().argmax(1) == d.argmax(1)).all()
+    np.testing.assert_array_equal(oh.numpy(), d)
     ref = orc.run_net(net, w, b, x[:2])
     assert rel_err(oh.numpy()[:2], ref) <= TOL["bf16"]
     assert np.isfinite(hh.numpy()).all() and (hh.numpy() >= 0).all()
@@ -336,3 +337,17 @@ def test_vgg16_tf32_bench_batch_sampled(orc):
     assert np.isfinite(out).all()
     ref = orc.run_net(net, w, b, x[17:18])
     assert rel_err(out[17:18], ref) <= TOL["tf32"]
+
+
+@pytest.mark.parametrize("name,B,half", [("alexnet", 64, 16), ("vgg16", 16, 8)])
+def test_per_image_logits_bitwise_batch_independent(name, B, half):
+    """configs[4]'s requirement: an image's logits do
+    not depend on how many images share its launch -- the FC K split is fixed
+    by the layer shape and no conv splits K once a tile shape fills the GPU --
+    so the per-rank shards B / W reproduce the W = 1 run bit for bit."""
+    net = synth.get_net(name)
+    w, b = params(net)
+    x = synth.images(0, B, net["in_shape"])
+    full = gpu_run(net, w, b, x, "bf16")["out"]
+    part = gpu_run(net, w, b, x[half:2 * half], "bf16")["out"]
+    np.testing.assert_array_equal(part, full[half:2 * half])
