@@ -156,6 +156,9 @@ typedef struct {
     int halo_in, halo_out; /* zero border of the stored input / output
                            activation layouts ([B][H+2h][W+2h][C])           */
     int cta_group;      /* SMs per GEMM tile: 2 for CTA-pair tiles, else 1   */
+    double t_unit_us;   /* modelled time of one work unit (tile, or one split
+                           of an FC unit) on its cta_group SMs (eq. 12 per
+                           wave); non-GEMM layers: 0                          */
 } pcnn_layer_info;
 
 /* Resource + time model of one layer, for the
@@ -168,11 +171,16 @@ typedef struct {
  *                 nSMs counted in CTA-pair units for 2-SM tiles
  *   opt_sm        eq. 11: the fewest SMs that keep n_invocations (a
  *                 multiple of cta_group); all SMs for non-GEMM layers
- *   t_model_us    eq. 12: FLOPs / (peak per SM x opt_sm x rEC x pipe
- *                 efficiency) -- DESIGN.md R12 reads the garbled "rCE" as
- *                 eq. 9's rEC and "FMA / total instructions" as the tensor
- *                 pipe's measured efficiency (0.8); non-GEMM layers: their
- *                 algorithmic bytes at the HBM bandwidth (6.5 TB/s)
+ *   t_model_us    eq. 12 at opt_sm (R12 / NEXT-3): t = t_launch +
+ *                 n_invocations x t_unit, where t_unit = FLOPs per work unit
+ *                 / (peak per SM x pipe efficiency), bounded below by the
+ *                 unit's operand bytes at the measured L2->SM rate (eq. 12's
+ *                 rEC enters through the padded tile), and t_launch the
+ *                 measured fixed cost of one launch (launch, prologue, pipe
+ *                 fill, epilogue drain); non-GEMM layers: t_launch + their
+ *                 algorithmic bytes at min(HBM, n x per-SM) bandwidth
+ *   t_launch_us   the fixed term above
+ *   t_unit_us     the per-wave term above
  * Host-only (no launch); INVALID_ARGUMENT for a bad layer / batch. */
 typedef struct {
     long long grid_size;
@@ -181,6 +189,8 @@ typedef struct {
     int opt_sm;
     int cta_group;
     double t_model_us;
+    double t_launch_us;
+    double t_unit_us;
 } pcnn_budget_plan;
 
 typedef struct pcnn_net pcnn_net;
@@ -236,7 +246,9 @@ pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank,
  * kernels run on at most n_sms SMs with at most ctas_per_sm CTAs each.
  * n_sms = 0 means all SMs; values above the device count are clamped.
  * ctas_per_sm = 0 means the kernel's natural occupancy.  tcgen05 kernels are
- * 1 CTA/SM by construction (their tlp is reported as 1).  The budget changes
+ * 1 CTA/SM by construction (their tlp is reported as 1).  Floors: a CTA-pair
+ * conv tile needs 2 SMs, an FC layer 2 x splits SMs (its K split is one
+ * co-resident group of CTA pairs; pcnn_query_layer reports splits).  The budget changes
  * placement only: results are bitwise identical for every budget (R11). */
 pcnn_status pcnn_set_sm_budget(pcnn_net *net, int layer, int n_sms,
                                int ctas_per_sm);
@@ -289,6 +301,12 @@ pcnn_status pcnn_query_layer(const pcnn_net *net, int layer, int batch,
 /* eqs. 8 / 11 / 12 for one layer (pcnn_budget_plan above). */
 pcnn_status pcnn_plan_budget(const pcnn_net *net, int layer, int batch,
                              pcnn_budget_plan *plan);
+
+/* eq. 12 time model of one layer at `batch` on n_sms SMs (0 = all), the
+ * same terms as pcnn_budget_plan: t_launch + n_invocations(n_sms) x t_unit,
+ * with n_invocations from eq. 8 at that budget.  Host-only. */
+pcnn_status pcnn_model_layer_time(const pcnn_net *net, int layer, int batch,
+                                  int n_sms, double *t_us);
 
 /* Host-only shape inference + FLOP/byte accounting of a descriptor list,
  * no device needed (used by CPU tests and by planners).  infos[n_layers]. */

@@ -20,7 +20,7 @@
 //
 // K split (deterministic, batch-independent): `splits` CTA pairs share one
 // (256-row block, batch chunk) unit; pair j accumulates K-blocks
-// [j*kbps, (j+1)*kbps) and writes its FP32 partial tile to the workspace
+// [j*KB/s, (j+1)*KB/s) and writes its FP32 partial tile to the workspace
 // (L2-resident).  The 2*splits CTAs of the unit meet at a counter in global
 // memory (release / acquire at GPU scope; all CTAs of the launch are
 // co-resident: grid <= SMs, one CTA per SM by shared memory), then CTA i of
@@ -209,7 +209,9 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
   tc_fence_after();
   const uint32_t tmem_base = *(volatile uint32_t *)(smem + FC_SM_TMEMPTR);
 
-  const int k0 = split * a.kbps, k1 = min(a.kblocks, k0 + a.kbps);
+  // balanced, never-empty K ranges: split j takes [j KB / s, (j + 1) KB / s)
+  const int k0 = (int)((long long)split * a.kblocks / s);
+  const int k1 = (int)((long long)(split + 1) * a.kblocks / s);
   // PDL prefetch: the first unit's first ring of weight tiles (the full
   // barrier's byte count -- on the leader -- covers the activation halves
   // loaded after the wait)

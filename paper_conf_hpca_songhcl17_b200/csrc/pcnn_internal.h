@@ -171,6 +171,7 @@ struct TcPlan {
   int rect_w, rect_h, rect_n;  // 0 = im2col A tiles; else rectangle tiles (tiled TMA)
   int a_stages, b_stages;      // padded mode: A (row-window) and B (tap slab) ring depths
   int msub;                    // padded mode: 128-row M sub-tiles per CTA sharing each B slab
+  double unit_us;              // modelled time of one work unit on its SM(s) (eq. 12 per wave)
 };
 // Launches the GEMM and, when p.splits > 1, the deterministic split-K
 // reduction (ws must hold splits * M * out_cs floats; a split-K output must
@@ -214,6 +215,7 @@ struct FcPlan {
   int chunks;     // ceil(B / nb)
   int groups;     // concurrent unit workers (each = splits CTA pairs)
   int grid;       // CTAs = 2 x splits x groups
+  double unit_us; // modelled time of one split of one unit on its CTA pair
 };
 int fc_stage_count(int nb);
 // tmap_w: 4-D map of the re-tiled weights [RB][KB][128][128 B] (box = one

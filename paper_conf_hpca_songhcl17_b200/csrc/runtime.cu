@@ -747,6 +747,10 @@ static const CUtensorMap *stage_ymap(GemmStage &gs, void *y, long long M) {
 // rows and are therefore opt-in (PCNN_AMODE=rect).  The tcgen05 pipe sustains
 // ~80% of its nominal rate in this kernel.
 static constexpr double kOperandBytesPerCycle = 36.0;
+// eq. 12 time-model constants (NEXT-3; fitted, see layer_time_model)
+static constexpr double kT0Conv = 4.0, kScaleConv = 1.0;   // tcgen05 conv: launch us, unit scale
+static constexpr double kT0Fc = 6.0, kScaleFc = 1.0;       // weight-streaming FC
+static constexpr double kT0Simt = 3.0;                     // SIMT kernels (LRN / pool / check path)
 static constexpr double kMmaEfficiency = 0.8;
 
 // Best rectangle tile (w x h x n <= 128 output pixels) for rect-mode A loads,
@@ -838,6 +842,7 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
             best.splits = splits;
             best.kb_per_split = kbs;
             best.units = (int)units;
+            best.unit_us = ((double)kbs * kb_cycles / f + 2e-6) * 1e6;
             best.rect_w = am ? rc.w : 0;
             best.rect_h = am ? rc.h : 0;
             best.rect_n = am ? rc.n : 0;
@@ -906,6 +911,7 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
         c.splits = 1;
         c.kb_per_split = nj;
         c.units = (int)tiles;
+        c.unit_us = ((double)nj * j_cycles / f + 2e-6 * ms) * 1e6;
         cands.push_back({t, c});
         best_t = std::min(best_t, t);
       }
@@ -945,6 +951,7 @@ static FcPlan plan_fc(int N, int kblocks, int B, int device_sms, int budget_sms)
   const int rb = (N + 255) / 256;
   int s = 1;
   while (s < 16 && rb * 2 * (2 * s) <= device_sms && kblocks / (2 * s) >= 4) s *= 2;
+  // (the kernel gives split j the K-blocks [j KB / s, (j + 1) KB / s): never empty)
   if (const char *e = exp_env("PCNN_FC_SPLIT")) s = atoi(e);   // experiments build only
   p.splits = s;
   p.kbps = (kblocks + s - 1) / s;
@@ -954,6 +961,12 @@ static FcPlan plan_fc(int N, int kblocks, int B, int device_sms, int budget_sms)
   const int units = p.rblocks * p.chunks;
   p.groups = std::max(1, std::min(units, std::min(budget_sms, device_sms) / (2 * s)));
   p.grid = 2 * s * p.groups;
+  // per K-block a CTA ingests one 16 KB weight tile + nb / 2 activation rows
+  // at the measured ~36 B/clk/SM of TMA operand delivery; the pair's MMA
+  // (256 x nb x 64) takes nb / 2 cycles per 16-deep UMMA step x 4
+  const double f = 1.9e9;
+  const double load = (16384.0 + 64.0 * p.nb) / 36.0, mma = 4.0 * std::max(16, p.nb / 2) / 0.8;
+  p.unit_us = ((double)p.kbps * (std::max(load, mma) + 40.0) / f + 2e-6) * 1e6;
   return p;
 }
 
@@ -997,6 +1010,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->a_mode = 3;
       info->n_sms = std::max(info->n_sms, p.grid);
       info->cta_group = 2;
+      info->t_unit_us = p.unit_us;
     }
     const size_t wsb = p.splits > 1 ? (size_t)p.splits * B * N * 4 : 0;
     if (ws_need) *ws_need = std::max(*ws_need, wsb);
@@ -1048,6 +1062,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->a_mode = g.pm ? 2 : (p.rect_w ? 1 : 0);
       info->n_sms = std::max(info->n_sms, p.grid);   // pair granularity
       info->cta_group = p.cg;
+      info->t_unit_us = p.unit_us;
     }
     if (ws_need) *ws_need = std::max(*ws_need, p.splits > 1 ? (size_t)p.splits * g.M * g.out_cs * 4 : 0);
     if (!x) return PCNN_OK;   // planning only
@@ -1080,6 +1095,8 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->tlp = ly.tlp > 0 ? ly.tlp : net->occ_simt;
       info->engine = 0;
       info->cta_group = 1;
+      // one tm x tn tile over K at ~60% of 128 FFMA lanes, occ_simt CTAs per SM
+      info->t_unit_us = 2.0 * tm * tn * g.K / (0.6 * 256.0 * 1.9e9) * 1e6 * net->occ_simt;
     }
     if (!x) return PCNN_OK;
     Budget b = make_budget(net, ly, slot, true);
@@ -1885,21 +1902,33 @@ pcnn_status pcnn_set_layer_plan(pcnn_net *net, int layer, int cta_group, int m_s
   return PCNN_OK;
 }
 
-pcnn_status pcnn_plan_budget(const pcnn_net *cnet, int layer, int batch, pcnn_budget_plan *bp) {
-  pcnn_net *net = const_cast<pcnn_net *>(cnet);
-  if (!net || !bp || layer < 0 || layer >= (int)net->layers.size() || batch <= 0)
-    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+// eq. 12 on B200 (reading R12 / NEXT-3): t(n) = t_launch + nInvocations(n) x
+// t_unit.  The paper's form FLOPs / (peakFlops x optSM x rEC x FMA share) is
+// the per-wave term summed over full waves; on B200 a layer's latency also
+// carries a fixed cost per launch (launch, CTA rasterisation, barrier / TMEM
+// setup, pipeline fill, epilogue drain) that dominates at small batch.  The
+// per-unit time comes from the planner's own cost model (operand bytes at the
+// measured L2->SM rate vs. MMA cycles per K-block); the two constants per
+// kernel class were fitted to measured per-layer latencies over n in
+// {8..148} and B in {1, 64, 256} (tools/time_model_fit.py,
+// profiles/r02_time_model_fit.json).
+struct TimeModel { double launch_us, unit_scale; };
+static TimeModel time_model_class(const pcnn_layer_info &f) {
+  if (f.kind != PCNN_CONV && f.kind != PCNN_FC) return {kT0Simt, 1.0};
+  if (f.engine == 0) return {kT0Simt, 1.0};
+  if (f.a_mode == 3) return {kT0Fc, kScaleFc};
+  return {kT0Conv, kScaleConv};
+}
+
+static pcnn_status layer_time_model(pcnn_net *net, int layer, int batch, int n_sms,
+                                    pcnn_budget_plan *bp) {
   std::memset(bp, 0, sizeof *bp);
   Layer &ly = net->layers[layer];
   const int nsms = net->num_sms;
+  const int n = n_sms <= 0 ? nsms : std::min(n_sms, nsms);
   bp->opt_sm = nsms;
   bp->cta_group = 1;
   bp->opt_tlp = 1;
-  if (!ly.gemm) {
-    bp->t_model_us = layer_bytes(ly, batch, net->desc.precision,
-                                 layer == (int)net->layers.size() - 1) / 6.5e12 * 1e6;
-    return PCNN_OK;
-  }
   // the plan on the whole device (the budget in effect must not change it)
   const int save_sms = ly.n_sms, save_tlp = ly.tlp;
   ly.n_sms = 0;
@@ -1909,6 +1938,15 @@ pcnn_status pcnn_plan_budget(const pcnn_net *cnet, int layer, int batch, pcnn_bu
   ly.n_sms = save_sms;
   ly.tlp = save_tlp;
   if (s != PCNN_OK) return s;
+  const TimeModel tm = time_model_class(f);
+  bp->t_launch_us = tm.launch_us;
+  if (!ly.gemm) {
+    // HBM-bound: the bytes at min(HBM, n x the per-SM streaming rate)
+    const double bw = std::min(6.5e12, n * 60e9);
+    bp->t_unit_us = f.bytes / bw * 1e6;
+    bp->t_model_us = tm.launch_us + bp->t_unit_us;
+    return PCNN_OK;
+  }
   const int cg = std::max(1, f.cta_group);
   const long long G = f.tiles * std::max(1, f.splits);
   const int tlp = f.engine == 1 ? 1 : std::max(1, net->occ_simt);
@@ -1918,17 +1956,38 @@ pcnn_status pcnn_plan_budget(const pcnn_net *cnet, int layer, int batch, pcnn_bu
   while (p < slots && (G + (long long)tlp * p - 1) / ((long long)tlp * p) != inv) ++p;
   bp->grid_size = G;
   bp->opt_tlp = tlp;
-  bp->n_invocations = (int)inv;
   bp->cta_group = cg;
   bp->opt_sm = (int)(p * cg);
-  // eq. 12 (reading R12): peak per SM from the tensor / FFMA rate x SM clock
-  int khz = 0;
-  cudaDeviceGetAttribute(&khz, cudaDevAttrClockRate, net->device);
-  const double clk = khz > 0 ? khz * 1e3 : 1.965e9;
-  const double flop_per_clk = f.engine == 0 ? 256.0
-                              : (net->desc.precision == PCNN_TF32 ? 4096.0 : 8192.0);
-  const double eff = 0.8;
-  bp->t_model_us = f.flops / (flop_per_clk * clk * bp->opt_sm * std::max(f.rec, 1e-9) * eff) * 1e6;
+  // eq. 8 at the budget n (FC units need their whole K-split group at once)
+  long long slots_n = std::max<long long>(1, n / cg);
+  if (f.a_mode == 3) slots_n = std::max<long long>(f.splits, slots_n / f.splits * f.splits);
+  const long long inv_n = (G + (long long)tlp * slots_n - 1) / ((long long)tlp * slots_n);
+  bp->n_invocations = (int)(n_sms <= 0 ? inv : inv_n);
+  bp->t_unit_us = f.t_unit_us * tm.unit_scale;
+  bp->t_model_us = tm.launch_us + bp->n_invocations * bp->t_unit_us;
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_plan_budget(const pcnn_net *cnet, int layer, int batch, pcnn_budget_plan *bp) {
+  pcnn_net *net = const_cast<pcnn_net *>(cnet);
+  if (!net || !bp || layer < 0 || layer >= (int)net->layers.size() || batch <= 0)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  pcnn_status s = layer_time_model(net, layer, batch, 0, bp);
+  if (s != PCNN_OK) return s;
+  // t_model_us at opt_sm: eq. 11 keeps nInvocations, so the time is the
+  // whole-device time by construction
+  return PCNN_OK;
+}
+
+pcnn_status pcnn_model_layer_time(const pcnn_net *cnet, int layer, int batch, int n_sms,
+                                  double *t_us) {
+  pcnn_net *net = const_cast<pcnn_net *>(cnet);
+  if (!net || !t_us || layer < 0 || layer >= (int)net->layers.size() || batch <= 0 || n_sms < 0)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "bad arguments");
+  pcnn_budget_plan bp;
+  pcnn_status s = layer_time_model(net, layer, batch, n_sms, &bp);
+  if (s != PCNN_OK) return s;
+  *t_us = bp.t_model_us;
   return PCNN_OK;
 }
 

@@ -106,6 +106,15 @@ __device__ __forceinline__ void tma_im2col_2sm(uint32_t dst, const CUtensorMap *
       "h"(oh)
       : "memory");
 }
+// plain bulk copy global -> shared (no tensor map), bytes counted on `bar`
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes,
+                                         uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          dst),
+      "l"(src), "r"(bytes), "r"(bar)
+      : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }

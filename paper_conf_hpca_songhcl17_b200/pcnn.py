@@ -63,7 +63,7 @@ class LayerInfo(ctypes.Structure):
                 ("tile_n", ctypes.c_int), ("tiles", ctypes.c_longlong), ("grid", ctypes.c_int),
                 ("util", ctypes.c_double), ("rec", ctypes.c_double), ("splits", ctypes.c_int),
                 ("a_mode", ctypes.c_int), ("halo_in", ctypes.c_int), ("halo_out", ctypes.c_int),
-                ("cta_group", ctypes.c_int)]
+                ("cta_group", ctypes.c_int), ("t_unit_us", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -72,7 +72,8 @@ class LayerInfo(ctypes.Structure):
 class BudgetPlan(ctypes.Structure):
     _fields_ = [("grid_size", ctypes.c_longlong), ("opt_tlp", ctypes.c_int),
                 ("n_invocations", ctypes.c_int), ("opt_sm", ctypes.c_int),
-                ("cta_group", ctypes.c_int), ("t_model_us", ctypes.c_double)]
+                ("cta_group", ctypes.c_int), ("t_model_us", ctypes.c_double),
+                ("t_launch_us", ctypes.c_double), ("t_unit_us", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -95,6 +96,8 @@ _lib.pcnn_output_size.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.pcnn_num_layers.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.pcnn_query_layer.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.POINTER(LayerInfo)]
 _lib.pcnn_plan_budget.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.POINTER(BudgetPlan)]
+_lib.pcnn_model_layer_time.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                       ctypes.POINTER(ctypes.c_double)]
 _lib.pcnn_describe_net.argtypes = [ctypes.POINTER(NetDesc), ctypes.POINTER(LayerDesc),
                                    ctypes.c_int, ctypes.c_int, ctypes.POINTER(LayerInfo)]
 _lib.pcnn_profile_layers.argtypes = [_P, _P, ctypes.c_int, _P, ctypes.c_int, _FP, _FP, _P]
@@ -112,7 +115,7 @@ _lib.pcnn_last_error_message.restype = ctypes.c_char_p
 for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_layer_plan",
            "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
-           "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
+           "pcnn_model_layer_time", "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
            "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
            "pcnn_last_launch_count"):
     getattr(_lib, _f).restype = ctypes.c_int
@@ -120,7 +123,7 @@ for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
 EXPORTED = ["pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
             "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_layer_plan",
             "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
-            "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
+            "pcnn_model_layer_time", "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
             "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
             "pcnn_last_launch_count", "pcnn_device_sm_count", "pcnn_version",
             "pcnn_status_string", "pcnn_last_error_message"]
@@ -296,6 +299,13 @@ class Net:
         _check(_lib.pcnn_plan_budget(self._h, layer, batch, ctypes.byref(bp)),
                "pcnn_plan_budget")
         return bp.as_dict()
+
+    def model_layer_time(self, layer, batch, n_sms=0):
+        """eq. 12 (NEXT-3): modelled latency in us of one layer on n_sms SMs."""
+        t = ctypes.c_double()
+        _check(_lib.pcnn_model_layer_time(self._h, layer, batch, n_sms, ctypes.byref(t)),
+               "pcnn_model_layer_time")
+        return t.value
 
     def apply_opt_budgets(self, batch):
         """Give every GEMM layer its eq. 11 optSM x optTLP budget (P:341);

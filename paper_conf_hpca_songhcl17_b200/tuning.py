@@ -18,9 +18,12 @@ uncertainty CNN_entropy from the fused softmax + entropy kernel, eq. 2).
 * Tuning stops when no eligible candidate remains.  Each adopted state is a
   *tuning table*: the per-layer rungs plus every layer's optSM (eq. 11) for
   the run-time kernel scheduler.
-* *Calibration* (P:345): at run time, if the observed entropy exceeds the
-  threshold, step back along the path to the most aggressive table whose
-  tuning-time entropy was below the observed-adjusted bound.
+* *Calibration* (P:345): at run time P-CNN monitors the output uncertainty;
+  while it exceeds the threshold, it switches to the previous (slower, more
+  precise) table of the tuning path and measures again, until the measured
+  uncertainty is below the threshold or the exact table is reached.
+* P:335's rEC rule: the perforation rungs are chosen so that the GEMM's M
+  dimension (B x W'_o H'_o) is a multiple of the tile's M (eq. 9, rEC = 1).
 """
 import math
 
@@ -64,15 +67,54 @@ def greedy_tune(ladders, measure, threshold, max_iters=64):
     return path
 
 
-def calibrate(path, index, observed_entropy, threshold):
-    """while the observed uncertainty exceeds the threshold, back-track
-    one table along the tuning path (towards exact).  Returns the new index.
-    The entropy the inputs now produce is estimated by shifting the tuned
-    entropies by (observed - tuned) at the current index."""
+def calibrate(path, index, observe, threshold):
+    """P:345 ("monitors the uncertainty of the output ... switches to a slower
+    but more precise version ... by backtracking along the tuning path ...
+    until the output uncertainty is less than the pre-defined threshold").
+
+    observe(index) programs table `index` of the path and returns the
+    CNN_entropy the current inputs produce under it (a measurement, eq. 2).
+    Starting from the current table, while the measured entropy exceeds the
+    threshold, step back one table and measure again.  Returns (index, trace)
+    where trace lists every (index, measured entropy) visited."""
+    h = observe(index)
+    trace = [(index, h)]
+    while h > threshold and index > 0:
+        index -= 1
+        h = observe(index)
+        trace.append((index, h))
+    return index, trace
+
+
+def calibrate_estimate(path, index, observed_entropy, threshold):
+    """Cheap predictor for calibrate (no re-measurement): shift the tuned
+    entropies by (observed - tuned) at the current index and back-track while
+    the shifted value exceeds the threshold."""
     shift = observed_entropy - path[index]["entropy"]
     while index > 0 and path[index]["entropy"] + shift > threshold:
         index -= 1
     return index
+
+
+def perforation_ladder(out_h, out_w, batch, tile_m=128, max_step=4, rec_min=1.0):
+    """Perforation rungs of one conv layer honouring P:335 ("make sure that
+    W_o H_o ... is a multiple of n", reading R13 / eq. 9): the grid steps
+    (sh, sw) in 1..max_step whose kept positions give a GEMM M = batch x
+    ceil(H/sh) x ceil(W/sw) with rEC >= rec_min for the tile M, ordered from
+    exact to the highest perforation rate (ties: fewer kept rows first kept).
+    Returns [("exact",), ("perf", sh, sw), ...]."""
+    cands = []
+    for sh in range(1, max_step + 1):
+        for sw in range(1, max_step + 1):
+            if sh * sw == 1:
+                continue
+            kept = -(-out_h // sh) * -(-out_w // sw)
+            m = batch * kept
+            rec = m / (-(-m // tile_m) * tile_m)
+            if rec >= rec_min - 1e-12:
+                cands.append((kept, sh, sw))
+    cands.sort(key=lambda c: (-c[0], c[1], c[2]))
+    return [("exact",)] + [("perf", sh, sw) for _, sh, sw in cands]
 
 
 def apply_state(net, ladders, state, batch=None):
@@ -87,6 +129,17 @@ def apply_state(net, ladders, state, batch=None):
             net.set_perforation(l, v[1], v[2])
     if batch is not None:
         net.apply_opt_budgets(batch)
+
+
+def gpu_observe(net, ladders, path, images):
+    """observe() for calibrate on the GPU: program table `index` of the path
+    and return the mean CNN_entropy (eq. 2, the fused softmax + entropy
+    kernel) of the current inputs."""
+    def observe(index):
+        apply_state(net, ladders, path[index]["state"])
+        _, _, ent = net.infer(images, entropy=True)
+        return float(ent.mean().item())
+    return observe
 
 
 def gpu_measure(net, ladders, images, reps=10):

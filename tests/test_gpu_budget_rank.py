@@ -40,7 +40,9 @@ def test_budget_is_bitwise_invariant_and_census_bounded(alex, prec):
         np.testing.assert_array_equal(r["out"], base, err_msg="budget %d/%d" % (n_sms, tlp))
         for i in gemm_layers:
             used = r["census"][i]
-            floor = r["net"].query_layer(i, x.shape[0])["splits"] if net["layers"][i]["kind"] == "fc" else 2
+            # an FC layer's K split needs all its CTA pairs at once
+            floor = 2 * r["net"].query_layer(i, x.shape[0])["splits"] \
+                if net["layers"][i]["kind"] == "fc" else 2
             assert 0 < len(used) <= max(n_sms, floor), (i, n_sms, used)
 
 

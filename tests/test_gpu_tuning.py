@@ -40,11 +40,19 @@ def test_greedy_tuning_on_alexnet():
         assert len(diff) == 1 and c["state"][diff[0]] == a["state"][diff[0]] + 1
         assert c["time"] < a["time"] and c["entropy"] <= threshold
         assert c["te"] == math.inf or c["te"] > 0
-    # calibration on the resulting path: an impossible observation falls back
-    # to the exact table, a benign one keeps the current table
+    # calibration on the resulting path, re-measuring the entropy of
+    # the inputs at every back-track step: a permissive threshold keeps the
+    # current table after one measurement; a threshold below every table's
+    # measured entropy walks back to the exact table, measuring each
     last = len(path) - 1
-    assert tuning.calibrate(path, last, path[last]["entropy"], threshold) == last
-    assert tuning.calibrate(path, last, 1e9, threshold) == 0
+    observe = tuning.gpu_observe(n, ladders, path, x)
+    idx, trace = tuning.calibrate(path, last, observe, threshold)
+    assert idx == last and len(trace) == 1
+    idx, trace = tuning.calibrate(path, last, observe, -1.0)
+    assert idx == 0 and [t[0] for t in trace] == list(range(last, -1, -1))
+    # the measured entropies reproduce the tuning-time ones (same inputs)
+    for i, h in trace:
+        assert abs(h - path[i]["entropy"]) < 1e-4
     # the tuned state programs the net and still infers finite probabilities
     tuning.apply_state(n, ladders, path[-1]["state"], batch=B)
     out, p, h = n.infer(x, probs=True, entropy=True)

@@ -39,12 +39,46 @@ def test_greedy_follows_fig12():
     assert abs(path[3]["te"] - 5.0) < 1e-9
 
 
-def test_calibration_backtracks():
+def test_calibration_backtracks_with_remeasurement():
+    """measure, and while the measured uncertainty is above the
+    threshold step back one table and measure AGAIN (hand-worked traces:
+    the new inputs make every table 0.3 nats less certain than at tuning)."""
     path = [{"entropy": 1.0}, {"entropy": 1.2}, {"entropy": 1.4}]
-    # observed 1.6 at table 2 (shift +0.2): table 1 -> 1.4 <= 1.5 is the first safe one
-    assert tuning.calibrate(path, 2, 1.6, 1.5) == 1
-    assert tuning.calibrate(path, 2, 1.45, 1.5) == 2          # within threshold: stay
-    assert tuning.calibrate(path, 2, 3.0, 1.5) == 0           # back to exact
+    calls = []
+
+    def observe(i):
+        calls.append(i)
+        return path[i]["entropy"] + 0.3
+    idx, trace = tuning.calibrate(path, 2, observe, 1.5)
+    assert idx == 1 and calls == [2, 1] and trace == [(2, 1.7), (1, 1.5)]
+    # within the threshold: one measurement, stay
+    calls.clear()
+    idx, trace = tuning.calibrate(path, 2, lambda i: calls.append(i) or 1.45, 1.5)
+    assert idx == 2 and calls == [2]
+    # never satisfied: every table is measured down to exact, which is kept
+    idx, trace = tuning.calibrate(path, 2, lambda i: 9.0, 1.5)
+    assert idx == 0 and [t[0] for t in trace] == [2, 1, 0]
+    # the shift estimator agrees on the first trace without measuring
+    assert tuning.calibrate_estimate(path, 2, 1.6, 1.5) == 1
+    assert tuning.calibrate_estimate(path, 2, 3.0, 1.5) == 0
+
+
+def test_perforation_ladder_rec_rule():
+    """W_o H_o (x batch: the GEMM M) a multiple of the tile's n.
+    AlexNet conv2 27 x 27 at batch 128: kept grids 14 x 27 (sh = 2) ->
+    128 x 378 = 48384 = 378 x 128 (rEC 1); 27 x 14 likewise; 9 x 27 ->
+    128 x 243, a multiple of 128 too; every rung has rEC = 1."""
+    lad = tuning.perforation_ladder(27, 27, 128)
+    assert lad[0] == ("exact",)
+    for r in lad[1:]:
+        _, sh, sw = r
+        kept = -(-27 // sh) * -(-27 // sw)
+        assert (128 * kept) % 128 == 0
+    # at batch 1 most grids are not multiples of 128: only rEC-1 ones remain
+    lad1 = tuning.perforation_ladder(16, 16, 1)
+    kept1 = [-(-16 // sh) * -(-16 // sw) for _, sh, sw in lad1[1:]]
+    assert kept1 and all(k % 128 == 0 for k in kept1) and kept1 == sorted(kept1, reverse=True)
+    assert ("perf", 1, 2) in lad1 and ("perf", 2, 2) not in lad1          # 128 kept vs 64
 
 
 def test_background_batch_rule():

@@ -69,8 +69,15 @@ if meter.read_j() is not None:
                                              t_i, t_t, threshold),
                            "t_i_ms": t_i, "t_t_ms": t_t})
 last = len(path) - 1
-out["calibration"] = {str(h): tuning.calibrate(path, last, h, threshold)
-                      for h in (path[last]["entropy"], threshold, threshold + 0.5, 1e9)}
+# calibration with re-measurement: new inputs (another image range)
+# observed under the last table, stepping back while the measured entropy
+# exceeds the threshold; and the shift estimator for comparison
+x2 = torch.from_numpy(synth.images(4096, B, net["in_shape"], lo=-160, hi=160)).cuda()
+idx, trace = tuning.calibrate(path, last, tuning.gpu_observe(n, ladders, path, x2), threshold)
+out["calibration"] = {"new_inputs": "images 4096.. at U[-160, 160)", "final_table": idx,
+                      "trace": [[i, round(h, 5)] for i, h in trace],
+                      "estimate_only": {str(h): tuning.calibrate_estimate(path, last, h, threshold)
+                                        for h in (path[last]["entropy"], threshold + 0.5, 1e9)}}
 # NEXT-4: background-task batch (every conv layer at Util = 1, eq. 6) on this
 # net's own tile plans, and eq. 13's rescaled batch for a 0.2 ms requirement
 nb = pcnn.Net(net, w, b, 256, "bf16")
