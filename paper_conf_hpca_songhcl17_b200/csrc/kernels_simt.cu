@@ -9,7 +9,6 @@
 #include "budget.cuh"
 #include "lrn_math.cuh"
 #include "pcnn_internal.h"
-#include "tc_ptx.cuh"
 
 namespace pcnn {
 
@@ -1574,228 +1573,6 @@ long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int
 }
 
 
-// LRN (size 5, across channels, R3) + pooling over bands of R output rows,
-// the band's input rows fetched by bulk copies into shared memory (one
-// mbarrier; the copies of one CTA overlap the other CTAs' compute on the SM).
-// The LRN runs in place in shared memory in rounds of whole pixels: a task =
-// one pixel x 4 chunks of 16 B (32 BF16 / 16 FP32 channels); every thread
-// first reads its chunks and the 2 channels on each side (the window's
-// neighbours in the adjacent tasks of the same pixel), the CTA syncs, then it
-// normalises (lrn_normalise: the same sum order and transcendental form as
-// every other LRN path) and writes its chunks back -- rounds cover whole
-// pixels, so no task reads a channel another round writes.  Then the band is
-// max / avg pooled from shared memory straight to the output layout (group
-// padding, halos).  Per element: ~9 FP32 ops + 2 MUFU (lg2, ex2), against ~26
-// instructions of the register-shuffle kernel; the input read is one bulk
-// copy per row instead of per-thread 16-B loads.
-template <int ST>
-__global__ void __launch_bounds__(256) lrn_bulk_kernel(const LrnPoolArgs a) {
-  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
-  extern __shared__ __align__(128) uint8_t lk_raw[];
-  constexpr int ESZ = ST == ST_BF16 ? 2 : 4;
-  constexpr int VN = Vec16<ST>::N;
-  constexpr int GC = 4 * VN;                    // channels per task
-  uint8_t *band = lk_raw + 128;                 // [nr][Wp][C] input rows, LRN in place
-  const uint32_t bar = smem_u32(lk_raw);
-  const int C = a.C, ngroups = C / GC, chunks = C / VN;
-  const int Hp = a.H + 2 * a.hi, Wp = a.W + 2 * a.hi;
-  const int Hop = a.Ho + 2 * a.ho, Wop = a.Wo + 2 * a.ho;
-  const int per_round = (256 / ngroups) * ngroups;
-  const float inv_ng = 1.f / (float)ngroups, inv_w = 1.f / (float)a.W;
-  const long long tiles = (long long)a.B * a.nbands;
-  const int tid = threadIdx.x;
-  if (tid == 0) {
-    mbar_init(bar, 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  uint32_t phase = 0;
-
-  for_each_tile(a.b, tiles, [&](long long t) {
-    const int bnd = (int)(t % a.nbands);
-    const long long n = t / a.nbands;
-    const int p0 = bnd * a.R, p1 = min(p0 + a.R, a.Ho);
-    const int h0 = p0 * a.s, h1 = min((p1 - 1) * a.s + a.k, a.H);
-    const int nr = h1 - h0;
-    __syncthreads();                     // the previous band's pooling is done with smem
-    if (tid == 0) {
-      const size_t rowb = (size_t)Wp * C * ESZ;
-      mbar_arrive_expect_tx(bar, (uint32_t)(rowb * nr));
-      const char *src = (const char *)a.x + ((size_t)n * Hp + h0 + a.hi) * rowb;
-      for (int r = 0; r < nr; ++r)
-        bulk_g2s(smem_u32(band) + (uint32_t)(r * rowb), src + r * rowb, (uint32_t)rowb, bar);
-    }
-    if (a.ho > 0) {                      // output halo zeros (the next conv's padding)
-      const int oc16 = a.Cout * ESZ / 16;
-      const uint4 z = make_uint4(0, 0, 0, 0);
-      uint4 *yb = (uint4 *)a.y;
-      if (p0 == 0)
-        for (int v = tid; v < a.ho * Wop * oc16; v += blockDim.x)
-          yb[(size_t)n * Hop * Wop * oc16 + v] = z;
-      if (p1 == a.Ho)
-        for (int v = tid; v < a.ho * Wop * oc16; v += blockDim.x)
-          yb[((size_t)n * Hop + a.Ho + a.ho) * Wop * oc16 + v] = z;
-      for (int v = tid; v < (p1 - p0) * 2 * a.ho * oc16; v += blockDim.x) {
-        const int rr = v / (2 * a.ho * oc16), e = v - rr * 2 * a.ho * oc16;
-        const int side = e / (a.ho * oc16), o = e - side * a.ho * oc16;
-        const size_t rowb = ((size_t)n * Hop + p0 + rr + a.ho) * Wop * oc16;
-        yb[rowb + (side ? (size_t)(a.Wo + a.ho) * oc16 : 0) + o] = z;
-      }
-    }
-    mbar_wait(bar, phase);
-    phase ^= 1;
-    // ---- LRN in place, rounds of whole pixels
-    const int ntasks = nr * a.W * ngroups;
-    for (int r0 = 0; r0 < ntasks; r0 += per_round) {
-      const int task = r0 + tid;
-      const bool mine = tid < per_round && task < ntasks;
-      uint4 raw[4];
-      float lb[2] = {0.f, 0.f}, rb[2] = {0.f, 0.f};
-      uint8_t *p = band;
-      if (mine) {
-        int pix, g, r, col;
-        fdivmod(task, ngroups, inv_ng, pix, g);
-        fdivmod(pix, a.W, inv_w, r, col);
-        p = band + ((size_t)(r * Wp + col + a.hi) * C + g * GC) * ESZ;
-#pragma unroll
-        for (int j = 0; j < 4; ++j) raw[j] = *(const uint4 *)(p + 16 * j);
-        if constexpr (ST == ST_BF16) {
-          if (g > 0) {
-            const uint32_t w = *(const uint32_t *)(p - 4);
-            lb[0] = __uint_as_float(w << 16);
-            lb[1] = __uint_as_float(w & 0xFFFF0000u);
-          }
-          if (g + 1 < ngroups) {
-            const uint32_t w = *(const uint32_t *)(p + GC * ESZ);
-            rb[0] = __uint_as_float(w << 16);
-            rb[1] = __uint_as_float(w & 0xFFFF0000u);
-          }
-        } else {
-          if (g > 0) {
-            const float2 w = *(const float2 *)(p - 8);
-            lb[0] = w.x;
-            lb[1] = w.y;
-          }
-          if (g + 1 < ngroups) {
-            const float2 w = *(const float2 *)(p + GC * ESZ);
-            rb[0] = w.x;
-            rb[1] = w.y;
-          }
-        }
-      }
-      __syncthreads();                   // every task has read its window
-      if (mine) {
-        float x[GC], sq[GC + 4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          Vec16<ST> v;
-          v.from_raw(raw[j]);
-#pragma unroll
-          for (int i = 0; i < VN; ++i) x[j * VN + i] = v.v[i];
-        }
-        sq[0] = lb[0] * lb[0];
-        sq[1] = lb[1] * lb[1];
-#pragma unroll
-        for (int i = 0; i < GC; ++i) sq[i + 2] = x[i] * x[i];
-        sq[GC + 2] = rb[0] * rb[0];
-        sq[GC + 3] = rb[1] * rb[1];
-        float o[GC];
-        lrn_normalise<ST == ST_BF16, 5, GC>(sq, x, a.lrn_k, a.lrn_alpha_over_n, a.lrn_beta, o);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          Vec16<ST> v;
-#pragma unroll
-          for (int i = 0; i < VN; ++i) v.v[i] = o[j * VN + i];
-          v.store(p + 16 * j, a.tf32_round);
-        }
-      }
-    }
-    __syncthreads();
-    // ---- pool (k = s = 1: copy) the normalised rows straight to the output
-    const float inv = 1.f / (float)(a.k * a.k);
-    const int ochunks = a.Cout / VN;
-    const float inv_oc = 1.f / (float)ochunks;
-    const int grp_real = a.ocg / VN, grp_pad = a.ocp / VN;
-    const int nq = a.Wo * ochunks;
-    const float inv_nq = 1.f / (float)nq;
-    for (int v = tid; v < (p1 - p0) * nq; v += blockDim.x) {
-      int rr, q, oc;
-      if (nq <= 1024) fdivmod(v, nq, inv_nq, rr, q);
-      else { rr = v / nq; q = v - rr * nq; }
-      fdivmod(q, ochunks, inv_oc, q, oc);
-      const int pp = p0 + rr;
-      int c = oc;
-      bool pad = false;
-      if (grp_pad > 0) {
-        const int gi = oc / grp_pad, j = oc - gi * grp_pad;
-        pad = j >= grp_real;
-        c = gi * grp_real + j;
-      }
-      char *dst = (char *)a.y + ((((size_t)n * Hop + pp + a.ho) * Wop + q + a.ho) * a.Cout + oc * VN) * ESZ;
-      const int rs = pp * a.s - h0, re = min(rs + a.k, nr);
-      const int cs = q * a.s, ce = min(cs + a.k, a.W);
-      auto at = [&](int r, int col) {
-        return band + ((size_t)(r * Wp + col + a.hi) * C + c * VN) * ESZ;
-      };
-      if (ST == ST_BF16 && a.is_max) {
-        __nv_bfloat162 m[4];
-        const __nv_bfloat162 ninf = __float2bfloat162_rn(-INFINITY);
-        const __nv_bfloat162 zero = __float2bfloat162_rn(0.f);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) m[j] = pad ? zero : ninf;
-        auto take = [&](int r, int col) {
-          const uint4 raw = *(const uint4 *)at(r, col);
-          const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
-#pragma unroll
-          for (int j = 0; j < 4; ++j) m[j] = __hmax2(m[j], h[j]);
-        };
-        if (!pad) {
-          if (re - rs == 3 && ce - cs == 3) {      // AlexNet's 3 x 3 windows, unclipped
-#pragma unroll
-            for (int dr = 0; dr < 3; ++dr)
-#pragma unroll
-              for (int dc = 0; dc < 3; ++dc) take(rs + dr, cs + dc);
-          } else {
-            for (int r = rs; r < re; ++r)
-              for (int col = cs; col < ce; ++col) take(r, col);
-          }
-        }
-        *(uint4 *)dst = *(const uint4 *)m;
-        continue;
-      }
-      Vec16<ST> acc, cur;
-#pragma unroll
-      for (int j = 0; j < VN; ++j) acc.v[j] = pad ? 0.f : (a.is_max ? -INFINITY : 0.f);
-      if (!pad) {
-        for (int r = rs; r < re; ++r)
-          for (int col = cs; col < ce; ++col) {
-            cur.load(at(r, col));
-#pragma unroll
-            for (int j = 0; j < VN; ++j)
-              acc.v[j] = a.is_max ? fmaxf(acc.v[j], cur.v[j]) : acc.v[j] + cur.v[j];
-          }
-        if (!a.is_max)
-#pragma unroll
-          for (int j = 0; j < VN; ++j) acc.v[j] *= inv;
-      }
-      acc.store(dst, a.is_max ? 0 : a.tf32_round);
-    }
-  });
-}
-
-// Output rows per band of lrn_bulk_kernel: the largest R whose staged input
-// rows fit ~100 KB (two CTAs per SM), 0 if the layout does not qualify
-// (LRN size 5, C a multiple of 4 x 16 B chunks, < 64 KB per row).
-static int lrn_bulk_rows(int st, int W, int C, int k, int s, int Ho, int halo) {
-  const int esz = st == ST_BF16 ? 2 : 4, gc = 4 * (16 / esz);
-  if (C % gc || C / gc > 256) return 0;
-  const size_t row = (size_t)(W + 2 * halo) * C * esz;
-  if (row % 16 || row > 64 * 1024) return 0;
-  int R = 0;
-  while (R < Ho && (size_t)(R * s + k) * row <= 100 * 1024) ++R;
-  return R;
-}
-
 // Plain pooling (no LRN, no group padding) straight from global memory: one
 // thread per (output pixel, 16 B channel chunk), chunk fastest, so each warp
 // reads whole runs of input pixels; K = 2 / 3 windows are unrolled (VGG 2x2
@@ -1921,30 +1698,6 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.ho = out_halo;
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
-  if (lrn_size == 5 && !exp_env("PCNN_LRN_REG")) {
-    // bulk-copy band kernel (the default for LRN size 5)
-    const int R = lrn_bulk_rows(st, W, C, k, s, Ho, in_halo);
-    if (R > 0) {
-      a.R = R;
-      a.nbands = (Ho + R - 1) / R;
-      const size_t smem =
-          128 + (size_t)min((R - 1) * s + k, H) * (W + 2 * in_halo) * C * esz;
-      auto go = [&](auto kern) -> cudaError_t {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        int g = grid;
-        if (!b.gated) {
-          int dev = 0, sms = 148, occ = 1;
-          cudaGetDevice(&dev);
-          cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 256, smem);
-          g = (int)std::min<long long>((long long)B * a.nbands, (long long)sms * std::max(occ, 1));
-        }
-        launch_pdl(kern, dim3(g), dim3(256), smem, stream, a);
-        return cudaGetLastError();
-      };
-      return st == ST_BF16 ? go(lrn_bulk_kernel<ST_BF16>) : go(lrn_bulk_kernel<ST_F32>);
-    }
-  }
   if (use_lrn_reg(st, C, lrn_size)) {
     a.R = lrn_band_rows(st, W, C, k, s, Ho, lrn_size);
     a.nbands = (Ho + a.R - 1) / a.R;

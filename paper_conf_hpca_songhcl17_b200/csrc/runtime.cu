@@ -748,8 +748,11 @@ static const CUtensorMap *stage_ymap(GemmStage &gs, void *y, long long M) {
 // ~80% of its nominal rate in this kernel.
 static constexpr double kOperandBytesPerCycle = 36.0;
 // eq. 12 time-model constants (NEXT-3; fitted, see layer_time_model)
-static constexpr double kT0Conv = 4.0, kScaleConv = 1.0;   // tcgen05 conv: launch us, unit scale
-static constexpr double kT0Fc = 6.0, kScaleFc = 1.0;       // weight-streaming FC
+static constexpr double kT0Conv = 13.07, kScaleConv = 0.534;   // tcgen05 conv: launch us, unit scale
+// (profiles/r02_time_model_fit.json; measured with live per-layer events,
+// which serialise launches -- inside a CUDA graph with PDL the launch term
+// mostly overlaps the previous layer)
+static constexpr double kT0Fc = 15.22, kScaleFc = 0.745;   // weight-streaming FC
 static constexpr double kT0Simt = 3.0;                     // SIMT kernels (LRN / pool / check path)
 static constexpr double kMmaEfficiency = 0.8;
 
@@ -961,12 +964,16 @@ static FcPlan plan_fc(int N, int kblocks, int B, int device_sms, int budget_sms)
   const int units = p.rblocks * p.chunks;
   p.groups = std::max(1, std::min(units, std::min(budget_sms, device_sms) / (2 * s)));
   p.grid = 2 * s * p.groups;
-  // per K-block a CTA ingests one 16 KB weight tile + nb / 2 activation rows
-  // at the measured ~36 B/clk/SM of TMA operand delivery; the pair's MMA
-  // (256 x nb x 64) takes nb / 2 cycles per 16-deep UMMA step x 4
+  // per K-block a CTA ingests one contiguous 16 KB weight tile + nb / 2
+  // activation rows at the measured ~60 B/clk/SM of this kernel's TMA stream
+  // (tools/time_model_fit.py: 5.4 us per 590 KB unit of fc6 at batch 1); the
+  // pair's MMA (256 x nb x 64) takes nb / 2 cycles per 16-deep UMMA step x 4
   const double f = 1.9e9;
-  const double load = (16384.0 + 64.0 * p.nb) / 36.0, mma = 4.0 * std::max(16, p.nb / 2) / 0.8;
-  p.unit_us = ((double)p.kbps * (std::max(load, mma) + 40.0) / f + 2e-6) * 1e6;
+  const double load = (16384.0 + 64.0 * p.nb) / 60.0, mma = 4.0 * std::max(16, p.nb / 2) / 0.8;
+  // + the split-K partial tile (written, then s slices of it read back by
+  // the reduction): 2 x 128 rows x nb x 4 B per CTA through L2
+  const double red = s > 1 ? 2.0 * 128.0 * p.nb * 4.0 / 36.0 : 0.0;
+  p.unit_us = ((double)p.kbps * (std::max(load, mma) + 40.0) / f + red / f + 2e-6) * 1e6;
   return p;
 }
 
