@@ -1582,23 +1582,32 @@ template <int ST, int K>
 __global__ void __launch_bounds__(256)
 pool_direct_kernel(const uint4 *__restrict__ x, uint4 *__restrict__ y, int B, int H, int W,
                    int chunks, int kk, int s, int is_max, int Ho, int Wo, int hi, int ho,
-                   int tf32_round, Budget bud) {
+                   int tf32_round, int ochunks, int grp_real, int grp_pad, Budget bud) {
   pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int VN = Vec16<ST>::N;
   const int k = K > 0 ? K : kk;
   const int Hp = H + 2 * hi, Wp = W + 2 * hi, Hop = Ho + 2 * ho, Wop = Wo + 2 * ho;
-  const long long total = (long long)B * Hop * Wop * chunks;
+  // output chunks: `chunks` input chunks, or (grp_pad > 0) each group's
+  // grp_real chunks padded with zeros to grp_pad (the layout a grouped conv
+  // reads with whole 128-B TMA slabs)
+  const long long total = (long long)B * Hop * Wop * ochunks;
   const float inv = 1.f / (float)(k * k);
   if (threadIdx.x == 0) census_mark(bud);
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
        i += (long long)gridDim.x * blockDim.x) {
-    const int ch = (int)(i % chunks);
-    const long long pix = i / chunks;
+    int ch = (int)(i % ochunks);
+    const long long pix = i / ochunks;
     const int q = (int)(pix % Wop) - ho;
     const long long t = pix / Wop;
     const int p = (int)(t % Hop) - ho;
     const long long n = t / Hop;
-    if (p < 0 || p >= Ho || q < 0 || q >= Wo) {
+    bool pad = false;
+    if (grp_pad > 0) {
+      const int gi = ch / grp_pad, j = ch - gi * grp_pad;
+      pad = j >= grp_real;
+      ch = gi * grp_real + j;
+    }
+    if (pad || p < 0 || p >= Ho || q < 0 || q >= Wo) {
       y[i] = make_uint4(0, 0, 0, 0);
       continue;
     }
@@ -1656,14 +1665,16 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   const int ocp = out_groups > 0 ? out_cg_pad : 0;
   if (out_groups > 0 && (C % out_groups || ocg % vn || ocp % vn || ocp < ocg))
     return cudaErrorInvalidValue;
-  if (lrn_size == 0 && out_groups == 0 && !b.gated && !exp_env("PCNN_OLD_POOL")) {
+  if (lrn_size == 0 && !b.gated && !exp_env("PCNN_OLD_POOL")) {
     const int chunks = C / vn;
-    const long long total = (long long)B * (Ho + 2 * out_halo) * (Wo + 2 * out_halo) * chunks;
+    const int gr = out_groups > 0 ? ocg / vn : 0, gp = out_groups > 0 ? ocp / vn : 0;
+    const int ochunks = out_groups > 0 ? out_groups * gp : chunks;
+    const long long total = (long long)B * (Ho + 2 * out_halo) * (Wo + 2 * out_halo) * ochunks;
     const int g = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
 #define PCNN_PD(STT, KK)                                                                       \
   launch_pdl(pool_direct_kernel<STT, KK>, dim3(g), dim3(256), 0, stream, (const uint4 *)x, (uint4 *)y, B, H, W,    \
                                                      chunks, k, s, is_max, Ho, Wo, in_halo,    \
-                                                     out_halo, tf32_round, b)
+                                                     out_halo, tf32_round, ochunks, gr, gp, b)
     if (st == ST_BF16) {
       if (k == 2) PCNN_PD(ST_BF16, 2); else if (k == 3) PCNN_PD(ST_BF16, 3); else PCNN_PD(ST_BF16, 0);
     } else {
