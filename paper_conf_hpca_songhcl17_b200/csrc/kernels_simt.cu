@@ -267,10 +267,11 @@ stage_im2col_kernel(const float *__restrict__ x, void *y, int H, int W, int Ho, 
   }
   asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
   __syncthreads();
-  // rows of a zero-haloed output grid (Ho + 2 halo) x (Wo + 2 halo): the
-  // interior only (the consumer never reads the halo rows of a 1x1 conv)
-  const int Wop = Wo + 2 * halo;
-  char *yrow = (char *)y + ((size_t)(n * (Ho + 2 * halo) + p + halo) * Wop + halo) * Kp * ESZ;
+  // rows of a zero-haloed output grid (Ho + halo) x (Wo + halo) (shared
+  // halo layout, interior at the origin): the interior only (the consumer
+  // never reads the halo rows of a 1x1 conv)
+  const int Wop = Wo + halo;
+  char *yrow = (char *)y + ((size_t)(n * (Ho + halo) + p) * Wop) * Kp * ESZ;
   for (int q = threadIdx.x; q < Wo; q += blockDim.x) {
     float v[K];
 #pragma unroll
@@ -369,11 +370,11 @@ stage_gather3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, 
   asm volatile("cp.async.commit_group;\ncp.async.wait_all;" ::: "memory");
   __syncthreads();
   // phase 2: thread = (pixel, 16 B output chunk)
-  const int Wop = Wo + 2 * halo;
+  const int Wop = Wo + halo;                         // shared-halo output grid
   const int ppi = blockDim.x / chunks;               // pixels per pass
   for (int hh = 0; hh < nh; ++hh) {
     const int h = h0 + hh;
-    char *yrow = (char *)y + ((size_t)(n * (Ho + 2 * halo) + h + halo) * Wop + halo) *
+    char *yrow = (char *)y + ((size_t)(n * (Ho + halo) + h) * Wop) *
                                  (size_t)Kp * (ST == ST_BF16 ? 2 : 4);
     // per channel of this thread's chunk: smem index of input column 0 of its
     // row in this output row, minus the pad (can be negative: the sentinel for
@@ -536,7 +537,7 @@ stage_im2c3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, in
   const long long tiles = (long long)B * bands;
   const uintptr_t xend = (uintptr_t)(x + (size_t)B * C * H * W);
   const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bar);
-  const int Hp = H + 2 * halo, Wp = W + 2 * halo;
+  const int Hp = H + halo, Wp = W + halo;        // shared-halo output grid
   if (threadIdx.x == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0));
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8));
@@ -575,7 +576,7 @@ stage_im2c3_kernel(const float *__restrict__ x, void *y, int B, int H, int W, in
             v[(r * S + s2) * C + c] = (o >= 0 && col >= 0 && col < W) ? rp[col] : 0.f;
           }
         }
-      char *py = (char *)y + ((((size_t)n * Hp + p0 + hr + halo) * Wp + q + halo) * (size_t)Kp) * ESZ;
+      char *py = (char *)y + ((((size_t)n * Hp + p0 + hr) * Wp + q) * (size_t)Kp) * ESZ;
       constexpr int NCH = (NREAL + VN - 1) / VN;
 #pragma unroll
       for (int ch = 0; ch < NCH; ++ch) {
@@ -993,7 +994,8 @@ struct LrnPoolArgs {
   int Cout;                // stored output channels
   int ocg, ocp;            // output group layout: ocg real channels padded to
                            // ocp per group (0 = compact, Cout == C)
-  int hi, ho;              // zero halo of the input / output layout (pixels per side)
+  int hi, ho;              // zero halo of the input / output layout: shared-halo grids
+                           // [H + h][W + h], interior at the origin
   int R, nbands;           // band kernel: output rows per tile, bands per image
   Budget b;
 };
@@ -1021,27 +1023,24 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
     const int h0 = p * a.s, h1 = min(h0 + a.k, a.H);
     const int w0 = q0 * a.s, w1 = min((q1 - 1) * a.s + a.k, a.W);
     const int nr = h1 - h0, wc = w1 - w0;
-    const int Hp = a.H + 2 * a.hi, Wp = a.W + 2 * a.hi;          // stored input grid
-    const int Hop = a.Ho + 2 * a.ho, Wop = a.Wo + 2 * a.ho;      // stored output grid
+    // shared-halo layouts ([H + h][W + h], interior at the origin, the zero
+    // rows / columns after it)
+    const int Hp = a.H + a.hi, Wp = a.W + a.hi;          // stored input grid
+    const int Hop = a.Ho + a.ho, Wop = a.Wo + a.ho;      // stored output grid
     if (a.ho > 0) {
-      // halo output: the edge tiles zero the border cells of their image
-      // (top rows with row 0, bottom rows with the last row, the left / right
-      // columns of this output row with the first / last column tile)
+      // halo output: the last row's first tile zeroes the bottom halo rows,
+      // the last column tile of every row that row's right halo columns
       const int oc16 = a.Cout * ESZ / 16;
       const uint4 z = make_uint4(0, 0, 0, 0);
       uint4 *yb = (uint4 *)a.y;
-      for (int e = 0; e < 2; ++e)
-        if (qt == 0 && p == (e == 0 ? 0 : a.Ho - 1)) {
-          const int r0 = e == 0 ? 0 : a.Ho + a.ho;
-          const size_t base = ((size_t)n * Hop + r0) * Wop * oc16;
-          for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x) yb[base + v] = z;
-        }
-      const size_t rowb = ((size_t)n * Hop + p + a.ho) * Wop * oc16;
-      if (qt == 0)
-        for (int v = threadIdx.x; v < a.ho * oc16; v += blockDim.x) yb[rowb + v] = z;
+      if (qt == 0 && p == a.Ho - 1) {
+        const size_t base = ((size_t)n * Hop + a.Ho) * Wop * oc16;
+        for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x) yb[base + v] = z;
+      }
+      const size_t rowb = ((size_t)n * Hop + p) * Wop * oc16;
       if (qt == a.nqt - 1)
         for (int v = threadIdx.x; v < a.ho * oc16; v += blockDim.x)
-          yb[rowb + (size_t)(a.Wo + a.ho) * oc16 + v] = z;
+          yb[rowb + (size_t)a.Wo * oc16 + v] = z;
     }
     __syncthreads();
     // stage rows [h0, h1) x cols [w0, w1): each row segment is contiguous;
@@ -1052,7 +1051,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
     for (int v = threadIdx.x; v < nr * vec_per_row; v += blockDim.x) {
       int r, rem;
       fdivmod(v, vec_per_row, inv_vpr, r, rem);
-      const size_t src = (((size_t)n * Hp + h0 + r + a.hi) * Wp + w0 + a.hi) * C + (size_t)rem * VN;
+      const size_t src = (((size_t)n * Hp + h0 + r) * Wp + w0) * C + (size_t)rem * VN;
       const uint32_t dst = tbase + (uint32_t)(((size_t)r * wc_max * C + (size_t)rem * VN) * ESZ);
       asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst),
                    "l"((const char *)a.x + src * ESZ)
@@ -1116,7 +1115,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
       Vec16<ST> acc, cur;
 #pragma unroll
       for (int j = 0; j < VN; ++j) acc.v[j] = pad ? 0.f : (a.is_max ? -INFINITY : 0.f);
-      char *dst = (char *)a.y + ((((size_t)n * Hop + p + a.ho) * Wop + q + a.ho) * a.Cout + oc * VN) * ESZ;
+      char *dst = (char *)a.y + ((((size_t)n * Hop + p) * Wop + q) * a.Cout + oc * VN) * ESZ;
       if (ST == ST_BF16 && a.is_max && !pad) {
         // max is exact in bf16: compare packed pairs, no conversions
         const int cs = q * a.s - w0, ce = min(cs + a.k, wc);
@@ -1172,8 +1171,8 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
   const int C = a.C, chunks = C / VN;
   const int pitch = C * ESZ + 16;
   const long long tiles = (long long)a.B * a.nbands;
-  const int Hp = a.H + 2 * a.hi, Wp = a.W + 2 * a.hi;
-  const int Hop = a.Ho + 2 * a.ho, Wop = a.Wo + 2 * a.ho;
+  const int Hp = a.H + a.hi, Wp = a.W + a.hi;             // shared-halo grids
+  const int Hop = a.Ho + a.ho, Wop = a.Wo + a.ho;
   const float inv_chunks = 1.f / (float)chunks;
 
   for_each_tile(a.b, tiles, [&](long long t) {
@@ -1188,17 +1187,13 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
       const int oc16 = a.Cout * ESZ / 16;
       const uint4 z = make_uint4(0, 0, 0, 0);
       uint4 *yb = (uint4 *)a.y;
-      if (p0 == 0)
+      if (p1 == a.Ho)                    // bottom halo rows
         for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
-          yb[(size_t)n * Hop * Wop * oc16 + v] = z;
-      if (p1 == a.Ho)
-        for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
-          yb[((size_t)n * Hop + a.Ho + a.ho) * Wop * oc16 + v] = z;
-      for (int v = threadIdx.x; v < (p1 - p0) * 2 * a.ho * oc16; v += blockDim.x) {
-        const int rr = v / (2 * a.ho * oc16), e = v - rr * 2 * a.ho * oc16;
-        const int side = e / (a.ho * oc16), o = e - side * a.ho * oc16;
-        const size_t rowb = ((size_t)n * Hop + p0 + rr + a.ho) * Wop * oc16;
-        yb[rowb + (side ? (size_t)(a.Wo + a.ho) * oc16 : 0) + o] = z;
+          yb[((size_t)n * Hop + a.Ho) * Wop * oc16 + v] = z;
+      for (int v = threadIdx.x; v < (p1 - p0) * a.ho * oc16; v += blockDim.x) {   // right columns
+        const int rr = v / (a.ho * oc16), o = v - rr * a.ho * oc16;
+        const size_t rowb = ((size_t)n * Hop + p0 + rr) * Wop * oc16;
+        yb[rowb + (size_t)a.Wo * oc16 + o] = z;
       }
     }
     __syncthreads();   // the previous band's pooling is done with smem
@@ -1208,7 +1203,7 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
       int pix, ch;
       fdivmod(v, chunks, inv_chunks, pix, ch);
       const int r = pix / a.W, col = pix - r * a.W;
-      const size_t src = (((size_t)n * Hp + h0 + r + a.hi) * Wp + col + a.hi) * C + (size_t)ch * VN;
+      const size_t src = (((size_t)n * Hp + h0 + r) * Wp + col) * C + (size_t)ch * VN;
       asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(
                        sbase + (uint32_t)(pix * pitch + ch * 16)),
                    "l"((const char *)a.x + src * ESZ)
@@ -1265,7 +1260,7 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
         pad = j >= grp_real;
         ch = gi * grp_real + j;
       }
-      char *dst = (char *)a.y + ((((size_t)n * Hop + pp + a.ho) * Wop + q + a.ho) * a.Cout + oc * VN) * ESZ;
+      char *dst = (char *)a.y + ((((size_t)n * Hop + pp) * Wop + q) * a.Cout + oc * VN) * ESZ;
       const int rs = pp * a.s - h0, re = min(rs + a.k, nr);
       const int cs = q * a.s, ce = min(cs + a.k, a.W);
       if (ST == ST_BF16 && a.is_max) {
@@ -1325,8 +1320,8 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
   constexpr bool SWZ = CPT == 8;
   const int C = a.C, chunks = C / VN, P = chunks / CPT;
   const long long tiles = (long long)a.B * a.nbands;
-  const int Hp = a.H + 2 * a.hi, Wp = a.W + 2 * a.hi;
-  const int Hop = a.Ho + 2 * a.ho, Wop = a.Wo + 2 * a.ho;
+  const int Hp = a.H + a.hi, Wp = a.W + a.hi;             // shared-halo grids
+  const int Hop = a.Ho + a.ho, Wop = a.Wo + a.ho;
   const int lane = threadIdx.x & 31;
   auto slot = [&](int pix, int c) -> int {
     return SWZ ? (c ^ ((pix * P + (c >> 3)) & 7)) : c;
@@ -1342,17 +1337,13 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
       const int oc16 = a.Cout * ESZ / 16;
       const uint4 z = make_uint4(0, 0, 0, 0);
       uint4 *yb = (uint4 *)a.y;
-      if (p0 == 0)
+      if (p1 == a.Ho)                    // bottom halo rows
         for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
-          yb[(size_t)n * Hop * Wop * oc16 + v] = z;
-      if (p1 == a.Ho)
-        for (int v = threadIdx.x; v < a.ho * Wop * oc16; v += blockDim.x)
-          yb[((size_t)n * Hop + a.Ho + a.ho) * Wop * oc16 + v] = z;
-      for (int v = threadIdx.x; v < (p1 - p0) * 2 * a.ho * oc16; v += blockDim.x) {
-        const int rr = v / (2 * a.ho * oc16), e = v - rr * 2 * a.ho * oc16;
-        const int side = e / (a.ho * oc16), o = e - side * a.ho * oc16;
-        const size_t rowb = ((size_t)n * Hop + p0 + rr + a.ho) * Wop * oc16;
-        yb[rowb + (side ? (size_t)(a.Wo + a.ho) * oc16 : 0) + o] = z;
+          yb[((size_t)n * Hop + a.Ho) * Wop * oc16 + v] = z;
+      for (int v = threadIdx.x; v < (p1 - p0) * a.ho * oc16; v += blockDim.x) {   // right columns
+        const int rr = v / (a.ho * oc16), o = v - rr * a.ho * oc16;
+        const size_t rowb = ((size_t)n * Hop + p0 + rr) * Wop * oc16;
+        yb[rowb + (size_t)a.Wo * oc16 + o] = z;
       }
     }
     __syncthreads();   // the previous band's pooling is done with smem
@@ -1365,7 +1356,7 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
       if (pix < npix) {
         const int r = pix / a.W, col = pix - r * a.W;
         const char *src = (const char *)a.x +
-            ((((size_t)n * Hp + h0 + r + a.hi) * Wp + col + a.hi) * C + (size_t)part * CPT * VN) * ESZ;
+            ((((size_t)n * Hp + h0 + r) * Wp + col) * C + (size_t)part * CPT * VN) * ESZ;
 #pragma unroll
         for (int j = 0; j < CPT; ++j) raw[j] = __ldg((const uint4 *)(src + j * 16));
       } else {
@@ -1433,7 +1424,7 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
         pad = j >= grp_real;
         c = gi * grp_real + j;
       }
-      char *dst = (char *)a.y + ((((size_t)n * Hop + pp + a.ho) * Wop + q + a.ho) * a.Cout + oc * VN) * ESZ;
+      char *dst = (char *)a.y + ((((size_t)n * Hop + pp) * Wop + q) * a.Cout + oc * VN) * ESZ;
       const int rs = pp * a.s - h0, re = min(rs + a.k, nr);
       const int cs = q * a.s, ce = min(cs + a.k, a.W);
       if (ST == ST_BF16 && a.is_max) {
@@ -1586,7 +1577,7 @@ pool_direct_kernel(const uint4 *__restrict__ x, uint4 *__restrict__ y, int B, in
   pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   constexpr int VN = Vec16<ST>::N;
   const int k = K > 0 ? K : kk;
-  const int Hp = H + 2 * hi, Wp = W + 2 * hi, Hop = Ho + 2 * ho, Wop = Wo + 2 * ho;
+  const int Hp = H + hi, Wp = W + hi, Hop = Ho + ho, Wop = Wo + ho;   // shared-halo grids
   // output chunks: `chunks` input chunks, or (grp_pad > 0) each group's
   // grp_real chunks padded with zeros to grp_pad (the layout a grouped conv
   // reads with whole 128-B TMA slabs)
@@ -1597,9 +1588,9 @@ pool_direct_kernel(const uint4 *__restrict__ x, uint4 *__restrict__ y, int B, in
        i += (long long)gridDim.x * blockDim.x) {
     int ch = (int)(i % ochunks);
     const long long pix = i / ochunks;
-    const int q = (int)(pix % Wop) - ho;
+    const int q = (int)(pix % Wop);
     const long long t = pix / Wop;
-    const int p = (int)(t % Hop) - ho;
+    const int p = (int)(t % Hop);
     const long long n = t / Hop;
     bool pad = false;
     if (grp_pad > 0) {
@@ -1613,7 +1604,7 @@ pool_direct_kernel(const uint4 *__restrict__ x, uint4 *__restrict__ y, int B, in
     }
     const int r0 = p * s, c0 = q * s;
     const int re = min(r0 + k, H), ce = min(c0 + k, W);
-    const uint4 *base = x + (((size_t)n * Hp + r0 + hi) * Wp + c0 + hi) * chunks + ch;
+    const uint4 *base = x + (((size_t)n * Hp + r0) * Wp + c0) * chunks + ch;
     if (ST == ST_BF16 && is_max) {
       __nv_bfloat162 m[4];
       const __nv_bfloat162 ninf = __float2bfloat162_rn(-INFINITY);
@@ -1669,7 +1660,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
     const int chunks = C / vn;
     const int gr = out_groups > 0 ? ocg / vn : 0, gp = out_groups > 0 ? ocp / vn : 0;
     const int ochunks = out_groups > 0 ? out_groups * gp : chunks;
-    const long long total = (long long)B * (Ho + 2 * out_halo) * (Wo + 2 * out_halo) * ochunks;
+    const long long total = (long long)B * (Ho + out_halo) * (Wo + out_halo) * ochunks;
     const int g = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
 #define PCNN_PD(STT, KK)                                                                       \
   launch_pdl(pool_direct_kernel<STT, KK>, dim3(g), dim3(256), 0, stream, (const uint4 *)x, (uint4 *)y, B, H, W,    \
@@ -1784,15 +1775,15 @@ perf_interp_kernel(const uint4 *__restrict__ t, uint4 *__restrict__ y, int B, in
                    int sh, int sw, int chunks, int ho) {
   pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
   const int Hk = (Ho + sh - 1) / sh, Wk = (Wo + sw - 1) / sw;
-  const int Hp = Ho + 2 * ho, Wp = Wo + 2 * ho;
+  const int Hp = Ho + ho, Wp = Wo + ho;               // shared-halo output grid
   const long long total = (long long)B * Hp * Wp * chunks;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
        i += (long long)gridDim.x * blockDim.x) {
     const int ch = (int)(i % chunks);
     const long long pix = i / chunks;
-    const int q = (int)(pix % Wp) - ho;
+    const int q = (int)(pix % Wp);
     const long long r = pix / Wp;
-    const int p = (int)(r % Hp) - ho;
+    const int p = (int)(r % Hp);
     const long long n = r / Hp;
     uint4 v = make_uint4(0, 0, 0, 0);
     if (p >= 0 && p < Ho && q >= 0 && q < Wo) {
@@ -1808,7 +1799,7 @@ cudaError_t launch_perf_interp(const void *t, void *y, int st, int B, int Ho, in
   const int esz = st == ST_BF16 ? 2 : 4;
   if ((Cs * esz) % 16) return cudaErrorInvalidValue;
   const int chunks = Cs * esz / 16;
-  const long long total = (long long)B * (Ho + 2 * ho) * (Wo + 2 * ho) * chunks;
+  const long long total = (long long)B * (Ho + ho) * (Wo + ho) * chunks;
   const int grid = (int)std::min<long long>((total + 255) / 256, 148LL * 16);
   launch_pdl(perf_interp_kernel, dim3(grid), dim3(256), 0, s, (const uint4 *)t, (uint4 *)y, B, Ho, Wo, sh, sw,
                                           chunks, ho);

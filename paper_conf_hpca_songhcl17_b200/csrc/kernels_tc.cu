@@ -529,7 +529,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
       // pm = 2: nseg segments of wv + 2 pad columns (grid columns -pad ..)
       const uint32_t pm_a_bytes = g.pm == 2 ? (uint32_t)(g.nseg * (g.wv + 2 * g.pad)) * slab_bytes
-                                            : (uint32_t)(TC_BM + 2 * g.pad) * slab_bytes;
+                                            : (uint32_t)(TC_BM + g.S - 1) * slab_bytes;
       uint32_t as = 0, aph = 0, bs = 0, bph = 0;
       WaitClock wc{TC_PROF(a) != 0};
       unsigned long long nkb = 0;
@@ -635,9 +635,10 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
           n0 = m0 / HoWo;
           const int pq = m0 % HoWo;
           // perforated variant: kept positions psh / psw output rows / cols
-          // apart; a zero-haloed input shifts every window by ih
-          w0 = (pq % g.Wo) * g.stride * max(g.psw, 1) - g.pad + g.ih;
-          h0 = (pq / g.Wo) * g.stride * max(g.psh, 1) - g.pad + g.ih;
+          // apart; a zero-haloed input (shared-halo grid, interior at the
+          // origin) only widens the map's extent
+          w0 = (pq % g.Wo) * g.stride * max(g.psw, 1) - g.pad;
+          h0 = (pq / g.Wo) * g.stride * max(g.psh, 1) - g.pad;
         }
         for (int kb = k0; kb < k1; ++kb) {
           wc.wait(sbase + SM_EMPTY + 8 * stage, phase ^ 1);
@@ -1169,7 +1170,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
     return cudaErrorInvalidValue;
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
-  if (g.pm && (p.splits != 1 || p.rect_w || g.stride != 1 || g.S != 2 * g.pad + 1 ||
+  if (g.pm && (p.splits != 1 || p.rect_w || g.stride != 1 || (g.S != 2 * g.pad + 1 && g.pad != 0) ||
                g.Cg % (args.slab_bytes / (st == ST_BF16 ? 2 : 4)) || p.a_stages < 2 ||
                p.b_stages < 2 || p.a_stages > TC_MAX_ASTAGES || p.b_stages > TC_MAX_BSTAGES))
     return cudaErrorInvalidValue;

@@ -110,17 +110,22 @@ struct ConvGeom {
   int relu;
   int out_mode;     // OutMode
   // padded-layout ("shifted window") mode, tcgen05 only (pm = 1): input and
-  // output share one zero-haloed grid hv x wv = (H + 2 vh) x (W + 2 vh) per
-  // image, M = B*hv*wv virtual rows, and the A rows of tap (r, s) for output
-  // row i are input rows i + (r - pad)*wv + (s - pad).  Rows outside the
-  // valid window [vh, vh + Ho) x [vh, vh + Wo) are written as zeros (they are
-  // the next layer's padding).  Requires stride 1 and S == 2*pad + 1.
+  // output share one zero-haloed grid hv x wv per image, M = B*hv*wv virtual
+  // rows, and the A rows of tap (r, s) for output row i are input rows
+  // i + (r - pad)*wv + (s - pad).  Rows outside the valid window
+  // [vh, vh + Ho) x [vh, vh + Wo) are written as zeros (they are the next
+  // layer's padding).  The runtime uses the shared-halo grid (vh = 0,
+  // hv = H + h, wv = W + h): the h zero columns after one row are the left
+  // padding of the next, the h zero rows after one image the top padding of
+  // the next (the first image's top padding is TMA's out-of-bounds zero fill).
+  // Requires stride 1 and S == 2*pad + 1.
   int pm;
   int hv, wv, vh;
   // perforated variant (NEXT-1, reading R13; im2col mode only): the GEMM rows
   // are the kept output positions of a psh x psw grid (Ho, Wo above are the
   // kept counts), i.e. input windows stride*psh / stride*psw apart; ih = zero
-  // border of the stored input ([B][H + 2ih][W + 2ih][Cs]); 0 = plain
+  // halo of the stored input (shared-halo grid [B][H + ih][W + ih][Cs],
+  // interior at the origin); 0 = plain
   int psh, psw, ih;
   // row-perforated padded mode (pm = 2): the kept output rows p' (p = psh p')
   // of each image form segments of wv virtual rows; a CTA tile is nseg

@@ -460,23 +460,28 @@ static pcnn_status build_stage(GemmStage &gs, const Layer &ly, int precision, in
     g.Kpad = round_up(g.K, k_align(precision));
     g.Creal = Cg_log;
     if (pm_halo > 0 && pm_valid) {
-      // a 'valid' stride-1 conv (pad 0, S = 2h + 1) read as a 'same' conv on
-      // its own input grid: the input is the halo-h grid of the output, the
-      // windows are shifted by the virtual pad h (layer 0 after space-to-depth)
+      // a 'valid' stride-1 conv (pad 0, S = 2h + 1) on its own input grid:
+      // output (p, q) sits at grid row p*wv + q and reads input rows
+      // (p + r)*wv + q + s; the output grid is the input grid, i.e. the
+      // shared-halo layout of the output with halo S - 1 (layer 0 after
+      // space-to-depth)
       if (gs.engine != 1 || stride != 1 || pad != 0 || S != 2 * pm_halo + 1)
         return fail(PCNN_ERR_UNSUPPORTED, "valid padded-layout mode needs pad 0, S = 2h + 1");
       g.pm = 1;
-      g.vh = pm_halo;
+      g.vh = 0;
       g.hv = in_h;
       g.wv = in_w;
-      g.pad = pm_halo;
+      g.pad = 0;
     } else if (pm_halo > 0) {
+      // shared-halo grid: [H + h][W + h] per image, interior at
+      // the origin; the zero columns / rows after a row / image are the left /
+      // top padding of the next one
       if (gs.engine != 1 || stride != 1 || S != 2 * pad + 1 || pad > pm_halo)
         return fail(PCNN_ERR_UNSUPPORTED, "padded-layout mode needs a stride-1 'same' conv");
       g.pm = 1;
-      g.vh = pm_halo;
-      g.hv = in_h + 2 * pm_halo;
-      g.wv = in_w + 2 * pm_halo;
+      g.vh = 0;
+      g.hv = in_h + pm_halo;
+      g.wv = in_w + pm_halo;
     }
     packed = pack_conv(w, Nf, Cg_log, Cg_st, S, g.Kpad);
     if (S > 1) {
@@ -628,12 +633,13 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, co
   if (!enc) return nullptr;
   // bounding box of the conv's input corners (square kernels: W and H equal);
   // a zero-haloed input (perforated variant of a padded-layout layer) is the
-  // grid [H + 2ih][W + 2ih] whose windows start ih - pad inside it
-  cuuint64_t dimsh[4] = {dims[0], dims[1] + 2 * (cuuint64_t)g.ih, dims[2] + 2 * (cuuint64_t)g.ih,
+  // shared-halo grid [H + ih][W + ih] (interior at the origin): only the
+  // extent grows, the traversal box still ends pad - (S - 1) past the interior
+  cuuint64_t dimsh[4] = {dims[0], dims[1] + (cuuint64_t)g.ih, dims[2] + (cuuint64_t)g.ih,
                          dims[3]};
   const cuuint64_t stridesh[3] = {(cuuint64_t)g.Cs * esz, dimsh[1] * g.Cs * esz,
                                   dimsh[2] * dimsh[1] * g.Cs * esz};
-  const int lower[2] = {g.ih - g.pad, g.ih - g.pad};
+  const int lower[2] = {-g.pad, -g.pad};
   const int upper[2] = {g.pad - (g.S - 1) - g.ih, g.pad - (g.S - 1) - g.ih};
   const cuuint32_t estr[4] = {1, (cuuint32_t)(g.stride * std::max(g.psw, 1)),
                               (cuuint32_t)(g.stride * std::max(g.psh, 1)), 1};
@@ -1193,7 +1199,7 @@ static pcnn_status run_layer(pcnn_net *net, int i, int B, const void *x, void *y
         const ConvGeom &g = ly.pf.g;
         const size_t rowb = (size_t)g.wv * ly.out_cs * esz_of(ly.pf.st);
         const size_t img = (size_t)g.hv * rowb;
-        CUDA_TRY(cudaMemset2DAsync(y, img, 0, (size_t)g.vh * rowb, B, s));
+        if (g.vh > 0) CUDA_TRY(cudaMemset2DAsync(y, img, 0, (size_t)g.vh * rowb, B, s));
         CUDA_TRY(cudaMemset2DAsync((char *)y + (size_t)(g.vh + g.Ho) * rowb, img, 0,
                                    (size_t)(g.hv - g.vh - g.Ho) * rowb, B, s));
         return PCNN_OK;
@@ -1566,7 +1572,8 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
         if (ly.d.stride != 1 || S != 2 * P + 1 || P < 1 || P > 3 || ly.in_cs % g) continue;
         const int sb = tc_slab_bytes(net->st, ly.in_cs / g);
         if (sb == 0 || (sb != 128 && !narrow_pm)) continue;
-        if ((double)(ly.in_h + 2 * P) * (ly.in_w + 2 * P) > pm_max_halo * ly.in_h * ly.in_w) continue;
+        // shared-halo grid: P zero rows / columns per image row / image
+        if ((double)(ly.in_h + P) * (ly.in_w + P) > pm_max_halo * ly.in_h * ly.in_w) continue;
         pmh[i] = P;
       }
       for (bool changed = true; changed;) {
@@ -1609,18 +1616,21 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
       Layer &ly = net->layers[i];
       ly.in_halo = i > 0 ? net->layers[i - 1].out_halo : (net->stage_blk > 1 ? 0 : pmh[0]);
       ly.pm_halo = pmh[i];
-      if (pmh[i]) ly.out_halo = pmh[i];
+      // shared-halo layouts: a 'same' pm conv keeps its grid (halo P); the
+      // 'valid' space-to-depth first conv computes its output on the staged
+      // grid, i.e. the output's halo is Sp - 1 = 2 pmh
+      if (pmh[i]) ly.out_halo = (i == 0 && net->stage_blk > 1) ? 2 * pmh[i] : pmh[i];
       else if (is_pool(i) && i + 1 < n && kind(i + 1) == PCNN_CONV) ly.out_halo = pmh[i + 1];
       else if (kind(i) == PCNN_LRN && i > 0 && pmh[i - 1] && i + 1 < n && is_pool(i + 1))
-        ly.out_halo = pmh[i - 1];   // keeps the conv's layout: conv + LRN may run fused
+        ly.out_halo = net->layers[i - 1].out_halo;   // keeps the conv's layout (conv + LRN may fuse)
       else ly.out_halo = 0;
     }
   }
   const int h0 = net->layers[0].in_halo;
-  size_t act = (size_t)B * (net->stage_h + 2 * h0) * (net->stage_w + 2 * h0) * net->in_cs * esz;
+  size_t act = (size_t)B * (net->stage_h + h0) * (net->stage_w + h0) * net->in_cs * esz;
   for (int i = 0; i < n; ++i) {
     Layer &ly = net->layers[i];
-    act = std::max(act, (size_t)B * (ly.out_h + 2 * ly.out_halo) * (ly.out_w + 2 * ly.out_halo) *
+    act = std::max(act, (size_t)B * (ly.out_h + ly.out_halo) * (ly.out_w + ly.out_halo) *
                             ly.out_cs * esz);
     if (ly.gemm) {
       const bool final_fc = (i == n - 1) && ly.d.kind == PCNN_FC;
@@ -1876,8 +1886,8 @@ pcnn_status pcnn_set_variant_factors(pcnn_net *net, int layer, int rank, const f
     if (rank > std::min(Nfg, K)) return fail(PCNN_ERR_INVALID_ARGUMENT, "rank out of [1, min(N_f/g, K)]");
     // stage 1 writes g * round_up(r, chunk) channels on the layer's output grid
     // into the arena's third buffer
-    const size_t s1 = (size_t)net->desc.max_batch * (ly.out_h + 2 * ly.out_halo) *
-                      (ly.out_w + 2 * ly.out_halo) * g *
+    const size_t s1 = (size_t)net->desc.max_batch * (ly.out_h + ly.out_halo) *
+                      (ly.out_w + ly.out_halo) * g *
                       round_up(rank, chunk_elems(net->desc.precision)) * esz_of(net->st);
     if (s1 > net->act_bytes)
       return fail(PCNN_ERR_UNSUPPORTED, "rank-r intermediate larger than the activation arena");
