@@ -707,6 +707,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     const uint32_t tempty_leader =
         CG == 2 ? mapa(sbase + SM_TEMPTY, 0) : sbase + SM_TEMPTY;
     uint32_t lt = 0;
+    uint32_t sbox = 0;   // bf16 TMA-store staging: two 2 KB boxes used alternately
     WaitClock wtf{TC_PROF(a) != 0 && lane == 0 && warp == 2};
     unsigned long long busy = 0;
     long long tb = 0;
@@ -763,12 +764,15 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         // 32-column passes; full chunks are staged in this warp's swizzled
         // box (SW64 rows for bf16, SW128 for fp32) and leave by one TMA
         // tensor store of the warp's 32 rows (rows past M are clipped by the
-        // map); a ragged last chunk falls back to row stores.
+        // map); a ragged last chunk falls back to row stores.  BF16 boxes
+        // (2 KB) are double-buffered: a chunk waits only for the store issued
+        // two chunks earlier, so the stores overlap the next chunk's TMEM
+        // load and conversion (the epilogue of narrow-N layers -- AlexNet
+        // conv1, VGG conv1_x -- was serialised on each store's smem read).
         const bool o16 = g.out_mode == OUT_BF16;
         const int split = ((a.bn / 2 + 31) / 32) * 32;
         const int cbeg = half == 0 ? 0 : split, cend = half == 0 ? split : a.bn;
         const int row0 = m - lane;                       // the warp's first row
-        const uint32_t sstage = smem_u32(stage);
         for (int c0 = cbeg; c0 < cend; c0 += 32) {
           const int n = nt * a.bn + c0;
           if (n >= g.Nfg) break;                         // warp-uniform
@@ -801,8 +805,12 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
             for (int i = 0; i < 32; ++i) f[i] = 0.f;
           const bool full = n + 32 <= g.Nfg && c0 + 32 <= cend;
           if (full) {
-            if (lane == 0) bulk_wait_read0();            // staging box free again
+            if (lane == 0) {                             // staging box free again
+              if (o16) bulk_wait_read1();
+              else bulk_wait_read0();
+            }
             __syncwarp();
+            uint8_t *box = o16 ? stage + sbox * 2048 : stage;
             if (o16) {
 #pragma unroll
               for (int q = 0; q < 4; ++q) {
@@ -813,7 +821,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
                   __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * q + 2 * i], f[8 * q + 2 * i + 1]);
                   pw[i] = *(uint32_t *)&b2;
                 }
-                *(uint4 *)(stage + lane * 64 + ((q ^ ((lane >> 1) & 3)) << 4)) = pk;
+                *(uint4 *)(box + lane * 64 + ((q ^ ((lane >> 1) & 3)) << 4)) = pk;
               }
             } else {
               const bool rnd = g.out_mode == OUT_F32_TF32;
@@ -830,9 +838,10 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
             fence_proxy_async();
             __syncwarp();
             if (lane == 0 && row0 < g.M) {
-              tma_store_2d(&tmap_y, sstage, col, row0);
+              tma_store_2d(&tmap_y, smem_u32(box), col, row0);
               bulk_commit();
             }
+            sbox ^= 1;
           } else {
             // ragged chunk: row stores of the np valid 16 B pieces
             uint4 pc[8];
