@@ -374,12 +374,15 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
   const bool leader = elect_one();
   WaitClock wfull{prof}, wtemp{prof};
   uint32_t as = 0, aph = 0, bs = 0, bph = 0, lt = 0;
+  const int tiles_all = a.mtiles * a.ntiles * a.g.groups, kbs = a.kb_per_split;
   for (int u = pair; u < units; u += npairs, ++lt) {
     const uint32_t buf = lt & 1, use = lt >> 1;
+    // split-K over the windows (small batches only): windows [j0, j1)
+    const int sp = u / tiles_all, j0 = sp * kbs, j1 = min(nj, j0 + kbs);
     wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
     tc_fence_after();
     const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
-    for (int j = 0; j < nj; ++j) {
+    for (int j = j0; j < j1; ++j) {
       wfull.wait(sbase + SM_AFULL + 8 * as, aph);
       const uint64_t ad = a_desc0 + as * a_st16;
       const int kk = j >= j_last ? kmma_last : KMMA;
@@ -394,7 +397,7 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
             for (int sb = 0; sb < MSUB; ++sb) {
               const uint64_t awb = aw + sb * sub16;
               const uint32_t dc = dcol + sb * (TC_BN_MAX / 2);
-              tc_mma<ST, CG>(dc, awb, bd, idesc, (j > 0 || s2 > 0) ? 1u : 0u);
+              tc_mma<ST, CG>(dc, awb, bd, idesc, (j > j0 || s2 > 0) ? 1u : 0u);
 #pragma unroll
               for (int k = 1; k < KMMA; ++k)
                 if (k < kk) tc_mma<ST, CG>(dc, awb + 2 * k, bd + 2 * k, idesc, 1u);
@@ -539,8 +542,10 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         nkb += pm_nj;
         const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
         const int i0 = (mt * CG + (int)rank) * TC_BM * a.msub;
-        int cb = 0, r = 0;
-        for (int j = 0; j < pm_nj; ++j) {
+        // split-K over the windows (small batches only): windows [j0, j1)
+        const int j0 = sp * a.kb_per_split, j1 = min(pm_nj, j0 + a.kb_per_split);
+        int cb = j0 / g.S, r = j0 - cb * g.S;
+        for (int j = j0; j < j1; ++j) {
           wc.wait(sbase + SM_AEMPTY + 8 * as, aph ^ 1);
           const uint32_t fa = sbase + SM_AFULL + 8 * as;
           if (rank == 0) mbar_arrive_expect_tx(fa, (a.skip & 1) ? 0 : CG * a.msub * pm_a_bytes);
@@ -1000,15 +1005,29 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
 }
 
 // Deterministic split-K reduction: y = act(sum_s ws[s] + bias), s ascending.
+// Padded-layout (pm) GEMMs: rows outside the valid window of the grid are
+// stored as zeros (pm_hv > 0: grid hv x wv per image, valid [vh, vh + Ho) x
+// [vh, vh + Wo)).
 __global__ void splitk_reduce_kernel(const float *__restrict__ ws, void *y,
                                      const float *__restrict__ bias, int M, int N, int splits,
-                                     int relu, int out_mode) {
+                                     int relu, int out_mode, int pm_hv, int pm_wv, int pm_vh,
+                                     int pm_ho, int pm_wo) {
   pdl_enter();
   const long long total = (long long)M * N / 4;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
        i += (long long)gridDim.x * blockDim.x) {
     const long long e = i * 4;
     const int col = (int)(e % N);
+    if (pm_hv > 0) {
+      const long long m = e / N;
+      const int rem = (int)(m % ((long long)pm_hv * pm_wv));
+      const int pv = rem / pm_wv, qv = rem - pv * pm_wv;
+      if (pv < pm_vh || pv >= pm_vh + pm_ho || qv < pm_vh || qv >= pm_vh + pm_wo) {
+        if (out_mode == OUT_BF16) *(uint2 *)((__nv_bfloat16 *)y + e) = make_uint2(0, 0);
+        else *(float4 *)((float *)y + e) = make_float4(0.f, 0.f, 0.f, 0.f);
+        continue;
+      }
+    }
     // partials summed in split order (fixed, so every SM budget gives the
     // same bits); the loads of three splits are issued before their adds so
     // a thread has three L2 round trips in flight instead of one
@@ -1179,7 +1198,8 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
     return cudaErrorInvalidValue;
   args.b = b;
   if (args.slab_bytes == 0) return cudaErrorInvalidValue;
-  if (g.pm && (p.splits != 1 || p.rect_w || g.stride != 1 || (g.S != 2 * g.pad + 1 && g.pad != 0) ||
+  if (g.pm && ((p.splits != 1 && g.pm != 1) || p.rect_w || g.stride != 1 ||
+               (g.S != 2 * g.pad + 1 && g.pad != 0) ||
                g.Cg % (args.slab_bytes / (st == ST_BF16 ? 2 : 4)) || p.a_stages < 2 ||
                p.b_stages < 2 || p.a_stages > TC_MAX_ASTAGES || p.b_stages > TC_MAX_BSTAGES))
     return cudaErrorInvalidValue;
@@ -1201,7 +1221,7 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   const long long total = (long long)g.M * g.out_cs / 4;
   const int grid = (int)std::min<long long>((total + 255) / 256, 148 * 8);
   launch_pdl(splitk_reduce_kernel, dim3(grid), dim3(256), 0, s, ws, y, bias, g.M, g.out_cs, p.splits, g.relu,
-                                            g.out_mode);
+             g.out_mode, g.pm == 1 ? g.hv : 0, g.wv, g.vh, g.Ho, g.Wo);
   return cudaGetLastError();
 }
 

@@ -880,6 +880,20 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
   const char *force_ms = exp_env("PCNN_PM_MSUB");           // 1 | 2 (experiments)
   if (want_cg > 0) force_cg = want_cg == 1 ? "1" : "2";
   if (want_msub > 0) force_ms = want_msub == 1 ? "1" : "2";
+  // split-K over the windows only when no tile shape fills the device (tiny
+  // batches; R17: the K order of an image is then batch-independent for every
+  // batch at which some tile shape fills it); row perforation (pm = 2) never
+  bool can_fill = false;
+  for (int ms = 1; ms <= 2; ++ms)
+    for (int cg = 1; cg <= 2; ++cg)
+      for (int bn = 32; bn <= std::max(32, nmax); bn += 32) {
+        if (ms == 2 && bn > 128) continue;
+        const long long t = ((g.M + 128LL * cg * ms - 1) / (128LL * cg * ms)) *
+                            ((g.Nfg + bn - 1) / bn) * g.groups;
+        if (t >= device_sms / cg) can_fill = true;
+      }
+  const int max_split = (can_fill || full_n || g.pm != 1) ? 1 : std::min(16, nj);
+  const double hbm = 6.0e12;
   for (int ms = 1; ms <= 2; ++ms) {
     if (force_ms && atoi(force_ms) != ms) continue;
     for (int cg = 1; cg <= 2; ++cg) {
@@ -908,21 +922,29 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
                                 kOperandBytesPerCycle + 64.0 * (ms + g.S);
         const double mma = ms * g.S * (slab / 128.0) * kfrac * 2.05 * bn / kMmaEfficiency;
         const double j_cycles = std::max(load, mma) + 40.0;
-        const long long waves = (tiles + slots - 1) / slots;
-        const double t = (double)waves * nj * j_cycles / f + 2e-6 * ms;
-        TcPlan c{};
-        c.cg = cg;
-        c.bn = bn;
-        c.msub = ms;
-        c.mtiles = mtiles;
-        c.ntiles = ntiles;
-        c.tiles = (int)tiles;
-        c.splits = 1;
-        c.kb_per_split = nj;
-        c.units = (int)tiles;
-        c.unit_us = ((double)nj * j_cycles / f + 2e-6 * ms) * 1e6;
-        cands.push_back({t, c});
-        best_t = std::min(best_t, t);
+        for (int want = 1; want <= max_split; ++want) {
+          const int kbs = (nj + want - 1) / want;
+          const int splits = (nj + kbs - 1) / kbs;
+          if (splits != want) continue;
+          const long long units = tiles * splits;
+          const long long waves = (units + slots - 1) / slots;
+          double t = (double)waves * kbs * j_cycles / f + 2e-6 * ms;
+          // partials written and summed by the reduction launch
+          if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
+          TcPlan c{};
+          c.cg = cg;
+          c.bn = bn;
+          c.msub = ms;
+          c.mtiles = mtiles;
+          c.ntiles = ntiles;
+          c.tiles = (int)tiles;
+          c.splits = splits;
+          c.kb_per_split = kbs;
+          c.units = (int)units;
+          c.unit_us = ((double)kbs * j_cycles / f + 2e-6 * ms) * 1e6;
+          cands.push_back({t, c});
+          best_t = std::min(best_t, t);
+        }
       }
     }
   }
