@@ -78,6 +78,13 @@ out["calibration"] = {"new_inputs": "images 4096.. at U[-160, 160)", "final_tabl
                       "trace": [[i, round(h, 5)] for i, h in trace],
                       "estimate_only": {str(h): tuning.calibrate_estimate(path, last, h, threshold)
                                         for h in (path[last]["entropy"], threshold + 0.5, 1e9)}}
+# a stricter requirement than at tuning time (a threshold below every table's
+# entropy): calibration walks back along the path to the exact table,
+# re-measuring the entropy after every step
+tight = min(p["entropy"] for p in path) - 1e-3
+idx, trace = tuning.calibrate(path, last, tuning.gpu_observe(n, ladders, path, x), tight)
+out["calibration_tight"] = {"threshold_nats": round(tight, 5), "final_table": idx,
+                            "trace": [[i, round(h, 5)] for i, h in trace]}
 # NEXT-4: background-task batch (every conv layer at Util = 1, eq. 6) on this
 # net's own tile plans, and eq. 13's rescaled batch for a 0.2 ms requirement
 nb = pcnn.Net(net, w, b, 256, "bf16")
