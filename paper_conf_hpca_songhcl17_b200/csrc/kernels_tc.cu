@@ -67,9 +67,10 @@ constexpr int SM_EPI = TC_STAGE_BUDGET;
 constexpr int SM_BAR = SM_EPI + 8 * EPI_WARP_BYTES;
 constexpr int SM_FULL = SM_BAR;
 constexpr int SM_EMPTY = SM_FULL + 8 * TC_MAX_BSTAGES;
+constexpr int TC_MAX_TBUF = 8;         // TMEM accumulator buffers (narrow N tiles)
 constexpr int SM_TFULL = SM_EMPTY + 8 * TC_MAX_BSTAGES;
-constexpr int SM_TEMPTY = SM_TFULL + 16;
-constexpr int SM_TMEMPTR = SM_TEMPTY + 16;
+constexpr int SM_TEMPTY = SM_TFULL + 8 * TC_MAX_TBUF;
+constexpr int SM_TMEMPTR = SM_TEMPTY + 8 * TC_MAX_TBUF;
 constexpr int TC_MAX_ASTAGES = 8;       // padded mode: A row-window ring
 constexpr int SM_AFULL = SM_TMEMPTR + 16;
 constexpr int SM_AEMPTY = SM_AFULL + 8 * TC_MAX_ASTAGES;
@@ -146,6 +147,10 @@ struct TcArgs {
   int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
   int a_stages, b_stages, pm_a_stage;   // padded mode rings (g.pm)
   int msub;             // padded mode: M sub-tiles of 128 rows per CTA sharing each B slab
+  // TMEM accumulator ring: nbuf buffers of tbw columns (512 / tbw), sub-tile
+  // sb at column tsub * sb of its buffer.  Narrow tiles get up to 8 buffers,
+  // so the MMA runs several tiles ahead of a latency-bound epilogue.
+  int nbuf, tbw, tsub;
   int kmma_last;        // padded mode: UMMAs (32 B of K each) of the last channel slab that
                         // touch real channels; the rest multiply zero padding and are skipped
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
@@ -321,10 +326,10 @@ __device__ __forceinline__ void mma_issuer_im2col(const TcArgs &a, uint32_t sbas
   for (int u = pair; u < units; u += npairs, ++lt) {
     const int sp = u / (mtiles * ntiles * groups);
     const int k0 = sp * kbs, k1 = min(kblocks, k0 + kbs);
-    const uint32_t buf = lt & 1, use = lt >> 1;
+    const uint32_t buf = lt % a.nbuf, use = lt / a.nbuf;
     wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
     tc_fence_after();
-    const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
+    const uint32_t dcol = tmem_base + buf * a.tbw;
     for (int kb = k0; kb < k1; ++kb) {
       wfull.wait(sbase + SM_FULL + 8 * stage, phase);
       tc_fence_after();
@@ -376,12 +381,12 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
   uint32_t as = 0, aph = 0, bs = 0, bph = 0, lt = 0;
   const int tiles_all = a.mtiles * a.ntiles * a.g.groups, kbs = a.kb_per_split;
   for (int u = pair; u < units; u += npairs, ++lt) {
-    const uint32_t buf = lt & 1, use = lt >> 1;
+    const uint32_t buf = lt % a.nbuf, use = lt / a.nbuf;
     // split-K over the windows (small batches only): windows [j0, j1)
     const int sp = u / tiles_all, j0 = sp * kbs, j1 = min(nj, j0 + kbs);
     wtemp.wait(sbase + SM_TEMPTY + 8 * buf, (use & 1) ^ 1);
     tc_fence_after();
-    const uint32_t dcol = tmem_base + buf * TC_BN_MAX;
+    const uint32_t dcol = tmem_base + buf * a.tbw;
     for (int j = j0; j < j1; ++j) {
       wfull.wait(sbase + SM_AFULL + 8 * as, aph);
       const uint64_t ad = a_desc0 + as * a_st16;
@@ -396,7 +401,7 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
 #pragma unroll
             for (int sb = 0; sb < MSUB; ++sb) {
               const uint64_t awb = aw + sb * sub16;
-              const uint32_t dc = dcol + sb * (TC_BN_MAX / 2);
+              const uint32_t dc = dcol + sb * a.tsub;
               tc_mma<ST, CG>(dc, awb, bd, idesc, (j > j0 || s2 > 0) ? 1u : 0u);
 #pragma unroll
               for (int k = 1; k < KMMA; ++k)
@@ -471,7 +476,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       mbar_init(sbase + SM_AFULL + 8 * s, 1);
       mbar_init(sbase + SM_AEMPTY + 8 * s, 1);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < a.nbuf; ++i) {
       mbar_init(sbase + SM_TFULL + 8 * i, 1);
       mbar_init(sbase + SM_TEMPTY + 8 * i, tc_nepi<LRN>() * CG);   // one arrive per epilogue warp
     }
@@ -719,14 +724,14 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     for (int u = pair; u < a.units; u += npairs, ++lt) {
       int mt, nt, grp, sp;
       decode(u, mt, nt, grp, sp);
-      const uint32_t buf = lt & 1, use = lt >> 1;
+      const uint32_t buf = lt % a.nbuf, use = lt / a.nbuf;
       if (wtf.on && tb) busy += clock64() - tb;
       wtf.wait(sbase + SM_TFULL + 8 * buf, use & 1);
       if (wtf.on) tb = clock64();
       tc_fence_after();
       for (int sb = 0; sb < a.msub; ++sb) {
       // TMEM columns of this sub-tile's accumulator
-      const uint32_t tcol = buf * TC_BN_MAX + sb * (TC_BN_MAX / 2);
+      const uint32_t tcol = buf * a.tbw + sb * a.tsub;
       int m;
       bool mok;
       if (rect) {
@@ -1181,6 +1186,17 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.a_stages = p.a_stages;
   args.b_stages = p.b_stages;
   args.msub = p.msub > 1 ? p.msub : 1;
+  {
+    // TMEM ring: sub-tile stride = the N tile rounded to 32 columns, buffer
+    // width = msub strides rounded up to a power of two (>= 64), as many
+    // buffers as fit the 512 allocated columns (2 .. 8)
+    args.tsub = (p.bn + 31) / 32 * 32;
+    int w = 64;
+    while (w < args.msub * args.tsub) w <<= 1;
+    args.tbw = w;
+    args.nbuf = std::min(TC_MAX_TBUF, TC_TMEM_COLS / w);
+    if (const char *e = exp_env("PCNN_TC_NBUF")) args.nbuf = std::max(2, std::min(args.nbuf, atoi(e)));
+  }
   {
     // padded mode: UMMAs of the last channel slab that reach real channels
     const int se = args.slab_bytes / (st == ST_BF16 ? 2 : 4);
