@@ -155,6 +155,7 @@ struct TcArgs {
                         // touch real channels; the rest multiply zero padding and are skipped
   int lrn;              // 1: fused across-channel LRN (size 5) in the epilogue
   int tma_y;            // 1: full 32-column output chunks leave by TMA tensor store
+  int tma_y64;          // 1: bf16 output, full 64-column chunks use the 128 B-row map
   float lrn_a_over_n, lrn_beta, lrn_k;
   Budget b;
 };
@@ -180,6 +181,46 @@ __device__ __forceinline__ void epi_store_rows(uint8_t *stage, const uint4 (&pc)
       *(uint4 *)(dst + 16 * j) = *(const uint4 *)(stage + r * EPI_PITCH + 16 * j);
   }
   __syncwarp();
+}
+
+// One 32-column epilogue step: bias (issued before the TMEM load so the
+// latencies overlap), TMEM load of the lane's row, ReLU, halo rows zeroed.
+__device__ __forceinline__ void epi_chunk32(const TcArgs &a, uint32_t taddr, int col, bool valid,
+                                            float (&f)[32]) {
+  const float4 *bp = (const float4 *)(a.bias + col);
+  float4 bb[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) bb[q] = __ldg(bp + q);
+  {
+    uint32_t v[32];
+    tmem_ld32(taddr, v);
+    tmem_ld_wait();
+#pragma unroll
+    for (int i = 0; i < 32; ++i) f[i] = __uint_as_float(v[i]);
+  }
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    f[4 * q] += bb[q].x;
+    f[4 * q + 1] += bb[q].y;
+    f[4 * q + 2] += bb[q].z;
+    f[4 * q + 3] += bb[q].w;
+  }
+  if (a.g.relu)
+#pragma unroll
+    for (int i = 0; i < 32; ++i) f[i] = fmaxf(f[i], 0.f);
+  if (!valid)
+#pragma unroll
+    for (int i = 0; i < 32; ++i) f[i] = 0.f;
+}
+__device__ __forceinline__ uint4 pack_bf16x8(const float *f) {
+  uint4 pk;
+  uint32_t *pw = (uint32_t *)&pk;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    __nv_bfloat162 b2 = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
+    pw[i] = *(uint32_t *)&b2;
+  }
+  return pk;
 }
 
 // Epilogue with the following LRN layer fused in (R3; Caffe size
@@ -262,7 +303,7 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
 //  0 producer waits on EMPTY   1 MMA waits on FULL   2 MMA waits on TEMPTY
 //  3 epilogue waits on TFULL   4 CTA lifetime        5 K-blocks issued
 //  6 epilogue busy cycles      7 CTAs
-__device__ unsigned long long g_tc_prof[8];
+__device__ unsigned long long g_tc_prof[16];
 
 // Role profiling is compiled in only with -DPCNN_TC_PROF=1 (tools/tc_roles.py
 // builds such a library): its clocks and 64-bit sums cost the issue loops
@@ -434,7 +475,8 @@ template <int ST, int CG, bool LRN>
 __global__ void __launch_bounds__(tc_threads<LRN>(), 1) __maxnreg__(LRN ? 255 : 200)
 conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
                const __grid_constant__ CUtensorMap tmap_x,
-               const __grid_constant__ CUtensorMap tmap_y, const TcArgs a) {
+               const __grid_constant__ CUtensorMap tmap_y,
+               const __grid_constant__ CUtensorMap tmap_y64, const TcArgs a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const uint32_t sbase = smem_u32(smem);
@@ -718,6 +760,16 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         CG == 2 ? mapa(sbase + SM_TEMPTY, 0) : sbase + SM_TEMPTY;
     uint32_t lt = 0;
     uint32_t sbox = 0;   // bf16 TMA-store staging: two 2 KB boxes used alternately
+    bool wide_prev = false;   // the last TMA store was a 64-column (4 KB) box
+    unsigned long long ep_cmp = 0, ep_box = 0, ep_st = 0, ep_fence = 0, ep_issue = 0, ep_n = 0;   // profile (warp 2)
+    // two warps per TMEM lane quarter: they split the N tile's columns at a
+    // 32 boundary, or -- bf16 TMA stores of an N tile <= 64 with two M
+    // sub-tiles -- take one sub-tile each with all its columns (64-column
+    // boxes instead of two 32-column ones)
+    const bool sub_split = a.tma_y && a.tma_y64 && a.msub == 2 && a.bn <= 64;
+    const int csplit = sub_split ? a.bn : ((a.bn / 2 + 31) / 32) * 32;
+    const int cbeg = sub_split || half == 0 ? 0 : csplit;
+    const int cend = sub_split || half != 0 ? a.bn : csplit;
     WaitClock wtf{TC_PROF(a) != 0 && lane == 0 && warp == 2};
     unsigned long long busy = 0;
     long long tb = 0;
@@ -730,6 +782,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       if (wtf.on) tb = clock64();
       tc_fence_after();
       for (int sb = 0; sb < a.msub; ++sb) {
+      if (sub_split && sb != half) continue;
       // TMEM columns of this sub-tile's accumulator
       const uint32_t tcol = buf * a.tbw + sb * a.tsub;
       int m;
@@ -771,101 +824,34 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         continue;
       }
       if (a.tma_y) {
-        // 32-column passes; full chunks are staged in this warp's swizzled
-        // box (SW64 rows for bf16, SW128 for fp32) and leave by one TMA
-        // tensor store of the warp's 32 rows (rows past M are clipped by the
-        // map); a ragged last chunk falls back to row stores.  BF16 boxes
-        // (2 KB) are double-buffered: a chunk waits only for the store issued
-        // two chunks earlier, so the stores overlap the next chunk's TMEM
-        // load and conversion (the epilogue of narrow-N layers -- AlexNet
-        // conv1, VGG conv1_x -- was serialised on each store's smem read).
+        // Full chunks are staged in this warp's swizzled box and leave by one
+        // TMA tensor store of the warp's 32 rows (rows past M are clipped by
+        // the map); a ragged last chunk falls back to row stores.  BF16
+        // chunks are 64 columns (128 B rows, SW128, 4 KB box) where the range
+        // allows, else 32 columns (SW64, 2 KB boxes used alternately, so a
+        // chunk waits only for the store issued two chunks earlier).  The
+        // TMA store cost grows with the box-row count, so narrow-N layers
+        // (AlexNet conv1, VGG conv1_x, the rank-r second stage) move 128 B
+        // per row request instead of 64 B.  FP32 chunks are 32 columns
+        // (128 B rows, SW128).
         const bool o16 = g.out_mode == OUT_BF16;
-        const int split = ((a.bn / 2 + 31) / 32) * 32;
-        const int cbeg = half == 0 ? 0 : split, cend = half == 0 ? split : a.bn;
         const int row0 = m - lane;                       // the warp's first row
-        for (int c0 = cbeg; c0 < cend; c0 += 32) {
+        const uint32_t trow = tmem_base + ((uint32_t)(quarter * 32) << 16) + tcol;
+        for (int c0 = cbeg; c0 < cend;) {
           const int n = nt * a.bn + c0;
           if (n >= g.Nfg) break;                         // warp-uniform
           const int col = grp * g.Nfg + n;
-          // bias loads issued before the TMEM load so their latencies overlap
-          const float4 *bp = (const float4 *)(a.bias + col);
-          float4 bb[8];
-#pragma unroll
-          for (int q = 0; q < 8; ++q) bb[q] = __ldg(bp + q);
-          float f[32];
-          {
-            uint32_t v[32];
-            tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + tcol + c0, v);
-            tmem_ld_wait();
-#pragma unroll
-            for (int i = 0; i < 32; ++i) f[i] = __uint_as_float(v[i]);
-          }
-#pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            f[4 * q] += bb[q].x;
-            f[4 * q + 1] += bb[q].y;
-            f[4 * q + 2] += bb[q].z;
-            f[4 * q + 3] += bb[q].w;
-          }
-          if (g.relu)
-#pragma unroll
-            for (int i = 0; i < 32; ++i) f[i] = fmaxf(f[i], 0.f);
-          if (!valid)
-#pragma unroll
-            for (int i = 0; i < 32; ++i) f[i] = 0.f;
-          const bool full = n + 32 <= g.Nfg && c0 + 32 <= cend;
-          if (full) {
-            if (lane == 0) {                             // staging box free again
-              if (o16) bulk_wait_read1();
-              else bulk_wait_read0();
-            }
-            __syncwarp();
-            uint8_t *box = o16 ? stage + sbox * 2048 : stage;
-            if (o16) {
-#pragma unroll
-              for (int q = 0; q < 4; ++q) {
-                uint4 pk;
-                uint32_t *pw = (uint32_t *)&pk;
-#pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                  __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * q + 2 * i], f[8 * q + 2 * i + 1]);
-                  pw[i] = *(uint32_t *)&b2;
-                }
-                *(uint4 *)(box + lane * 64 + ((q ^ ((lane >> 1) & 3)) << 4)) = pk;
-              }
-            } else {
-              const bool rnd = g.out_mode == OUT_F32_TF32;
-#pragma unroll
-              for (int q = 0; q < 8; ++q) {
-                float t[4];
-#pragma unroll
-                for (int i = 0; i < 4; ++i) t[i] = rnd ? tf32_rna_tc(f[4 * q + i]) : f[4 * q + i];
-                *(uint4 *)(stage + lane * 128 + ((q ^ (lane & 7)) << 4)) =
-                    make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]),
-                               __float_as_uint(t[2]), __float_as_uint(t[3]));
-              }
-            }
-            fence_proxy_async();
-            __syncwarp();
-            if (lane == 0 && row0 < g.M) {
-              tma_store_2d(&tmap_y, smem_u32(box), col, row0);
-              bulk_commit();
-            }
-            sbox ^= 1;
-          } else {
+          const bool w64 = a.tma_y64 && c0 + 64 <= cend && n + 64 <= g.Nfg;
+          const bool full = w64 || (n + 32 <= g.Nfg && c0 + 32 <= cend);
+          if (!full) {
             // ragged chunk: row stores of the np valid 16 B pieces
+            float f[32];
+            epi_chunk32(a, trow + c0, col, valid, f);
             uint4 pc[8];
             const int eb = o16 ? 2 : 4;
             if (o16) {
 #pragma unroll
-              for (int q = 0; q < 4; ++q) {
-                uint32_t *pw = (uint32_t *)&pc[q];
-#pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                  __nv_bfloat162 b2 = __floats2bfloat162_rn(f[8 * q + 2 * i], f[8 * q + 2 * i + 1]);
-                  pw[i] = *(uint32_t *)&b2;
-                }
-              }
+              for (int q = 0; q < 4; ++q) pc[q] = pack_bf16x8(f + 8 * q);
             } else {
               const bool rnd = g.out_mode == OUT_F32_TF32;
 #pragma unroll
@@ -882,7 +868,63 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
             const int np = min(o16 ? 4 : 8, (min(g.Nfg - n, cend - c0) * eb) / 16);
             char *rowp = mok ? (char *)a.y + ((size_t)m * g.out_cs + col) * eb : nullptr;
             epi_store_rows(stage, pc, np, rowp, lane);
+            c0 += 32;
+            continue;
           }
+          // first 32 columns computed while earlier stores drain, then the
+          // staging box must be free: a 64-column box (or any chunk after
+          // one) needs every earlier store to have read its source
+          const bool pon = TC_PROF(a) && warp == 2;
+          long long pt = pon ? clock64() : 0;
+          float f[32];
+          epi_chunk32(a, trow + c0, col, valid, f);
+          if (pon) { const long long t = clock64(); ep_cmp += t - pt; pt = t; }
+          if (lane == 0) {
+            if (o16 && !w64 && !wide_prev) bulk_wait_read1();
+            else bulk_wait_read0();
+          }
+          __syncwarp();
+          if (pon) { const long long t = clock64(); ep_box += t - pt; pt = t; }
+          if (w64) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              *(uint4 *)(stage + lane * 128 + ((q ^ (lane & 7)) << 4)) = pack_bf16x8(f + 8 * q);
+            if (pon) { const long long t = clock64(); ep_st += t - pt; pt = t; }
+            epi_chunk32(a, trow + c0 + 32, col + 32, valid, f);
+            if (pon) { const long long t = clock64(); ep_cmp += t - pt; pt = t; }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              *(uint4 *)(stage + lane * 128 + (((4 + q) ^ (lane & 7)) << 4)) = pack_bf16x8(f + 8 * q);
+          } else if (o16) {
+            uint8_t *box = stage + sbox * 2048;
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              *(uint4 *)(box + lane * 64 + ((q ^ ((lane >> 1) & 3)) << 4)) = pack_bf16x8(f + 8 * q);
+          } else {
+            const bool rnd = g.out_mode == OUT_F32_TF32;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              float t[4];
+#pragma unroll
+              for (int i = 0; i < 4; ++i) t[i] = rnd ? tf32_rna_tc(f[4 * q + i]) : f[4 * q + i];
+              *(uint4 *)(stage + lane * 128 + ((q ^ (lane & 7)) << 4)) =
+                  make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]),
+                             __float_as_uint(t[2]), __float_as_uint(t[3]));
+            }
+          }
+          if (pon) { const long long t = clock64(); ep_st += t - pt; pt = t; }
+          fence_proxy_async();
+          __syncwarp();
+          if (pon) { const long long t = clock64(); ep_fence += t - pt; pt = t; }
+          if (lane == 0 && row0 < g.M) {
+            if (w64) tma_store_2d(&tmap_y64, smem_u32(stage), col, row0);
+            else tma_store_2d(&tmap_y, smem_u32(o16 ? stage + sbox * 2048 : stage), col, row0);
+            bulk_commit();
+          }
+          if (pon) { ep_issue += clock64() - pt; ++ep_n; }
+          if (o16 && !w64) sbox ^= 1;
+          wide_prev = w64;
+          c0 += w64 ? 64 : 32;
         }
         continue;
       }
@@ -894,9 +936,6 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       char *obase = partial ? (char *)(a.ws + (size_t)sp * g.M * g.out_cs)
                             : (char *)a.y;
       const int eb = out16 ? 2 : 4;
-      // the two warps of a lane quarter split the tile's columns at a 32 boundary
-      const int split = ((a.bn / 2 + 31) / 32) * 32;
-      const int cbeg = half == 0 ? 0 : split, cend = half == 0 ? split : a.bn;
       for (int c0 = cbeg; c0 < cend; c0 += pass_cols) {
         const int n = nt * a.bn + c0;          // column within the group
         if (n >= g.Nfg) break;                 // warp-uniform
@@ -986,6 +1025,14 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     if (wtf.on && tb) busy += clock64() - tb;
     wtf_acc_out = wtf.acc;
     busy_out = busy;
+    if (TC_PROF(a) && warp == 2 && lane == 0) {
+      atomicAdd(&g_tc_prof[8], ep_cmp);
+      atomicAdd(&g_tc_prof[9], ep_box);
+      atomicAdd(&g_tc_prof[10], ep_st);
+      atomicAdd(&g_tc_prof[11], ep_n);
+      atomicAdd(&g_tc_prof[12], ep_fence);
+      atomicAdd(&g_tc_prof[13], ep_issue);
+    }
   }
 
   if (TC_PROF(a) && warp == 2 && lane == 0) {
@@ -1101,8 +1148,8 @@ int tc_slab_bytes(int st, int cg_channels) {
 
 template <int ST, int CG, bool LRN>
 static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_x,
-                             const CUtensorMap *tmap_y, const TcArgs &args, int grid,
-                             cudaStream_t s) {
+                             const CUtensorMap *tmap_y, const CUtensorMap *tmap_y64,
+                             const TcArgs &args, int grid, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(tc_threads<LRN>());
@@ -1117,16 +1164,17 @@ static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 2;
-  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG, LRN>, *tmap_w, *tmap_x, *tmap_y, args);
+  return cudaLaunchKernelEx(&cfg, conv_tc_kernel<ST, CG, LRN>, *tmap_w, *tmap_x, *tmap_y, *tmap_y64,
+                            args);
 }
 
-cudaError_t tc_profile(int reset, unsigned long long out[8]) {
+cudaError_t tc_profile(int reset, unsigned long long out[16]) {
   cudaError_t e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return e;
-  if (out) e = cudaMemcpyFromSymbol(out, g_tc_prof, sizeof(unsigned long long) * 8);
+  if (out) e = cudaMemcpyFromSymbol(out, g_tc_prof, sizeof(unsigned long long) * 16);
   if (e != cudaSuccess) return e;
   if (reset) {
-    unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    unsigned long long z[16] = {};
     e = cudaMemcpyToSymbol(g_tc_prof, z, sizeof(z));
   }
   return e;
@@ -1135,7 +1183,8 @@ cudaError_t tc_profile(int reset, unsigned long long out[8]) {
 cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias, void *y,
                            const int *ktab, const TcPlan &p, float *ws, const Budget &b,
-                           cudaStream_t s, const float *lrn, const CUtensorMap *tmap_y) {
+                           cudaStream_t s, const float *lrn, const CUtensorMap *tmap_y,
+                           const CUtensorMap *tmap_y64) {
   TcArgs args;
   static const int prof_env = [] {
     const char *e = exp_env("PCNN_TC_PROFILE");
@@ -1166,6 +1215,9 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   args.fd_w.init(g.pm == 2 ? g.wv + 2 * g.pad : g.pm ? g.wv : 1);
   args.y = y;
   args.tma_y = (tmap_y != nullptr && !lrn && p.splits == 1 && p.rect_w == 0 && g.pm != 2) ? 1 : 0;
+  args.tma_y64 = args.tma_y && tmap_y64 != nullptr && g.out_mode == OUT_BF16 ? 1 : 0;
+  const CUtensorMap *ym = tmap_y ? tmap_y : tmap_x;
+  const CUtensorMap *ym64 = args.tma_y64 ? tmap_y64 : ym;
   args.ws = ws;
   args.bias = bias;
   args.ktab = ktab;
@@ -1222,15 +1274,15 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
   cudaError_t e;
   const bool L = args.lrn != 0;
   if (st == ST_BF16)
-    e = p.cg == 2 ? (L ? launch_tc<ST_BF16, 2, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
-                       : launch_tc<ST_BF16, 2, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s))
-                  : (L ? launch_tc<ST_BF16, 1, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
-                       : launch_tc<ST_BF16, 1, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s));
+    e = p.cg == 2 ? (L ? launch_tc<ST_BF16, 2, true>(tmap_w, tmap_x, ym, ym64, args, p.grid, s)
+                       : launch_tc<ST_BF16, 2, false>(tmap_w, tmap_x, ym, ym64, args, p.grid, s))
+                  : (L ? launch_tc<ST_BF16, 1, true>(tmap_w, tmap_x, ym, ym64, args, p.grid, s)
+                       : launch_tc<ST_BF16, 1, false>(tmap_w, tmap_x, ym, ym64, args, p.grid, s));
   else
-    e = p.cg == 2 ? (L ? launch_tc<ST_F32, 2, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
-                       : launch_tc<ST_F32, 2, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s))
-                  : (L ? launch_tc<ST_F32, 1, true>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s)
-                       : launch_tc<ST_F32, 1, false>(tmap_w, tmap_x, tmap_y ? tmap_y : tmap_x, args, p.grid, s));
+    e = p.cg == 2 ? (L ? launch_tc<ST_F32, 2, true>(tmap_w, tmap_x, ym, ym64, args, p.grid, s)
+                       : launch_tc<ST_F32, 2, false>(tmap_w, tmap_x, ym, ym64, args, p.grid, s))
+                  : (L ? launch_tc<ST_F32, 1, true>(tmap_w, tmap_x, ym, ym64, args, p.grid, s)
+                       : launch_tc<ST_F32, 1, false>(tmap_w, tmap_x, ym, ym64, args, p.grid, s));
   if (e != cudaSuccess) return e;
   e = cudaGetLastError();
   if (e != cudaSuccess || p.splits <= 1) return e;

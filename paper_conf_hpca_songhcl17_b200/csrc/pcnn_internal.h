@@ -188,10 +188,13 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
                            const CUtensorMap *tmap_w, const float *bias,
                            void *y, const int *ktab, const TcPlan &p, float *ws,
                            const Budget &b, cudaStream_t s, const float *lrn = nullptr,
-                           const CUtensorMap *tmap_y = nullptr);
+                           const CUtensorMap *tmap_y = nullptr,
+                           const CUtensorMap *tmap_y64 = nullptr);
 // tmap_y (optional): tiled map of the output [M][out_cs] (box 32 columns x
 // 32 rows, SW64 for bf16 / SW128 for fp32); full 32-column chunks are then
 // written by TMA tensor stores from the epilogue's staging boxes.
+// tmap_y64 (optional, bf16 output): the same matrix with 64-column boxes
+// (128 B rows, SW128), used for full 64-column chunks.
 // lrn (optional) = {size, alpha, beta, k} of a following LRN layer fused into
 // the epilogue (size 5, one N tile holding all channels, no split-K).
 // A-slab width in bytes (128 / 64 / 32) for Cg channels per group, 0 if the
@@ -202,7 +205,7 @@ int tc_stages_for(int bn, int cg);
 void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages,
                   int *b_stages);
 // debug: per-role barrier-wait cycle totals accumulated while PCNN_TC_PROFILE=1
-cudaError_t tc_profile(int reset, unsigned long long out[8]);
+cudaError_t tc_profile(int reset, unsigned long long out[16]);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)
 cudaError_t tc_init();                 // sets the kernels' smem attributes
 size_t tc_smem_bytes();

@@ -112,7 +112,8 @@ struct GemmStage {           // one implicit-GEMM launch
   std::map<int, CUtensorMap> tmaps;  // weight maps by box rows
   std::map<std::tuple<const void *, int, int, int, int>, CUtensorMap> xmaps;   // A maps by
                                                  // (input, batch, rect w, h, n)
-  std::map<std::pair<const void *, long long>, CUtensorMap> ymaps;   // output maps by (y, M)
+  // output maps by (y, M): 32-column boxes, and 64-column boxes (bf16)
+  std::map<std::pair<const void *, long long>, std::pair<CUtensorMap, CUtensorMap>> ymaps;
   size_t w_bytes = 0;
   void release() {
     if (d_w) cudaFree(d_w);
@@ -703,31 +704,49 @@ static const CUtensorMap *stage_fcxmap(GemmStage &gs, const void *x, int batch, 
   return &(gs.xmaps[key] = m);
 }
 
-// Output map for the epilogue's TMA tensor stores: the [M][out_cs] output
+// Output maps for the epilogue's TMA tensor stores: the [M][out_cs] output
 // matrix (rows = output pixels, padded grid in pm mode), boxes of 32 columns
-// x 32 rows, swizzle = the box row width (64 B bf16 / 128 B fp32).  nullptr
-// when the layout does not meet TMA's alignment rules (row stores are used).
-static const CUtensorMap *stage_ymap(GemmStage &gs, void *y, long long M) {
+// x 32 rows, swizzle = the box row width (64 B bf16 / 128 B fp32), and for
+// bf16 a second map with 64-column boxes (128 B rows, SW128; *y64 = nullptr
+// when out_cs < 64).  nullptr when the layout does not meet TMA's alignment
+// rules (row stores are used).
+static const CUtensorMap *stage_ymap(GemmStage &gs, void *y, long long M,
+                                     const CUtensorMap **y64) {
   const ConvGeom &g = gs.g;
   const int eszo = g.out_mode == OUT_BF16 ? 2 : 4;
+  *y64 = nullptr;
   if (((uintptr_t)y & 15) || ((long long)g.out_cs * eszo) % 16 || g.out_cs < 32) return nullptr;
+  const bool wide = eszo == 2 && g.out_cs >= 64;
   const auto key = std::make_pair((const void *)y, M);
   auto it = gs.ymaps.find(key);
-  if (it != gs.ymaps.end()) return &it->second;
+  if (it != gs.ymaps.end()) {
+    if (wide) *y64 = &it->second.second;
+    return &it->second.first;
+  }
   auto enc = get_encode_tiled();
   if (!enc) return nullptr;
-  CUtensorMap m;
+  std::pair<CUtensorMap, CUtensorMap> m;
   const cuuint64_t dims[2] = {(cuuint64_t)g.out_cs, (cuuint64_t)M};
   const cuuint64_t strides[1] = {(cuuint64_t)g.out_cs * eszo};
   const cuuint32_t box[2] = {32, 32};
   const cuuint32_t estr[2] = {1, 1};
-  CUresult r = enc(&m, eszo == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+  CUresult r = enc(&m.first, eszo == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
                    2, y, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                    eszo == 2 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return nullptr;
+  m.second = m.first;
+  if (wide) {
+    const cuuint32_t box64[2] = {64, 32};
+    r = enc(&m.second, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, y, dims, strides, box64, estr,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return nullptr;
+  }
   if (gs.ymaps.size() > 64) gs.ymaps.clear();
-  return &(gs.ymaps[key] = m);
+  auto &slot = gs.ymaps[key] = m;
+  if (wide) *y64 = &slot.second;
+  return &slot.first;
 }
 
 // ------------------------------------------------------------------ planning
@@ -1111,10 +1130,16 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       const char *e = exp_env("PCNN_NO_TMA_STORE");
       return e && e[0] == '1';
     }();
+    static const bool no_wide = [] {
+      const char *e = exp_env("PCNN_NO_WIDE_STORE");
+      return e && e[0] == '1';
+    }();
+    const CUtensorMap *ym64 = nullptr;
     const CUtensorMap *ym = (p.splits == 1 && !lrn && !p.rect_w && !no_tma_store && g.pm != 2)
-                                ? stage_ymap(gs, y, g.M) : nullptr;
+                                ? stage_ymap(gs, y, g.M, &ym64) : nullptr;
+    if (no_wide) ym64 = nullptr;
     CUDA_TRY(counted(launch_conv_tc(g, gs.st, xm, tm, gs.d_bias, y, gs.d_ktab, p, net->d_ws,
-                                    b, s, lrn, ym)));
+                                    b, s, lrn, ym, ym64)));
   } else {
     const int tiles = conv_simt_tiles(g);
     const bool gated = is_gated(net, ly);
@@ -2263,7 +2288,7 @@ pcnn_status pcnn_last_launch_count(const pcnn_net *net, int *launches) {
 }
 
 // Debug export (not part of include/pcnn.h): tcgen05 kernel role-wait counters.
-pcnn_status pcnn_debug_tc_profile(int reset, unsigned long long out[8]) {
+pcnn_status pcnn_debug_tc_profile(int reset, unsigned long long out[16]) {
   CUDA_TRY(tc_profile(reset, out));
   return PCNN_OK;
 }

@@ -22,6 +22,7 @@ SHAPES = {  # name: (in_shape, layer)
     "conv1s": ((48, 57, 57), dict(kind="conv", out=96, k=3, stride=1, pad=0, groups=1, relu=True, in_c=48)),
     "vgg1_2": ((64, 224, 224), dict(kind="conv", out=64, k=3, stride=1, pad=1, groups=1, relu=True, in_c=64)),
     "vgg1_1s": ((32, 224, 224), dict(kind="conv", out=64, k=1, stride=1, pad=0, groups=1, relu=True, in_c=32)),
+    "rank2": ((128, 27, 27), dict(kind="conv", out=256, k=1, stride=1, pad=0, groups=2, relu=True, in_c=128)),
     "vgg2_2": ((128, 112, 112), dict(kind="conv", out=128, k=3, stride=1, pad=1, groups=1, relu=True, in_c=128)),
     "vgg5_2": ((512, 14, 14), dict(kind="conv", out=512, k=3, stride=1, pad=1, groups=1, relu=True, in_c=512)),
     "norm1pool1": ((96, 55, 55), [dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0), dict(kind="maxpool", k=3, stride=2)]),

@@ -20,7 +20,7 @@ n = pcnn.Net(net, w, b, B, "bf16")
 x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
 lib = pcnn.library()
 lib.pcnn_debug_tc_profile.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_ulonglong)]
-out = (ctypes.c_ulonglong * 8)()
+out = (ctypes.c_ulonglong * 16)()
 n.infer(x); torch.cuda.synchronize()
 lib.pcnn_debug_tc_profile(1, out)
 for _ in range(3):
@@ -33,3 +33,6 @@ print("%s B=%d plan %s" % (name, B, {k: v for k, v in n.query_layer(li, B).items
 print("  per CTA: lifetime %.0f cyc, K-blocks %.1f (%.0f cyc/kb)" % (life, c[5] / ctas, life / max(c[5] / ctas, 1)))
 for i, lab in [(0, "producer wait EMPTY"), (1, "MMA wait FULL"), (2, "MMA wait TEMPTY"), (3, "epi wait TFULL"), (6, "epi busy")]:
     print("  %-22s %5.1f%%" % (lab, 100.0 * c[i] / ctas / life))
+if c[11]:
+    print("  epilogue TMA-store chunks (warp 2): %.1f per CTA; per chunk: compute %.0f cyc, "
+          "box wait %.0f, st.shared %.0f, fence %.0f, issue %.0f cyc" % (c[11] / ctas, c[8] / c[11], c[9] / c[11], c[10] / c[11], c[12] / c[11], c[13] / c[11]))
