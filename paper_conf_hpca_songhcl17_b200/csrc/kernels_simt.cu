@@ -636,6 +636,10 @@ cudaError_t launch_stage_im2col(const float *x, void *y, int st, int B, int C, i
   return cudaGetLastError();
 }
 
+// Band kernels (staging, LRN + pool) shorten their bands at small batches
+// until a launch has about two CTAs per SM.
+constexpr long long kBandTargetCtas = 2 * 148;
+
 // Space-to-depth staging for 3-channel inputs, block 4, no padding (AlexNet
 // conv1 11x11/4 -> 3x3/1 on 48 channels).  A persistent CTA walks bands of R
 // staged rows; one thread copies each needed input row (all W floats of one
@@ -737,10 +741,12 @@ stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int
 
 static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int H, int W,
                                      int Hs, int Ws, int Cs, int tf32_round, cudaStream_t s) {
-  static const int R = [] {                          // staged rows per band
+  static const int R3 = [] {                         // staged rows per band
     const char *e = exp_env("PCNN_S2D_ROWS");
     return e && atoi(e) > 0 ? atoi(e) : 3;
   }();
+  int R = R3;                                        // small batches: shorter bands
+  while (R > 1 && (long long)B * ((Hs + R - 1) / R) < kBandTargetCtas) --R;
   const int pitch = ((W + 3) / 4 + 1) * 4;
   const size_t smem = (size_t)2 * R * 12 * pitch * 4 + 16 + 2 * R * 12 * 4;
   if (smem > 200 * 1024) return cudaErrorInvalidValue;
@@ -1501,13 +1507,16 @@ static bool use_lrn_reg(int st, int C, int lrn) {
   return lrn == 5 && !off && lrn_reg_cpt(st, C) > 0;
 }
 
-static int lrn_band_rows(int st, int W, int C, int k, int s, int Ho, int lrn) {
+// Small batches: fewer rows per band until the launch has ~2 CTAs per SM (the
+// bands overlap by k - s input rows, recomputed; results do not depend on R).
+static int lrn_band_rows(int st, int B, int W, int C, int k, int s, int Ho, int lrn) {
   const int esz = st == ST_BF16 ? 2 : 4;
   const size_t row = (size_t)W * (C * esz + (use_lrn_reg(st, C, lrn) ? 0 : 16));
   const char *e = exp_env("PCNN_LB_KB");          // tuning experiments
   const size_t budget = e ? (size_t)atoi(e) * 1024 : (size_t)LB_SMEM_BUDGET;
   int R = 1;
   while (R < Ho && (size_t)((R) * s + k) * row <= budget) ++R;
+  while (R > 1 && (long long)B * ((Ho + R - 1) / R) < kBandTargetCtas) --R;
   return R;
 }
 
@@ -1556,7 +1565,7 @@ static cudaError_t lrn_pool_dispatch(const LrnPoolArgs &a, int grid, size_t smem
 
 long long lrn_pool_tiles(int st, int B, int W, int C, int lrn, int k, int s, int Ho, int Wo) {
   if (lrn) {
-    const int R = lrn_band_rows(st, W, C, k, s, Ho, lrn);
+    const int R = lrn_band_rows(st, B, W, C, k, s, Ho, lrn);
     return (long long)B * ((Ho + R - 1) / R);
   }
   const int Q = lrn_pool_cols(st, W, C, lrn, k, s, Wo);
@@ -1701,7 +1710,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
   if (use_lrn_reg(st, C, lrn_size)) {
-    a.R = lrn_band_rows(st, W, C, k, s, Ho, lrn_size);
+    a.R = lrn_band_rows(st, B, W, C, k, s, Ho, lrn_size);
     a.nbands = (Ho + a.R - 1) / a.R;
     const size_t smem = (size_t)(min((a.R - 1) * s + k, H)) * W * C * esz;
     if (smem > 200 * 1024) return cudaErrorInvalidValue;
@@ -1734,7 +1743,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   }
   if (lrn_size > 0 && (lrn_size == 5 || lrn_size == 3)) {
     // band kernel (every LRN, fused with a following pool or not)
-    a.R = lrn_band_rows(st, W, C, k, s, Ho, lrn_size);
+    a.R = lrn_band_rows(st, B, W, C, k, s, Ho, lrn_size);
     a.nbands = (Ho + a.R - 1) / a.R;
     const size_t smem = (size_t)(min((a.R - 1) * s + k, H)) * W * (C * esz + 16);
     if (smem > 200 * 1024) return cudaErrorInvalidValue;

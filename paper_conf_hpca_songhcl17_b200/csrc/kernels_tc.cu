@@ -303,7 +303,16 @@ __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bo
 //  0 producer waits on EMPTY   1 MMA waits on FULL   2 MMA waits on TEMPTY
 //  3 epilogue waits on TFULL   4 CTA lifetime        5 K-blocks issued
 //  6 epilogue busy cycles      7 CTAs
-__device__ unsigned long long g_tc_prof[16];
+//  16.. timeline (globaltimer ns, summed over CTAs): 16 setup + PDL wait,
+//  17 wait -> first accumulator ready (epilogue warp 2), 18 wait -> epilogue
+//  done, 19 wait -> exit, 20 CTAs, 21 ~min entry, 22 max exit, 23 ~min wait,
+//  24 max wait
+__device__ unsigned long long g_tc_prof[32];
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 
 // Role profiling is compiled in only with -DPCNN_TC_PROF=1 (tools/tc_roles.py
 // builds such a library): its clocks and 64-bit sums cost the issue loops
@@ -478,6 +487,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
                const __grid_constant__ CUtensorMap tmap_y,
                const __grid_constant__ CUtensorMap tmap_y64, const TcArgs a) {
   extern __shared__ uint8_t smem_raw[];
+  const unsigned long long tl_entry = TC_PROF(a) ? gtimer() : 0;
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const uint32_t sbase = smem_u32(smem);
   const int tid = threadIdx.x;
@@ -544,12 +554,6 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   if constexpr (CG == 2) cluster_sync(); else __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *(volatile uint32_t *)(smem + SM_TMEMPTR);
-  // PDL: setup above overlapped the previous kernel's tail; activations are
-  // read (and outputs written) only after its completion
-  pdl_enter();
-  const long long t_start = TC_PROF(a) ? clock64() : 0;
-  unsigned long long wtf_acc_out = 0, busy_out = 0;   // epilogue profile (warp 2)
-
   const int HoWo = g.Ho * g.Wo;
   // work unit u -> (m tile, n tile, group, split); m fastest so CTAs running
   // concurrently share one weight slice in L2.
@@ -565,6 +569,36 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     k0 = sp * a.kb_per_split;
     k1 = min(a.kblocks, k0 + a.kb_per_split);
   };
+
+  // L2 prefetch of the first unit's weight boxes: the weights do not depend on
+  // the previous layer, so at small batches their first HBM touch overlaps its
+  // tail (the A operand is read only after the PDL wait)
+  if (warp == 0 && lane == 0 && pair < a.units) {
+    int mt, nt, grp, sp;
+    decode(pair, mt, nt, grp, sp);
+    const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
+    if (g.pm) {
+      const int pm_se0 = slab_bytes / ESZ, nj = (g.Cg / pm_se0) * g.S;
+      const int j0 = sp * a.kb_per_split, j1 = min(nj, j0 + a.kb_per_split);
+      for (int j = j0, n = 0; j < j1 && n < 64; ++j) {
+        const int cb = j / g.S, r = j - cb * g.S;
+        for (int s2 = 0; s2 < g.S; ++s2, ++n)
+          tma_prefetch_2d(&tmap_w, (r * g.S + s2) * g.Cg + cb * pm_se0, nrow);
+      }
+    } else {
+      int k0, k1;
+      kb_range(sp, k0, k1);
+      for (int kb = k0; kb < k1 && kb < k0 + 64; ++kb)
+        tma_prefetch_2d(&tmap_w, kb * (TC_ROW_BYTES / ESZ), nrow);
+    }
+  }
+  // PDL: setup above overlapped the previous kernel's tail; activations are
+  // read (and outputs written) only after its completion
+  pdl_enter();
+  const long long t_start = TC_PROF(a) ? clock64() : 0;
+  const unsigned long long tl_wait = TC_PROF(a) ? gtimer() : 0;
+  unsigned long long tl_first = 0;
+  unsigned long long wtf_acc_out = 0, busy_out = 0;   // epilogue profile (warp 2)
 
   // padded mode: K runs over (channel slab cb, filter row r) windows, each
   // feeding the S taps (r, s) of that row by shifting the A descriptor s rows
@@ -780,6 +814,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       if (wtf.on && tb) busy += clock64() - tb;
       wtf.wait(sbase + SM_TFULL + 8 * buf, use & 1);
       if (wtf.on) tb = clock64();
+      if (TC_PROF(a) && tl_first == 0) tl_first = gtimer();
       tc_fence_after();
       for (int sb = 0; sb < a.msub; ++sb) {
       if (sub_split && sb != half) continue;
@@ -1026,6 +1061,8 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     wtf_acc_out = wtf.acc;
     busy_out = busy;
     if (TC_PROF(a) && warp == 2 && lane == 0) {
+      atomicAdd(&g_tc_prof[17], tl_first - tl_wait);
+      atomicAdd(&g_tc_prof[18], gtimer() - tl_wait);
       atomicAdd(&g_tc_prof[8], ep_cmp);
       atomicAdd(&g_tc_prof[9], ep_box);
       atomicAdd(&g_tc_prof[10], ep_st);
@@ -1045,6 +1082,14 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   if (TC_PROF(a) && tid == 0) {
     atomicAdd(&g_tc_prof[4], (unsigned long long)(clock64() - t_start));
     atomicAdd(&g_tc_prof[7], 1ULL);
+    const unsigned long long tl_exit = gtimer();
+    atomicAdd(&g_tc_prof[16], tl_wait - tl_entry);
+    atomicAdd(&g_tc_prof[19], tl_exit - tl_wait);
+    atomicAdd(&g_tc_prof[20], 1ULL);
+    atomicMax(&g_tc_prof[21], ~tl_entry);
+    atomicMax(&g_tc_prof[22], tl_exit);
+    atomicMax(&g_tc_prof[23], ~tl_wait);
+    atomicMax(&g_tc_prof[24], tl_wait);
   }
   if (warp == 1) {
     if constexpr (CG == 1)
@@ -1168,13 +1213,13 @@ static cudaError_t launch_tc(const CUtensorMap *tmap_w, const CUtensorMap *tmap_
                             args);
 }
 
-cudaError_t tc_profile(int reset, unsigned long long out[16]) {
+cudaError_t tc_profile(int reset, unsigned long long out[32]) {
   cudaError_t e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return e;
-  if (out) e = cudaMemcpyFromSymbol(out, g_tc_prof, sizeof(unsigned long long) * 16);
+  if (out) e = cudaMemcpyFromSymbol(out, g_tc_prof, sizeof(unsigned long long) * 32);
   if (e != cudaSuccess) return e;
   if (reset) {
-    unsigned long long z[16] = {};
+    unsigned long long z[32] = {};
     e = cudaMemcpyToSymbol(g_tc_prof, z, sizeof(z));
   }
   return e;

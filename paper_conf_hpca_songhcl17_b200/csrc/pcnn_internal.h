@@ -205,7 +205,7 @@ int tc_stages_for(int bn, int cg);
 void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages,
                   int *b_stages);
 // debug: per-role barrier-wait cycle totals accumulated while PCNN_TC_PROFILE=1
-cudaError_t tc_profile(int reset, unsigned long long out[16]);
+cudaError_t tc_profile(int reset, unsigned long long out[32]);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)
 cudaError_t tc_init();                 // sets the kernels' smem attributes
 size_t tc_smem_bytes();

@@ -2288,7 +2288,7 @@ pcnn_status pcnn_last_launch_count(const pcnn_net *net, int *launches) {
 }
 
 // Debug export (not part of include/pcnn.h): tcgen05 kernel role-wait counters.
-pcnn_status pcnn_debug_tc_profile(int reset, unsigned long long out[16]) {
+pcnn_status pcnn_debug_tc_profile(int reset, unsigned long long out[32]) {
   CUDA_TRY(tc_profile(reset, out));
   return PCNN_OK;
 }

@@ -1,0 +1,1 @@
+for L in fc6 fc7 fc8; do timeout 120 python tools/fc_diag.py $L 1 64 256 2>&1 | grep -v "clusters of"; done

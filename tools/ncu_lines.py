@@ -1,15 +1,22 @@
-"""Per-source-line stall summary of the kernel in an .ncu-rep (read here, not
-on the GPU box):  python tools/ncu_lines.py report.ncu-rep [top]
+"""Per-source-line stall summary of the kernels in an .ncu-rep (read here, not
+on the GPU box):  python tools/ncu_lines.py report.ncu-rep [top] [function-substring]
 Aggregates the SASS rows under each CUDA source line (--print-source cuda,sass)."""
 import csv, io, subprocess, sys
 rep = sys.argv[1]
 top = int(sys.argv[2]) if len(sys.argv) > 2 else 25
+want = sys.argv[3] if len(sys.argv) > 3 else None
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                      capture_output=True, text=True).stdout
 agg, src, cur, fname = {}, {}, None, ""
 hdr = None
+keep = True
 for r in csv.reader(io.StringIO(out)):
     if not r:
+        continue
+    if r[0] == "Function Name":
+        keep = want is None or want in r[1]
+        continue
+    if not keep:
         continue
     if r[0] == "File Path":
         fname = r[1].split("/")[-1]

@@ -17,6 +17,7 @@ SHAPES = {  # name: (in_shape, layer)
     "vgg4_2": ((512, 28, 28), dict(kind="conv", out=512, k=3, stride=1, pad=1, groups=1, relu=True, in_c=512)),
     "fc6": ((256, 6, 6), dict(kind="fc", out=4096, in_f=9216, relu=True)),
     "fc7": ((4096, 1, 1), dict(kind="fc", out=4096, in_f=4096, relu=True)),
+    "fc8": ((4096, 1, 1), dict(kind="fc", out=1000, in_f=4096, relu=False)),
     "conv2p": ((128, 27, 27), dict(kind="conv", out=256, k=5, stride=1, pad=2, groups=2, relu=True, in_c=128)),
     "conv1p": ((64, 57, 57), dict(kind="conv", out=96, k=3, stride=1, pad=0, groups=1, relu=True, in_c=64)),
     "conv1s": ((48, 57, 57), dict(kind="conv", out=96, k=3, stride=1, pad=0, groups=1, relu=True, in_c=48)),

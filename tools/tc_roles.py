@@ -20,10 +20,10 @@ n = pcnn.Net(net, w, b, B, "bf16")
 x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
 lib = pcnn.library()
 lib.pcnn_debug_tc_profile.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_ulonglong)]
-out = (ctypes.c_ulonglong * 16)()
+out = (ctypes.c_ulonglong * 32)()
 n.infer(x); torch.cuda.synchronize()
 lib.pcnn_debug_tc_profile(1, out)
-for _ in range(3):
+for _ in range(1):
     n.infer(x)
 lib.pcnn_debug_tc_profile(1, out)
 c = list(out)
@@ -36,3 +36,13 @@ for i, lab in [(0, "producer wait EMPTY"), (1, "MMA wait FULL"), (2, "MMA wait T
 if c[11]:
     print("  epilogue TMA-store chunks (warp 2): %.1f per CTA; per chunk: compute %.0f cyc, "
           "box wait %.0f, st.shared %.0f, fence %.0f, issue %.0f cyc" % (c[11] / ctas, c[8] / c[11], c[9] / c[11], c[10] / c[11], c[12] / c[11], c[13] / c[11]))
+
+if c[20]:
+    M = (1 << 64) - 1
+    k = c[20]
+    span = (c[22] - (M - c[21])) / 1e3
+    print("  timeline (us, per CTA from its PDL wait): setup+wait %.2f, first accumulator %.2f, "
+          "epilogue done %.2f, exit %.2f; launch span %.2f us, wait release spread %.2f us, "
+          "first wait -> last exit %.2f us (one launch)" % (
+              c[16] / k / 1e3, c[17] / k / 1e3, c[18] / k / 1e3, c[19] / k / 1e3, span,
+              (c[24] - (M - c[23])) / 1e3, (c[22] - (M - c[23])) / 1e3))
