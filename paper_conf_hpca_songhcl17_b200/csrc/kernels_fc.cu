@@ -57,7 +57,22 @@ constexpr int FC_SM_TOTAL = FC_SM_TMEMPTR + 16;
 constexpr size_t FC_SMEM_BYTES = FC_SM_TOTAL + 1024;
 constexpr int FC_ROWS = 256;                  // weight rows per CTA pair (UMMA M)
 
+#ifndef PCNN_TC_PROF
+#define PCNN_TC_PROF 0
+#endif
+// Debug timeline (prof build, PCNN_TC_PROFILE=1; globaltimer ns summed over
+// CTAs, from each CTA's PDL wait): 0 entry -> wait, 1 accumulator ready,
+// 2 partial stored, 3 split-K peers met, 4 reduction done, 5 exit, 6 CTAs,
+// 7 ~min entry, 8 max exit, 9 ~min wait
+__device__ unsigned long long g_fc_prof[16];
+__device__ __forceinline__ unsigned long long fc_gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 struct FcArgs {
+  int prof;
   int N, B;              // output features (weight rows), batch rows of X
   int kblocks, kbps;     // K-blocks of Kpad, K-blocks per split
   int splits;            // CTA pairs per unit (K split)
@@ -107,45 +122,46 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
 // Split-K reduction of one unit by CTA `idx` (0 .. 2s-1) of the unit: rows
 // [idx * 256 / (2s), ...) for every image of the chunk, each output the sum of
 // the s partials in split order 0..s-1 (+ bias, activation, rounding).  Four
-// consecutive rows per thread (16-B loads) and all partials of two images in
-// flight before any add: the loads are L2-latency bound.
+// consecutive rows per thread (16-B loads); the partials of 16 / s images are
+// all in flight before the first add (the loads are L2-latency bound).
+template <int S>
 __device__ __forceinline__ void fc_reduce(const FcArgs &a, int rb, int ch, int idx, int t) {
-  const int s = a.splits, rows = FC_ROWS / (2 * s);
+  constexpr int s = S, rows = FC_ROWS / (2 * S);
+  constexpr int IMG = S >= 16 ? 1 : 16 / S;
   const int b0 = ch * a.nb, ncols = min(a.nb, a.B - b0);
   const size_t sBN = (size_t)a.B * a.N;
   const int nbase = rb * FC_ROWS + idx * rows;
-  if ((a.N & 3) == 0 && (rows & 3) == 0) {
-    const int r4 = rows / 4, bstep = 128 / r4;
+  if ((a.N & 3) == 0) {
+    constexpr int r4 = rows / 4, bstep = 128 / r4;
     const int q = t % r4, bsub = t / r4;
     const int n = nbase + 4 * q;
     if (bsub >= bstep || n >= a.N) return;
     const float4 bias = *(const float4 *)(a.bias + n);
-    for (int bi = bsub; bi < ncols; bi += 2 * bstep) {
-      const bool two = bi + bstep < ncols;
-      const size_t o0 = (size_t)(b0 + bi) * a.N + n, o1 = o0 + (size_t)bstep * a.N;
-      float4 v0[16], v1[16];
+    for (int bi0 = bsub; bi0 < ncols; bi0 += IMG * bstep) {
+      float4 v[IMG][S];
 #pragma unroll
-      for (int j = 0; j < 16; ++j) {
-        if (j < s) {
-          v0[j] = __ldcg((const float4 *)(a.ws + (size_t)j * sBN + o0));   // L2: peers' writes
-          if (two) v1[j] = __ldcg((const float4 *)(a.ws + (size_t)j * sBN + o1));
+      for (int h = 0; h < IMG; ++h) {
+        const int bi = bi0 + h * bstep;
+        if (bi < ncols) {
+          const size_t o = (size_t)(b0 + bi) * a.N + n;
+#pragma unroll
+          for (int j = 0; j < S; ++j)
+            v[h][j] = __ldcg((const float4 *)(a.ws + (size_t)j * sBN + o));   // L2: peers' writes
         }
       }
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        if (h == 1 && !two) break;
-        float4 acc = h ? v1[0] : v0[0];
+      for (int h = 0; h < IMG; ++h) {
+        const int bi = bi0 + h * bstep;
+        if (bi >= ncols) break;
+        float4 acc = v[h][0];
 #pragma unroll
-        for (int j = 1; j < 16; ++j) {
-          if (j < s) {
-            const float4 v = h ? v1[j] : v0[j];
-            acc.x += v.x;
-            acc.y += v.y;
-            acc.z += v.z;
-            acc.w += v.w;
-          }
+        for (int j = 1; j < S; ++j) {
+          acc.x += v[h][j].x;
+          acc.y += v[h][j].y;
+          acc.z += v[h][j].z;
+          acc.w += v[h][j].w;
         }
-        const size_t yo = (size_t)(b0 + bi + h * bstep) * a.ldy + n;
+        const size_t yo = (size_t)(b0 + bi) * a.ldy + n;
         fc_store(a.y, yo, fc_act(acc.x + bias.x, a.relu), a.out_mode);
         fc_store(a.y, yo + 1, fc_act(acc.y + bias.y, a.relu), a.out_mode);
         fc_store(a.y, yo + 2, fc_act(acc.z + bias.z, a.relu), a.out_mode);
@@ -159,14 +175,12 @@ __device__ __forceinline__ void fc_reduce(const FcArgs &a, int rb, int ch, int i
     const int n = nbase + r;
     if (n >= a.N) continue;
     const size_t off = (size_t)(b0 + bi) * a.N + n;
-    float v[16];
+    float v[S];
 #pragma unroll
-    for (int j = 0; j < 16; ++j)
-      if (j < s) v[j] = __ldcg(a.ws + (size_t)j * sBN + off);
+    for (int j = 0; j < S; ++j) v[j] = __ldcg(a.ws + (size_t)j * sBN + off);
     float acc = v[0];
 #pragma unroll
-    for (int j = 1; j < 16; ++j)
-      if (j < s) acc += v[j];
+    for (int j = 1; j < S; ++j) acc += v[j];
     fc_store(a.y, (size_t)(b0 + bi) * a.ldy + n, fc_act(acc + __ldg(&a.bias[n]), a.relu),
              a.out_mode);
   }
@@ -177,6 +191,9 @@ __global__ void __launch_bounds__(FC_THREADS, 1)
 fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__ CUtensorMap tmap_x,
              const FcArgs a) {
   extern __shared__ uint8_t smem_raw[];
+  const bool prof = PCNN_TC_PROF && a.prof;
+  const unsigned long long t_entry = prof ? fc_gtimer() : 0;
+  unsigned long long t_full = 0, t_st = 0, t_met = 0, t_red = 0;
   uint8_t *smem = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   const uint32_t sbase = smem_u32(smem);
   const int tid = threadIdx.x;
@@ -228,6 +245,7 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
     }
   }
   pdl_enter();
+  const unsigned long long t_wait = prof ? fc_gtimer() : 0;
 
   uint32_t stage = 0, phase = 0;
   int lt = 0;
@@ -281,6 +299,7 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
       const int q = warp & 3;
       mbar_wait(sbase + FC_SM_TFULL, lt & 1);
       tc_fence_after();
+      if (prof && t_full == 0) t_full = fc_gtimer();
       const int b0 = ch * a.nb;
       const int ncols = min(a.nb, a.B - b0);
       const bool partial = s > 1;
@@ -315,6 +334,7 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
       }
       if (partial) {
         // meet the unit's other 2s - 1 CTAs, then reduce this CTA's row slice
+        if (prof && t_st == 0) t_st = fc_gtimer();
         epi_bar();
         const int t = tid - 64;
         if (t == 0) {
@@ -323,8 +343,14 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
           while (ld_acquire(&a.sem[u]) < 2u * s) __nanosleep(64);
         }
         epi_bar();
-        fc_reduce(a, rb, ch, split * 2 + (int)rank, t);
+        if (prof && t_met == 0) t_met = fc_gtimer();
+        const int idx = split * 2 + (int)rank;
+        if (s == 2) fc_reduce<2>(a, rb, ch, idx, t);
+        else if (s == 4) fc_reduce<4>(a, rb, ch, idx, t);
+        else if (s == 8) fc_reduce<8>(a, rb, ch, idx, t);
+        else fc_reduce<16>(a, rb, ch, idx, t);
         epi_bar();
+        if (prof && t_red == 0) t_red = fc_gtimer();
         if (t == 0) {   // the last CTA out re-arms the unit's counters for the next launch
           if (atomicAdd(&a.sem[a.units + u], 1u) == 2u * s - 1) {
             a.sem[u] = 0;
@@ -338,6 +364,19 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
   __syncthreads();
   cluster_sync();
   tc_fence_after();
+  if (prof && warp == 2 && lane == 0) {
+    const unsigned long long t_exit = fc_gtimer();
+    atomicAdd(&g_fc_prof[0], t_wait - t_entry);
+    atomicAdd(&g_fc_prof[1], t_full - t_wait);
+    atomicAdd(&g_fc_prof[2], (t_st ? t_st : t_full) - t_wait);
+    atomicAdd(&g_fc_prof[3], (t_met ? t_met : t_full) - t_wait);
+    atomicAdd(&g_fc_prof[4], (t_red ? t_red : t_full) - t_wait);
+    atomicAdd(&g_fc_prof[5], t_exit - t_wait);
+    atomicAdd(&g_fc_prof[6], 1ULL);
+    atomicMax(&g_fc_prof[7], ~t_entry);
+    atomicMax(&g_fc_prof[8], t_exit);
+    atomicMax(&g_fc_prof[9], ~t_wait);
+  }
   if (warp == 1)
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
                  "r"(a.tmem_cols));
@@ -376,6 +415,19 @@ int fc_stage_count(int nb) {
   return std::min(FC_MAX_STAGES, FC_STAGE_BUDGET / per);
 }
 
+// Debug: the FC timeline counters (prof build)
+cudaError_t fc_profile(int reset, unsigned long long out[16]) {
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return e;
+  if (out) e = cudaMemcpyFromSymbol(out, g_fc_prof, sizeof(unsigned long long) * 16);
+  if (e != cudaSuccess) return e;
+  if (reset) {
+    unsigned long long z[16] = {};
+    e = cudaMemcpyToSymbol(g_fc_prof, z, sizeof(z));
+  }
+  return e;
+}
+
 cudaError_t launch_fc_tc(const FcPlan &p, int st, const CUtensorMap *tmap_w,
                          const CUtensorMap *tmap_x, const float *bias, void *y, float *ws,
                          unsigned *sem, int N, int B, int kblocks, int relu, int out_mode,
@@ -384,6 +436,11 @@ cudaError_t launch_fc_tc(const FcPlan &p, int st, const CUtensorMap *tmap_w,
       p.nb % 16 || (p.splits > 1 && (!ws || !sem)) || p.grid != 2 * p.splits * p.groups)
     return cudaErrorInvalidValue;
   FcArgs a;
+  static const int prof_env = [] {
+    const char *e = exp_env("PCNN_TC_PROFILE");
+    return e && e[0] == '1' ? 1 : 0;
+  }();
+  a.prof = prof_env;
   a.N = N;
   a.B = B;
   a.kblocks = kblocks;

@@ -2293,6 +2293,12 @@ pcnn_status pcnn_debug_tc_profile(int reset, unsigned long long out[32]) {
   return PCNN_OK;
 }
 
+// Debug export: FC kernel timeline counters (prof build)
+pcnn_status pcnn_debug_fc_profile(int reset, unsigned long long out[16]) {
+  CUDA_TRY(fc_profile(reset, out));
+  return PCNN_OK;
+}
+
 pcnn_status pcnn_enable_sm_census(pcnn_net *net, int enable) {
   if (!net) return fail(PCNN_ERR_INVALID_ARGUMENT, "null net");
   net->census = enable != 0;

@@ -11,11 +11,8 @@ from paper_conf_hpca_songhcl17_b200 import pcnn
 from tools.one_layer import make_net
 
 lib = pcnn.library()
-lib.pcnn_debug_fc_profile.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_ulonglong)]
+lib.pcnn_debug_fc_profile.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_ulonglong)]
 out = (ctypes.c_ulonglong * 16)()
-for size in (2, 4, 8, 16):
-    lib.pcnn_debug_fc_profile(0, size, out)
-    print("clusters of %d FC CTAs resident at once: %d" % (size, out[15]))
 name = sys.argv[1] if len(sys.argv) > 1 else "fc6"
 for B in [int(b) for b in sys.argv[2:]] or [1, 256]:
     shape, net, li = make_net(name)
@@ -23,15 +20,16 @@ for B in [int(b) for b in sys.argv[2:]] or [1, 256]:
     n = pcnn.Net(net, w, b, B, "bf16")
     x = torch.from_numpy(synth.images(0, B, shape, lo=-1, hi=1)).cuda()
     n.infer(x); torch.cuda.synchronize()
-    lib.pcnn_debug_fc_profile(1, 2, out)
+    lib.pcnn_debug_fc_profile(1, out)
     n.infer(x)
-    lib.pcnn_debug_fc_profile(1, 2, out)
+    lib.pcnn_debug_fc_profile(1, out)
     c = list(out)
-    k = max(c[5], 1)
+    k = max(c[6], 1)
     M = (1 << 64) - 1
     info = n.query_layer(li, B)
     print("%s B=%d splits %d grid %d: per CTA from PDL wait (us): entry->wait %.2f, acc ready %.2f, "
-          "parked %.2f, reduced %.2f, exit %.2f; first wait -> last exit %.2f, span %.2f" % (
-              name, B, info["splits"], info["grid"], c[0] / k / 1e3, c[1] / k / 1e3, c[2] / k / 1e3,
-              c[3] / k / 1e3, c[4] / k / 1e3, (c[7] - (M - c[8])) / 1e3, (c[7] - (M - c[6])) / 1e3))
+          "partial stored %.2f, peers met %.2f, reduced %.2f, exit %.2f; first wait -> last exit %.2f, "
+          "span %.2f" % (name, B, info["splits"], info["grid"], c[0] / k / 1e3, c[1] / k / 1e3,
+                         c[2] / k / 1e3, c[3] / k / 1e3, c[4] / k / 1e3, c[5] / k / 1e3,
+                         (c[8] - (M - c[9])) / 1e3, (c[8] - (M - c[7])) / 1e3))
     n.close()
