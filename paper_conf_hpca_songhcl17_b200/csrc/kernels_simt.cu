@@ -1092,7 +1092,7 @@ __global__ void __launch_bounds__(256) lrn_pool_kernel(const LrnPoolArgs a) {
         for (int j = 0; j < VN + 2 * HALF; ++j) {
           const int t = j - HALF;            // channel offset from the chunk start
           const float xv = t < 0 ? prev.v[VN + t] : (t < VN ? cur.v[t] : next.v[t - VN]);
-          sq[j] = xv * xv;
+          sq[j] = __fmul_rn(xv, xv);
         }
         Vec16<ST> out;
         lrn_normalise<ST == ST_BF16, LS, VN>(sq, cur.v, a.lrn_k, a.lrn_alpha_over_n, a.lrn_beta,
@@ -1235,7 +1235,7 @@ __global__ void __launch_bounds__(256) lrn_band_kernel(const LrnPoolArgs a) {
           for (int j = 0; j < VN + 2 * HALF; ++j) {
             const int o = j - HALF;
             const float xv = o < 0 ? tail[HALF + o] : (o < VN ? cur.v[o] : nxt.v[o - VN]);
-            sq[j] = xv * xv;
+            sq[j] = __fmul_rn(xv, xv);
           }
           Vec16<ST> out;
           lrn_normalise<ST == ST_BF16, LS, VN>(sq, cur.v, a.lrn_k, a.lrn_alpha_over_n,
@@ -1400,7 +1400,7 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
             if (o < 0) xv = j > 0 ? ch[j - 1].v[VN + o] : tail[HALF + o];
             else if (o < VN) xv = ch[j].v[o];
             else xv = j + 1 < CPT ? ch[j + 1].v[o - VN] : head[o - VN];
-            sq[q] = xv * xv;
+            sq[q] = __fmul_rn(xv, xv);
           }
           Vec16<ST> out;
           lrn_normalise<ST == ST_BF16, 2 * HALF + 1, VN>(sq, ch[j].v, a.lrn_k, a.lrn_alpha_over_n,

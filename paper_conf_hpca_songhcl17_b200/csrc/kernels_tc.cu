@@ -51,10 +51,9 @@ constexpr int EPI_PITCH = 144;          // epilogue staging row: 128 B + 16 B pa
 // per-warp staging slot: 32 rows x 144 B (st.global path) or one 32-row x
 // 32-column swizzled TMA-store box (<= 4 KB); 1024-aligned slots
 constexpr int EPI_WARP_BYTES = 5120;
-// warps: 0 TMA producer, 1 MMA issuer, then NEPI epilogue warps (8, two per
-// TMEM lane quarter splitting the columns; 4 for the LRN-fused variant, whose
-// per-row channel vector needs ~255 registers)
-template <bool LRN> __host__ __device__ constexpr int tc_nepi() { return LRN ? 4 : 8; }
+// warps: 0 TMA producer, 1 MMA issuer, then NEPI = 8 epilogue warps (two per
+// TMEM lane quarter splitting the columns, also in the LRN-fused variant)
+template <bool LRN> __host__ __device__ constexpr int tc_nepi() { return 8; }
 template <bool LRN> __host__ __device__ constexpr int tc_threads() { return 64 + 32 * tc_nepi<LRN>(); }
 constexpr int TC_TMEM_COLS = 512;       // 2 accumulator buffers x 256 columns
 
@@ -225,77 +224,113 @@ __device__ __forceinline__ uint4 pack_bf16x8(const float *f) {
 
 // Epilogue with the following LRN layer fused in (R3; Caffe size
 // 5).  The tile holds every channel of its pixels (bn == Nfg <= 128, one N
-// tile), so each thread normalises its own pixel's channel vector in
-// registers: bias, ReLU, rounding to the storage precision, then exactly the
-// stand-alone LRN kernel's arithmetic (same sum order and transcendental
-// form), so the result is bitwise identical to conv -> store -> LRN.
+// tile).  The two warps of a TMEM lane quarter split the channels in halves
+// (16-aligned); each thread streams its pixel's half through 16-column TMEM
+// loads, 8 channels (one 16 B bf16 piece) at a time, with the window's 2
+// channels on either side taken from the neighbouring columns (the other
+// half's at the boundary).  Per value: bias, ReLU, rounding to the storage
+// precision -- the value the stand-alone conv would have stored -- then the
+// stand-alone LRN kernels' arithmetic (squares by __fmul_rn, lrn_normalise),
+// so the result is the one of conv -> store -> LRN.
+template <int ST>
+__device__ __forceinline__ void lrn_x16(const TcArgs &a, uint32_t taddr, int c0, bool valid,
+                                        float (&f)[16]) {
+  const ConvGeom &g = a.g;
+  if (c0 >= g.Nfg) {                                   // past the channels: zero
+#pragma unroll
+    for (int i = 0; i < 16; ++i) f[i] = 0.f;
+    return;
+  }
+  uint32_t v[16];
+  tmem_ld16(taddr + c0, v);
+  const float4 *bp = (const float4 *)(a.bias + c0);
+  float4 bb[4];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) bb[q] = __ldg(bp + q);
+  tmem_ld_wait();
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {
+    const float b = i % 4 == 0 ? bb[i / 4].x : i % 4 == 1 ? bb[i / 4].y : i % 4 == 2 ? bb[i / 4].z : bb[i / 4].w;
+    float x = __uint_as_float(v[i]) + b;
+    if (g.relu) x = fmaxf(x, 0.f);
+    if constexpr (ST == ST_BF16) x = __bfloat162float(__float2bfloat16_rn(x));
+    else if (g.out_mode == OUT_F32_TF32) x = tf32_rna_tc(x);
+    f[i] = (c0 + i < g.Nfg && valid) ? x : 0.f;        // halo rows are stored as zeros
+  }
+}
+
 template <int ST>
 __device__ __forceinline__ void epilogue_lrn(const TcArgs &a, uint32_t taddr, bool mok,
                                              bool valid, size_t orow, uint8_t *stage,
-                                             int lane) {
+                                             int lane, int half) {
   const ConvGeom &g = a.g;
-  constexpr int MAXC = 128;
-  float f[MAXC];
-#pragma unroll
-  for (int c0 = 0; c0 < MAXC; c0 += 32) {
-    if (c0 < a.bn) {                       // warp-uniform
-      uint32_t v[32];
-      tmem_ld32(taddr + c0, v);
-      tmem_ld_wait();
-#pragma unroll
-      for (int i = 0; i < 32; ++i) f[c0 + i] = __uint_as_float(v[i]);
-    }
-  }
   const int C = g.Nfg;
-#pragma unroll
-  for (int i = 0; i < MAXC; ++i) {
-    float x = f[i] + __ldg(&a.bias[i]);
-    if (g.relu) x = fmaxf(x, 0.f);
-    // the value the stand-alone conv would have stored
-    if constexpr (ST == ST_BF16) x = __bfloat162float(__float2bfloat16_rn(x));
-    else if (g.out_mode == OUT_F32_TF32) x = tf32_rna_tc(x);
-    f[i] = (i < C && valid) ? x : 0.f;   // padded-layout halo rows are stored as zeros
-  }
-  float sq[MAXC + 4];
-  sq[0] = sq[1] = sq[MAXC + 2] = sq[MAXC + 3] = 0.f;
-#pragma unroll
-  for (int i = 0; i < MAXC; ++i) sq[i + 2] = f[i] * f[i];
-  // normalised outputs, 8 channels = one 16 B piece (bf16) / two (fp32)
+  const int ch = ((C + 1) / 2 + 15) & ~15;             // channels per half (16-aligned)
+  const int lo = half * ch, hi = min(C, lo + ch);
+  if (lo >= hi) return;                                // warp-uniform
   constexpr int EB = ST == ST_BF16 ? 2 : 4;
-  const int row_bytes = C * EB;
-  char *rowp = mok ? (char *)a.y + orow * EB : nullptr;
+  constexpr int PER = 16 / EB;                         // channels per 16 B piece
+  float A[16], Bv[16];
+  float l0 = 0.f, l1 = 0.f;                            // channels c - 2, c - 1
+  if (lo > 0) {
+    lrn_x16<ST>(a, taddr, lo - 16, valid, A);
+    l0 = A[14];
+    l1 = A[15];
+  }
+  lrn_x16<ST>(a, taddr, lo, valid, A);
+  lrn_x16<ST>(a, taddr, lo + 16, valid, Bv);
+  char *rowp = mok ? (char *)a.y + (orow + lo) * EB : nullptr;
+  uint4 pc[8];
+  // ch <= 64: at most 8 steps of 8 channels, unrolled so every register
+  // index is static; BF16 flushes its 128 B row piece once, FP32 every 4 steps
 #pragma unroll
-  for (int pass = 0; pass < MAXC * EB / 128; ++pass) {   // 128 B of the row per pass
-    if (pass * 128 >= row_bytes) break;                  // warp-uniform
-    uint4 pc[8];
+  for (int p = 0; p < 8; ++p) {
+    const int c = lo + 8 * p;
+    if (c >= hi) break;                                // warp-uniform
+    const bool odd = (p & 1) != 0;
+    float w[12];
+    w[0] = l0;
+    w[1] = l1;
 #pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      constexpr int PER = 16 / EB;                       // channels per piece
-      const int c0 = (pass * 128 + q * 16) / EB;
-      float o[PER];
-      float sq8[PER + 4], x8[PER];
+    for (int i = 0; i < 8; ++i) w[2 + i] = odd ? A[8 + i] : A[i];
+    w[10] = odd ? Bv[0] : A[8];
+    w[11] = odd ? Bv[1] : A[9];
+    float sq[12];
 #pragma unroll
-      for (int t = 0; t < PER + 4; ++t) sq8[t] = sq[(c0 + t) < MAXC + 4 ? c0 + t : MAXC + 3];
+    for (int i = 0; i < 12; ++i) sq[i] = __fmul_rn(w[i], w[i]);
+    float o[8];
+    lrn_normalise<ST == ST_BF16, 5, 8>(sq, w + 2, a.lrn_k, a.lrn_a_over_n, a.lrn_beta, o);
+    if constexpr (ST == ST_BF16) {
+      pc[p] = pack_bf16x8(o);
+    } else {
+      float t[8];
 #pragma unroll
-      for (int j = 0; j < PER; ++j) x8[j] = c0 + j < MAXC ? f[c0 + j < MAXC ? c0 + j : 0] : 0.f;
-      lrn_normalise<ST == ST_BF16, 5, PER>(sq8, x8, a.lrn_k, a.lrn_a_over_n, a.lrn_beta, o);
-      if constexpr (ST == ST_BF16) {
-        uint32_t *pw = (uint32_t *)&pc[q];
+      for (int i = 0; i < 8; ++i) t[i] = g.out_mode == OUT_F32_TF32 ? tf32_rna_tc(o[i]) : o[i];
+      pc[(2 * p) % 8] = make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]),
+                                   __float_as_uint(t[2]), __float_as_uint(t[3]));
+      pc[(2 * p + 1) % 8] = make_uint4(__float_as_uint(t[4]), __float_as_uint(t[5]),
+                                       __float_as_uint(t[6]), __float_as_uint(t[7]));
+    }
+    l0 = w[8];
+    l1 = w[9];
+    if (odd) {                                         // next 16 columns
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          __nv_bfloat162 b2 = __floats2bfloat162_rn(o[2 * i], o[2 * i + 1]);
-          pw[i] = *(uint32_t *)&b2;
-        }
-      } else {
-        float t[4];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) t[i] = g.out_mode == OUT_F32_TF32 ? tf32_rna_tc(o[i]) : o[i];
-        pc[q] = make_uint4(__float_as_uint(t[0]), __float_as_uint(t[1]), __float_as_uint(t[2]),
-                           __float_as_uint(t[3]));
+      for (int i = 0; i < 16; ++i) A[i] = Bv[i];
+      lrn_x16<ST>(a, taddr, c + 24, valid, Bv);
+    }
+    const bool last = c + 8 >= hi;
+    if constexpr (ST == ST_BF16) {
+      if (p == 7 || last) {
+        const int np = min(p + 1, (hi - lo + PER - 1) / PER);
+        epi_store_rows(stage, pc, np, rowp, lane);
+      }
+    } else {
+      if (p % 4 == 3 || last) {
+        const int base = (p / 4) * 8;                  // pieces already stored
+        const int np = min(2 * (p % 4 + 1), (hi - lo + PER - 1) / PER - base);
+        epi_store_rows(stage, pc, np, rowp ? rowp + base * 16 : nullptr, lane);
       }
     }
-    const int np = min(8, (row_bytes - pass * 128) / 16);
-    epi_store_rows(stage, pc, np, rowp ? rowp + pass * 128 : nullptr, lane);
   }
 }
 
@@ -481,7 +516,7 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
 }
 
 template <int ST, int CG, bool LRN>
-__global__ void __launch_bounds__(tc_threads<LRN>(), 1) __maxnreg__(LRN ? 255 : 200)
+__global__ void __launch_bounds__(tc_threads<LRN>(), 1) __maxnreg__(LRN ? 200 : 200)
 conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
                const __grid_constant__ CUtensorMap tmap_x,
                const __grid_constant__ CUtensorMap tmap_y,
@@ -855,7 +890,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       const size_t orow = (size_t)m * g.out_cs;
       if constexpr (LRN) {
         epilogue_lrn<ST>(a, tmem_base + ((uint32_t)(quarter * 32) << 16) + tcol, mok,
-                         valid, orow, stage, lane);
+                         valid, orow, stage, lane, half);
         continue;
       }
       if (a.tma_y) {

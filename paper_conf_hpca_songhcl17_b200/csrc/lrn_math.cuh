@@ -8,7 +8,8 @@ namespace pcnn {
 
 // The LRN of N consecutive channels: out[j] = x[j] * (k + a_n *
 // sum_{w<LS} sq[j+w])^(-beta), with sq[t] = the square of channel j0 + t -
-// LS/2 (zero outside the tensor).  Every LRN path (the stand-alone kernels and
+// LS/2 (zero outside the tensor), computed by every caller as __fmul_rn(x, x)
+// so no caller's compiler can contract it into the window sum.  Every LRN path (the stand-alone kernels and
 // the conv epilogue) calls this, so they agree bit for bit.
 //   * size 5: the window is summed as ((sq0 + sq1) + (sq2 + sq3)) + sq4, so
 //     neighbouring channels share the pair sums and the dependency chain is

@@ -1175,8 +1175,10 @@ static bool fuse_conv_lrn(const pcnn_net *net, int i) {
   if (!net->fuse_lrn_pool || i + 1 >= (int)net->layers.size()) return false;
   const Layer &c = net->layers[i], &l = net->layers[i + 1];
   // padded-layout convs fuse LRN only on request (PCNN_FLAG_CONV_LRN_EPILOGUE):
-  // the LRN epilogue (4 warps, one pixel's channel vector per thread) made
-  // AlexNet conv1 279 us against 79 us conv + 92 us register-LRN/pool kernel
+  // even the 8-warp streaming LRN epilogue makes AlexNet conv1 161 us (+ 49 us
+  // for the then stand-alone pool1) against 84 us conv + 90 us LRN+pool kernel
+  // at B = 256: two epilogue warps per SM sub-partition cannot hide the
+  // per-element MUFU work (round 1's 4-warp epilogue: 279 us)
   const bool pm_lrn = net->conv_lrn_pm;
   return c.d.kind == PCNN_CONV && l.d.kind == PCNN_LRN && l.d.kernel == 5 &&
          (c.pm_halo == 0 || pm_lrn) && c.perf_sh * c.perf_sw == 1 &&

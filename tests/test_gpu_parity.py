@@ -205,13 +205,17 @@ def test_infer_host_matches_device(orc):
 
 
 # ------------------------------------------------------------ layout transforms
-def test_fused_lrn_pool_bitwise_equals_unfused(orc):
+@pytest.mark.parametrize("shape", [(96, 27, 27), (96, 55, 55), (256, 27, 27), (48, 19, 71)])
+def test_fused_lrn_pool_bitwise_equals_unfused(orc, shape):
     """norm -> pool fusion changes scheduling only: the LRN output is rounded
-    to the storage precision before the max in both paths."""
-    net = dict(in_shape=(96, 27, 27), layers=[
+    to the storage precision before the max in both paths.  The fused pair
+    runs the register-only walk kernel (3 x 3 / 2 max pool; strips of 30
+    columns, 71 -> 3 strips), the unfused one the LRN kernel + the pooling
+    kernel: bitwise equal."""
+    net = dict(in_shape=shape, layers=[
         dict(kind="lrn", size=5, alpha=1e-4, beta=0.75, k=1.0),
         dict(kind="maxpool", k=3, stride=2)])
-    x = small_inputs((96, 27, 27), 3, lo=-128, hi=128)
+    x = small_inputs(shape, 3, lo=-128, hi=128)
     for prec in PRECS:
         fr = gpu_run(net, [None, None], [None, None], x, prec)
         fused = fr["out"]
