@@ -419,32 +419,50 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
         "logits_sha256": hashlib.sha256(np.ascontiguousarray(logits, np.float32).tobytes()).hexdigest(),
     }
     if e2e:
-        # end to end through the host-buffer C-ABI call (pinned host memory,
-        # H2D of the images and D2H of logits / probs / entropy every step)
-        xh = torch.from_numpy(x_host).pin_memory()
+        # end to end through the host-buffer C-ABI calls (pinned host memory,
+        # H2D of the images and D2H of logits / probs / entropy every step).
+        # Headline: 8-bit pixels (the images' native format, pcnn_infer_host_u8,
+        # network input = pixel - 128 on the device); also the fp32 form.
         oh = torch.empty((B, n.out_elems)).pin_memory()
         ph = torch.empty((B, n.out_elems)).pin_memory()
         hh = torch.empty((B,)).pin_memory()
         og = torch.empty((B, n.out_elems), device="cuda") if world > 1 else None
-        for _ in range(2):
-            n.infer_host(xh, oh, ph, hh, stream=ctx.stream)
-        ctx.barrier()
-        te0 = time.perf_counter()
-        e2e_steps = max(3, min(steps, 20))
-        for _ in range(e2e_steps):
-            n.infer_host(xh, oh, ph, hh, stream=ctx.stream)
-            if world > 1:   # gather THIS step's logits (re-uploaded from the host result)
-                og.copy_(oh, non_blocking=True)
-                ctx.dist.all_gather_into_tensor(gathered, og)
-                torch.cuda.synchronize()
-        te = time.perf_counter() - te0
-        ctx.barrier()
-        te = ctx.max_over_ranks(te)
-        res["e2e"] = {"value": round(world * B * e2e_steps / te, 1), "unit": "images/sec",
-                      "h2d_bytes_per_step": int(x_host.nbytes + (oh.numel() * 4 if world > 1 else 0)),
-                      "d2h_bytes_per_step": int(oh.numel() * 4 + ph.numel() * 4 + hh.numel() * 4),
-                      "api": "pcnn_infer_host (pinned host buffers)" +
-                             (" + all_gather of the step's logits" if world > 1 else "")}
+        px_host = synth.pixels(start, B, net["in_shape"])
+        forms = {
+            "u8": (torch.from_numpy(px_host).pin_memory(),
+                   "pcnn_infer_host_u8 (pinned uint8 pixels, mean 128 subtracted on the device)"),
+            "f32": (torch.from_numpy(x_host).pin_memory(), "pcnn_infer_host (pinned fp32 images)"),
+        }
+        e2e_res = {}
+        for form, (xh, api) in forms.items():
+            def call():
+                if form == "u8":
+                    n.infer_host_u8(xh, oh, mean=[128.0] * net["in_shape"][0], probs=ph, entropy=hh,
+                                    stream=ctx.stream)
+                else:
+                    n.infer_host(xh, oh, ph, hh, stream=ctx.stream)
+            for _ in range(2):
+                call()
+            ctx.barrier()
+            te0 = time.perf_counter()
+            e2e_steps = max(3, min(steps, 20))
+            for _ in range(e2e_steps):
+                call()
+                if world > 1:   # gather THIS step's logits (re-uploaded from the host result)
+                    og.copy_(oh, non_blocking=True)
+                    ctx.dist.all_gather_into_tensor(gathered, og)
+                    torch.cuda.synchronize()
+            te = time.perf_counter() - te0
+            ctx.barrier()
+            te = ctx.max_over_ranks(te)
+            e2e_res[form] = {
+                "value": round(world * B * e2e_steps / te, 1), "unit": "images/sec",
+                "h2d_bytes_per_step": int(xh.numel() * xh.element_size() +
+                                          (oh.numel() * 4 if world > 1 else 0)),
+                "d2h_bytes_per_step": int(oh.numel() * 4 + ph.numel() * 4 + hh.numel() * 4),
+                "api": api + (" + all_gather of the step's logits" if world > 1 else "")}
+        res["e2e"] = dict(e2e_res["u8"])
+        res["e2e"]["fp32_images"] = e2e_res["f32"]
     return res, n, (net, w, b), (x, out, probs, ent)
 
 

@@ -291,6 +291,19 @@ pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch,
                             float *h_out, float *h_probs, float *h_entropy,
                             void *stream);
 
+/* pcnn_infer_host for 8-bit images, the pixels' native format: h_pixels
+ * [batch][C][H][W] uint8 (host, pinned for full PCIe bandwidth).  The network
+ * input is x = (pixel - mean[c]) * scale (mean: C floats, NULL = 0), computed
+ * on the device (exact for integer pixels and mean, scale 1); everything else
+ * as pcnn_infer_host -- PCIe carries 1 B per pixel instead of 4.  The batch
+ * runs as 4 pipelined chunks when the copy per image exceeds a quarter of
+ * the modelled compute per image.  Per-image results are bitwise those of
+ * pcnn_infer on the converted images. */
+pcnn_status pcnn_infer_host_u8(pcnn_net *net, const unsigned char *h_pixels,
+                               const float *mean, float scale, int batch,
+                               float *h_out, float *h_probs, float *h_entropy,
+                               void *stream);
+
 /* Elements per image of d_out (C*H*W of the last layer). */
 pcnn_status pcnn_output_size(const pcnn_net *net, int *out_elems);
 

@@ -819,6 +819,45 @@ cudaError_t launch_stage_input(const float *x, void *y, int st, int B, int C, in
   return cudaGetLastError();
 }
 
+// pcnn_infer_host_u8: uint8 NCHW pixels -> fp32 network input
+// (pixel - mean[c]) * scale, 16 pixels per thread (one 16 B load, four 16 B
+// stores).  HW % 16 == 0 takes the vector path; else one pixel per step.
+__global__ void pixels_u8_kernel(const unsigned char *__restrict__ px, const float *__restrict__ mean,
+                                 float scale, float *__restrict__ y, long long total, int C, int HW) {
+  pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  if ((HW & 15) == 0) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < total / 16; v += stride) {
+      const long long e = v * 16;
+      const int c = (int)((e / HW) % C);
+      const float m = mean[c];
+      const uint4 raw = __ldg((const uint4 *)(px + e));
+      const uint32_t w[4] = {raw.x, raw.y, raw.z, raw.w};
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        float4 o;
+        o.x = ((float)(w[q] & 0xFF) - m) * scale;
+        o.y = ((float)((w[q] >> 8) & 0xFF) - m) * scale;
+        o.z = ((float)((w[q] >> 16) & 0xFF) - m) * scale;
+        o.w = ((float)(w[q] >> 24) - m) * scale;
+        *(float4 *)(y + e + 4 * q) = o;
+      }
+    }
+    return;
+  }
+  for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < total; e += stride)
+    y[e] = ((float)px[e] - mean[(e / HW) % C]) * scale;
+}
+
+cudaError_t launch_pixels_u8(const unsigned char *px, const float *mean, float scale, float *y,
+                             int B, int C, int HW, cudaStream_t s) {
+  const long long total = (long long)B * C * HW;
+  const long long work = (HW & 15) == 0 ? total / 16 : total;
+  const int grid = (int)std::max<long long>(1, std::min<long long>((work + 255) / 256, 148LL * 8));
+  launch_pdl(pixels_u8_kernel, dim3(grid), dim3(256), 0, s, px, mean, scale, y, total, C, HW);
+  return cudaGetLastError();
+}
+
 // final NHWC storage -> NCHW fp32 flatten (C,H,W order, reading R5)
 __global__ void unstage_output_kernel(const void *x, int st, float *y, int B,
                                       int C, int H, int W, int Cs) {

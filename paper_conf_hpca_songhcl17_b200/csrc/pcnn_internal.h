@@ -226,6 +226,9 @@ struct FcPlan {
   double unit_us; // modelled time of one split of one unit on its CTA pair
 };
 int fc_stage_count(int nb);
+// uint8 NCHW pixels -> fp32 network input (pixel - mean[c]) * scale
+cudaError_t launch_pixels_u8(const unsigned char *px, const float *mean, float scale, float *y,
+                             int B, int C, int HW, cudaStream_t s);
 cudaError_t fc_profile(int reset, unsigned long long out[16]);   // debug timeline (prof build)
 // tmap_w: 4-D map of the re-tiled weights [RB][KB][128][128 B] (box = one
 // 16 KB tile, SW128); tmap_x: tiled map of the input [B][K] (box 128 B x

@@ -170,6 +170,8 @@ struct pcnn_net {
   void *d_act[3] = {nullptr, nullptr, nullptr};
   float *d_host_in = nullptr, *d_host_out = nullptr, *d_host_p = nullptr,
         *d_host_h = nullptr;
+  unsigned char *d_host_u8 = nullptr;   // pcnn_infer_host_u8 pixels
+  float *d_mean = nullptr;              // per-channel mean (C floats)
   // pcnn_infer_host pipelining: host->device copies of later chunks on their
   // own stream while earlier chunks compute
   cudaStream_t copy_stream = nullptr;
@@ -1759,6 +1761,8 @@ pcnn_status pcnn_destroy_net(pcnn_net *net) {
   for (auto &e : net->ev_copy)
     if (e) cudaEventDestroy(e);
   if (net->d_host_in) cudaFree(net->d_host_in);
+  if (net->d_host_u8) cudaFree(net->d_host_u8);
+  if (net->d_mean) cudaFree(net->d_mean);
   if (net->d_host_out) cudaFree(net->d_host_out);
   if (net->d_host_p) cudaFree(net->d_host_p);
   if (net->d_host_h) cudaFree(net->d_host_h);
@@ -2155,13 +2159,20 @@ pcnn_status pcnn_infer(pcnn_net *net, const float *d_images, int batch, float *d
   return PCNN_OK;
 }
 
-pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch, float *h_out,
-                            float *h_probs, float *h_entropy, void *stream) {
-  if (!net || !h_images || !h_out) return fail(PCNN_ERR_INVALID_ARGUMENT, "null pointer");
+// pcnn_infer_host / pcnn_infer_host_u8: host images (fp32, or uint8 pixels
+// converted on the device) -> library device buffers -> pcnn_infer, chunked
+// so that the host->device copies overlap inference when they dominate.
+static pcnn_status infer_host_impl(pcnn_net *net, const float *h_images,
+                                   const unsigned char *h_pixels, const float *mean, float scale,
+                                   int batch, float *h_out, float *h_probs, float *h_entropy,
+                                   void *stream) {
+  if (!net || !(h_images || h_pixels) || !h_out)
+    return fail(PCNN_ERR_INVALID_ARGUMENT, "null pointer");
   if (batch <= 0 || batch > net->desc.max_batch)
     return fail(PCNN_ERR_BATCH_TOO_LARGE, "bad batch");
   CUDA_TRY(cudaSetDevice(net->device));
-  const size_t in_elems = (size_t)net->desc.in_channels * net->desc.in_height * net->desc.in_width;
+  const int C = net->desc.in_channels;
+  const size_t in_elems = (size_t)C * net->desc.in_height * net->desc.in_width;
   const size_t maxb = net->desc.max_batch;
   if (!net->d_host_in) {
     CUDA_TRY(cudaMalloc(&net->d_host_in, sizeof(float) * in_elems * maxb));
@@ -2170,14 +2181,25 @@ pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch, flo
     CUDA_TRY(cudaMalloc(&net->d_host_h, sizeof(float) * maxb));
   }
   cudaStream_t s = (cudaStream_t)stream;
-  // When the images take much longer to cross PCIe (~50 GB/s) than to infer
-  // (FLOPs at ~700 TFLOP/s), split the batch into 4 chunks: chunk i+1's
-  // host->device copy (own stream) overlaps chunk i's inference.  Images are
-  // independent, so the chunks compute the same per-image results.
+  const bool u8 = h_pixels != nullptr;
+  if (u8) {
+    if (!net->d_host_u8) {
+      CUDA_TRY(cudaMalloc(&net->d_host_u8, in_elems * maxb));
+      CUDA_TRY(cudaMalloc(&net->d_mean, sizeof(float) * C));
+    }
+    std::vector<float> m(C, 0.f);
+    if (mean) m.assign(mean, mean + C);
+    CUDA_TRY(cudaMemcpyAsync(net->d_mean, m.data(), sizeof(float) * C, cudaMemcpyHostToDevice, s));
+  }
+  const size_t in_bytes = u8 ? 1 : sizeof(float);
+  // When the images take long to cross PCIe (~50 GB/s) compared with the
+  // inference (FLOPs at ~700 TFLOP/s), split the batch into 4 chunks: chunk
+  // i+1's host->device copy (own stream) overlaps chunk i's inference.
+  // Images are independent, so the chunks compute the same per-image results.
   double flops = 0;
   for (auto &ly : net->layers) flops += layer_flops_exact(ly, 1);
-  const double h2d_img = sizeof(float) * in_elems / 50e9, comp_img = flops / 7e14;
-  const int k = (batch >= 64 && h2d_img > 2.0 * comp_img) ? 4 : 1;
+  const double h2d_img = in_bytes * in_elems / 50e9, comp_img = flops / 7e14;
+  const int k = (batch >= 64 && h2d_img > (u8 ? 0.25 : 2.0) * comp_img) ? 4 : 1;
   const int chunk = (batch + k - 1) / k;
   if (k > 1 && !net->copy_stream) {
     CUDA_TRY(cudaStreamCreateWithFlags(&net->copy_stream, cudaStreamNonBlocking));
@@ -2189,14 +2211,22 @@ pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch, flo
   }
   for (int c = 0, b0 = 0; b0 < batch; ++c, b0 += chunk) {
     const int nb = std::min(chunk, batch - b0);
-    CUDA_TRY(cudaMemcpyAsync(net->d_host_in + (size_t)b0 * in_elems, h_images + (size_t)b0 * in_elems,
-                             sizeof(float) * in_elems * nb, cudaMemcpyHostToDevice,
-                             k > 1 ? net->copy_stream : s));
+    if (u8)
+      CUDA_TRY(cudaMemcpyAsync(net->d_host_u8 + (size_t)b0 * in_elems, h_pixels + (size_t)b0 * in_elems,
+                               in_elems * nb, cudaMemcpyHostToDevice, k > 1 ? net->copy_stream : s));
+    else
+      CUDA_TRY(cudaMemcpyAsync(net->d_host_in + (size_t)b0 * in_elems, h_images + (size_t)b0 * in_elems,
+                               sizeof(float) * in_elems * nb, cudaMemcpyHostToDevice,
+                               k > 1 ? net->copy_stream : s));
     if (k > 1) CUDA_TRY(cudaEventRecord(net->ev_copy[c], net->copy_stream));
   }
   for (int c = 0, b0 = 0; b0 < batch; ++c, b0 += chunk) {
     const int nb = std::min(chunk, batch - b0);
     if (k > 1) CUDA_TRY(cudaStreamWaitEvent(s, net->ev_copy[c], 0));
+    if (u8)
+      CUDA_TRY(counted(launch_pixels_u8(net->d_host_u8 + (size_t)b0 * in_elems, net->d_mean, scale,
+                                        net->d_host_in + (size_t)b0 * in_elems, nb, C,
+                                        (int)(in_elems / C), s)));
     const size_t oo = (size_t)b0 * net->out_elems;
     pcnn_status r = pcnn_infer(net, net->d_host_in + (size_t)b0 * in_elems, nb,
                                net->d_host_out + oo, h_probs ? net->d_host_p + oo : nullptr,
@@ -2213,6 +2243,20 @@ pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch, flo
   }
   CUDA_TRY(cudaStreamSynchronize(s));
   return PCNN_OK;
+}
+
+pcnn_status pcnn_infer_host(pcnn_net *net, const float *h_images, int batch, float *h_out,
+                            float *h_probs, float *h_entropy, void *stream) {
+  return infer_host_impl(net, h_images, nullptr, nullptr, 1.f, batch, h_out, h_probs, h_entropy,
+                         stream);
+}
+
+pcnn_status pcnn_infer_host_u8(pcnn_net *net, const unsigned char *h_pixels, const float *mean,
+                               float scale, int batch, float *h_out, float *h_probs,
+                               float *h_entropy, void *stream) {
+  if (!h_pixels) return fail(PCNN_ERR_INVALID_ARGUMENT, "null pointer");
+  return infer_host_impl(net, nullptr, h_pixels, mean, scale, batch, h_out, h_probs, h_entropy,
+                         stream);
 }
 
 pcnn_status pcnn_profile_layers(pcnn_net *net, const float *d_images, int batch, float *d_out,

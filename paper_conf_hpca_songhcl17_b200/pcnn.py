@@ -92,6 +92,7 @@ _lib.pcnn_set_layer_plan.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_in
 _lib.pcnn_set_perforation.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.c_int]
 _lib.pcnn_infer.argtypes = [_P, _P, ctypes.c_int, _P, _P, _P, _P]
 _lib.pcnn_infer_host.argtypes = [_P, _P, ctypes.c_int, _P, _P, _P, _P]
+_lib.pcnn_infer_host_u8.argtypes = [_P, _P, _P, ctypes.c_float, ctypes.c_int, _P, _P, _P, _P]
 _lib.pcnn_output_size.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.pcnn_num_layers.argtypes = [_P, ctypes.POINTER(ctypes.c_int)]
 _lib.pcnn_query_layer.argtypes = [_P, ctypes.c_int, ctypes.c_int, ctypes.POINTER(LayerInfo)]
@@ -114,7 +115,7 @@ _lib.pcnn_status_string.restype = ctypes.c_char_p
 _lib.pcnn_last_error_message.restype = ctypes.c_char_p
 for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
            "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_layer_plan",
-           "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
+           "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_infer_host_u8", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
            "pcnn_model_layer_time", "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
            "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
            "pcnn_last_launch_count"):
@@ -122,7 +123,7 @@ for _f in ("pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
 
 EXPORTED = ["pcnn_create_net", "pcnn_destroy_net", "pcnn_set_variant",
             "pcnn_set_variant_factors", "pcnn_set_sm_budget", "pcnn_set_layer_plan",
-            "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
+            "pcnn_set_perforation", "pcnn_infer", "pcnn_infer_host", "pcnn_infer_host_u8", "pcnn_output_size", "pcnn_num_layers", "pcnn_query_layer", "pcnn_plan_budget",
             "pcnn_model_layer_time", "pcnn_describe_net", "pcnn_profile_layers", "pcnn_enable_sm_census",
             "pcnn_get_sm_census", "pcnn_set_layer_timing", "pcnn_read_layer_timing",
             "pcnn_last_launch_count", "pcnn_device_sm_count", "pcnn_version",
@@ -285,6 +286,19 @@ class Net:
         B = images.shape[0]
         _check(_lib.pcnn_infer_host(self._h, _ptr(images), B, _ptr(out), _ptr(probs),
                                     _ptr(entropy), _stream_ptr(stream)), "pcnn_infer_host")
+        return out
+
+    def infer_host_u8(self, pixels, out, mean=None, scale=1.0, probs=None, entropy=None,
+                      stream=None):
+        """pixels: CPU uint8 tensor [B][C][H][W] (pinned for speed); the network
+        input is (pixel - mean[c]) * scale, converted on the device."""
+        B = pixels.shape[0]
+        m = None
+        if mean is not None:
+            m = (ctypes.c_float * len(mean))(*[float(v) for v in mean])
+        _check(_lib.pcnn_infer_host_u8(self._h, _ptr(pixels), m, ctypes.c_float(scale), B,
+                                       _ptr(out), _ptr(probs), _ptr(entropy),
+                                       _stream_ptr(stream)), "pcnn_infer_host_u8")
         return out
 
     def query_layer(self, layer, batch):

@@ -12,13 +12,13 @@ FC or softmax, and no output-size formulas).  It only defines
 Both ``oracle/`` and ``paper_conf_hpca_songhcl17_b200/`` consume these plain
 arrays; neither imports the other.
 """
-from .rng import (counter_u64, uniform, normal, round_to_bf16, images,
+from .rng import (counter_u64, uniform, normal, round_to_bf16, images, pixels,
                   he_weights, biases, net_params, IMAGE_TENSOR_ID,
                   WEIGHT_SEED, IMAGE_SEED, prototypes, planted_images)
 from .nets import NETS, alexnet, vgg16, cifar_quick, weight_shapes, get_net
 
 __all__ = [
-    "counter_u64", "uniform", "normal", "round_to_bf16", "images", "he_weights",
+    "counter_u64", "uniform", "normal", "round_to_bf16", "images", "pixels", "he_weights",
     "biases", "net_params", "IMAGE_TENSOR_ID", "WEIGHT_SEED", "IMAGE_SEED",
     "NETS", "alexnet", "vgg16", "cifar_quick", "weight_shapes", "get_net",
     "prototypes", "planted_images",

@@ -79,6 +79,15 @@ def images(n_start, count, shape, seed=IMAGE_SEED, lo=-128.0, hi=128.0, bf16=Tru
     return round_to_bf16(v).reshape((count,) + tuple(shape))
 
 
+def pixels(n_start, count, shape, seed=IMAGE_SEED):
+    """8-bit images [count, C, H, W] uint8, uniform over 0..255: the pixels'
+    native format (pcnn_infer_host_u8).  Same counters as ``images``, so
+    ``pixels - 128`` is an integer-valued image on Caffe's ±128 scale."""
+    per = int(np.prod(shape))
+    v = uniform(seed, IMAGE_TENSOR_ID, n_start * per, count * per, 0.0, 256.0)
+    return np.minimum(np.floor(v), 255).astype(np.uint8).reshape((count,) + tuple(shape))
+
+
 def he_weights(shape, fan_in, layer_index, seed=WEIGHT_SEED, bf16=True):
     """He-normal N(0, 2/fan_in), BF16-representable float32 (bf16=False: full
     FP32 values)."""

@@ -25,7 +25,7 @@ def _declared_symbols():
     with open(os.path.join(ROOT, "include", "pcnn.h")) as f:
         src = f.read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"\b(pcnn_[a-z_]+)\s*\(", src)))
+    return sorted(set(re.findall(r"\b(pcnn_[a-z0-9_]+)\s*\(", src)))
 
 
 def test_every_declared_symbol_is_exported(pcnn):

@@ -311,6 +311,35 @@ def test_infer_host_pipelined_chunks(orc):
     assert np.isfinite(hh.numpy()).all() and (hh.numpy() >= 0).all()
 
 
+@pytest.mark.parametrize("name,B", [("alexnet", 64), ("tiny", 3)])
+def test_infer_host_u8_equals_device_call(orc, name, B):
+    """pcnn_infer_host_u8 (8-bit pixels over PCIe, (pixel - mean) * scale on
+    the device): bitwise the device call on the converted float images.
+    AlexNet B = 64 takes the pipelined 4-chunk path and the 16-pixel vector
+    conversion; the tiny net (H*W = 63) the scalar conversion."""
+    import torch
+    from paper_conf_hpca_songhcl17_b200 import pcnn
+    if name == "alexnet":
+        net = synth.alexnet()
+        mean, scale = [128.0, 117.0, 104.0], 1.0
+    else:
+        net = dict(in_shape=(3, 9, 7), layers=[conv_layer(16, 3, 3, 1, 1, 1, relu=True)])
+        mean, scale = [120.5, 100.25, 90.0], 0.5
+    w, b = params(net)
+    px = synth.pixels(0, B, net["in_shape"])
+    x = ((px.astype(np.float32) - np.array(mean, np.float32)[None, :, None, None]) *
+         np.float32(scale)).astype(np.float32)
+    n = pcnn.Net(net, w, b, B, "bf16")
+    dev, _, _ = n.infer(torch.from_numpy(x).cuda())
+    torch.cuda.synchronize()
+    ph = torch.from_numpy(px).pin_memory()
+    oh = torch.empty(tuple(dev.shape)).pin_memory()
+    n.infer_host_u8(ph, oh, mean=mean, scale=scale)
+    np.testing.assert_array_equal(oh.numpy(), dev.cpu().numpy())
+    ref = orc.run_net(net, w, b, x[:2]).reshape(2, -1)
+    assert rel_err(oh.numpy()[:2].reshape(2, -1), ref) <= TOL["bf16"]
+
+
 # ------------------------------------------------------------ bench configurations, full size
 @pytest.mark.parametrize("name,B,samples", [("alexnet", 256, (0, 131, 255)), ("vgg16", 64, (0, 63))])
 def test_bench_workload_sampled_parity(orc, name, B, samples):
