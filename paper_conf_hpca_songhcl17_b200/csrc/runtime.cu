@@ -914,6 +914,10 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
         if (t >= device_sms / cg) can_fill = true;
       }
   const int max_split = (can_fill || full_n || g.pm != 1) ? 1 : std::min(16, nj);
+  static const int force_split = [] {              // tuning experiments
+    const char *e = exp_env("PCNN_FORCE_SPLIT");
+    return e ? atoi(e) : 0;
+  }();
   const double hbm = 6.0e12;
   for (int ms = 1; ms <= 2; ++ms) {
     if (force_ms && atoi(force_ms) != ms) continue;
@@ -947,6 +951,7 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
           const int kbs = (nj + want - 1) / want;
           const int splits = (nj + kbs - 1) / kbs;
           if (splits != want) continue;
+          if (force_split > 0 && splits != force_split && max_split >= force_split) continue;
           const long long units = tiles * splits;
           const long long waves = (units + slots - 1) / slots;
           double t = (double)waves * kbs * j_cycles / f + 2e-6 * ms;
