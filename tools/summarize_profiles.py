@@ -100,4 +100,30 @@ if os.path.exists(full):
         "source": "ncu --set full --clock-control none (one capture of each kernel)"}
     json.dump(allj, open(js, "w"), indent=1)
     summary["ncu_full_alexnet_b256"] = out
+other = os.path.join(RAW, "full_alexnet_b256_other_%s.ncu-rep" % RND)
+if os.path.exists(other):
+    # memory-bound kernels (LRN + pool, staging, pooling, softmax): DRAM bytes
+    # and throughput, issue activity and occupancy
+    raw = subprocess.run(["ncu", "-i", other, "--page", "raw", "--csv"], capture_output=True,
+                         text=True).stdout.splitlines()
+    rows = list(csv.reader(raw))
+    h = rows[0]
+    keys = ["Kernel Name", "Grid Size", "gpu__time_duration.sum", "dram__bytes_read.sum",
+            "dram__bytes_write.sum", "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
+            "sm__inst_issued.avg.pct_of_peak_sustained_active",
+            "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread"]
+    idx = [h.index(k) if k in h else -1 for k in keys]
+    units = [rows[1][i] if i >= 0 else "" for i in idx]
+    with open(os.path.join(OUT, "%s_ncu_full_alexnet_b256_other.csv" % RND), "w") as f:
+        f.write("kernel,grid,dur_us,dram_bytes,dram_pct,issue_active_pct,warps_active_pct,regs\n")
+        for r in rows[2:]:
+            d = {k: (r[i] if i >= 0 else "0") for k, i in zip(keys, idx)}
+            mb = lambda x: float(x) * (1e6 if "Mbyte" in units[3] else 1e9 if "Gbyte" in units[3] else 1e3)
+            f.write("%s,\"%s\",%.2f,%d,%.1f,%.1f,%.1f,%d\n" % (
+                short(d["Kernel Name"]), d["Grid Size"], float(d["gpu__time_duration.sum"]),
+                int(mb(d["dram__bytes_read.sum"]) + mb(d["dram__bytes_write.sum"])),
+                float(d["gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"]),
+                float(d["sm__inst_issued.avg.pct_of_peak_sustained_active"]),
+                float(d["sm__warps_active.avg.pct_of_peak_sustained_active"]),
+                int(float(d["launch__registers_per_thread"]))))
 print(json.dumps(summary, indent=1))
