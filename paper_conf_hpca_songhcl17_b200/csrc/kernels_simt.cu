@@ -649,8 +649,14 @@ constexpr long long kBandTargetCtas = 2 * 148;
 // pixel reads its 4 x 3 row segments as 16 B vectors (re-aligned by the row's
 // start offset), permutes them into the (dr, ds, c) channel order and writes
 // the whole pixel (Cs channels, zero padded) with 16 B stores.
+#ifndef PCNN_S2D_MINB
+#define PCNN_S2D_MINB 1
+#endif
+#ifndef PCNN_S2D_ROWS_DEFAULT
+#define PCNN_S2D_ROWS_DEFAULT 4
+#endif
 template <int ST>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(256, PCNN_S2D_MINB)
 stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Hs, int Ws,
                   int Cs, int R, int tf32_round) {
   pdl_enter();   // PDL: wait for the previous kernel, let the next one launch
@@ -743,7 +749,7 @@ static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int
                                      int Hs, int Ws, int Cs, int tf32_round, cudaStream_t s) {
   static const int R3 = [] {                         // staged rows per band
     const char *e = exp_env("PCNN_S2D_ROWS");
-    return e && atoi(e) > 0 ? atoi(e) : 3;
+    return e && atoi(e) > 0 ? atoi(e) : PCNN_S2D_ROWS_DEFAULT;
   }();
   int R = R3;                                        // small batches: shorter bands
   while (R > 1 && (long long)B * ((Hs + R - 1) / R) < kBandTargetCtas) --R;
