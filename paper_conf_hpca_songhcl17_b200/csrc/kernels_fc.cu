@@ -33,8 +33,9 @@
 // PDL: the weights do not depend on the previous layer, so the producer
 // streams the first ring of weight tiles before griddepcontrol.wait.
 //
-// CTA = 6 warps: warp 0 TMA producer, warp 1 TMEM allocator + MMA issuer
-// (leader CTA), warps 2..5 epilogue / reduction (TMEM lane quarter = warp % 4).
+// CTA = 10 warps: warp 0 TMA producer, warp 1 TMEM allocator + MMA issuer
+// (leader CTA), warps 2..9 epilogue / reduction (TMEM lane quarter = warp % 4,
+// two warps per quarter taking alternate 32-column chunks).
 #include <algorithm>
 
 #include "budget.cuh"
@@ -43,7 +44,8 @@
 
 namespace pcnn {
 
-constexpr int FC_THREADS = 192;
+constexpr int FC_THREADS = 320;        // producer, MMA, 8 epilogue / reduction warps
+constexpr int FC_EPI = FC_THREADS - 64; // epilogue threads
 constexpr int FC_STAGE_BUDGET = 200 * 1024;
 constexpr int FC_MAX_STAGES = 16;
 constexpr int FC_W_TILE = 128 * 128;          // one weight tile: 128 rows x 128 B
@@ -110,8 +112,8 @@ __device__ __forceinline__ void fc_store(void *y, size_t idx, float v, int out_m
   }
 }
 
-__device__ __forceinline__ void epi_bar() {          // the 4 epilogue warps only
-  asm volatile("bar.sync 1, 128;" ::: "memory");
+__device__ __forceinline__ void epi_bar() {          // the 8 epilogue warps only
+  asm volatile("bar.sync 1, %0;" ::"n"(FC_EPI) : "memory");
 }
 __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
   unsigned v;
@@ -122,17 +124,17 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
 // Split-K reduction of one unit by CTA `idx` (0 .. 2s-1) of the unit: rows
 // [idx * 256 / (2s), ...) for every image of the chunk, each output the sum of
 // the s partials in split order 0..s-1 (+ bias, activation, rounding).  Four
-// consecutive rows per thread (16-B loads); the partials of 16 / s images are
+// consecutive rows per thread (16-B loads); the partials of 8 / s images are
 // all in flight before the first add (the loads are L2-latency bound).
 template <int S>
 __device__ __forceinline__ void fc_reduce(const FcArgs &a, int rb, int ch, int idx, int t) {
   constexpr int s = S, rows = FC_ROWS / (2 * S);
-  constexpr int IMG = S >= 16 ? 1 : 16 / S;
+  constexpr int IMG = S >= 8 ? 1 : 8 / S;
   const int b0 = ch * a.nb, ncols = min(a.nb, a.B - b0);
   const size_t sBN = (size_t)a.B * a.N;
   const int nbase = rb * FC_ROWS + idx * rows;
   if ((a.N & 3) == 0) {
-    constexpr int r4 = rows / 4, bstep = 128 / r4;
+    constexpr int r4 = rows / 4, bstep = FC_EPI / r4;
     const int q = t % r4, bsub = t / r4;
     const int n = nbase + 4 * q;
     if (bsub >= bstep || n >= a.N) return;
@@ -170,7 +172,7 @@ __device__ __forceinline__ void fc_reduce(const FcArgs &a, int rb, int ch, int i
     }
     return;
   }
-  for (int e = t; e < rows * ncols; e += 128) {          // general N: one output per step
+  for (int e = t; e < rows * ncols; e += FC_EPI) {       // general N: one output per step
     const int r = e % rows, bi = e / rows;
     const int n = nbase + r;
     if (n >= a.N) continue;
@@ -211,7 +213,7 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
       mbar_init(sbase + FC_SM_EMPTY + 8 * i, 1);
     }
     mbar_init(sbase + FC_SM_TFULL, 1);
-    mbar_init(sbase + FC_SM_TEMPTY, 8);                    // epilogue warps of both CTAs
+    mbar_init(sbase + FC_SM_TEMPTY, 2 * (FC_EPI / 32));     // epilogue warps of both CTAs
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     census_mark(a.b);
   }
@@ -296,7 +298,8 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
       }
     } else {
       // ------------------------------------------------ epilogue: TMEM -> y / partials
-      const int q = warp & 3;
+      // two warps per TMEM lane quarter (warp % 4), alternating 32-column chunks
+      const int q = warp & 3, half = (warp - 2) >> 2;
       mbar_wait(sbase + FC_SM_TFULL, lt & 1);
       tc_fence_after();
       if (prof && t_full == 0) t_full = fc_gtimer();
@@ -306,7 +309,7 @@ fc_tc_kernel(const __grid_constant__ CUtensorMap tmap_w, const __grid_constant__
       const int n = rb * FC_ROWS + (int)rank * 128 + q * 32 + lane;
       const bool nok = n < a.N;
       const float bias = (!partial && nok) ? __ldg(&a.bias[n]) : 0.f;
-      for (int c0 = 0; c0 < ncols; c0 += 32) {                 // warp-uniform
+      for (int c0 = 32 * half; c0 < ncols; c0 += 64) {         // warp-uniform
         uint32_t v[32];
         tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + c0, v);
         tmem_ld_wait();
