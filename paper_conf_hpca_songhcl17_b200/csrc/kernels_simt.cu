@@ -1370,6 +1370,8 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
   constexpr int HALF = 2;                      // LRN size 5
   constexpr bool SWZ = CPT == 8;
   const int C = a.C, chunks = C / VN, P = chunks / CPT;
+  const int lp = __ffs(P) - 1;                 // P is a power of two (lrn_reg_cpt)
+  const float inv_w = 1.f / (float)a.W;
   const long long tiles = (long long)a.B * a.nbands;
   const int Hp = a.H + a.hi, Wp = a.W + a.hi;             // shared-halo grids
   const int Hop = a.Ho + a.ho, Wop = a.Wo + a.ho;
@@ -1403,9 +1405,10 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
     // the next item's chunks are loaded before the current one is normalised,
     // so every thread keeps two items' global loads in flight
     auto load_item = [&](int v, uint4 (&raw)[CPT]) {
-      const int pix = v / P, part = v - pix * P;
+      const int pix = v >> lp, part = v & (P - 1);
       if (pix < npix) {
-        const int r = pix / a.W, col = pix - r * a.W;
+        int r, col;
+        fdivmod(pix, a.W, inv_w, r, col);           // pix < 2^22, W <= 1024: exact
         const char *src = (const char *)a.x +
             ((((size_t)n * Hp + h0 + r) * Wp + col) * C + (size_t)part * CPT * VN) * ESZ;
 #pragma unroll
@@ -1418,7 +1421,7 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
     uint4 nraw[CPT];
     if ((int)threadIdx.x < nv) load_item(threadIdx.x, nraw);
     for (int v = threadIdx.x; v < nv; v += blockDim.x) {
-      const int pix = v / P, part = v - pix * P;
+      const int pix = v >> lp, part = v & (P - 1);
       const bool ok = pix < npix;
       Vec16<ST> ch[CPT];
 #pragma unroll
@@ -1460,6 +1463,7 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
     const int ochunks = a.Cout / VN;
     const float inv_oc = 1.f / (float)ochunks;
     const int grp_real = a.ocg / VN, grp_pad = a.ocp / VN;
+    const float inv_gp = grp_pad > 0 ? 1.f / (float)grp_pad : 0.f;
     const int nq = a.Wo * ochunks;
     const float inv_nq = 1.f / (float)nq;
     for (int v = threadIdx.x; v < (p1 - p0) * nq; v += blockDim.x) {
@@ -1471,7 +1475,8 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
       int c = oc;
       bool pad = false;
       if (grp_pad > 0) {
-        const int gi = oc / grp_pad, j = oc - gi * grp_pad;
+        int gi, j;
+        fdivmod(oc, grp_pad, inv_gp, gi, j);
         pad = j >= grp_real;
         c = gi * grp_real + j;
       }
@@ -1546,7 +1551,8 @@ static int lrn_reg_cpt(int st, int C) {
 constexpr int LB_SMEM_BUDGET = 100 * 1024;
 
 // output rows per band so that the band's staged rows fit LB_SMEM_BUDGET
-static bool use_lrn_reg(int st, int C, int lrn) {
+static bool use_lrn_reg(int st, int C, int lrn, int W) {
+  if (W > 1024) return false;                    // fdivmod's exact range (pixel -> row, col)
   const char *e = exp_env("PCNN_LRN_BAND");     // A/B tests: the staged band kernel
   const bool off = e && e[0] == '1';
   return lrn == 5 && !off && lrn_reg_cpt(st, C) > 0;
@@ -1556,7 +1562,7 @@ static bool use_lrn_reg(int st, int C, int lrn) {
 // bands overlap by k - s input rows, recomputed; results do not depend on R).
 static int lrn_band_rows(int st, int B, int W, int C, int k, int s, int Ho, int lrn) {
   const int esz = st == ST_BF16 ? 2 : 4;
-  const size_t row = (size_t)W * (C * esz + (use_lrn_reg(st, C, lrn) ? 0 : 16));
+  const size_t row = (size_t)W * (C * esz + (use_lrn_reg(st, C, lrn, W) ? 0 : 16));
   const char *e = exp_env("PCNN_LB_KB");          // tuning experiments
   const size_t budget = e ? (size_t)atoi(e) * 1024 : (size_t)LB_SMEM_BUDGET;
   int R = 1;
@@ -1754,7 +1760,7 @@ cudaError_t launch_lrn_pool(const void *x, void *y, int st, int tf32_round, int 
   a.ho = out_halo;
   a.b = b;
   const int esz = st == ST_BF16 ? 2 : 4;
-  if (use_lrn_reg(st, C, lrn_size)) {
+  if (use_lrn_reg(st, C, lrn_size, W)) {
     a.R = lrn_band_rows(st, B, W, C, k, s, Ho, lrn_size);
     a.nbands = (Ho + a.R - 1) / a.R;
     const size_t smem = (size_t)(min((a.R - 1) * s + k, H)) * W * C * esz;
