@@ -107,8 +107,11 @@ typedef enum {
     PCNN_FLAG_NARROW_SLABS = 16,        /* grouped convs with channels per
                                            group not a multiple of 128 B keep
                                            them unpadded (SW64 / SW32 slabs) */
-    PCNN_FLAG_PERFORATION_IM2COL = 32   /* row perforation of padded-layout
+    PCNN_FLAG_PERFORATION_IM2COL = 32,  /* row perforation of padded-layout
                                            layers in im2col mode (NEXT-1)    */
+    PCNN_FLAG_PER_ROW_WINDOWS = 64      /* padded-layout convs load one A
+                                           window per filter row (never one
+                                           whole-slab window for all taps)   */
 } pcnn_net_flag;
 
 typedef struct {
@@ -159,6 +162,10 @@ typedef struct {
     double t_unit_us;   /* modelled time of one work unit (tile, or one split
                            of an FC unit) on its cta_group SMs (eq. 12 per
                            wave); non-GEMM layers: 0                          */
+    int whole_window;   /* a_mode 2 only: 1 = one TMA window of 128 + (S-1) x
+                           (grid width + 1) rows per channel slab feeds all
+                           S x S taps (fewer A bytes for narrow grids), 0 =
+                           one window per filter row                          */
 } pcnn_layer_info;
 
 /* Resource + time model of one layer, for the

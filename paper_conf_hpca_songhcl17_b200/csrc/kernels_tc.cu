@@ -88,19 +88,24 @@ int tc_block_k_elems(int st) { return st == ST_BF16 ? 64 : 32; }
 // rows from one sub-tile's window to the next: a whole number of 8-row
 // swizzle atoms, so every window starts swizzle-aligned
 __host__ __device__ constexpr int pm_sub_rows(int S) { return (TC_BM + S - 1 + 7) / 8 * 8; }
-static int pm_a_stage_bytes(int slab_bytes, int S, int msub) {
-  return ((msub - 1) * pm_sub_rows(S) * slab_bytes + (TC_BM + S - 1) * slab_bytes + 1023) /
-         1024 * 1024;
+// A window rows per sub-tile: per filter row (ww = 0) or whole (ww = 1)
+int pm_window_rows(int S, int wv, int ww) { return ww ? TC_BM + (S - 1) * (wv + 1) : TC_BM + S - 1; }
+static int pm_a_stage_bytes(int slab_bytes, int rows, int msub) {
+  const int sub = (rows + 7) / 8 * 8;
+  return ((msub - 1) * sub * slab_bytes + rows * slab_bytes + 1023) / 1024 * 1024;
 }
-void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages, int *b_stages) {
-  const int as_bytes = pm_a_stage_bytes(slab_bytes, S, msub);
+void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages, int *b_stages,
+                  int rows, int ww) {
+  const int as_bytes = pm_a_stage_bytes(slab_bytes, rows, msub);
   const int bs_bytes = bn / cg * slab_bytes;
   // 128 B slabs keep the tuned ring depths (4 windows, 12 tap slabs); narrow
-  // slabs carry 2-4x less work per stage and get deeper rings
+  // slabs carry 2-4x less work per stage and get deeper rings.  Whole windows
+  // keep >= 8 tap slabs in flight (a window's S*S slabs stream through them).
   int na = slab_bytes == 128 ? 4 : TC_MAX_ASTAGES;
-  while (na > 2 && na * as_bytes + 2 * S * bs_bytes > TC_STAGE_BUDGET) --na;
+  const int bmin = ww ? 8 : 2 * S;
+  while (na > 2 && na * as_bytes + bmin * bs_bytes > TC_STAGE_BUDGET) --na;
   int nb = (TC_STAGE_BUDGET - na * as_bytes) / bs_bytes;
-  const int nb_max = slab_bytes == 128 ? TC_MAX_STAGES : TC_MAX_BSTAGES;
+  const int nb_max = slab_bytes == 128 && !ww ? TC_MAX_STAGES : TC_MAX_BSTAGES;
   if (nb > nb_max) nb = nb_max;
   *a_stages = na;
   *b_stages = nb;
@@ -145,6 +150,12 @@ struct TcArgs {
   int prof;             // 1: accumulate per-role barrier-wait cycles (debug)
   int skip;             // debug: 1 skip A loads, 2 skip B loads, 4 skip MMAs
   int a_stages, b_stages, pm_a_stage;   // padded mode rings (g.pm)
+  // padded mode, whole windows (ww = 1): ONE A window of pm_rows = 128 +
+  // (S-1)(wv+1) rows per channel slab feeds all S x S taps (tap (r, s) = a
+  // descriptor shift of r*wv + s rows) instead of one (128 + S - 1)-row
+  // window per filter row; pm_sub = rows from one M sub-tile's window to the
+  // next in the A stage (a whole number of 8-row swizzle atoms)
+  int ww, pm_rows, pm_sub;
   int msub;             // padded mode: M sub-tiles of 128 rows per CTA sharing each B slab
   // TMEM accumulator ring: nbuf buffers of tbw columns (512 / tbw), sub-tile
   // sb at column tsub * sb of its buffer.  Narrow tiles get up to 8 buffers,
@@ -457,9 +468,10 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
   const uint64_t b_desc0 = umma_desc(sBp, SLAB);
   const uint32_t a_st16 = (uint32_t)a.pm_a_stage / 16, b_st16 = pm_b_bytes / 16;
   const int a_stages = a.a_stages, b_stages = a.b_stages, units = a.units, S = a.g.S;
-  const int j_last = nj - S, kmma_last = a.kmma_last;   // windows of the last channel slab
-  // sub-tile 1's window starts pm_sub_rows(S) rows into the A stage
-  const uint32_t sub16 = (uint32_t)pm_sub_rows(S) * ROW16;
+  const int ww = a.ww, taps = ww ? S * S : S, wv = a.g.wv;
+  const int j_last = ww ? nj - 1 : nj - S, kmma_last = a.kmma_last;   // windows of the last channel slab
+  // sub-tile 1's window starts pm_sub rows into the A stage
+  const uint32_t sub16 = (uint32_t)a.pm_sub * ROW16;
   const bool prof = TC_PROF(a) != 0, skip_mma = (a.skip & 4) != 0;
   const bool leader = elect_one();
   WaitClock wfull{prof}, wtemp{prof};
@@ -476,10 +488,11 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
       wfull.wait(sbase + SM_AFULL + 8 * as, aph);
       const uint64_t ad = a_desc0 + as * a_st16;
       const int kk = j >= j_last ? kmma_last : KMMA;
-      for (int s2 = 0; s2 < S; ++s2) {
+      for (int t = 0, r = 0, s2 = 0; t < taps; ++t) {
         wfull.wait(sbase + SM_FULL + 8 * bs, bph);
         tc_fence_after();
-        const uint64_t aw = ad + s2 * ROW16;
+        // tap (r, s2): the window shifted by r*wv + s2 rows (ww) or s2 rows
+        const uint64_t aw = ad + (uint32_t)(r * wv + s2) * ROW16;
         const uint64_t bd = b_desc0 + bs * b_st16;
         if (leader) {
           if (!skip_mma) {
@@ -487,7 +500,7 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
             for (int sb = 0; sb < MSUB; ++sb) {
               const uint64_t awb = aw + sb * sub16;
               const uint32_t dc = dcol + sb * a.tsub;
-              tc_mma<ST, CG>(dc, awb, bd, idesc, (j > j0 || s2 > 0) ? 1u : 0u);
+              tc_mma<ST, CG>(dc, awb, bd, idesc, (j > j0 || t > 0) ? 1u : 0u);
 #pragma unroll
               for (int k = 1; k < KMMA; ++k)
                 if (k < kk) tc_mma<ST, CG>(dc, awb + 2 * k, bd + 2 * k, idesc, 1u);
@@ -499,6 +512,10 @@ __device__ __forceinline__ void mma_issuer_pm(const TcArgs &a, uint32_t sbase, u
         if (++bs == (uint32_t)b_stages) {
           bs = 0;
           bph ^= 1;
+        }
+        if (++s2 == S) {
+          s2 = 0;
+          ++r;
         }
       }
       if (leader) tc_commit<CG>(sbase + SM_AEMPTY + 8 * as);
@@ -613,12 +630,14 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
     decode(pair, mt, nt, grp, sp);
     const int nrow = grp * g.Nfg + nt * a.bn + (int)rank * b_rows;
     if (g.pm) {
-      const int pm_se0 = slab_bytes / ESZ, nj = (g.Cg / pm_se0) * g.S;
+      const int pm_se0 = slab_bytes / ESZ, rw = a.ww ? g.S : 1;   // filter rows per window
+      const int nj = (g.Cg / pm_se0) * g.S / rw;
       const int j0 = sp * a.kb_per_split, j1 = min(nj, j0 + a.kb_per_split);
       for (int j = j0, n = 0; j < j1 && n < 64; ++j) {
-        const int cb = j / g.S, r = j - cb * g.S;
-        for (int s2 = 0; s2 < g.S; ++s2, ++n)
-          tma_prefetch_2d(&tmap_w, (r * g.S + s2) * g.Cg + cb * pm_se0, nrow);
+        const int cb = j * rw / g.S, r0 = j * rw - cb * g.S;
+        for (int r = r0; r < r0 + rw; ++r)
+          for (int s2 = 0; s2 < g.S; ++s2, ++n)
+            tma_prefetch_2d(&tmap_w, (r * g.S + s2) * g.Cg + cb * pm_se0, nrow);
       }
     } else {
       int k0, k1;
@@ -638,7 +657,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
   // padded mode: K runs over (channel slab cb, filter row r) windows, each
   // feeding the S taps (r, s) of that row by shifting the A descriptor s rows
   const int pm_se = slab_bytes / ESZ;                  // channels per slab
-  const int pm_nj = g.pm ? (g.Cg / pm_se) * g.S : 0;   // A windows per tile
+  const int pm_nj = g.pm ? (g.Cg / pm_se) * (a.ww ? 1 : g.S) : 0;   // A windows per tile
   const uint32_t sBp = sbase + (uint32_t)a.a_stages * (uint32_t)a.pm_a_stage;
   const uint32_t pm_b_bytes = (uint32_t)b_rows * slab_bytes;
   if (warp == 0 && g.pm) {
@@ -648,7 +667,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
       asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_x) : "memory");
       // pm = 2: nseg segments of wv + 2 pad columns (grid columns -pad ..)
       const uint32_t pm_a_bytes = g.pm == 2 ? (uint32_t)(g.nseg * (g.wv + 2 * g.pad)) * slab_bytes
-                                            : (uint32_t)(TC_BM + g.S - 1) * slab_bytes;
+                                            : (uint32_t)a.pm_rows * slab_bytes;
       uint32_t as = 0, aph = 0, bs = 0, bph = 0;
       WaitClock wc{TC_PROF(a) != 0};
       unsigned long long nkb = 0;
@@ -660,7 +679,7 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
         const int i0 = (mt * CG + (int)rank) * TC_BM * a.msub;
         // split-K over the windows (small batches only): windows [j0, j1)
         const int j0 = sp * a.kb_per_split, j1 = min(pm_nj, j0 + a.kb_per_split);
-        int cb = j0 / g.S, r = j0 - cb * g.S;
+        int cb = a.ww ? j0 : j0 / g.S, r = a.ww ? 0 : j0 - cb * g.S;
         for (int j = j0; j < j1; ++j) {
           wc.wait(sbase + SM_AEMPTY + 8 * as, aph ^ 1);
           const uint32_t fa = sbase + SM_AFULL + 8 * as;
@@ -675,31 +694,35 @@ conv_tc_kernel(const __grid_constant__ CUtensorMap tmap_w,
               const int T = (mt * CG + (int)rank) * a.msub + sb, n = T / g.tpi,
                         tb = T - n * g.tpi;
               const int grow = n * g.hv + g.vh + g.psh * tb * g.nseg + r - g.pad;
-              tma_load_3d<CG>(dA + (uint32_t)(sb * pm_sub_rows(g.S) * slab_bytes), &tmap_x, fa,
+              tma_load_3d<CG>(dA + (uint32_t)(sb * a.pm_sub * slab_bytes), &tmap_x, fa,
                               cc, -g.pad, grow);
             }
           } else if (!(a.skip & 1)) {
             const uint32_t dA = sA + as * (uint32_t)a.pm_a_stage;
             const int cc = grp * g.Cg + cb * pm_se, row = i0 + (r - g.pad) * g.wv - g.pad;
             for (int sb = 0; sb < a.msub; ++sb) {
-              const uint32_t d = dA + (uint32_t)(sb * pm_sub_rows(g.S) * slab_bytes);
+              const uint32_t d = dA + (uint32_t)(sb * a.pm_sub * slab_bytes);
               if constexpr (CG == 1) tma_load_2d(d, &tmap_x, fa, cc, row + sb * TC_BM);
               else tma_load_2d_2sm(d, &tmap_x, fa, cc, row + sb * TC_BM);
             }
           }
           advance(as, aph, a.a_stages);
-          for (int s2 = 0; s2 < g.S; ++s2) {
-            wc.wait(sbase + SM_EMPTY + 8 * bs, bph ^ 1);
-            const uint32_t fb = sbase + SM_FULL + 8 * bs;
-            if (rank == 0) mbar_arrive_expect_tx(fb, (a.skip & 2) ? 0 : CG * pm_b_bytes);
-            if (!(a.skip & 2)) {
-              const int kk = (r * g.S + s2) * g.Cg + cb * pm_se;
-              if constexpr (CG == 1) tma_load_2d(sBp + bs * pm_b_bytes, &tmap_w, fb, kk, nrow);
-              else tma_load_2d_2sm(sBp + bs * pm_b_bytes, &tmap_w, fb, kk, nrow);
+          // the window's tap slabs: filter row r (per-row windows) or rows
+          // 0 .. S-1 (whole windows), taps s2 = 0 .. S-1 of each
+          for (int rr = r; rr < (a.ww ? g.S : r + 1); ++rr)
+            for (int s2 = 0; s2 < g.S; ++s2) {
+              wc.wait(sbase + SM_EMPTY + 8 * bs, bph ^ 1);
+              const uint32_t fb = sbase + SM_FULL + 8 * bs;
+              if (rank == 0) mbar_arrive_expect_tx(fb, (a.skip & 2) ? 0 : CG * pm_b_bytes);
+              if (!(a.skip & 2)) {
+                const int kk = (rr * g.S + s2) * g.Cg + cb * pm_se;
+                if constexpr (CG == 1) tma_load_2d(sBp + bs * pm_b_bytes, &tmap_w, fb, kk, nrow);
+                else tma_load_2d_2sm(sBp + bs * pm_b_bytes, &tmap_w, fb, kk, nrow);
+              }
+              advance(bs, bph, a.b_stages);
             }
-            advance(bs, bph, a.b_stages);
-          }
-          if (++r == g.S) { r = 0; ++cb; }
+          if (a.ww) ++cb;
+          else if (++r == g.S) { r = 0; ++cb; }
         }
       }
       if (TC_PROF(a)) {
@@ -1340,7 +1363,11 @@ cudaError_t launch_conv_tc(const ConvGeom &g, int st, const CUtensorMap *tmap_x,
     if (!(ek && ek[0] == '1') && valid_b > 0)
       args.kmma_last = std::min(args.slab_bytes / 32, (valid_b + 31) / 32);
   }
-  args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, g.S, args.msub) : 0;
+  args.ww = g.pm == 1 ? p.ww : 0;
+  args.pm_rows = g.pm ? pm_window_rows(g.S, g.wv, args.ww) : 0;
+  args.pm_sub = (args.pm_rows + 7) / 8 * 8;
+  args.pm_a_stage = g.pm ? pm_a_stage_bytes(args.slab_bytes, args.pm_rows, args.msub) : 0;
+  if (args.ww && (p.splits != 1 || args.pm_rows > 256)) return cudaErrorInvalidValue;
   if (args.msub > 2 || (args.msub == 2 && (!g.pm || p.bn > TC_BN_MAX / 2)) ||
       (g.pm == 2 && (g.nseg < 1 || g.nseg * (g.wv + 2 * g.pad) > TC_BM || g.tpi < 1)))
     return cudaErrorInvalidValue;

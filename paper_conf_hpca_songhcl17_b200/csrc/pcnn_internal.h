@@ -176,6 +176,7 @@ struct TcPlan {
   int rect_w, rect_h, rect_n;  // 0 = im2col A tiles; else rectangle tiles (tiled TMA)
   int a_stages, b_stages;      // padded mode: A (row-window) and B (tap slab) ring depths
   int msub;                    // padded mode: 128-row M sub-tiles per CTA sharing each B slab
+  int ww;                      // padded mode: whole-slab A windows (all S x S taps; no split-K)
   double unit_us;              // modelled time of one work unit on its SM(s) (eq. 12 per wave)
 };
 // Launches the GEMM and, when p.splits > 1, the deterministic split-K
@@ -203,7 +204,10 @@ int tc_slab_bytes(int st, int cg_channels);
 int tc_stages_for(int bn, int cg);
 // padded mode: ring depths for an N tile, CTA grouping, slab width and kernel size
 void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages,
-                  int *b_stages);
+                  int *b_stages, int rows, int ww);
+// padded mode: A window rows per sub-tile, per filter row (ww = 0) or whole
+// (ww = 1: 128 + (S - 1)(wv + 1) rows feed all S x S taps)
+int pm_window_rows(int S, int wv, int ww);
 // debug: per-role barrier-wait cycle totals accumulated while PCNN_TC_PROFILE=1
 cudaError_t tc_profile(int reset, unsigned long long out[32]);
 int tc_block_k_elems(int st);          // K-block in elements (128 B)

@@ -183,6 +183,7 @@ struct pcnn_net {
   int stage_im2col = 0;     // 1: layer 0 input staged as im2col rows (1x1 conv)
   bool fuse_lrn_pool = true;
   bool conv_lrn_pm = false;    // PCNN_FLAG_CONV_LRN_EPILOGUE
+  bool per_row_windows = false; // PCNN_FLAG_PER_ROW_WINDOWS
   bool perf_im2col = false;    // PCNN_FLAG_PERFORATION_IM2COL
   bool census = false;
   // CUDA graph cache
@@ -559,7 +560,8 @@ static const CUtensorMap *stage_tmap(GemmStage &gs, int rows, int slab = 128) {
 
 // TMA im2col map of a stage's NHWC input for `batch` images.
 static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, const TcPlan &p) {
-  const auto key = std::make_tuple(x, batch, p.rect_w, p.rect_h, p.rect_n);
+  // (padded-layout plans have no rectangle: rect_n carries the whole-window flag)
+  const auto key = std::make_tuple(x, batch, p.rect_w, p.rect_h, gs.g.pm ? -1 - p.ww : p.rect_n);
   auto it = gs.xmaps.find(key);
   if (it != gs.xmaps.end()) return &it->second;
   const ConvGeom &g = gs.g;
@@ -595,7 +597,7 @@ static const CUtensorMap *stage_xmap(GemmStage &gs, const void *x, int batch, co
     if (!enct) return nullptr;
     const cuuint64_t d2[2] = {(cuuint64_t)g.Cs, (cuuint64_t)batch * g.hv * g.wv};
     const cuuint64_t s2[1] = {(cuuint64_t)g.Cs * esz};
-    const cuuint32_t box[2] = {(cuuint32_t)(slab / esz), (cuuint32_t)(128 + g.S - 1)};
+    const cuuint32_t box[2] = {(cuuint32_t)(slab / esz), (cuuint32_t)pm_window_rows(g.S, g.wv, p.ww)};
     const cuuint32_t estr[2] = {1, 1};
     const CUtensorMapSwizzle sw = slab == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
                                   : slab == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
@@ -888,7 +890,7 @@ static TcPlan plan_tc(const ConvGeom &g, int device_sms, int kblocks, int esz,
 // (128 + S - 1) A rows once plus S weight slabs and issues S x slab/32 UMMAs;
 // no split-K (a split would need the halo zeroing in the reduction).
 static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n = false,
-                         int want_cg = 0, int want_msub = 0) {
+                         int want_cg = 0, int want_msub = 0, bool per_row = false) {
   TcPlan best{};
   double best_t = 1e300;
   std::vector<std::pair<double, TcPlan>> cands;
@@ -918,6 +920,10 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
     const char *e = exp_env("PCNN_FORCE_SPLIT");
     return e ? atoi(e) : 0;
   }();
+  static const int force_ww = [] {                 // A/B experiments: 0 off, 1 forced
+    const char *e = exp_env("PCNN_WW");
+    return e ? atoi(e) : -1;
+  }();
   const double hbm = 6.0e12;
   for (int ms = 1; ms <= 2; ++ms) {
     if (force_ms && atoi(force_ms) != ms) continue;
@@ -943,33 +949,54 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
         const double last_frac =
             std::min(1.0, std::ceil((double)(creal - (ncb - 1) * se) * esz / 32.0) / (slab / 32.0));
         const double kfrac = ((ncb - 1) + last_frac) / ncb;
-        const double load = (ms * (128.0 + g.S - 1) * slab + (double)g.S * slab * bn / cg) /
-                                kOperandBytesPerCycle + 64.0 * (ms + g.S);
-        const double mma = ms * g.S * (slab / 128.0) * kfrac * 2.05 * bn / kMmaEfficiency;
-        const double j_cycles = std::max(load, mma) + 40.0;
-        for (int want = 1; want <= max_split; ++want) {
-          const int kbs = (nj + want - 1) / want;
-          const int splits = (nj + kbs - 1) / kbs;
-          if (splits != want) continue;
-          if (force_split > 0 && splits != force_split && max_split >= force_split) continue;
-          const long long units = tiles * splits;
-          const long long waves = (units + slots - 1) / slots;
-          double t = (double)waves * kbs * j_cycles / f + 2e-6 * ms;
-          // partials written and summed by the reduction launch
-          if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
-          TcPlan c{};
-          c.cg = cg;
-          c.bn = bn;
-          c.msub = ms;
-          c.mtiles = mtiles;
-          c.ntiles = ntiles;
-          c.tiles = (int)tiles;
-          c.splits = splits;
-          c.kb_per_split = kbs;
-          c.units = (int)units;
-          c.unit_us = ((double)kbs * j_cycles / f + 2e-6 * ms) * 1e6;
-          cands.push_back({t, c});
-          best_t = std::min(best_t, t);
+        // whole windows (ww = 1, no split-K): one A window of 128 + (S-1)(wv+1)
+        // rows per channel slab feeds all S x S taps, instead of S windows of
+        // 128 + S - 1 rows (one per filter row) -- fewer A bytes when wv is
+        // small against 128 (AlexNet conv1-5, VGG-16 conv2-5)
+        for (int ww = 0; ww <= 1; ++ww) {
+          if (ww && (per_row || g.pm != 1 || pm_window_rows(g.S, g.wv, 1) > 256 || g.S < 2 ||
+                     pm_window_rows(g.S, g.wv, 1) >= g.S * (128 + g.S - 1) || force_ww == 0))
+            continue;
+          if (!ww && force_ww == 1 && g.pm == 1 && pm_window_rows(g.S, g.wv, 1) <= 256) continue;
+          const int rows = pm_window_rows(g.S, g.wv, ww);
+          const int taps = ww ? g.S * g.S : g.S, nwin = ww ? nj / g.S : nj;
+          {   // the A ring must hold 2 windows next to 8 tap slabs
+            int na = 0, nb = 0;
+            tc_pm_stages(bn, cg, slab, g.S, ms, &na, &nb, rows, ww);
+            if (na < 2 || nb < (ww ? 8 : 2)) continue;
+          }
+          const double load = (ms * (double)rows * slab + (double)taps * slab * bn / cg) /
+                                  kOperandBytesPerCycle + 64.0 * (ms + taps);
+          const double mma = ms * taps * (slab / 128.0) * kfrac * 2.05 * bn / kMmaEfficiency;
+          // + the issuer's per-tap cost (full-barrier wait, fence, commit; ~100
+          // cycles measured: without it narrow-N whole-window plans, e.g.
+          // AlexNet conv4 512 x 64, model faster than the 256 x 192 that wins)
+          const double j_cycles = std::max(load, mma) + 40.0 + 100.0 * taps;
+          for (int want = 1; want <= (ww ? 1 : max_split); ++want) {
+            const int kbs = (nwin + want - 1) / want;
+            const int splits = (nwin + kbs - 1) / kbs;
+            if (splits != want) continue;
+            if (force_split > 0 && splits != force_split && max_split >= force_split) continue;
+            const long long units = tiles * splits;
+            const long long waves = (units + slots - 1) / slots;
+            double t = (double)waves * kbs * j_cycles / f + 2e-6 * ms;
+            // partials written and summed by the reduction launch
+            if (splits > 1) t += (double)g.M * g.Nfg * g.groups * 4.0 * (splits + 1) / hbm + 3e-6;
+            TcPlan c{};
+            c.cg = cg;
+            c.bn = bn;
+            c.msub = ms;
+            c.ww = ww;
+            c.mtiles = mtiles;
+            c.ntiles = ntiles;
+            c.tiles = (int)tiles;
+            c.splits = splits;
+            c.kb_per_split = kbs;
+            c.units = (int)units;
+            c.unit_us = ((double)kbs * j_cycles / f + 2e-6 * ms) * 1e6;
+            cands.push_back({t, c});
+            best_t = std::min(best_t, t);
+          }
         }
       }
     }
@@ -988,7 +1015,8 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
       best = pc.second;
     }
   }
-  tc_pm_stages(best.bn, best.cg, slab, g.S, best.msub, &best.a_stages, &best.b_stages);
+  tc_pm_stages(best.bn, best.cg, slab, g.S, best.msub, &best.a_stages, &best.b_stages,
+               pm_window_rows(g.S, g.wv, best.ww), best.ww);
   return best;
 }
 
@@ -1102,7 +1130,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
   }
   if (gs.engine == 1) {
     TcPlan p = g.pm ? plan_tc_pm(g, net->num_sms, esz_of(gs.st), lrn != nullptr, ly.plan_cg,
-                                 ly.plan_msub)
+                                 ly.plan_msub, net->per_row_windows)
                     : plan_tc(g, net->num_sms, g.Kpad / tc_block_k_elems(gs.st), esz_of(gs.st),
                               lrn != nullptr, ly.plan_cg);
     // the budget caps concurrent units; a CTA pair needs at least 2 SMs
@@ -1121,6 +1149,7 @@ static pcnn_status run_stage(pcnn_net *net, Layer &ly, GemmStage &gs, int B, con
       info->engine = 1;
       info->splits = p.splits;
       info->a_mode = g.pm ? 2 : (p.rect_w ? 1 : 0);
+      info->whole_window = p.ww;
       info->n_sms = std::max(info->n_sms, p.grid);   // pair granularity
       info->cta_group = p.cg;
       info->t_unit_us = p.unit_us;
@@ -1525,6 +1554,7 @@ pcnn_status pcnn_create_net(const pcnn_net_desc *desc, const pcnn_layer_desc *la
   net->fuse_lrn_pool = !(desc->flags & PCNN_FLAG_NO_LRN_POOL_FUSION);
   net->conv_lrn_pm = (desc->flags & PCNN_FLAG_CONV_LRN_EPILOGUE) != 0;
   net->perf_im2col = (desc->flags & PCNN_FLAG_PERFORATION_IM2COL) != 0;
+  net->per_row_windows = (desc->flags & PCNN_FLAG_PER_ROW_WINDOWS) != 0;
   if (desc->precision != PCNN_FP32_SIMT) {
     if (!get_encode_tiled() || !get_encode_im2col())
       return fail(PCNN_ERR_CUDA, "driver entry points cuTensorMapEncode{Tiled,Im2col} unavailable");

@@ -30,6 +30,7 @@ FLAG_NO_SPACE_TO_DEPTH = 1
 FLAG_NO_PADDED_LAYOUT = 2
 FLAG_NO_LRN_POOL_FUSION = 4
 FLAG_CONV_LRN_EPILOGUE = 8
+FLAG_PER_ROW_WINDOWS = 64
 FLAG_NARROW_SLABS = 16
 FLAG_PERFORATION_IM2COL = 32
 PRECISIONS = {"fp32": FP32_SIMT, "fp32_simt": FP32_SIMT, "tf32": TF32, "bf16": BF16}
@@ -63,7 +64,8 @@ class LayerInfo(ctypes.Structure):
                 ("tile_n", ctypes.c_int), ("tiles", ctypes.c_longlong), ("grid", ctypes.c_int),
                 ("util", ctypes.c_double), ("rec", ctypes.c_double), ("splits", ctypes.c_int),
                 ("a_mode", ctypes.c_int), ("halo_in", ctypes.c_int), ("halo_out", ctypes.c_int),
-                ("cta_group", ctypes.c_int), ("t_unit_us", ctypes.c_double)]
+                ("cta_group", ctypes.c_int), ("t_unit_us", ctypes.c_double),
+                ("whole_window", ctypes.c_int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

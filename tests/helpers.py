@@ -11,6 +11,7 @@ FLAG_NO_SPACE_TO_DEPTH = 1
 FLAG_NO_PADDED_LAYOUT = 2
 FLAG_NO_LRN_POOL_FUSION = 4
 FLAG_CONV_LRN_EPILOGUE = 8
+FLAG_PER_ROW_WINDOWS = 64
 FLAG_NARROW_SLABS = 16
 FLAG_PERFORATION_IM2COL = 32
 

@@ -6,8 +6,8 @@ import numpy as np
 import pytest
 
 from tests.helpers import (FLAG_CONV_LRN_EPILOGUE, FLAG_NARROW_SLABS, FLAG_NO_LRN_POOL_FUSION,
-                           FLAG_NO_PADDED_LAYOUT, FLAG_PERFORATION_IM2COL, TOL, conv_layer,
-                           gpu_run, params, rel_err, small_inputs)
+                           FLAG_NO_PADDED_LAYOUT, FLAG_PER_ROW_WINDOWS, FLAG_PERFORATION_IM2COL,
+                           TOL, conv_layer, gpu_run, params, rel_err, small_inputs)
 
 pytestmark = pytest.mark.gpu
 
@@ -187,3 +187,30 @@ def test_padded_mode_skips_channel_padding(orc, prec):
     assert rel_err(fast["out"], ref) <= TOL[prec] / 2
     narrow = gpu_run(net, w, b, x, prec, flags=FLAG_NARROW_SLABS)["out"]
     assert rel_err(fast["out"], narrow) <= TOL[prec] / 8
+
+
+@pytest.mark.parametrize("prec", ["bf16", "tf32"])
+@pytest.mark.parametrize("shape,cout,k,groups,B", [
+    ((256, 13, 13), 384, 3, 1, 16),     # AlexNet conv3 (14-wide shared-halo grid)
+    ((384, 13, 13), 256, 3, 2, 16),     # conv5, grouped
+    ((64, 23, 23), 96, 3, 1, 24),       # narrow N, several windows per image row
+])
+def test_whole_window_bitwise_equals_per_row_windows(orc, prec, shape, cout, k, groups, B):
+    """Whole-slab A windows (one TMA window of 128 + (S-1)(wv+1) rows feeds
+    all S x S taps) change only which shared-memory rows each tap's UMMA
+    reads: the K order (slab, filter row, tap) is the per-row mode's, so the
+    result is bitwise the same; and the oracle's tolerance."""
+    C = shape[0]
+    net = dict(in_shape=shape, layers=[dict(kind="maxpool", k=1, stride=1),
+                                       conv_layer(cout, k, C, 1, k // 2, groups),
+                                       dict(kind="maxpool", k=1, stride=1)])
+    w, b = params(net, seed=31)
+    x = small_inputs(shape, B, lo=-4, hi=4)
+    ww = gpu_run(net, w, b, x, prec)
+    pr = gpu_run(net, w, b, x, prec, flags=FLAG_PER_ROW_WINDOWS)
+    fw, fr = ww["net"].query_layer(1, B), pr["net"].query_layer(1, B)
+    assert fw["a_mode"] == 2 and fr["a_mode"] == 2
+    assert fw["whole_window"] == 1 and fr["whole_window"] == 0
+    np.testing.assert_array_equal(ww["out"], pr["out"])
+    ref = orc.run_net(net, w, b, x[:2]).reshape(2, -1)
+    assert rel_err(ww["out"][:2], ref) <= TOL[prec] / 4

@@ -32,7 +32,7 @@ def run(li):
 
 for name in names:
     li = idx[name]
-    for cg, ms_ in [(0, 0), (2, 1), (2, 2), (1, 1), (1, 2)]:
+    for cg, ms_ in [(0, 0), (2, 1), (2, 2), (1, 1), (1, 2)]:  # (0, 0): the planner's choice
         try:
             n.set_layer_plan(li, cg, ms_)
         except Exception as e:
