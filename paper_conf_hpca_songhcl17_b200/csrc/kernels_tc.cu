@@ -102,7 +102,7 @@ void tc_pm_stages(int bn, int cg, int slab_bytes, int S, int msub, int *a_stages
   // slabs carry 2-4x less work per stage and get deeper rings.  Whole windows
   // keep >= 8 tap slabs in flight (a window's S*S slabs stream through them).
   int na = slab_bytes == 128 ? 4 : TC_MAX_ASTAGES;
-  const int bmin = ww ? 8 : 2 * S;
+  const int bmin = ww ? 6 : 2 * S;
   while (na > 2 && na * as_bytes + bmin * bs_bytes > TC_STAGE_BUDGET) --na;
   int nb = (TC_STAGE_BUDGET - na * as_bytes) / bs_bytes;
   const int nb_max = slab_bytes == 128 && !ww ? TC_MAX_STAGES : TC_MAX_BSTAGES;

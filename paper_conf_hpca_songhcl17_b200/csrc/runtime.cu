@@ -963,7 +963,7 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
           {   // the A ring must hold 2 windows next to 8 tap slabs
             int na = 0, nb = 0;
             tc_pm_stages(bn, cg, slab, g.S, ms, &na, &nb, rows, ww);
-            if (na < 2 || nb < (ww ? 8 : 2)) continue;
+            if (na < 2 || nb < (ww ? 6 : 2)) continue;
           }
           const double load = (ms * (double)rows * slab + (double)taps * slab * bn / cg) /
                                   kOperandBytesPerCycle + 64.0 * (ms + taps);
