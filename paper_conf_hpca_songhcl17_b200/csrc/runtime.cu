@@ -915,11 +915,16 @@ static TcPlan plan_tc_pm(const ConvGeom &g, int device_sms, int esz, bool full_n
                             ((g.Nfg + bn - 1) / bn) * g.groups;
         if (t >= device_sms / cg) can_fill = true;
       }
-  const int max_split = (can_fill || full_n || g.pm != 1) ? 1 : std::min(16, nj);
+  // Measured (tools/exp_b1_split.sh, AlexNet B = 1, graph replay): the
+  // split-K plans' partial epilogues and reduction launches cost more than the
+  // extra CTAs gain (0.124 vs 0.1205 ms per pass), so padded-layout plans do
+  // not split K; the experiments build can still force a split.
   static const int force_split = [] {              // tuning experiments
     const char *e = exp_env("PCNN_FORCE_SPLIT");
     return e ? atoi(e) : 0;
   }();
+  const int max_split =
+      (can_fill || full_n || g.pm != 1 || force_split <= 1) ? 1 : std::min(16, nj);
   static const int force_ww = [] {                 // A/B experiments: 0 off, 1 forced
     const char *e = exp_env("PCNN_WW");
     return e ? atoi(e) : -1;
