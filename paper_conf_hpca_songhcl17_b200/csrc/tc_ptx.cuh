@@ -53,6 +53,14 @@ __device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap *map, int c0, 
                : "memory");
 }
 
+__device__ __forceinline__ void tma_prefetch_4d(const CUtensorMap *map, int c0, int c1, int c2,
+                                                int c3) {
+  asm volatile("cp.async.bulk.prefetch.tensor.4d.L2.global.tile [%0, {%1, %2, %3, %4}];" ::"l"(
+                   (uint64_t)map),
+               "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
+
 // TMA im2col load of one A slab: 128 output pixels starting at (w, h, n)
 // (input-space corner of the first pixel), channels [c, c + slab), filter tap
 // offsets (ow, oh); padding / out-of-range pixels are zero-filled.
@@ -178,16 +186,6 @@ __device__ __forceinline__ void tc_commit(uint32_t bar) {
         "h"((uint16_t)0x3)
         : "memory");
   }
-}
-
-// cta_group::2 commit arriving on the barrier at this offset in both CTAs of
-// the pair whose leader has cluster rank `lead` (clusters of several pairs)
-__device__ __forceinline__ void tc_commit_pair(uint32_t bar, uint32_t lead) {
-  asm volatile(
-      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
-      " [%0], %1;" ::"r"(bar),
-      "h"((uint16_t)(0x3u << lead))
-      : "memory");
 }
 
 __device__ __forceinline__ uint32_t cluster_ctarank() {
