@@ -72,6 +72,9 @@ def parse():
                     help="profiling: only the warm-up and the timed steps of the main workload "
                          "(no graph-replay pass, e2e, energy, sweep or extras)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--nccl", action="store_true",
+                    help="run the NCCL data path (weight broadcast, logits all-gather) even on "
+                         "one rank")
     a = ap.parse_args()
     if a.batch is None:
         a.batch = 256 if a.net == "alexnet" else 64
@@ -246,21 +249,22 @@ def run_reference(a):
 class Ctx:
     """Process-group state shared by the measurements."""
 
-    def __init__(self, world, rank, local):
+    def __init__(self, world, rank, local, dist_on=None):
         import torch
         import torch.distributed as dist
         self.torch, self.dist = torch, dist
         self.world, self.rank, self.local = world, rank, local
+        self.dist_on = world > 1 if dist_on is None else dist_on   # NCCL group initialised
         self.stream = torch.cuda.current_stream()
         self.peaks, self.peak_src = measured_peaks()
 
     def barrier(self):
-        if self.world > 1:
+        if self.dist_on:
             self.dist.barrier()
 
     def max_over_ranks(self, v):
         t = self.torch.tensor([float(v)], device="cuda")
-        if self.world > 1:
+        if self.dist_on:
             self.dist.all_reduce(t, op=self.dist.ReduceOp.MAX)
         return float(t.item())
 
@@ -360,7 +364,7 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
             raise SystemExit("--global-batch must be a multiple of the GPU count")
     else:
         start = rank * B
-    if world > 1:
+    if ctx.dist_on:
         w, b, bcast_ms = pdist.broadcast_params(net, rank)
     else:
         w, b = synth.net_params(net)
@@ -371,11 +375,11 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
     out = torch.empty((B, n.out_elems), device="cuda")
     probs = torch.empty_like(out)
     ent = torch.empty((B,), device="cuda")
-    gathered = torch.empty((world * B, n.out_elems), device="cuda") if world > 1 else None
+    gathered = torch.empty((world * B, n.out_elems), device="cuda") if ctx.dist_on else None
 
     def step():
         n.infer(x, out, probs, ent, stream=ctx.stream)
-        if world > 1:
+        if ctx.dist_on:
             ctx.dist.all_gather_into_tensor(gathered, out)        # C3: logits gather
 
     for _ in range(warmup):
@@ -395,7 +399,7 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
     n.set_layer_timing(False)
     layer_ms, nsteps = n.read_layer_timing()
     torch.cuda.synchronize()
-    logits = (gathered if world > 1 else out).cpu().numpy()
+    logits = (gathered if ctx.dist_on else out).cpu().numpy()
     infos = [n.query_layer(i, B) for i in range(n.n_layers)]
     per_layer = layer_rooflines(n, net, infos, layer_ms, nsteps, precision, ctx.peaks,
                                 ctx.peak_src)
@@ -426,7 +430,7 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
         oh = torch.empty((B, n.out_elems)).pin_memory()
         ph = torch.empty((B, n.out_elems)).pin_memory()
         hh = torch.empty((B,)).pin_memory()
-        og = torch.empty((B, n.out_elems), device="cuda") if world > 1 else None
+        og = torch.empty((B, n.out_elems), device="cuda") if ctx.dist_on else None
         px_host = synth.pixels(start, B, net["in_shape"])
         forms = {
             "u8": (torch.from_numpy(px_host).pin_memory(),
@@ -448,7 +452,7 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
             e2e_steps = max(3, min(steps, 20))
             for _ in range(e2e_steps):
                 call()
-                if world > 1:   # gather THIS step's logits (re-uploaded from the host result)
+                if ctx.dist_on:   # gather THIS step's logits (re-uploaded from the host result)
                     og.copy_(oh, non_blocking=True)
                     ctx.dist.all_gather_into_tensor(gathered, og)
                     torch.cuda.synchronize()
@@ -458,9 +462,9 @@ def measure(ctx, net_name, precision, B, steps, warmup, sampler=None, e2e=False,
             e2e_res[form] = {
                 "value": round(world * B * e2e_steps / te, 1), "unit": "images/sec",
                 "h2d_bytes_per_step": int(xh.numel() * xh.element_size() +
-                                          (oh.numel() * 4 if world > 1 else 0)),
+                                          (oh.numel() * 4 if ctx.dist_on else 0)),
                 "d2h_bytes_per_step": int(oh.numel() * 4 + ph.numel() * 4 + hh.numel() * 4),
-                "api": api + (" + all_gather of the step's logits" if world > 1 else "")}
+                "api": api + (" + all_gather of the step's logits" if ctx.dist_on else "")}
         res["e2e"] = dict(e2e_res["u8"])
         res["e2e"]["fp32_images"] = e2e_res["f32"]
     return res, n, (net, w, b), (x, out, probs, ent)
@@ -518,14 +522,18 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
-    if world > 1:
+    use_dist = world > 1 or a.nccl
+    if use_dist:
+        if "MASTER_ADDR" not in os.environ:     # --nccl without torchrun: a 1-rank group
+            os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=os.environ.get("MASTER_PORT", "29533"),
+                              RANK="0", WORLD_SIZE="1", LOCAL_RANK="0")
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     from paper_conf_hpca_songhcl17_b200 import dist as pdist
     from paper_conf_hpca_songhcl17_b200 import tuning as ptuning
     pdist.check_world(a.gpus) if world > 1 else None
     if world == 1 and a.gpus != 1:
         raise SystemExit("--gpus %d but WORLD_SIZE=1" % a.gpus)
-    ctx = Ctx(world, rank, local)
+    ctx = Ctx(world, rank, local, dist_on=use_dist)
 
     sampler = ClockSampler(local)
     sampler.start()
@@ -539,7 +547,7 @@ def main():
                               "ms_per_step": main_res["ms_per_step"], "minimal": True,
                               "per_layer": main_res["per_layer"]}))
         n.close()
-        if world > 1:
+        if use_dist:
             dist.destroy_process_group()
         return
     B = main_res["batch_per_gpu"]
@@ -570,6 +578,7 @@ def main():
         "unit": "images/sec",
         "n_gpus": world,
         "gpus_active": world,
+        "nccl": bool(use_dist),
         "steps": a.steps,
         "warmup": a.warmup,
         "ms_per_step": main_res["ms_per_step"],
@@ -626,7 +635,7 @@ def main():
         res["cpu_baseline"] = cpu_baseline(net, w, b, a.cpu_seconds)
     if rank == 0:
         print(json.dumps(res))
-    if world > 1:
+    if use_dist:
         dist.destroy_process_group()
 
 
