@@ -2232,14 +2232,15 @@ static pcnn_status infer_host_impl(pcnn_net *net, const float *h_images,
     CUDA_TRY(cudaMemcpyAsync(net->d_mean, m.data(), sizeof(float) * C, cudaMemcpyHostToDevice, s));
   }
   const size_t in_bytes = u8 ? 1 : sizeof(float);
-  // When the images take long to cross PCIe (~50 GB/s) compared with the
+  // When the images take long to cross PCIe (25-50 GB/s pinned) compared with the
   // inference (FLOPs at ~700 TFLOP/s), split the batch into 4 chunks: chunk
   // i+1's host->device copy (own stream) overlaps chunk i's inference.
   // Images are independent, so the chunks compute the same per-image results.
   double flops = 0;
   for (auto &ly : net->layers) flops += layer_flops_exact(ly, 1);
   const double h2d_img = in_bytes * in_elems / 50e9, comp_img = flops / 7e14;
-  const int k = (batch >= 64 && h2d_img > (u8 ? 0.25 : 2.0) * comp_img) ? 4 : 1;
+  int k = (batch >= 64 && h2d_img > (u8 ? 0.25 : 2.0) * comp_img) ? 4 : 1;
+  if (const char *e = exp_env("PCNN_H2D_CHUNKS")) k = std::max(1, std::min(4, atoi(e)));   // experiments
   const int chunk = (batch + k - 1) / k;
   if (k > 1 && !net->copy_stream) {
     CUDA_TRY(cudaStreamCreateWithFlags(&net->copy_stream, cudaStreamNonBlocking));
