@@ -1466,6 +1466,59 @@ __global__ void __launch_bounds__(256, MINB) lrn_reg_kernel(const LrnPoolArgs a)
     const float inv_gp = grp_pad > 0 ? 1.f / (float)grp_pad : 0.f;
     const int nq = a.Wo * ochunks;
     const float inv_nq = 1.f / (float)nq;
+    if (ST == ST_BF16 && a.is_max && a.k == 3 && a.s == 2 && (a.Wo - 1) * 2 + 3 <= a.W &&
+        (p1 - 1) * 2 + 3 - h0 <= nr) {
+      // AlexNet's 3 x 3 / 2 max pool, no window clipped in this band: a thread
+      // owns one output column chunk and walks down the band's output rows;
+      // the horizontal 3-max of a window's last row is the next window's
+      // first (6 instead of 9 smem reads per output; max is exact, so the
+      // result is the general path's bit for bit)
+      const size_t orow = (size_t)Wop * a.Cout * ESZ;
+      for (int v = threadIdx.x; v < nq; v += blockDim.x) {
+        int q, oc;
+        fdivmod(v, ochunks, inv_oc, q, oc);
+        int c = oc;
+        bool pad = false;
+        if (grp_pad > 0) {
+          int gi, j;
+          fdivmod(oc, grp_pad, inv_gp, gi, j);
+          pad = j >= grp_real;
+          c = gi * grp_real + j;
+        }
+        char *dst = (char *)a.y + ((((size_t)n * Hop + p0) * Wop + q) * a.Cout + oc * VN) * ESZ;
+        if (pad) {
+          for (int pp = p0; pp < p1; ++pp, dst += orow) *(uint4 *)dst = make_uint4(0, 0, 0, 0);
+          continue;
+        }
+        auto hrow = [&](int r) {                // max over the window's 3 columns of row r
+          __nv_bfloat162 m[4];
+#pragma unroll
+          for (int dc = 0; dc < 3; ++dc) {
+            const int pix = r * a.W + 2 * q + dc;
+            const uint4 raw = *(const uint4 *)(lr_smem + ((size_t)pix * chunks + slot(pix, c)) * 16);
+            const __nv_bfloat162 *h = (const __nv_bfloat162 *)&raw;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) m[j] = dc ? __hmax2(m[j], h[j]) : h[j];
+          }
+          return *(const uint4 *)m;
+        };
+        auto max4 = [](uint4 x, uint4 y) {
+          __nv_bfloat162 *a2 = (__nv_bfloat162 *)&x;
+          const __nv_bfloat162 *b2 = (const __nv_bfloat162 *)&y;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) a2[j] = __hmax2(a2[j], b2[j]);
+          return x;
+        };
+        uint4 carry = hrow(p0 * 2 - h0);
+        for (int pp = p0; pp < p1; ++pp, dst += orow) {
+          const int r0 = pp * 2 - h0;
+          const uint4 r2 = hrow(r0 + 2);
+          *(uint4 *)dst = max4(max4(carry, hrow(r0 + 1)), r2);
+          carry = r2;
+        }
+      }
+      return;
+    }
     for (int v = threadIdx.x; v < (p1 - p0) * nq; v += blockDim.x) {
       int rr, q, oc;
       if (nq <= 1024) fdivmod(v, nq, inv_nq, rr, q);   // fdivmod's exact range
