@@ -655,6 +655,7 @@ constexpr long long kBandTargetCtas = 2 * 148;
 #ifndef PCNN_S2D_ROWS_DEFAULT
 #define PCNN_S2D_ROWS_DEFAULT 4
 #endif
+
 template <int ST>
 __global__ void __launch_bounds__(256, PCNN_S2D_MINB)
 stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int Hs, int Ws,
