@@ -59,7 +59,7 @@ for tag in ("alexnet_b256", "alexnet_b1", "vgg16_b64"):
     with open(os.path.join(OUT, "%s_launches_%s.csv" % (RND, tag)), "w") as f:
         f.write("kernel,us_median,share_of_step\n")
         for k, v in step:
-            f.write("%s,%.2f,%.4f\n" % (k, v, v / tot))
+            f.write("\"%s\",%.2f,%.4f\n" % (k, v, v / tot))
     summary[tag] = {"steps": nsteps, "launches_per_step": len(step), "sum_us": round(tot, 1),
                     "kernels": [[k, round(v, 2)] for k, v in step]}
 
@@ -87,7 +87,7 @@ if os.path.exists(full):
     with open(os.path.join(OUT, "%s_ncu_full_alexnet_b256.csv" % RND), "w") as f:
         f.write("kernel,grid,dur_us,dram_bytes,tensor_pipe_pct,dram_pct,regs\n")
         for d in out:
-            f.write("%s,\"%s\",%.2f,%d,%.1f,%.1f,%d\n" % (d["kernel"], d["grid"], d["dur_us"],
+            f.write("\"%s\",\"%s\",%.2f,%d,%.1f,%.1f,%d\n" % (d["kernel"], d["grid"], d["dur_us"],
                                                         d["dram_bytes"], d["tensor_pct"],
                                                         d["dram_pct"], d["regs"]))
     conv = [d for d in out if d["kernel"].startswith("conv_tc")]
@@ -119,7 +119,7 @@ if os.path.exists(other):
         for r in rows[2:]:
             d = {k: (r[i] if i >= 0 else "0") for k, i in zip(keys, idx)}
             mb = lambda x: float(x) * (1e6 if "Mbyte" in units[3] else 1e9 if "Gbyte" in units[3] else 1e3)
-            f.write("%s,\"%s\",%.2f,%d,%.1f,%.1f,%.1f,%d\n" % (
+            f.write("\"%s\",\"%s\",%.2f,%d,%.1f,%.1f,%.1f,%d\n" % (
                 short(d["Kernel Name"]), d["Grid Size"], float(d["gpu__time_duration.sum"]),
                 int(mb(d["dram__bytes_read.sum"]) + mb(d["dram__bytes_write.sum"])),
                 float(d["gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"]),
