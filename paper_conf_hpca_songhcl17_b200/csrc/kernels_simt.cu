@@ -655,6 +655,9 @@ constexpr long long kBandTargetCtas = 2 * 148;
 #ifndef PCNN_S2D_ROWS_DEFAULT
 #define PCNN_S2D_ROWS_DEFAULT 4
 #endif
+#ifndef PCNN_S2D_NBUF
+#define PCNN_S2D_NBUF 2
+#endif
 
 template <int ST>
 __global__ void __launch_bounds__(256, PCNN_S2D_MINB)
@@ -667,16 +670,17 @@ stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int
   extern __shared__ __align__(128) uint8_t s2_smem[];
   const int pitch = ((W + 3) / 4 + 1) * 4;            // floats per smem row (16 B multiple)
   const int rows = R * BLK * C;
-  float *bufs = (float *)s2_smem;                     // [2][rows][pitch]
-  uint64_t *bar = (uint64_t *)(s2_smem + (size_t)2 * rows * pitch * 4);
-  int *shift = (int *)(bar + 2);                      // [2][rows]: start offset, -1 = zero row
+  constexpr int NB = PCNN_S2D_NBUF;                   // band buffers in flight
+  float *bufs = (float *)s2_smem;                     // [NB][rows][pitch]
+  uint64_t *bar = (uint64_t *)(s2_smem + (size_t)NB * rows * pitch * 4);
+  int *shift = (int *)(bar + NB);                     // [NB][rows]: start offset, -1 = zero row
   const int bands = (Hs + R - 1) / R;
   const long long tiles = (long long)B * bands;
   const uintptr_t xend = (uintptr_t)(x + (size_t)B * C * H * W);
   const uint32_t bar0 = (uint32_t)__cvta_generic_to_shared(bar);
   if (threadIdx.x == 0) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0));
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8));
+#pragma unroll
+    for (int i = 0; i < NB; ++i) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar0 + 8 * i));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -687,10 +691,16 @@ stage_s2d4_kernel(const float *__restrict__ x, void *y, int B, int H, int W, int
               shift + b * rows, pitch, bar0 + 8 * b);
   };
   long long t = blockIdx.x;
-  if (threadIdx.x < 32 && t < tiles) issue(t, 0);
-  uint32_t phase[2] = {0, 0};
-  for (int b = 0; t < tiles; t += gridDim.x, b ^= 1) {
-    if (threadIdx.x < 32 && t + gridDim.x < tiles) issue(t + gridDim.x, b ^ 1);
+  if (threadIdx.x < 32)
+    for (int i = 0; i < NB - 1; ++i)
+      if (t + (long long)i * gridDim.x < tiles) issue(t + (long long)i * gridDim.x, i);
+  uint32_t phase[NB] = {};
+  for (int b = 0; t < tiles; t += gridDim.x, b = b + 1 == NB ? 0 : b + 1) {
+    {   // the band NB - 1 tiles ahead goes into the buffer freed last iteration
+      const long long ta = t + (long long)(NB - 1) * gridDim.x;
+      const int ba = (b + NB - 1) % NB;
+      if (threadIdx.x < 32 && ta < tiles) issue(ta, ba);
+    }
     {
       const uint32_t bb = bar0 + 8 * b, par = phase[b];
       asm volatile(
@@ -755,7 +765,7 @@ static cudaError_t launch_stage_s2d4(const float *x, void *y, int st, int B, int
   int R = R3;                                        // small batches: shorter bands
   while (R > 1 && (long long)B * ((Hs + R - 1) / R) < kBandTargetCtas) --R;
   const int pitch = ((W + 3) / 4 + 1) * 4;
-  const size_t smem = (size_t)2 * R * 12 * pitch * 4 + 16 + 2 * R * 12 * 4;
+  const size_t smem = (size_t)PCNN_S2D_NBUF * (R * 12 * pitch * 4 + 8 + R * 12 * 4);
   if (smem > 200 * 1024) return cudaErrorInvalidValue;
   const long long tiles = (long long)B * ((Hs + R - 1) / R);
   int dev = 0, sms = 148, occ = 1;
