@@ -33,7 +33,13 @@ SHAPES = {  # name: (in_shape, layer)
 }
 def make_net(name):
     """name[+pm]: '+pm' wraps the conv between identity pools so the runtime
-    may choose the padded-layout mode (it needs pool / pm-conv neighbours)."""
+    may choose the padded-layout mode (it needs pool / pm-conv neighbours).
+    'alexnet_head': AlexNet's conv1 -> norm1 -> pool1 as the full net runs them
+    (space-to-depth staging, padded-layout conv1)."""
+    if name == "alexnet_head":
+        import synth
+        net = synth.alexnet()
+        return net["in_shape"], dict(in_shape=net["in_shape"], layers=net["layers"][:3]), 0
     wrap = name.endswith("+pm")
     shape, L = SHAPES[name[:-3] if wrap else name]
     layers = L if isinstance(L, list) else [L]
