@@ -777,11 +777,11 @@ static const CUtensorMap *stage_ymap(GemmStage &gs, void *y, long long M,
 // ~80% of its nominal rate in this kernel.
 static constexpr double kOperandBytesPerCycle = 36.0;
 // eq. 12 time-model constants (NEXT-3; fitted, see layer_time_model)
-static constexpr double kT0Conv = 13.07, kScaleConv = 0.534;   // tcgen05 conv: launch us, unit scale
+static constexpr double kT0Conv = 14.58, kScaleConv = 0.4985;   // tcgen05 conv: launch us, unit scale
 // (profiles/r02_time_model_fit.json; measured with live per-layer events,
 // which serialise launches -- inside a CUDA graph with PDL the launch term
 // mostly overlaps the previous layer)
-static constexpr double kT0Fc = 15.22, kScaleFc = 0.745;   // weight-streaming FC
+static constexpr double kT0Fc = 15.08, kScaleFc = 0.699;   // weight-streaming FC
 static constexpr double kT0Simt = 3.0;                     // SIMT kernels (LRN / pool / check path)
 static constexpr double kMmaEfficiency = 0.8;
 
